@@ -1,0 +1,362 @@
+#!/usr/bin/env python
+"""Benchmark of the GPU Dedup hot path (Rabin CDC -> SHA-1 -> global dedup).
+
+Contract (README / DESIGN.md "Measurement"):
+  python bench.py --gpus N --steps K --warmup W [--impl b200|reference]
+prints ONE JSON line on rank 0.
+
+A step is one pass of the whole hot path (rows A1-A9 of SURVEY 8(a)) over
+one GPU batch of the BASELINE.json configs[1] workload: the 184 MiB
+simlarge-sized synthetic stream (1 MiB items, ~50 % duplicate chunks),
+cycled; at every wrap of the stream a new dedup stream (fresh digest table)
+starts.  `value` is input GB/s (1e9 B/s) with the stream resident in HBM
+(device-timed with CUDA events around submit..drain); `e2e` is the same
+metric through dedup_submit_batch with pinned HOST buffers (H2D and the
+result read-back inside the timed region).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+import synthgen  # noqa: E402
+
+MiB = 1 << 20
+ITEM_BYTES = MiB                 # the paper's fixed 1 MB batches
+BATCH_BYTES = 32 * MiB           # GPU batch (step); C2 batch sweep 1-64 MiB
+BATCH_ITEMS = 64
+SLOTS = 6
+WORKLOAD = "C2"
+METRIC = "input GB/s & chunks/s (dedup hot path) at 1/2/4/8 B200; % of HBM/INT roofline"
+
+# SHA-1 algorithmic 32-bit integer ops per 64-byte block (FIPS 180-4 6.1.2,
+# counting a 3-input logic/add as one op and a rotate as one op):
+#   80 rounds x (f 1 + rotl5 1 + adds 2 + rotl30 1) + 64 x schedule 3 + 5.
+SHA1_OPS_PER_BLOCK = 80 * 5 + 64 * 3 + 5
+# alu-pipe peak (LOP3/SHF/IADD3/PRMT): 148 SM x 4 SMSP x 16 lanes/clk
+ALU_LANES_PER_SM_CLK = 64
+
+
+def engine_kwargs(stream_bytes: int) -> dict:
+    return dict(batch_bytes=BATCH_BYTES, batch_items=BATCH_ITEMS, slots=SLOTS,
+                table_capacity=max(1 << 16, stream_bytes // 2048), host_fed=True)
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d, "measured"
+    return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}, "fallback"
+
+
+class ClockSampler:
+    """NVML sampling of SM clock + throttle reasons during the timed region."""
+
+    REASONS = {
+        0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+        0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+        0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
+        0x100: "display_clock_setting"}
+
+    def __init__(self, device: int):
+        self.samples, self.reasons, self._stop = [], set(), threading.Event()
+        self.max_mhz = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(device)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.nv = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksThrottleReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit and bit != 0x1:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(0.005)
+
+    def __enter__(self):
+        if self.nv is not None:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self.nv is not None:
+            self._t.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
+                    "samples": 0}
+        return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def plan_batches(off):
+    out, k, n = [], 0, len(off) - 1
+    while k < n:
+        j = k + 1
+        while j < n and j - k < BATCH_ITEMS and int(off[j + 1]) - int(off[k]) <= BATCH_BYTES:
+            j += 1
+        out.append((k, j))
+        k = j
+    return out
+
+
+def run_steps(d, submit, n_batches, steps, first_step):
+    """Submit `steps` consecutive steps (batches, cycling the stream)."""
+    for s in range(first_step, first_step + steps):
+        b = s % n_batches
+        if b == 0 and s > 0:
+            d.end_stream()
+        while True:
+            try:
+                submit(b)
+                break
+            except Exception as e:
+                if "EAGAIN" not in str(e):
+                    raise
+                d.drain_raw(wait_ms=-1)
+    while d.pending():
+        d.drain_raw(wait_ms=-1)
+
+
+def stat_delta(a, b):
+    return {k: b[k] - a[k] for k in a if isinstance(a[k], (int, float))}
+
+
+def cpu_baseline(data, off, seconds_budget=12.0):
+    """The oracle as it stands, 1 host thread, on a bounded prefix sample."""
+    import oracle
+    t_total, nbytes, items = 0.0, 0, 0
+    st = oracle.Stream()
+    k = 0
+    n = len(off) - 1
+    while k < n and t_total < seconds_budget:
+        it = data[int(off[k]):int(off[k + 1])]
+        t0 = time.perf_counter()
+        st.item(k, it)
+        t_total += time.perf_counter() - t0
+        nbytes += len(it)
+        items += 1
+        k += 1
+    c = st.counts()
+    st.close()
+    return {"value": nbytes / t_total / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle",
+            "sample": f"first {items} items ({nbytes / MiB:.0f} MiB) of the {WORKLOAD} stream, "
+                      f"sequential C++ oracle (chunk+SHA-1+dedup), {c['chunks']} chunks",
+            "chunks_per_s": c["chunks"] / t_total}
+
+
+def reference_arm(args, data, off):
+    """--impl reference: the oracle on the host cores, same metric/config."""
+    import oracle
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    n = len(off) - 1
+    total_steps = args.steps + args.warmup
+    budget_bytes = 60.0 * 60e6       # ~60 s of oracle work (~60 MB/s) over the whole run
+    per_step_items = max(1, min(BATCH_ITEMS, int(budget_bytes / max(total_steps, 1) / ITEM_BYTES)))
+    st = oracle.Stream()
+    k, seq = 0, 0
+    t_timed, bytes_timed, chunks_timed = 0.0, 0, 0
+    for s in range(total_steps):
+        t0 = time.perf_counter()
+        nb = nc = 0
+        for _ in range(per_step_items):
+            if k == n:
+                st.close()
+                st = oracle.Stream()
+                k = 0
+            it = data[int(off[k]):int(off[k + 1])]
+            r = st.item(seq, it)
+            nb += len(it)
+            nc += len(r.chunk_start)
+            k += 1
+            seq += 1
+        dt = time.perf_counter() - t0
+        if s >= args.warmup:
+            t_timed += dt
+            bytes_timed += nb
+            chunks_timed += nc
+    st.close()
+    v = bytes_timed / t_timed / 1e9
+    line = {
+        "impl": "reference", "metric": METRIC, "value": v, "unit": "GB/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": 1e3 * t_timed / max(args.steps, 1), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "chunks_per_s": chunks_timed / t_timed,
+        "config": {"workload": f"{WORKLOAD}: 184 MiB simlarge-sized stream, 1 MiB items, "
+                               "dup_frac 0.52", "step_sample_items": per_step_items},
+        "cpu_baseline": {"value": v, "unit": "GB/s", "cores": 1, "kind": "oracle",
+                         "sample": f"{per_step_items} x 1 MiB items per step, cycling the "
+                                   f"{WORKLOAD} stream"},
+        "e2e": {"value": v, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=600)
+    ap.add_argument("--warmup", type=int, default=12)
+    ap.add_argument("--impl", default="b200", choices=["b200", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=0, help="0 = min(steps, 120)")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+
+    data = synthgen.config_stream(WORKLOAD)
+    off = synthgen.split_items(data, ITEM_BYTES)
+
+    if args.impl == "reference":
+        return reference_arm(args, data, off)
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if world > 1 or args.gpus > 1:
+        from paper_conf_ipps_rockenbachsgmtd19_b200 import dist_bench
+        return dist_bench.main(args, data, off)
+
+    import torch
+
+    from paper_conf_ipps_rockenbachsgmtd19_b200 import Dedup
+
+    dev = torch.device("cuda:0")
+    torch.cuda.set_device(dev)
+    plan = plan_batches(off)
+    nb = len(plan)
+    dd = torch.from_numpy(data).to(dev)
+    subs = []
+    for k, j in plan:
+        subs.append((dd[int(off[k]):int(off[j])], (off[k:j + 1] - off[k]).copy()))
+    batch_bytes = [int(off[j]) - int(off[k]) for k, j in plan]
+
+    d = Dedup(0, **engine_kwargs(len(data)))
+    submit_dev = lambda b: d.submit_device(subs[b][0], subs[b][1])  # noqa: E731
+    torch.cuda.synchronize()
+
+    # ---- device-resident (value) ----
+    run_steps(d, submit_dev, nb, args.warmup, 0)
+    torch.cuda.synchronize()
+    s0 = d.stats()
+    l0 = d.kernel_launches()
+    start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(0) as clk:
+        start.record()
+        run_steps(d, submit_dev, nb, args.steps, args.warmup)
+        d.join()
+        end.record()
+        end.synchronize()
+    ms = start.elapsed_time(end)
+    s1 = d.stats()
+    launches = d.kernel_launches() - l0
+    ds = stat_delta(s0, s1)
+    step_ids = [(args.warmup + s) % nb for s in range(args.steps)]
+    bytes_timed = sum(batch_bytes[b] for b in step_ids)
+    assert ds["bytes"] == bytes_timed, (ds["bytes"], bytes_timed)
+    value = bytes_timed / (ms / 1e3) / 1e9
+    chunks_per_s = ds["chunks"] / (ms / 1e3)
+
+    # ---- roofline of the dominant kernel (live CUDA-event stage times) ----
+    pk, src = peaks()
+    clocks = clk.summary()
+    sm_mhz = pk.get("sm_max_mhz", 1965.0)
+    alu_peak = 148 * ALU_LANES_PER_SM_CLK * sm_mhz * 1e6 / 1e12      # Tops/s
+    sha_achieved = ds["sha1_blocks"] * SHA1_OPS_PER_BLOCK / (ds["ms_sha1"] / 1e3) / 1e12
+    scan_achieved = (bytes_timed * (1 + 1 / 8)) / (ds["ms_scan"] / 1e3) / 1e9
+    kernels = {
+        "sha1": {"ms_per_step": ds["ms_sha1"] / args.steps, "bound": "alu",
+                 "achieved": sha_achieved, "peak": alu_peak, "unit": "Tops/s",
+                 "frac": sha_achieved / alu_peak},
+        "rabin_scan": {"ms_per_step": ds["ms_scan"] / args.steps, "bound": "hbm",
+                       "achieved": scan_achieved, "peak": pk["hbm_gbs"], "unit": "GB/s",
+                       "frac": scan_achieved / pk["hbm_gbs"]},
+        "select+meta": {"ms_per_step": ds["ms_select"] / args.steps},
+        "table": {"ms_per_step": ds["ms_table"] / args.steps},
+        "pack_d2h": {"ms_per_step": ds["ms_d2h"] / args.steps},
+    }
+    dom = "sha1" if ds["ms_sha1"] >= ds["ms_scan"] else "rabin_scan"
+    kd = kernels[dom]
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tp):
+        traffic = json.load(open(tp)).get(dom)
+    roofline = {"kernel": dom, "bound": kd["bound"], "achieved": kd["achieved"],
+                "peak": kd["peak"], "unit": kd["unit"], "frac": kd["frac"], "traffic": traffic,
+                "peak_source": f"{src} (MEASURED_PEAKS.json)" if kd["bound"] == "hbm" else
+                f"derived: 148 SM x 64 alu lanes/clk x {sm_mhz:.0f} MHz ({src} max clock)"}
+
+    # ---- end-to-end through the host-fed C ABI ----
+    e2e_steps = args.e2e_steps or min(args.steps, 120)
+    pin = d.host_empty(len(data))
+    pin[:] = data
+    submit_host = lambda b: d.submit_buffer(  # noqa: E731
+        pin[int(off[plan[b][0]]):int(off[plan[b][1]])], subs[b][1])
+    d.end_stream()
+    run_steps(d, submit_host, nb, args.warmup, 0)
+    torch.cuda.synchronize()
+    e0 = d.stats()
+    start.record()
+    run_steps(d, submit_host, nb, e2e_steps, args.warmup)
+    d.join()
+    end.record()
+    end.synchronize()
+    ems = start.elapsed_time(end)
+    e1 = d.stats()
+    de = stat_delta(e0, e1)
+    e2e_value = de["bytes"] / (ems / 1e3) / 1e9
+    items_per_step = de["items"] / e2e_steps
+    e2e = {"value": e2e_value, "unit": "GB/s",
+           "h2d_bytes_per_step": (de["bytes"] + 8 * (de["items"] + de["batches"])) / e2e_steps,
+           "d2h_bytes_per_step": (33 * de["chunks"] + 4 * de["items"] + 8 * de["batches"])
+           / e2e_steps,
+           "steps": e2e_steps, "items_per_step": items_per_step,
+           "api": "dedup_submit_batch (pinned host buffers) + dedup_drain"}
+    d.close()
+
+    line = {
+        "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": 1, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "chunks_per_s": chunks_per_s,
+        "dup_ratio": ds["dup_chunks"] / max(ds["chunks"], 1),
+        "config": {"workload": f"{WORKLOAD}: 184 MiB simlarge-sized synthetic stream (seed 2), "
+                               "1 MiB items, dup_frac 0.52, device-resident",
+                   "batch_bytes": BATCH_BYTES, "batch_items": BATCH_ITEMS, "slots": SLOTS,
+                   "batches_per_stream": nb, "parallelism": "1 GPU",
+                   "l2": "inputs larger than L2 (184 MiB stream cycled, 126 MB L2)"},
+        "clocks": clocks, "gpu_launches": launches, "roofline": roofline, "kernels": kernels,
+        "e2e": e2e,
+    }
+    if not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline(data, off)
+    print(json.dumps(line), flush=True)
+
+
+if __name__ == "__main__":
+    main()

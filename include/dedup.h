@@ -1,0 +1,275 @@
+/*
+ * dedup.h -- C ABI of the B200-native GPU Dedup hot path.
+ *
+ * The hot path is the data-parallel core of the GPU Dedup of Rockenbach et
+ * al., "Stream Processing on Multi-Cores with GPUs: Parallel Programming
+ * Models' Challenges" (IPDPSW 2019), Section IV-B.  "P:NNN" = line NNN of the
+ * paper text:
+ *   - P:197  fixed-size batches; Rabin fingerprint fragmentation; "saved all
+ *            the indexes where the algorithm would fragment the data".
+ *   - P:199  Fig. 2: startPos = chunk start indexes of a batch.
+ *   - P:213  stage 1: batches of 1 MB, Rabin blocks.
+ *   - P:214  stage 2: SHA-1 of every block on the GPU, results in an array.
+ *   - P:215  stage 3: check whether blocks are duplicated.
+ *   - P:217  stage 5: reorder batches (results in sequence order).
+ * A stream item is one of the paper's batches (an "item" here); a GPU batch
+ * groups whole items and never changes results (reading O8).
+ *
+ * Method parameters (readings O1-O7): window 32 bytes,
+ * P(t) = t^32 + poly (0x45c2b6a1), cut iff (fp & anchor_mask) == anchor_value
+ * (0xFFF / 0), minimum chunk = window (restart semantics), no maximum chunk.
+ *
+ * Two layers:
+ *   1. Streaming API (dedup_init / dedup_submit_batch / dedup_submit_device /
+ *      dedup_drain / dedup_stats / dedup_end_stream / dedup_destroy): items
+ *      in, per-item results out in sequence order.  One ctx per GPU.
+ *   2. Stream-ordered device operations (dedup_op_*): the individual hot-path
+ *      steps on caller-owned DEVICE buffers, enqueued on a caller-provided
+ *      cudaStream_t (passed as void*).  Used by the multi-GPU orchestrator
+ *      (digest all-to-all between the route / owner / scatter steps) and by
+ *      the per-kernel parity tests.
+ *
+ * Conventions for every call:
+ *   - Return value: dedup_status, 0 = DEDUP_OK, < 0 = error.  DEDUP_ECUDA is
+ *     sticky: afterwards the ctx accepts only dedup_stats, dedup_last_error
+ *     and dedup_destroy.
+ *   - A ctx is NOT thread-safe: calls on one ctx must be serialised by the
+ *     caller (the paper's multi-thread GPU pitfall).
+ *   - "device pointer" arguments must be allocations on the ctx's device;
+ *     "host pointer" arguments are ordinary process memory.
+ *   - No function here allocates memory that the caller must free, except
+ *     dedup_host_alloc (freed by dedup_host_free).
+ */
+#ifndef DEDUP_B200_H
+#define DEDUP_B200_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef int32_t dedup_status;
+#define DEDUP_OK 0
+#define DEDUP_EINVAL (-1)       /* bad config or arguments; nothing enqueued */
+#define DEDUP_EAGAIN (-2)       /* in-flight window full: drain first */
+#define DEDUP_ENOMEM (-3)       /* device or pinned allocation failed */
+#define DEDUP_ETABLEFULL (-4)   /* digest table overflow (sticky) */
+#define DEDUP_EUNSUPPORTED (-5) /* config valid for the method, not for GPU v1 */
+#define DEDUP_ECUDA (-6)        /* CUDA error (sticky) */
+#define DEDUP_ETIMEDOUT (-7)    /* dedup_drain: nothing completed within wait_ms */
+
+#define DEDUP_ABI_VERSION 1
+
+typedef struct dedup_ctx dedup_ctx; /* opaque; owns its device buffers and tables */
+
+typedef struct {
+    uint32_t struct_size;    /* = sizeof(dedup_config) */
+    uint32_t window;         /* 32 (GPU v1 requires 32) */
+    uint32_t poly;           /* P(t) = t^32 + poly over GF(2) */
+    uint32_t anchor_mask;    /* cut iff (fp & anchor_mask) == anchor_value */
+    uint32_t anchor_value;
+    uint32_t min_chunk;      /* GPU v1 requires == window */
+    uint32_t max_chunk;      /* 0 = none; GPU v1 requires 0 */
+    int32_t device;          /* CUDA device ordinal of this ctx */
+    uint32_t slots;          /* in-flight batches ("memory spaces"), 1..16 */
+    uint32_t batch_items;    /* max items per GPU batch */
+    uint64_t batch_bytes;    /* max bytes per GPU batch (<= 1 GiB) */
+    uint64_t table_capacity; /* expected distinct digests per stream (this owner's share) */
+    uint32_t owner_rank;     /* digest-prefix owner index of this ctx's table shard */
+    uint32_t num_owners;     /* number of table shards (GPUs); 1 = single GPU */
+    uint32_t host_fed;       /* 1: allocate device input slots for dedup_submit_batch */
+    uint32_t reserved[7];
+} dedup_config;
+
+/* Fills *cfg with the defaults above (struct_size set). */
+void dedup_config_default(dedup_config* cfg);
+
+/* Creates a ctx on cfg->device: copies the config, builds the Rabin tables,
+ * allocates `slots` batch slots (device + pinned host result buffers) and two
+ * digest tables of >= 2 * table_capacity slots (power of two).
+ * Errors: EINVAL (bad config), EUNSUPPORTED (window/min/max_chunk not
+ * supported by the GPU kernels), ENOMEM, ECUDA.  *out is NULL on error. */
+dedup_status dedup_init(const dedup_config* cfg, dedup_ctx** out);
+
+/* Releases everything; waits for in-flight work.  Accepts NULL. */
+void dedup_destroy(dedup_ctx* c);
+
+/* Human-readable description of the last error on c (never NULL). */
+const char* dedup_last_error(const dedup_ctx* c);
+
+/* ------------------------------------------------------------------------ */
+/* 1. Streaming API                                                         */
+/* ------------------------------------------------------------------------ */
+
+/* Submits n_items host items (item k = item_len[k] bytes at item_ptr[k]).
+ * Items receive consecutive sequence numbers *first_seq_out + k.  Items are
+ * packed in order into GPU batches of <= batch_bytes / batch_items; every
+ * batch needs a free slot, otherwise nothing is submitted and DEDUP_EAGAIN is
+ * returned.  An item longer than batch_bytes or 2^32-1 is EINVAL.
+ * Ownership: item buffers are BORROWED until the item is returned by
+ * dedup_drain (copies are asynchronous).  Buffers from dedup_host_alloc (or
+ * otherwise pinned) are DMA'd directly; other memory goes through the CUDA
+ * driver's staging copy (slower).  Requires cfg.host_fed = 1. */
+dedup_status dedup_submit_batch(dedup_ctx* c, uint32_t n_items, const uint8_t* const* item_ptr,
+                                const uint64_t* item_len, uint64_t* first_seq_out);
+
+/* Submits ONE GPU batch whose bytes are already resident on the device:
+ * d_bytes (device pointer, 16-byte aligned, readable up to nbytes rounded up
+ * to 16) holds n_items items back to back; item_off (HOST pointer,
+ * n_items + 1 entries, item_off[0] = 0, non-decreasing, item_off[n_items] =
+ * nbytes) gives their offsets.  `producer` (cudaStream_t as void*, NULL =
+ * legacy default stream) is the stream that wrote d_bytes: the batch starts
+ * after the work enqueued on it so far.  item_off is copied before return;
+ * d_bytes is borrowed until the items are drained.  nbytes <= batch_bytes and
+ * n_items <= batch_items, else EINVAL; EAGAIN if no slot is free. */
+dedup_status dedup_submit_device(dedup_ctx* c, const uint8_t* d_bytes, uint64_t nbytes,
+                                 const uint64_t* item_off, uint32_t n_items, void* producer,
+                                 uint64_t* first_seq_out);
+
+/* Makes `stream` (cudaStream_t as void*) wait for all work submitted so far
+ * (no host synchronisation).  Used to bracket the engine with CUDA events. */
+dedup_status dedup_join(dedup_ctx* c, void* stream);
+
+/* Marks the end of the current dedup stream: items submitted afterwards are
+ * checked against a fresh (empty) digest table.  Sequence numbers continue. */
+dedup_status dedup_end_stream(dedup_ctx* c);
+
+typedef struct {
+    uint64_t seq;             /* sequence number (submission order) */
+    uint64_t item_len;        /* bytes */
+    uint32_t n_chunks;        /* 0 for an empty item */
+    uint32_t reserved;
+    const uint32_t* chunk_start; /* [n_chunks] item-relative starts, [0] = 0, increasing (startPos) */
+    const uint8_t* digest;    /* [n_chunks * 20] SHA-1, FIPS byte order */
+    const uint8_t* is_dup;    /* [n_chunks] 1 iff an earlier chunk of the stream has the same digest */
+    const uint64_t* first_id; /* [n_chunks] (seq << 32) | chunk index of the first occurrence */
+} dedup_item_result;
+
+/* Returns up to max_items completed items, strictly in sequence order
+ * (P:217).  wait_ms < 0 waits without limit for the next item, 0 polls,
+ * > 0 waits up to wait_ms milliseconds.  *n_out = number returned (0 with
+ * DEDUP_ETIMEDOUT when nothing completed in time; 0 with DEDUP_OK when
+ * nothing is in flight).  Result arrays are ctx-owned and valid until the
+ * next dedup_drain / dedup_destroy on c. */
+dedup_status dedup_drain(dedup_ctx* c, uint32_t max_items, int32_t wait_ms,
+                         dedup_item_result* out, uint32_t* n_out);
+
+/* Number of submitted items not yet returned by dedup_drain. */
+uint64_t dedup_pending(const dedup_ctx* c);
+
+typedef struct {
+    uint64_t items, bytes, chunks, dup_chunks, dup_bytes, unique_chunks;
+    uint64_t batches, table_used, table_slots, kernel_launches;
+    uint32_t num_owners, owner_rank;
+    /* summed CUDA-event stage times over drained batches (ms): H2D of the
+     * input, Rabin scan kernel, cut selection + chunk metadata, SHA-1 kernel,
+     * table insert + lookup, pack of results into pinned host memory */
+    double ms_h2d, ms_scan, ms_select, ms_sha1, ms_table, ms_d2h;
+    uint64_t sha1_blocks; /* 64-byte SHA-1 compressions over drained batches */
+} dedup_stats_t;
+
+/* Counters over all drained batches of the ctx (all streams). */
+dedup_status dedup_stats(const dedup_ctx* c, dedup_stats_t* out);
+
+/* Pinned, portable host memory usable as zero-copy DMA source for
+ * dedup_submit_batch.  Returns NULL on failure. */
+void* dedup_host_alloc(dedup_ctx* c, size_t bytes);
+void dedup_host_free(dedup_ctx* c, void* p);
+
+/* ------------------------------------------------------------------------ */
+/* 2. Stream-ordered device operations (caller-owned device buffers)        */
+/* ------------------------------------------------------------------------ */
+/* All pointers below are DEVICE pointers unless marked (host).  `stream` is a
+ * cudaStream_t of the ctx's device (NULL = legacy default stream).  The calls
+ * only enqueue work; outputs are valid once the stream reaches that point.
+ * Device-side counts (d_n_*) are read by the kernels, so no host
+ * synchronisation is needed between steps.  Ops on one ctx use one internal
+ * workspace and must not overlap in time on different streams. */
+
+/* Rows A2+A3: Rabin candidate scan over the whole batch
+ * (d_bytes[0..nbytes), 16-byte aligned, readable to nbytes rounded up to 16)
+ * with items at d_item_off[0..n_items] (u64, item_off[0] = 0,
+ * item_off[n_items] = nbytes), then greedy cut selection with forced cuts at
+ * every non-empty item start.  Writes the batch-relative chunk starts
+ * d_cut_pos[0..n) (u32, increasing) and n to *d_n_chunks (u32).
+ * cap = capacity of d_cut_pos; if n would exceed cap, *d_n_chunks = n but
+ * only cap entries are written and the call returns DEDUP_OK (check n).
+ * nbytes <= cfg.batch_bytes (workspace size), else EINVAL. */
+dedup_status dedup_op_chunk(dedup_ctx* c, void* stream, const uint8_t* d_bytes, uint64_t nbytes,
+                            const uint64_t* d_item_off, uint32_t n_items, uint32_t* d_cut_pos,
+                            uint64_t cap, uint32_t* d_n_chunks);
+
+/* Per-chunk metadata from the cuts: item-relative d_chunk_start (u32),
+ * d_chunk_id = ((first_seq + item) << 32) | index within item (u64), and
+ * d_item_first_chunk[item] (u32, 0xFFFFFFFF for empty items). cap as above. */
+dedup_status dedup_op_chunk_meta(dedup_ctx* c, void* stream, const uint64_t* d_item_off,
+                                 uint32_t n_items, const uint32_t* d_cut_pos,
+                                 const uint32_t* d_n_chunks, uint64_t cap, uint64_t first_seq,
+                                 uint32_t* d_chunk_start, uint64_t* d_chunk_id,
+                                 uint32_t* d_item_first_chunk);
+
+/* Row A4: SHA-1 (FIPS 180-4) of every chunk k = d_bytes[cut[k],
+ * cut[k+1]) (last chunk ends at nbytes) for k < min(*d_n_chunks, cap);
+ * writes d_digest[20k..20k+20).  Any increasing cut list starting at 0
+ * describes a valid partition. */
+dedup_status dedup_op_sha1(dedup_ctx* c, void* stream, const uint8_t* d_bytes, uint64_t nbytes,
+                           const uint32_t* d_cut_pos, const uint32_t* d_n_chunks, uint64_t cap,
+                           uint8_t* d_digest);
+
+/* Row A7 on this ctx's table of the CURRENT stream: insert every
+ * record (d_digest[20r..], d_id[r]) keeping the minimum id per digest, then
+ * look each one up: d_first_id[r] = min id over all records inserted so far
+ * with that digest; d_is_dup[r] = (d_first_id[r] != d_id[r]).  Records are
+ * r < min(*d_n, cap).  Results equal the sequential stream-order answer
+ * provided every record with a smaller id was inserted earlier or in this
+ * call.  d_is_dup may be NULL.  Table overflow sets a sticky device flag
+ * reported by dedup_op_table_status. */
+dedup_status dedup_op_table_insert_lookup(dedup_ctx* c, void* stream, const uint8_t* d_digest,
+                                          const uint64_t* d_id, const uint32_t* d_n, uint64_t cap,
+                                          uint64_t* d_first_id, uint8_t* d_is_dup);
+
+/* Clears the current stream's table (stream-ordered). */
+dedup_status dedup_op_table_reset(dedup_ctx* c, void* stream);
+
+/* Reads table occupancy and the overflow flag (synchronises `stream`). */
+dedup_status dedup_op_table_status(dedup_ctx* c, void* stream, uint64_t* used, uint64_t* slots,
+                                   int32_t* overflow);
+
+/* 32-byte digest record exchanged between GPUs (rows A5/A6). */
+typedef struct {
+    uint8_t digest[20];
+    uint32_t pad;
+    uint64_t id;
+} dedup_record;
+
+/* Row A5: owner(r) = floor(BE32(digest[0..3]) * num_owners / 2^32).
+ * Writes records grouped by owner into d_send (capacity cap records):
+ * owner o's records occupy d_send[d_send_off[o] .. d_send_off[o+1]) (u32
+ * exclusive offsets, num_owners + 1 entries); d_send_pos[r] = slot of record r
+ * in d_send.  num_owners <= 64. */
+dedup_status dedup_op_route(dedup_ctx* c, void* stream, const uint8_t* d_digest,
+                            const uint64_t* d_id, const uint32_t* d_n, uint64_t cap,
+                            uint32_t num_owners, dedup_record* d_send, uint32_t* d_send_off,
+                            uint32_t* d_send_pos);
+
+/* Row A7 on the owner: insert all n_recv (host count) received records into
+ * this ctx's table shard, then write d_reply[i] = first id of record i. */
+dedup_status dedup_op_owner(dedup_ctx* c, void* stream, const dedup_record* d_recv,
+                            uint64_t n_recv, uint64_t* d_reply);
+
+/* Row A8: d_first_id[r] = d_reply_back[d_send_pos[r]],
+ * d_is_dup[r] = (d_first_id[r] != d_id[r]). */
+dedup_status dedup_op_scatter(dedup_ctx* c, void* stream, const uint64_t* d_reply_back,
+                              const uint32_t* d_send_pos, const uint64_t* d_id,
+                              const uint32_t* d_n, uint64_t cap, uint64_t* d_first_id,
+                              uint8_t* d_is_dup);
+
+/* Number of kernels this ctx has launched so far (all layers). */
+uint64_t dedup_kernel_launches(const dedup_ctx* c);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DEDUP_B200_H */

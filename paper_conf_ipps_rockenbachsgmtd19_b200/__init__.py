@@ -1,0 +1,10 @@
+"""B200-native GPU Dedup hot path (Rockenbach et al., IPDPSW 2019, Sec. IV-B).
+
+Rabin content-defined chunking -> SHA-1 per chunk -> global duplicate check,
+as hand-written sm_100a CUDA kernels behind the C ABI of include/dedup.h.
+This package is the thin Python binding (argument marshalling only).
+"""
+from ._native import DedupError, lib  # noqa: F401
+from .api import Dedup, ItemResult, result_from_c  # noqa: F401
+
+__all__ = ["Dedup", "DedupError", "ItemResult", "lib", "result_from_c"]

@@ -1,0 +1,264 @@
+"""Thin Python binding of the C ABI (include/dedup.h): argument marshalling only.
+
+Every step of the hot path runs in the CUDA kernels of libdedup_b200.so.
+PyTorch is used only to hand device buffers and streams to the library.
+"""
+from __future__ import annotations
+
+import collections
+import ctypes
+from dataclasses import dataclass
+
+import numpy as np
+
+from . import _native as N
+
+_u64 = ctypes.c_uint64
+_vp = ctypes.c_void_p
+
+
+@dataclass
+class ItemResult:
+    """Per-item output (P:199 startPos, P:214 digests, P:215 dup flags)."""
+    seq: int
+    item_len: int
+    chunk_start: np.ndarray  # u32 [n]
+    digest: np.ndarray       # u8 [n, 20]
+    is_dup: np.ndarray       # u8 [n]
+    first_id: np.ndarray     # u64 [n]
+
+    @property
+    def n_chunks(self) -> int:
+        return len(self.chunk_start)
+
+
+def _ptr(t) -> int:
+    """Device pointer of a torch tensor (or raw int)."""
+    if t is None:
+        return 0
+    if isinstance(t, int):
+        return t
+    return t.data_ptr()
+
+
+def _stream(stream) -> int:
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream().cuda_stream
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+def result_from_c(r: N.ItemResult, copy: bool = True) -> ItemResult:
+    n = int(r.n_chunks)
+    if n == 0:
+        z = np.zeros(0, np.uint32)
+        return ItemResult(int(r.seq), int(r.item_len), z, np.zeros((0, 20), np.uint8),
+                          np.zeros(0, np.uint8), np.zeros(0, np.uint64))
+    cs = np.ctypeslib.as_array(r.chunk_start, (n,))
+    dg = np.ctypeslib.as_array(r.digest, (n * 20,)).reshape(n, 20)
+    dup = np.ctypeslib.as_array(r.is_dup, (n,))
+    fid = np.ctypeslib.as_array(r.first_id, (n,))
+    if copy:
+        cs, dg, dup, fid = cs.copy(), dg.copy(), dup.copy(), fid.copy()
+    return ItemResult(int(r.seq), int(r.item_len), cs, dg, dup, fid)
+
+
+class Dedup:
+    """One dedup context on one GPU (streaming API of include/dedup.h)."""
+
+    def __init__(self, device: int = 0, *, slots: int = 4, batch_bytes: int = 64 << 20,
+                 batch_items: int = 4096, table_capacity: int = 1 << 20, host_fed: bool = True,
+                 window: int = 32, poly: int = 0x45C2B6A1, anchor_mask: int = 0xFFF,
+                 anchor_value: int = 0, min_chunk: int = 32, max_chunk: int = 0,
+                 owner_rank: int = 0, num_owners: int = 1, max_drain: int = 65536):
+        L = N.lib()
+        cfg = N.Config()
+        L.dedup_config_default(ctypes.byref(cfg))
+        for k, v in dict(device=device, slots=slots, batch_bytes=batch_bytes,
+                         batch_items=batch_items, table_capacity=table_capacity,
+                         host_fed=int(host_fed), window=window, poly=poly,
+                         anchor_mask=anchor_mask, anchor_value=anchor_value,
+                         min_chunk=min_chunk, max_chunk=max_chunk, owner_rank=owner_rank,
+                         num_owners=num_owners).items():
+            setattr(cfg, k, v)
+        self.cfg = cfg
+        self._ctx = _vp()
+        st = L.dedup_init(ctypes.byref(cfg), ctypes.byref(self._ctx))
+        if st != N.DEDUP_OK:
+            raise N.DedupError(st, "dedup_init failed")
+        self._res = (N.ItemResult * max_drain)()
+        self._max_drain = max_drain
+        self._borrowed = collections.deque()  # (last_seq_exclusive, objects)
+        self._next_out = 0
+        self._pinned = []
+
+    # -- lifetime --------------------------------------------------------
+    @property
+    def ctx(self):
+        return self._ctx
+
+    def close(self):
+        if self._ctx:
+            L = N.lib()
+            L.dedup_destroy(self._ctx)
+            for p in self._pinned:
+                L.dedup_host_free(None, p)
+            self._pinned.clear()
+            self._ctx = _vp()
+            self._borrowed.clear()
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def _check(self, st):
+        N.check(st, self._ctx)
+
+    # -- submission --------------------------------------------------------
+    def submit(self, items) -> int:
+        """Submit host items (bytes / uint8 arrays); returns the first seq."""
+        arrs = []
+        for x in items:
+            if isinstance(x, (bytes, bytearray, memoryview)):
+                x = np.frombuffer(x, np.uint8)
+            arrs.append(np.ascontiguousarray(x, dtype=np.uint8).reshape(-1))
+        n = len(arrs)
+        ptrs = (_vp * max(n, 1))(*[a.ctypes.data for a in arrs])
+        lens = (_u64 * max(n, 1))(*[a.nbytes for a in arrs])
+        seq = _u64()
+        self._check(N.lib().dedup_submit_batch(self._ctx, n, ptrs, lens, ctypes.byref(seq)))
+        self._borrowed.append((seq.value + n, arrs))
+        return seq.value
+
+    def submit_buffer(self, buf: np.ndarray, item_off) -> int:
+        """Submit items that are slices buf[item_off[k]:item_off[k+1]] of one
+        host buffer (pinned buffers from host_empty() are DMA'd directly)."""
+        off = np.asarray(item_off, np.uint64)
+        n = len(off) - 1
+        base = buf.ctypes.data
+        ptrs = (_vp * max(n, 1))(*[base + int(o) for o in off[:-1]])
+        lens = (_u64 * max(n, 1))(*[int(b - a) for a, b in zip(off[:-1], off[1:])])
+        seq = _u64()
+        self._check(N.lib().dedup_submit_batch(self._ctx, n, ptrs, lens, ctypes.byref(seq)))
+        self._borrowed.append((seq.value + n, buf))
+        return seq.value
+
+    def submit_device(self, data, item_off, producer=None) -> int:
+        """Submit ONE GPU batch already resident in device memory: ``data`` is
+        a CUDA uint8 tensor (or device pointer int + nbytes via item_off[-1]);
+        the batch waits for ``producer`` (default: torch's current stream)."""
+        off = np.ascontiguousarray(item_off, np.uint64)
+        n = len(off) - 1
+        seq = _u64()
+        self._check(N.lib().dedup_submit_device(
+            self._ctx, _ptr(data), int(off[-1]), off.ctypes.data_as(ctypes.POINTER(_u64)), n,
+            _stream(producer), ctypes.byref(seq)))
+        self._borrowed.append((seq.value + n, data))
+        return seq.value
+
+    def join(self, stream=None):
+        """Make ``stream`` (default: torch's current stream) wait for all work."""
+        self._check(N.lib().dedup_join(self._ctx, _stream(stream)))
+
+    def end_stream(self):
+        self._check(N.lib().dedup_end_stream(self._ctx))
+
+    # -- results -----------------------------------------------------------
+    def drain_raw(self, max_items: int | None = None, wait_ms: int = -1) -> int:
+        """Drain into the internal result array; returns the count (no copies)."""
+        m = min(max_items or self._max_drain, self._max_drain)
+        n = ctypes.c_uint32()
+        st = N.lib().dedup_drain(self._ctx, m, wait_ms, self._res, ctypes.byref(n))
+        if st == N.DEDUP_ETIMEDOUT:
+            return 0
+        self._check(st)
+        got = n.value
+        if got:
+            self._next_out = self._res[got - 1].seq + 1
+            while self._borrowed and self._borrowed[0][0] <= self._next_out:
+                self._borrowed.popleft()
+        return got
+
+    def drain(self, max_items: int | None = None, wait_ms: int = -1) -> list[ItemResult]:
+        got = self.drain_raw(max_items, wait_ms)
+        return [result_from_c(self._res[i]) for i in range(got)]
+
+    def drain_all(self) -> list[ItemResult]:
+        out = []
+        while self.pending():
+            out.extend(self.drain(wait_ms=-1))
+        return out
+
+    def pending(self) -> int:
+        return int(N.lib().dedup_pending(self._ctx))
+
+    def stats(self) -> dict:
+        s = N.Stats()
+        self._check(N.lib().dedup_stats(self._ctx, ctypes.byref(s)))
+        return {k: getattr(s, k) for k, _ in N.Stats._fields_}
+
+    def kernel_launches(self) -> int:
+        return int(N.lib().dedup_kernel_launches(self._ctx))
+
+    def host_empty(self, nbytes: int) -> np.ndarray:
+        """Pinned host buffer (zero-copy DMA source), freed by close()."""
+        p = N.lib().dedup_host_alloc(self._ctx, max(nbytes, 1))
+        if not p:
+            raise MemoryError("dedup_host_alloc failed")
+        self._pinned.append(p)
+        buf = (ctypes.c_uint8 * max(nbytes, 1)).from_address(p)
+        return np.frombuffer(buf, np.uint8, count=nbytes)
+
+    # -- stream-ordered device operations (dedup_op_*) ---------------------
+    def op_chunk(self, data, nbytes, item_off, n_items, cut_pos, cap, n_chunks, stream=None):
+        self._check(N.lib().dedup_op_chunk(self._ctx, _stream(stream), _ptr(data), nbytes,
+                                           _ptr(item_off), n_items, _ptr(cut_pos), cap,
+                                           _ptr(n_chunks)))
+
+    def op_chunk_meta(self, item_off, n_items, cut_pos, n_chunks, cap, first_seq, chunk_start,
+                      chunk_id, item_first_chunk, stream=None):
+        self._check(N.lib().dedup_op_chunk_meta(
+            self._ctx, _stream(stream), _ptr(item_off), n_items, _ptr(cut_pos), _ptr(n_chunks),
+            cap, first_seq, _ptr(chunk_start), _ptr(chunk_id), _ptr(item_first_chunk)))
+
+    def op_sha1(self, data, nbytes, cut_pos, n_chunks, cap, digest, stream=None):
+        self._check(N.lib().dedup_op_sha1(self._ctx, _stream(stream), _ptr(data), nbytes,
+                                          _ptr(cut_pos), _ptr(n_chunks), cap, _ptr(digest)))
+
+    def op_table(self, digest, ids, n, cap, first_id, is_dup=None, stream=None):
+        self._check(N.lib().dedup_op_table_insert_lookup(
+            self._ctx, _stream(stream), _ptr(digest), _ptr(ids), _ptr(n), cap, _ptr(first_id),
+            _ptr(is_dup)))
+
+    def op_table_reset(self, stream=None):
+        self._check(N.lib().dedup_op_table_reset(self._ctx, _stream(stream)))
+
+    def op_table_status(self, stream=None):
+        used, slots, ovf = _u64(), _u64(), ctypes.c_int32()
+        self._check(N.lib().dedup_op_table_status(self._ctx, _stream(stream), ctypes.byref(used),
+                                                  ctypes.byref(slots), ctypes.byref(ovf)))
+        return used.value, slots.value, ovf.value
+
+    def op_route(self, digest, ids, n, cap, num_owners, send, send_off, send_pos, stream=None):
+        self._check(N.lib().dedup_op_route(self._ctx, _stream(stream), _ptr(digest), _ptr(ids),
+                                           _ptr(n), cap, num_owners, _ptr(send), _ptr(send_off),
+                                           _ptr(send_pos)))
+
+    def op_owner(self, recv, n_recv, reply, stream=None):
+        self._check(N.lib().dedup_op_owner(self._ctx, _stream(stream), _ptr(recv), n_recv,
+                                           _ptr(reply)))
+
+    def op_scatter(self, reply_back, send_pos, ids, n, cap, first_id, is_dup=None, stream=None):
+        self._check(N.lib().dedup_op_scatter(self._ctx, _stream(stream), _ptr(reply_back),
+                                             _ptr(send_pos), _ptr(ids), _ptr(n), cap,
+                                             _ptr(first_id), _ptr(is_dup)))

@@ -1,0 +1,819 @@
+// api.cpp -- C ABI (include/dedup.h) and the per-GPU streaming engine.
+//
+// Engine (rows A1 + A9 of the hot path): a ring of `slots` batch slots, each
+// with its own CUDA stream, device buffers and a mapped pinned result buffer
+// ("memory spaces" used round-robin).  Per batch,
+// everything is enqueued asynchronously on the slot's stream:
+//   H2D (host-fed only) -> rabin_scan -> select -> chunk_meta -> sha1
+//   -> [wait previous batch's table event] -> table insert -> lookup
+//   -> pack (kernel stores results straight into pinned host memory)
+// Table work of consecutive batches of one dedup stream is chained with
+// events, so every lookup sees the inserts of all earlier batches (the
+// sequential stream-order answer, reading O12).  No host synchronisation
+// happens between steps; dedup_drain waits on the slot's completion event and
+// hands items out strictly in sequence order.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstring>
+#include <deque>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "dedup.h"
+#include "internal.h"
+
+using namespace dd;
+
+namespace {
+
+struct Workspace {
+    uint32_t* bitmap = nullptr;   // candidate bitmap, one bit per byte
+    uint64_t* desc = nullptr;     // look-back descriptors
+    uint32_t* counters = nullptr; // [0] tile counter, [1] sha1 work counter, [64..191] route
+    uint32_t* slot_idx = nullptr; // table slot per record
+    uint64_t n_desc_tiles = 0;
+    uint32_t epoch = 0;
+};
+
+struct Slot {
+    cudaStream_t stream = nullptr;
+    cudaEvent_t ev_start = nullptr, ev_h2d = nullptr, ev_scan = nullptr, ev_chunk = nullptr,
+                ev_sha = nullptr, ev_table = nullptr, ev_done = nullptr;
+    cudaEvent_t ev_prod = nullptr;  // producer-stream dependency (no timing)
+    uint8_t* d_bytes = nullptr;  // host-fed input copy
+    uint64_t* d_item_off = nullptr;
+    Workspace ws;
+    uint32_t* d_cut_pos = nullptr;
+    uint32_t* d_chunk_start = nullptr;
+    uint32_t* d_item_first = nullptr;
+    uint32_t* d_n_chunks = nullptr;
+    uint64_t* d_chunk_id = nullptr;
+    uint64_t* d_first_id = nullptr;
+    uint8_t* d_digest = nullptr;
+    uint8_t* d_is_dup = nullptr;
+    uint64_t* h_item_off = nullptr;  // pinned staging of item offsets
+    uint8_t* h_res = nullptr;        // mapped pinned results
+    HostResultLayout hdev{};         // device view of h_res
+    HostResultLayout hhost{};        // host view of h_res
+    // batch in flight
+    bool busy = false;
+    bool parsed = false;
+    bool host_fed = false;
+    uint64_t first_seq = 0;
+    uint32_t n_items = 0;
+    uint64_t nbytes = 0;
+    std::vector<uint64_t> item_len;
+    std::vector<uint32_t> item_first, item_n;
+    uint32_t next_item = 0;  // next item of this batch to hand out
+};
+
+struct TableBuf {
+    TableSlot* slots = nullptr;
+    uint32_t* status = nullptr;
+    uint64_t capacity = 0;
+    cudaEvent_t last_use = nullptr;
+    bool used = false;
+};
+
+}  // namespace
+
+struct dedup_ctx {
+    dedup_config cfg{};
+    int num_sms = 0;
+    uint32_t* d_tab = nullptr;  // R[256] then W256[256]
+    std::vector<Slot> slots;
+    TableBuf tables[2];
+    int cur_table = 0;
+    bool stream_fresh = true;            // next batch starts a new dedup stream
+    cudaEvent_t chain_ev = nullptr;      // table event of the previous batch of this stream
+    bool chain_valid = false;
+    Workspace op_ws;
+    uint64_t chunk_cap = 0;              // chunks per slot
+    std::deque<int> inflight;            // slot indices in seq order
+    std::vector<int> to_release;         // slots fully handed out by the last drain
+    uint64_t next_seq = 0;
+    uint64_t pending_items = 0;
+    dedup_status sticky = DEDUP_OK;
+    std::string err = "no error";
+    uint64_t launches = 0;
+    dedup_stats_t st{};
+};
+
+namespace {
+
+dedup_status fail(dedup_ctx* c, dedup_status s, const std::string& msg) {
+    if (c) {
+        c->err = msg;
+        if (s == DEDUP_ECUDA || s == DEDUP_ETABLEFULL) c->sticky = s;
+    }
+    return s;
+}
+
+#define CU(call)                                                                        \
+    do {                                                                                \
+        cudaError_t e_ = (call);                                                        \
+        if (e_ != cudaSuccess)                                                          \
+            return fail(c, DEDUP_ECUDA, std::string(#call ": ") + cudaGetErrorString(e_)); \
+    } while (0)
+
+// ---- product-side Rabin tables (independent of the oracle) ----------------
+// Multiply a degree<32 polynomial by t^k modulo P(t) = t^32 + poly.
+uint32_t mul_tk(uint32_t x, unsigned k, uint32_t poly) {
+    while (k--) x = (x & 0x80000000u) ? ((x << 1) ^ poly) : (x << 1);
+    return x;
+}
+
+uint64_t next_pow2(uint64_t v) {
+    uint64_t p = 1;
+    while (p < v) p <<= 1;
+    return p;
+}
+
+template <class T>
+dedup_status dalloc(dedup_ctx* c, T** p, uint64_t count) {
+    if (count == 0) count = 1;
+    cudaError_t e = cudaMalloc(reinterpret_cast<void**>(p), sizeof(T) * count);
+    if (e != cudaSuccess) return fail(c, DEDUP_ENOMEM, std::string("cudaMalloc: ") + cudaGetErrorString(e));
+    return DEDUP_OK;
+}
+
+#define TRY(x)                            \
+    do {                                  \
+        dedup_status s_ = (x);            \
+        if (s_ != DEDUP_OK) return s_;    \
+    } while (0)
+
+dedup_status ws_alloc(dedup_ctx* c, Workspace& w, uint64_t batch_bytes, uint64_t cap) {
+    w.n_desc_tiles = (batch_bytes + kSelTile - 1) / kSelTile + 1;
+    TRY(dalloc(c, &w.bitmap, batch_bytes / 32 + 2));
+    TRY(dalloc(c, &w.desc, w.n_desc_tiles * kDescWords));
+    TRY(dalloc(c, &w.counters, 256));
+    TRY(dalloc(c, &w.slot_idx, cap));
+    CU(cudaMemset(w.desc, 0, sizeof(uint64_t) * w.n_desc_tiles * kDescWords));
+    CU(cudaMemset(w.counters, 0, sizeof(uint32_t) * 256));
+    return DEDUP_OK;
+}
+
+void ws_free(Workspace& w) {
+    cudaFree(w.bitmap);
+    cudaFree(w.desc);
+    cudaFree(w.counters);
+    cudaFree(w.slot_idx);
+    w = Workspace{};
+}
+
+bool usable(const dedup_ctx* c) { return c != nullptr && c->sticky == DEDUP_OK; }
+
+TableView table_view(dedup_ctx* c) {
+    TableBuf& t = c->tables[c->cur_table];
+    return TableView{t.slots, t.capacity - 1, t.status};
+}
+
+// Enqueue rows A2-A3 on stream s (optionally recording `mid` after the scan).
+dedup_status enqueue_chunk(dedup_ctx* c, Workspace& w, cudaStream_t s, const uint8_t* d_bytes,
+                           uint64_t nbytes, const uint64_t* d_item_off, uint32_t n_items,
+                           uint32_t* d_cut_pos, uint64_t cap, uint32_t* d_n,
+                           cudaEvent_t mid = nullptr) {
+    if (++w.epoch == 0) ++w.epoch;
+    launch_rabin_scan(d_bytes, nbytes, c->d_tab, c->cfg.anchor_mask, c->cfg.anchor_value,
+                      w.bitmap, c->num_sms, s);
+    if (mid) CU(cudaEventRecord(mid, s));
+    launch_select(w.bitmap, nbytes, d_item_off, n_items, w.desc, w.counters, w.epoch, d_cut_pos,
+                  cap, d_n, c->num_sms, s);
+    c->launches += nbytes ? 2 : 0;
+    CU(cudaGetLastError());
+    return DEDUP_OK;
+}
+
+dedup_status enqueue_table(dedup_ctx* c, Workspace& w, cudaStream_t s, const uint8_t* d_digest,
+                           const uint64_t* d_id, const uint32_t* d_n, uint64_t cap,
+                           uint64_t* d_first_id, uint8_t* d_is_dup) {
+    TableView tv = table_view(c);
+    launch_table_insert(tv, d_digest, d_id, nullptr, d_n, 0, cap, w.slot_idx, c->num_sms, s);
+    launch_table_lookup(tv, d_id, nullptr, d_n, 0, cap, w.slot_idx, d_first_id, d_is_dup,
+                        c->num_sms, s);
+    c->launches += cap ? 2 : 0;
+    CU(cudaGetLastError());
+    return DEDUP_OK;
+}
+
+dedup_status slot_alloc(dedup_ctx* c, Slot& sl) {
+    const dedup_config& g = c->cfg;
+    const uint64_t cap = c->chunk_cap;
+    CU(cudaStreamCreateWithFlags(&sl.stream, cudaStreamNonBlocking));
+    for (cudaEvent_t* e : {&sl.ev_start, &sl.ev_h2d, &sl.ev_scan, &sl.ev_chunk, &sl.ev_sha,
+                           &sl.ev_table, &sl.ev_done})
+        CU(cudaEventCreate(e));
+    CU(cudaEventCreateWithFlags(&sl.ev_prod, cudaEventDisableTiming));
+    if (g.host_fed) TRY(dalloc(c, &sl.d_bytes, g.batch_bytes + 256));
+    TRY(dalloc(c, &sl.d_item_off, (uint64_t)g.batch_items + 1));
+    TRY(ws_alloc(c, sl.ws, g.batch_bytes, cap));
+    TRY(dalloc(c, &sl.d_cut_pos, cap));
+    TRY(dalloc(c, &sl.d_chunk_start, cap));
+    TRY(dalloc(c, &sl.d_item_first, g.batch_items));
+    TRY(dalloc(c, &sl.d_n_chunks, 4));
+    TRY(dalloc(c, &sl.d_chunk_id, cap));
+    TRY(dalloc(c, &sl.d_first_id, cap));
+    TRY(dalloc(c, &sl.d_digest, cap * 20));
+    TRY(dalloc(c, &sl.d_is_dup, cap));
+    CU(cudaHostAlloc(reinterpret_cast<void**>(&sl.h_item_off),
+                     sizeof(uint64_t) * ((uint64_t)g.batch_items + 1), cudaHostAllocPortable));
+    // results: header 64 B | chunk_start 4*cap | first_id 8*cap | digest 20*cap | is_dup cap
+    //          | item_first 4*items
+    const uint64_t o_cs = 64, o_fid = o_cs + ((4 * cap + 63) & ~63ull),
+                   o_dg = o_fid + 8 * cap, o_dup = o_dg + 20 * cap,
+                   o_if = (o_dup + cap + 63) & ~63ull, total = o_if + 4ull * g.batch_items + 64;
+    CU(cudaHostAlloc(reinterpret_cast<void**>(&sl.h_res), total,
+                     cudaHostAllocMapped | cudaHostAllocPortable));
+    uint8_t* dres = nullptr;
+    CU(cudaHostGetDevicePointer(reinterpret_cast<void**>(&dres), sl.h_res, 0));
+    auto lay = [&](uint8_t* b) {
+        HostResultLayout h;
+        h.header = reinterpret_cast<uint32_t*>(b);
+        h.chunk_start = reinterpret_cast<uint32_t*>(b + o_cs);
+        h.first_id = reinterpret_cast<uint64_t*>(b + o_fid);
+        h.digest = b + o_dg;
+        h.is_dup = b + o_dup;
+        h.item_first_chunk = reinterpret_cast<uint32_t*>(b + o_if);
+        return h;
+    };
+    sl.hdev = lay(dres);
+    sl.hhost = lay(sl.h_res);
+    return DEDUP_OK;
+}
+
+void slot_free(Slot& sl) {
+    if (sl.stream) cudaStreamSynchronize(sl.stream);
+    for (cudaEvent_t e : {sl.ev_start, sl.ev_h2d, sl.ev_scan, sl.ev_chunk, sl.ev_sha, sl.ev_table,
+                          sl.ev_done, sl.ev_prod})
+        if (e) cudaEventDestroy(e);
+    cudaFree(sl.d_bytes);
+    cudaFree(sl.d_item_off);
+    ws_free(sl.ws);
+    cudaFree(sl.d_cut_pos);
+    cudaFree(sl.d_chunk_start);
+    cudaFree(sl.d_item_first);
+    cudaFree(sl.d_n_chunks);
+    cudaFree(sl.d_chunk_id);
+    cudaFree(sl.d_first_id);
+    cudaFree(sl.d_digest);
+    cudaFree(sl.d_is_dup);
+    if (sl.h_item_off) cudaFreeHost(sl.h_item_off);
+    if (sl.h_res) cudaFreeHost(sl.h_res);
+    if (sl.stream) cudaStreamDestroy(sl.stream);
+    sl = Slot{};
+}
+
+int free_slot_count(const dedup_ctx* c) {
+    int n = 0;
+    for (const Slot& s : c->slots) n += s.busy ? 0 : 1;
+    return n;
+}
+
+int take_free_slot(dedup_ctx* c) {
+    for (size_t i = 0; i < c->slots.size(); ++i)
+        if (!c->slots[i].busy) return (int)i;
+    return -1;
+}
+
+// Enqueue one batch on slot i.  Input is either the slot's own device copy
+// (host-fed, already enqueued) or an external device pointer.
+dedup_status launch_batch(dedup_ctx* c, int i, const uint8_t* d_bytes) {
+    Slot& sl = c->slots[i];
+    cudaStream_t s = sl.stream;
+    const uint64_t cap = c->chunk_cap;
+    // item offsets -> device (from pinned staging)
+    CU(cudaMemcpyAsync(sl.d_item_off, sl.h_item_off, sizeof(uint64_t) * (sl.n_items + 1),
+                       cudaMemcpyHostToDevice, s));
+    CU(cudaEventRecord(sl.ev_h2d, s));
+    TRY(enqueue_chunk(c, sl.ws, s, d_bytes, sl.nbytes, sl.d_item_off, sl.n_items, sl.d_cut_pos,
+                      cap, sl.d_n_chunks, sl.ev_scan));
+    launch_chunk_meta(sl.d_item_off, sl.n_items, sl.d_cut_pos, sl.d_n_chunks, cap, sl.first_seq,
+                      sl.d_chunk_start, sl.d_chunk_id, sl.d_item_first, c->num_sms, s);
+    c->launches += (cap && sl.n_items) ? 1 : 0;
+    CU(cudaEventRecord(sl.ev_chunk, s));
+    launch_sha1(d_bytes, sl.nbytes, sl.d_cut_pos, sl.d_n_chunks, cap, sl.ws.counters + 1,
+                sl.d_digest, c->num_sms, s);
+    c->launches += 1;
+    CU(cudaEventRecord(sl.ev_sha, s));
+    // table: chain after the previous batch of this dedup stream
+    TableBuf& tb = c->tables[c->cur_table];
+    if (c->stream_fresh) {
+        if (tb.used) CU(cudaStreamWaitEvent(s, tb.last_use, 0));
+        CU(cudaMemsetAsync(tb.slots, 0, sizeof(TableSlot) * tb.capacity, s));
+        CU(cudaMemsetAsync(tb.status, 0, sizeof(uint32_t) * 4, s));
+        c->stream_fresh = false;
+        tb.used = true;
+    } else if (c->chain_valid) {
+        CU(cudaStreamWaitEvent(s, c->chain_ev, 0));
+    }
+    TRY(enqueue_table(c, sl.ws, s, sl.d_digest, sl.d_chunk_id, sl.d_n_chunks, cap,
+                      sl.d_first_id, sl.d_is_dup));
+    CU(cudaEventRecord(sl.ev_table, s));
+    CU(cudaEventRecord(tb.last_use, s));
+    c->chain_ev = sl.ev_table;
+    c->chain_valid = true;
+    launch_pack(sl.d_n_chunks, cap, sl.n_items, sl.d_chunk_start, sl.d_first_id, sl.d_digest,
+                sl.d_is_dup, sl.d_item_first, tb.status, sl.hdev, c->num_sms, s);
+    c->launches += 1;
+    CU(cudaGetLastError());
+    CU(cudaEventRecord(sl.ev_done, s));
+    sl.busy = true;
+    sl.parsed = false;
+    sl.next_item = 0;
+    c->inflight.push_back(i);
+    c->pending_items += sl.n_items;
+    c->st.batches += 1;
+    return DEDUP_OK;
+}
+
+dedup_status check_cfg(const dedup_config* g) {
+    if (g == nullptr || g->struct_size != sizeof(dedup_config)) return DEDUP_EINVAL;
+    if (g->window == 0 || g->window > 64 || g->min_chunk < g->window) return DEDUP_EINVAL;
+    if (g->max_chunk != 0 && g->max_chunk < g->min_chunk) return DEDUP_EINVAL;
+    if (g->slots < 1 || g->slots > 16 || g->batch_items < 1) return DEDUP_EINVAL;
+    if (g->batch_bytes < 1 || g->batch_bytes > (1ull << 30)) return DEDUP_EINVAL;
+    if (g->num_owners < 1 || g->num_owners > 64 || g->owner_rank >= g->num_owners)
+        return DEDUP_EINVAL;
+    if (g->table_capacity < 1 || g->table_capacity > (1ull << 31)) return DEDUP_EINVAL;
+    if (g->window != 32 || g->min_chunk != 32 || g->max_chunk != 0) return DEDUP_EUNSUPPORTED;
+    return DEDUP_OK;
+}
+
+// Turn a completed slot's host results into per-item views + stats.
+dedup_status parse_slot(dedup_ctx* c, Slot& sl) {
+    const uint32_t n = sl.hhost.header[0];
+    if (sl.hhost.header[1] != 0)
+        return fail(c, DEDUP_ETABLEFULL, "digest table overflow: raise table_capacity");
+    if (n > c->chunk_cap) return fail(c, DEDUP_ECUDA, "chunk capacity exceeded");
+    sl.item_first.assign(sl.n_items, 0);
+    sl.item_n.assign(sl.n_items, 0);
+    uint32_t next = n;
+    for (int64_t k = (int64_t)sl.n_items - 1; k >= 0; --k) {
+        uint32_t f = sl.hhost.item_first_chunk[k];
+        if (f == 0xFFFFFFFFu) {
+            sl.item_first[k] = next;
+            sl.item_n[k] = 0;
+        } else {
+            sl.item_first[k] = f;
+            sl.item_n[k] = next - f;
+            next = f;
+        }
+    }
+    // stats
+    uint64_t dups = 0, dup_bytes = 0, blocks = 0;
+    for (uint32_t k = 0; k < sl.n_items; ++k) {
+        const uint32_t f = sl.item_first[k], m = sl.item_n[k];
+        for (uint32_t j = 0; j < m; ++j) {
+            const uint64_t s0 = sl.hhost.chunk_start[f + j];
+            const uint64_t s1 = j + 1 < m ? sl.hhost.chunk_start[f + j + 1] : sl.item_len[k];
+            blocks += (s1 - s0 + 9 + 63) / 64;
+            if (sl.hhost.is_dup[f + j]) {
+                ++dups;
+                dup_bytes += s1 - s0;
+            }
+        }
+    }
+    c->st.sha1_blocks += blocks;
+    c->st.chunks += n;
+    c->st.dup_chunks += dups;
+    c->st.unique_chunks += n - dups;
+    c->st.dup_bytes += dup_bytes;
+    c->st.items += sl.n_items;
+    c->st.bytes += sl.nbytes;
+    float ms = 0;
+    if (sl.host_fed && cudaEventElapsedTime(&ms, sl.ev_start, sl.ev_h2d) == cudaSuccess)
+        c->st.ms_h2d += ms;
+    if (cudaEventElapsedTime(&ms, sl.ev_h2d, sl.ev_scan) == cudaSuccess) c->st.ms_scan += ms;
+    if (cudaEventElapsedTime(&ms, sl.ev_scan, sl.ev_chunk) == cudaSuccess) c->st.ms_select += ms;
+    if (cudaEventElapsedTime(&ms, sl.ev_chunk, sl.ev_sha) == cudaSuccess) c->st.ms_sha1 += ms;
+    if (cudaEventElapsedTime(&ms, sl.ev_sha, sl.ev_table) == cudaSuccess) c->st.ms_table += ms;
+    if (cudaEventElapsedTime(&ms, sl.ev_table, sl.ev_done) == cudaSuccess) c->st.ms_d2h += ms;
+    sl.parsed = true;
+    return DEDUP_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+void dedup_config_default(dedup_config* g) {
+    std::memset(g, 0, sizeof(*g));
+    g->struct_size = sizeof(dedup_config);
+    g->window = 32;
+    g->poly = 0x45C2B6A1u;
+    g->anchor_mask = 0xFFFu;
+    g->anchor_value = 0;
+    g->min_chunk = 32;
+    g->max_chunk = 0;
+    g->device = 0;
+    g->slots = 4;
+    g->batch_items = 4096;
+    g->batch_bytes = 64ull << 20;
+    g->table_capacity = 1ull << 20;
+    g->owner_rank = 0;
+    g->num_owners = 1;
+    g->host_fed = 1;
+}
+
+dedup_status dedup_init(const dedup_config* cfg, dedup_ctx** out) {
+    if (out == nullptr) return DEDUP_EINVAL;
+    *out = nullptr;
+    dedup_status s = check_cfg(cfg);
+    if (s != DEDUP_OK) return s;
+    dedup_ctx* c = new dedup_ctx();
+    c->cfg = *cfg;
+    auto bail = [&](dedup_status r) {
+        dedup_destroy(c);
+        return r;
+    };
+    if (cudaSetDevice(cfg->device) != cudaSuccess) return bail(DEDUP_ECUDA);
+    if (cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, cfg->device) !=
+        cudaSuccess)
+        return bail(DEDUP_ECUDA);
+    c->chunk_cap = cfg->batch_bytes / 32 + cfg->batch_items + 2;
+    uint32_t tab[512];
+    for (uint32_t b = 0; b < 256; ++b) {
+        tab[b] = mul_tk(b, 32, cfg->poly);         // R[b]    = b t^32  mod P
+        tab[256 + b] = mul_tk(b, 256, cfg->poly);  // W256[b] = b t^256 mod P
+    }
+    if ((s = dalloc(c, &c->d_tab, 512)) != DEDUP_OK) return bail(s);
+    if (cudaMemcpy(c->d_tab, tab, sizeof(tab), cudaMemcpyHostToDevice) != cudaSuccess)
+        return bail(DEDUP_ECUDA);
+    for (TableBuf& t : c->tables) {
+        t.capacity = next_pow2(2 * cfg->table_capacity);
+        if ((s = dalloc(c, &t.slots, t.capacity)) != DEDUP_OK) return bail(s);
+        if ((s = dalloc(c, &t.status, 4)) != DEDUP_OK) return bail(s);
+        if (cudaMemset(t.slots, 0, sizeof(TableSlot) * t.capacity) != cudaSuccess ||
+            cudaMemset(t.status, 0, 16) != cudaSuccess ||
+            cudaEventCreateWithFlags(&t.last_use, cudaEventDisableTiming) != cudaSuccess)
+            return bail(DEDUP_ECUDA);
+    }
+    c->tables[0].used = true;  // stream 0 starts on table 0 (cleared above)
+    c->stream_fresh = false;
+    if ((s = ws_alloc(c, c->op_ws, cfg->batch_bytes, c->chunk_cap)) != DEDUP_OK) return bail(s);
+    c->slots.resize(cfg->slots);
+    for (Slot& sl : c->slots)
+        if ((s = slot_alloc(c, sl)) != DEDUP_OK) return bail(s);
+    if (cudaDeviceSynchronize() != cudaSuccess) return bail(DEDUP_ECUDA);
+    c->st.table_slots = c->tables[0].capacity;
+    c->st.num_owners = cfg->num_owners;
+    c->st.owner_rank = cfg->owner_rank;
+    *out = c;
+    return DEDUP_OK;
+}
+
+void dedup_destroy(dedup_ctx* c) {
+    if (c == nullptr) return;
+    cudaSetDevice(c->cfg.device);
+    for (Slot& sl : c->slots) slot_free(sl);
+    ws_free(c->op_ws);
+    for (TableBuf& t : c->tables) {
+        cudaFree(t.slots);
+        cudaFree(t.status);
+        if (t.last_use) cudaEventDestroy(t.last_use);
+    }
+    cudaFree(c->d_tab);
+    delete c;
+}
+
+const char* dedup_last_error(const dedup_ctx* c) {
+    return c == nullptr ? "null ctx" : c->err.c_str();
+}
+
+dedup_status dedup_submit_batch(dedup_ctx* c, uint32_t n_items, const uint8_t* const* item_ptr,
+                                const uint64_t* item_len, uint64_t* first_seq_out) {
+    if (c == nullptr) return DEDUP_EINVAL;
+    if (!usable(c)) return c->sticky;
+    if (!c->cfg.host_fed) return fail(c, DEDUP_EINVAL, "ctx was created with host_fed = 0");
+    if (c->cfg.num_owners != 1)
+        return fail(c, DEDUP_EUNSUPPORTED, "num_owners > 1: use the dedup_op_* orchestration");
+    if (n_items > 0 && (item_ptr == nullptr || item_len == nullptr))
+        return fail(c, DEDUP_EINVAL, "null item arrays");
+    CU(cudaSetDevice(c->cfg.device));
+    // plan batches
+    std::vector<std::pair<uint32_t, uint32_t>> plan;  // [first, last) item ranges
+    uint32_t b0 = 0;
+    uint64_t bytes = 0;
+    for (uint32_t k = 0; k < n_items; ++k) {
+        const uint64_t L = item_len[k];
+        if (L > c->cfg.batch_bytes || L > 0xFFFFFFFFull)
+            return fail(c, DEDUP_EINVAL, "item larger than batch_bytes");
+        if (L > 0 && item_ptr[k] == nullptr) return fail(c, DEDUP_EINVAL, "null item pointer");
+        if (k > b0 && (bytes + L > c->cfg.batch_bytes || k - b0 >= c->cfg.batch_items)) {
+            plan.emplace_back(b0, k);
+            b0 = k;
+            bytes = 0;
+        }
+        bytes += L;
+    }
+    if (n_items > b0) plan.emplace_back(b0, n_items);
+    if ((int)plan.size() > free_slot_count(c))
+        return fail(c, DEDUP_EAGAIN, "no free batch slot");
+    if (first_seq_out) *first_seq_out = c->next_seq;
+    for (auto& r : plan) {
+        const int i = take_free_slot(c);
+        Slot& sl = c->slots[i];
+        sl.host_fed = true;
+        sl.first_seq = c->next_seq;
+        sl.n_items = r.second - r.first;
+        sl.item_len.assign(item_len + r.first, item_len + r.second);
+        uint64_t off = 0;
+        sl.h_item_off[0] = 0;
+        for (uint32_t k = 0; k < sl.n_items; ++k) sl.h_item_off[k + 1] = (off += sl.item_len[k]);
+        sl.nbytes = off;
+        CU(cudaEventRecord(sl.ev_start, sl.stream));
+        // H2D of the items (row A1), merging contiguous host ranges
+        uint32_t k = 0;
+        while (k < sl.n_items) {
+            const uint8_t* p = item_ptr[r.first + k];
+            uint64_t dst = sl.h_item_off[k], len = sl.item_len[k];
+            uint32_t j = k + 1;
+            while (j < sl.n_items && item_ptr[r.first + j] == p + len) len += sl.item_len[j++];
+            if (len) CU(cudaMemcpyAsync(sl.d_bytes + dst, p, len, cudaMemcpyHostToDevice,
+                                        sl.stream));
+            k = j;
+        }
+        TRY(launch_batch(c, i, sl.d_bytes));
+        c->next_seq += sl.n_items;
+    }
+    return DEDUP_OK;
+}
+
+dedup_status dedup_submit_device(dedup_ctx* c, const uint8_t* d_bytes, uint64_t nbytes,
+                                 const uint64_t* item_off, uint32_t n_items, void* producer,
+                                 uint64_t* first_seq_out) {
+    if (c == nullptr) return DEDUP_EINVAL;
+    if (!usable(c)) return c->sticky;
+    if (c->cfg.num_owners != 1)
+        return fail(c, DEDUP_EUNSUPPORTED, "num_owners > 1: use the dedup_op_* orchestration");
+    if (item_off == nullptr || (nbytes > 0 && d_bytes == nullptr))
+        return fail(c, DEDUP_EINVAL, "null argument");
+    if (reinterpret_cast<uintptr_t>(d_bytes) & 15)
+        return fail(c, DEDUP_EINVAL, "d_bytes must be 16-byte aligned");
+    if (nbytes > c->cfg.batch_bytes || n_items > c->cfg.batch_items)
+        return fail(c, DEDUP_EINVAL, "batch larger than batch_bytes / batch_items");
+    if (item_off[0] != 0 || item_off[n_items] != nbytes)
+        return fail(c, DEDUP_EINVAL, "item_off must start at 0 and end at nbytes");
+    for (uint32_t k = 0; k < n_items; ++k)
+        if (item_off[k + 1] < item_off[k]) return fail(c, DEDUP_EINVAL, "item_off decreasing");
+    const int i = take_free_slot(c);
+    if (i < 0) return fail(c, DEDUP_EAGAIN, "no free batch slot");
+    CU(cudaSetDevice(c->cfg.device));
+    Slot& sl = c->slots[i];
+    sl.host_fed = false;
+    sl.first_seq = c->next_seq;
+    sl.n_items = n_items;
+    sl.nbytes = nbytes;
+    sl.item_len.resize(n_items);
+    for (uint32_t k = 0; k < n_items; ++k) sl.item_len[k] = item_off[k + 1] - item_off[k];
+    std::memcpy(sl.h_item_off, item_off, sizeof(uint64_t) * (n_items + 1));
+    CU(cudaEventRecord(sl.ev_prod, static_cast<cudaStream_t>(producer)));
+    CU(cudaStreamWaitEvent(sl.stream, sl.ev_prod, 0));
+    CU(cudaEventRecord(sl.ev_start, sl.stream));
+    if (first_seq_out) *first_seq_out = c->next_seq;
+    TRY(launch_batch(c, i, d_bytes));
+    c->next_seq += n_items;
+    return DEDUP_OK;
+}
+
+dedup_status dedup_join(dedup_ctx* c, void* stream) {
+    if (c == nullptr) return DEDUP_EINVAL;
+    if (!usable(c)) return c->sticky;
+    CU(cudaSetDevice(c->cfg.device));
+    for (int i : c->inflight)
+        CU(cudaStreamWaitEvent(static_cast<cudaStream_t>(stream), c->slots[i].ev_done, 0));
+    return DEDUP_OK;
+}
+
+dedup_status dedup_end_stream(dedup_ctx* c) {
+    if (c == nullptr) return DEDUP_EINVAL;
+    if (!usable(c)) return c->sticky;
+    c->cur_table ^= 1;
+    c->stream_fresh = true;
+    c->chain_valid = false;
+    return DEDUP_OK;
+}
+
+dedup_status dedup_drain(dedup_ctx* c, uint32_t max_items, int32_t wait_ms,
+                         dedup_item_result* out, uint32_t* n_out) {
+    if (c == nullptr || n_out == nullptr || (max_items > 0 && out == nullptr)) return DEDUP_EINVAL;
+    *n_out = 0;
+    if (!usable(c)) return c->sticky;
+    CU(cudaSetDevice(c->cfg.device));
+    for (int i : c->to_release) c->slots[i].busy = false;
+    c->to_release.clear();
+    uint32_t got = 0;
+    const auto deadline = std::chrono::steady_clock::now() + std::chrono::milliseconds(wait_ms);
+    while (got < max_items && !c->inflight.empty()) {
+        const int i = c->inflight.front();
+        Slot& sl = c->slots[i];
+        if (!sl.parsed) {
+            cudaError_t q = cudaEventQuery(sl.ev_done);
+            if (q == cudaErrorNotReady) {
+                if (got > 0 || wait_ms == 0) break;
+                if (wait_ms < 0) {
+                    q = cudaEventSynchronize(sl.ev_done);
+                } else {
+                    while ((q = cudaEventQuery(sl.ev_done)) == cudaErrorNotReady &&
+                           std::chrono::steady_clock::now() < deadline)
+                        std::this_thread::sleep_for(std::chrono::microseconds(20));
+                    if (q == cudaErrorNotReady)
+                        return fail(c, DEDUP_ETIMEDOUT, "no batch completed within wait_ms");
+                }
+            }
+            if (q != cudaSuccess)
+                return fail(c, DEDUP_ECUDA, std::string("batch failed: ") + cudaGetErrorString(q));
+            TRY(parse_slot(c, sl));
+        }
+        while (got < max_items && sl.next_item < sl.n_items) {
+            const uint32_t k = sl.next_item++;
+            dedup_item_result& r = out[got++];
+            r.seq = sl.first_seq + k;
+            r.item_len = sl.item_len[k];
+            r.n_chunks = sl.item_n[k];
+            r.reserved = 0;
+            if (r.n_chunks) {
+                const uint32_t f = sl.item_first[k];
+                r.chunk_start = sl.hhost.chunk_start + f;
+                r.digest = sl.hhost.digest + 20ull * f;
+                r.is_dup = sl.hhost.is_dup + f;
+                r.first_id = sl.hhost.first_id + f;
+            } else {
+                r.chunk_start = nullptr;
+                r.digest = nullptr;
+                r.is_dup = nullptr;
+                r.first_id = nullptr;
+            }
+            --c->pending_items;
+        }
+        if (sl.next_item == sl.n_items) {
+            c->inflight.pop_front();
+            c->to_release.push_back(i);  // results stay valid until the next drain
+        }
+    }
+    *n_out = got;
+    return DEDUP_OK;
+}
+
+uint64_t dedup_pending(const dedup_ctx* c) { return c ? c->pending_items : 0; }
+
+dedup_status dedup_stats(const dedup_ctx* c, dedup_stats_t* out) {
+    if (c == nullptr || out == nullptr) return DEDUP_EINVAL;
+    *out = c->st;
+    out->kernel_launches = c->launches;
+    return DEDUP_OK;
+}
+
+void* dedup_host_alloc(dedup_ctx* c, size_t bytes) {
+    if (c == nullptr) return nullptr;
+    cudaSetDevice(c->cfg.device);
+    void* p = nullptr;
+    if (cudaHostAlloc(&p, bytes, cudaHostAllocPortable) != cudaSuccess) return nullptr;
+    return p;
+}
+
+void dedup_host_free(dedup_ctx* c, void* p) {
+    (void)c;
+    if (p) cudaFreeHost(p);
+}
+
+uint64_t dedup_kernel_launches(const dedup_ctx* c) { return c ? c->launches : 0; }
+
+// ---------------------------------------------------------------------------
+// Stream-ordered device operations
+// ---------------------------------------------------------------------------
+dedup_status dedup_op_chunk(dedup_ctx* c, void* stream, const uint8_t* d_bytes, uint64_t nbytes,
+                            const uint64_t* d_item_off, uint32_t n_items, uint32_t* d_cut_pos,
+                            uint64_t cap, uint32_t* d_n_chunks) {
+    if (c == nullptr) return DEDUP_EINVAL;
+    if (!usable(c)) return c->sticky;
+    if (nbytes > c->cfg.batch_bytes) return fail(c, DEDUP_EINVAL, "nbytes > batch_bytes");
+    if (reinterpret_cast<uintptr_t>(d_bytes) & 15)
+        return fail(c, DEDUP_EINVAL, "d_bytes must be 16-byte aligned");
+    CU(cudaSetDevice(c->cfg.device));
+    return enqueue_chunk(c, c->op_ws, static_cast<cudaStream_t>(stream), d_bytes, nbytes,
+                         d_item_off, n_items, d_cut_pos, cap, d_n_chunks);
+}
+
+dedup_status dedup_op_chunk_meta(dedup_ctx* c, void* stream, const uint64_t* d_item_off,
+                                 uint32_t n_items, const uint32_t* d_cut_pos,
+                                 const uint32_t* d_n_chunks, uint64_t cap, uint64_t first_seq,
+                                 uint32_t* d_chunk_start, uint64_t* d_chunk_id,
+                                 uint32_t* d_item_first_chunk) {
+    if (c == nullptr) return DEDUP_EINVAL;
+    if (!usable(c)) return c->sticky;
+    CU(cudaSetDevice(c->cfg.device));
+    launch_chunk_meta(d_item_off, n_items, d_cut_pos, d_n_chunks, cap, first_seq, d_chunk_start,
+                      d_chunk_id, d_item_first_chunk, c->num_sms,
+                      static_cast<cudaStream_t>(stream));
+    c->launches += (cap && n_items) ? 1 : 0;
+    CU(cudaGetLastError());
+    return DEDUP_OK;
+}
+
+dedup_status dedup_op_sha1(dedup_ctx* c, void* stream, const uint8_t* d_bytes, uint64_t nbytes,
+                           const uint32_t* d_cut_pos, const uint32_t* d_n_chunks, uint64_t cap,
+                           uint8_t* d_digest) {
+    if (c == nullptr) return DEDUP_EINVAL;
+    if (!usable(c)) return c->sticky;
+    if (reinterpret_cast<uintptr_t>(d_bytes) & 15)
+        return fail(c, DEDUP_EINVAL, "d_bytes must be 16-byte aligned");
+    if (reinterpret_cast<uintptr_t>(d_digest) & 3)
+        return fail(c, DEDUP_EINVAL, "d_digest must be 4-byte aligned");
+    CU(cudaSetDevice(c->cfg.device));
+    launch_sha1(d_bytes, nbytes, d_cut_pos, d_n_chunks, cap, c->op_ws.counters + 1, d_digest,
+                c->num_sms, static_cast<cudaStream_t>(stream));
+    c->launches += 1;
+    CU(cudaGetLastError());
+    return DEDUP_OK;
+}
+
+dedup_status dedup_op_table_insert_lookup(dedup_ctx* c, void* stream, const uint8_t* d_digest,
+                                          const uint64_t* d_id, const uint32_t* d_n, uint64_t cap,
+                                          uint64_t* d_first_id, uint8_t* d_is_dup) {
+    if (c == nullptr) return DEDUP_EINVAL;
+    if (!usable(c)) return c->sticky;
+    if (cap > c->chunk_cap) return fail(c, DEDUP_EINVAL, "cap larger than the ctx workspace");
+    CU(cudaSetDevice(c->cfg.device));
+    return enqueue_table(c, c->op_ws, static_cast<cudaStream_t>(stream), d_digest, d_id, d_n, cap,
+                         d_first_id, d_is_dup);
+}
+
+dedup_status dedup_op_table_reset(dedup_ctx* c, void* stream) {
+    if (c == nullptr) return DEDUP_EINVAL;
+    if (!usable(c)) return c->sticky;
+    CU(cudaSetDevice(c->cfg.device));
+    TableBuf& t = c->tables[c->cur_table];
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    CU(cudaMemsetAsync(t.slots, 0, sizeof(TableSlot) * t.capacity, s));
+    CU(cudaMemsetAsync(t.status, 0, 16, s));
+    return DEDUP_OK;
+}
+
+dedup_status dedup_op_table_status(dedup_ctx* c, void* stream, uint64_t* used, uint64_t* slots,
+                                   int32_t* overflow) {
+    if (c == nullptr) return DEDUP_EINVAL;
+    CU(cudaSetDevice(c->cfg.device));
+    TableBuf& t = c->tables[c->cur_table];
+    uint32_t st[4];
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    CU(cudaMemcpyAsync(st, t.status, 16, cudaMemcpyDeviceToHost, s));
+    CU(cudaStreamSynchronize(s));
+    if (used) *used = st[1];
+    if (slots) *slots = t.capacity;
+    if (overflow) *overflow = (int32_t)st[0];
+    return DEDUP_OK;
+}
+
+dedup_status dedup_op_route(dedup_ctx* c, void* stream, const uint8_t* d_digest,
+                            const uint64_t* d_id, const uint32_t* d_n, uint64_t cap,
+                            uint32_t num_owners, dedup_record* d_send, uint32_t* d_send_off,
+                            uint32_t* d_send_pos) {
+    if (c == nullptr) return DEDUP_EINVAL;
+    if (!usable(c)) return c->sticky;
+    if (num_owners < 1 || num_owners > 64) return fail(c, DEDUP_EINVAL, "num_owners in 1..64");
+    CU(cudaSetDevice(c->cfg.device));
+    launch_route(d_digest, d_id, d_n, cap, num_owners, d_send, d_send_off, d_send_pos,
+                 c->op_ws.counters + 64, c->num_sms, static_cast<cudaStream_t>(stream));
+    c->launches += cap ? 3 : 1;
+    CU(cudaGetLastError());
+    return DEDUP_OK;
+}
+
+dedup_status dedup_op_owner(dedup_ctx* c, void* stream, const dedup_record* d_recv,
+                            uint64_t n_recv, uint64_t* d_reply) {
+    if (c == nullptr) return DEDUP_EINVAL;
+    if (!usable(c)) return c->sticky;
+    if (n_recv > c->chunk_cap) return fail(c, DEDUP_EINVAL, "n_recv larger than the workspace");
+    CU(cudaSetDevice(c->cfg.device));
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    TableView tv = table_view(c);
+    launch_table_insert(tv, nullptr, nullptr, d_recv, nullptr, n_recv, n_recv,
+                        c->op_ws.slot_idx, c->num_sms, s);
+    launch_table_lookup(tv, nullptr, d_recv, nullptr, n_recv, n_recv, c->op_ws.slot_idx, d_reply,
+                        nullptr, c->num_sms, s);
+    c->launches += n_recv ? 2 : 0;
+    CU(cudaGetLastError());
+    return DEDUP_OK;
+}
+
+dedup_status dedup_op_scatter(dedup_ctx* c, void* stream, const uint64_t* d_reply_back,
+                              const uint32_t* d_send_pos, const uint64_t* d_id,
+                              const uint32_t* d_n, uint64_t cap, uint64_t* d_first_id,
+                              uint8_t* d_is_dup) {
+    if (c == nullptr) return DEDUP_EINVAL;
+    if (!usable(c)) return c->sticky;
+    CU(cudaSetDevice(c->cfg.device));
+    launch_scatter(d_reply_back, d_send_pos, d_id, d_n, cap, d_first_id, d_is_dup, c->num_sms,
+                   static_cast<cudaStream_t>(stream));
+    c->launches += cap ? 1 : 0;
+    CU(cudaGetLastError());
+    return DEDUP_OK;
+}
+
+}  // extern "C"

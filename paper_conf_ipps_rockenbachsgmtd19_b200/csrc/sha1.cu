@@ -1,0 +1,211 @@
+// sha1.cu -- row A4 of the hot path: SHA-1 (FIPS 180-4) of every chunk.
+// "each GPU thread calculates the SHA-1 of one block. The
+// result is saved in an array".
+//
+// Kept from the paper: one lane owns one chunk (SHA-1 is a sequential chain
+// of 64-byte compressions, so a chunk cannot be split).  Changed for sm_100a:
+//   * persistent warps pull chunks from a device work counter with one
+//     warp-aggregated atomic; a lane that finishes its chunk picks up the next
+//     one at the following 64-byte step, so lanes of a warp stay busy even
+//     though chunk lengths vary from 32 B to megabytes (block-granular load
+//     balancing instead of one launch thread per chunk);
+//   * the 16-word message schedule lives in registers (fully unrolled
+//     rounds, circular W[16]) and rotates are funnel shifts (SHF);
+//   * unaligned chunk data is read with five 16-byte loads and realigned with
+//     two select stages + one PRMT per word (PRMT also does the big-endian
+//     byte swap).
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "internal.h"
+
+namespace dd {
+
+namespace {
+
+constexpr int kShaThreads = 128;
+constexpr uint32_t kFull = 0xFFFFFFFFu;
+
+__device__ __forceinline__ uint32_t rotl(uint32_t x, int s) { return __funnelshift_l(x, x, s); }
+
+__device__ __forceinline__ void sha1_compress(uint32_t H[5], uint32_t W[16]) {
+    uint32_t a = H[0], b = H[1], c = H[2], d = H[3], e = H[4];
+#pragma unroll
+    for (int t = 0; t < 80; ++t) {
+        uint32_t w;
+        if (t < 16) {
+            w = W[t];
+        } else {
+            w = rotl(W[(t - 3) & 15] ^ W[(t - 8) & 15] ^ W[(t - 14) & 15] ^ W[t & 15], 1);
+            W[t & 15] = w;
+        }
+        uint32_t f, K;
+        if (t < 20) {
+            f = (b & c) ^ (~b & d);
+            K = 0x5A827999u;
+        } else if (t < 40) {
+            f = b ^ c ^ d;
+            K = 0x6ED9EBA1u;
+        } else if (t < 60) {
+            f = (b & c) ^ (b & d) ^ (c & d);
+            K = 0x8F1BBCDCu;
+        } else {
+            f = b ^ c ^ d;
+            K = 0xCA62C1D6u;
+        }
+        const uint32_t T = rotl(a, 5) + f + e + K + w;
+        e = d;
+        d = c;
+        c = rotl(b, 30);
+        b = a;
+        a = T;
+    }
+    H[0] += a;
+    H[1] += b;
+    H[2] += c;
+    H[3] += d;
+    H[4] += e;
+}
+
+// 64 message bytes starting at byte offset p (any alignment) as 16
+// big-endian words.  Reads the 16-byte-aligned window [p & ~15, +80); with
+// guard, vectors at or beyond lim16 read as zero.
+template <bool kGuard>
+__device__ __forceinline__ void load_block(const uint8_t* __restrict__ bytes, uint64_t p,
+                                           uint64_t lim16, uint32_t M[16]) {
+    const uint64_t base = p & ~uint64_t(15);
+    const uint32_t o = (uint32_t)(p & 15);
+    uint32_t v[20];
+#pragma unroll
+    for (int i = 0; i < 5; ++i) {
+        uint4 x = make_uint4(0, 0, 0, 0);
+        const uint64_t a = base + 16 * i;
+        bool ok = (i < 4) || (o != 0);
+        if (kGuard) ok = ok && (a < lim16);
+        if (ok) x = __ldg(reinterpret_cast<const uint4*>(bytes + a));
+        v[4 * i] = x.x;
+        v[4 * i + 1] = x.y;
+        v[4 * i + 2] = x.z;
+        v[4 * i + 3] = x.w;
+    }
+    const uint32_t wsh = o >> 2;
+    if (wsh & 2) {
+#pragma unroll
+        for (int i = 0; i < 18; ++i) v[i] = v[i + 2];
+    }
+    if (wsh & 1) {
+#pragma unroll
+        for (int i = 0; i < 17; ++i) v[i] = v[i + 1];
+    }
+    const uint32_t sel = 0x0123u + (o & 3) * 0x1111u;
+#pragma unroll
+    for (int j = 0; j < 16; ++j) M[j] = __byte_perm(v[j], v[j + 1], sel);
+}
+
+__global__ void __launch_bounds__(kShaThreads, 8)
+sha1_kernel(const uint8_t* __restrict__ bytes, uint64_t nbytes,
+            const uint32_t* __restrict__ cut_pos, const uint32_t* __restrict__ n_chunks_p,
+            uint64_t cap, uint32_t* work_counter, uint8_t* __restrict__ digest) {
+    const uint32_t n = (uint32_t)min((uint64_t)*n_chunks_p, cap);
+    const uint32_t lane = threadIdx.x & 31;
+    const uint64_t lim16 = (nbytes + 15) & ~uint64_t(15);
+    int64_t k = -1;      // chunk owned by this lane
+    uint64_t p = 0;      // next byte of the chunk to consume
+    uint32_t rem = 0;    // chunk bytes not yet consumed
+    uint32_t len = 0;    // chunk length
+    uint32_t phase = 0;  // 1: only the length block is left
+    bool done = false;
+    uint32_t H[5] = {0, 0, 0, 0, 0};
+    while (true) {
+        const bool need = !done && k < 0;
+        const uint32_t m = __ballot_sync(kFull, need);
+        if (m) {
+            const int leader = __ffs(m) - 1;
+            uint32_t base = 0;
+            if ((int)lane == leader) base = atomicAdd(work_counter, (uint32_t)__popc(m));
+            base = __shfl_sync(kFull, base, leader);
+            if (need) {
+                const uint32_t idx = base + __popc(m & ((1u << lane) - 1u));
+                if (idx < n) {
+                    k = idx;
+                    const uint32_t s = cut_pos[idx];
+                    const uint64_t e = (idx + 1 < n) ? (uint64_t)cut_pos[idx + 1] : nbytes;
+                    p = s;
+                    rem = len = (uint32_t)(e - s);
+                    phase = 0;
+                    H[0] = 0x67452301u;
+                    H[1] = 0xEFCDAB89u;
+                    H[2] = 0x98BADCFEu;
+                    H[3] = 0x10325476u;
+                    H[4] = 0xC3D2E1F0u;
+                } else {
+                    done = true;
+                }
+            }
+        }
+        if (__all_sync(kFull, done)) break;
+        if (!done) {
+            uint32_t M[16];
+            bool fin = false;
+            if (phase == 0 && rem >= 64) {
+                load_block<false>(bytes, p, lim16, M);
+                p += 64;
+                rem -= 64;
+            } else if (phase == 0) {
+                // final data block: rem (0..63) bytes, 0x80, zeros [, length]
+                load_block<true>(bytes, p, lim16, M);
+#pragma unroll
+                for (int j = 0; j < 16; ++j) {
+                    const int nv = (int)rem - 4 * j;
+                    uint32_t w = M[j];
+                    if (nv < 4) {
+                        if (nv >= 0) {
+                            const uint32_t keep = nv == 0 ? 0u : (0xFFFFFFFFu << (32 - 8 * nv));
+                            w = (w & keep) | (0x80u << (24 - 8 * nv));
+                        } else {
+                            w = 0;
+                        }
+                    }
+                    M[j] = w;
+                }
+                if (rem <= 55) {
+                    M[14] = len >> 29;
+                    M[15] = len << 3;
+                    fin = true;
+                } else {
+                    phase = 1;
+                }
+                rem = 0;
+            } else {
+#pragma unroll
+                for (int j = 0; j < 14; ++j) M[j] = 0;
+                M[14] = len >> 29;
+                M[15] = len << 3;
+                fin = true;
+            }
+            sha1_compress(H, M);
+            if (fin) {
+                uint32_t* out = reinterpret_cast<uint32_t*>(digest + 20 * (uint64_t)k);
+#pragma unroll
+                for (int i = 0; i < 5; ++i) out[i] = __byte_perm(H[i], 0, 0x0123);
+                k = -1;
+            }
+        }
+    }
+}
+
+}  // namespace
+
+void launch_sha1(const uint8_t* bytes, uint64_t nbytes, const uint32_t* cut_pos,
+                 const uint32_t* n_chunks, uint64_t cap, uint32_t* work_counter,
+                 uint8_t* digest, int num_sms, cudaStream_t s) {
+    cudaMemsetAsync(work_counter, 0, sizeof(uint32_t), s);
+    if (cap == 0) return;
+    uint64_t blocks = (cap + kShaThreads - 1) / kShaThreads;
+    const uint64_t max_blocks = (uint64_t)num_sms * 8;
+    if (blocks > max_blocks) blocks = max_blocks;
+    sha1_kernel<<<(unsigned)blocks, kShaThreads, 0, s>>>(bytes, nbytes, cut_pos, n_chunks, cap,
+                                                         work_counter, digest);
+}
+
+}  // namespace dd

@@ -1,0 +1,266 @@
+// table.cu -- rows A5 (route by digest owner), A7 (global digest table:
+// insert + lookup), A8 (reply scatter) and A9 (results into pinned host
+// memory).  PAPER.md P:215: "it checks if blocks in the batch are
+// duplicated"; results are reordered by sequence on the host.
+//
+// The table is a GPU-resident open-addressing hash table of 32-byte slots
+// (one L2 sector each): 20-byte digest key, a state word claimed by atomic
+// CAS (0 empty -> 1 writing -> 2 published), and ~min_id updated with
+// atomicMax, so the recorded first occurrence is the minimum (seq, index)
+// id -- the sequential stream-order answer -- independent of thread timing
+// (reading O12).  Linear probing from 64 digest bits that are
+// independent of the owner-routing prefix.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "internal.h"
+
+namespace dd {
+
+namespace {
+
+__device__ __forceinline__ uint32_t ld_acquire(const uint32_t* p) {
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ void load_key(const uint8_t* digest, const uint64_t* id,
+                                         const void* rec, uint64_t r, uint32_t key[5],
+                                         uint64_t& myid) {
+    if (rec != nullptr) {
+        const uint32_t* p = reinterpret_cast<const uint32_t*>(
+            static_cast<const uint8_t*>(rec) + 32 * r);
+#pragma unroll
+        for (int i = 0; i < 5; ++i) key[i] = p[i];
+        myid = *reinterpret_cast<const uint64_t*>(p + 6);
+    } else {
+        const uint32_t* p = reinterpret_cast<const uint32_t*>(digest + 20 * r);
+#pragma unroll
+        for (int i = 0; i < 5; ++i) key[i] = p[i];
+        myid = id != nullptr ? id[r] : 0;
+    }
+}
+
+__device__ __forceinline__ uint64_t record_count(const uint32_t* d_n, uint64_t n_host,
+                                                 uint64_t cap) {
+    return d_n != nullptr ? min((uint64_t)*d_n, cap) : n_host;
+}
+
+__global__ void table_insert_kernel(TableView t, const uint8_t* __restrict__ digest,
+                                    const uint64_t* __restrict__ id, const void* rec,
+                                    const uint32_t* d_n, uint64_t n_host, uint64_t cap,
+                                    uint32_t* __restrict__ slot_idx) {
+    const uint64_t n = record_count(d_n, n_host, cap);
+    for (uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; r < n;
+         r += (uint64_t)gridDim.x * blockDim.x) {
+        uint32_t key[5];
+        uint64_t myid;
+        load_key(digest, id, rec, r, key, myid);
+        // bytes 4..11 of the digest; bytes 0..3 pick the owner GPU
+        uint64_t idx = (((uint64_t)key[2] << 32) | key[1]) & t.mask;
+        uint32_t found = 0xFFFFFFFFu;
+        for (uint64_t probe = 0; probe <= t.mask; ++probe) {
+            TableSlot* s = t.slots + idx;
+            uint32_t st = ld_acquire(&s->state);
+            if (st == 0) {
+                const uint32_t old = atomicCAS(&s->state, 0u, 1u);
+                if (old == 0) {
+#pragma unroll
+                    for (int i = 0; i < 5; ++i) s->key[i] = key[i];
+                    __threadfence();
+                    atomicExch(&s->state, 2u);
+                    atomicAdd(&t.status[1], 1u);
+                    atomicMax(reinterpret_cast<unsigned long long*>(&s->inv_min),
+                              (unsigned long long)~myid);
+                    found = (uint32_t)idx;
+                    break;
+                }
+                st = old;
+            }
+            while (st == 1) st = ld_acquire(&s->state);
+            bool eq = true;
+#pragma unroll
+            for (int i = 0; i < 5; ++i) eq = eq && (ld_acquire(&s->key[i]) == key[i]);
+            if (eq) {
+                atomicMax(reinterpret_cast<unsigned long long*>(&s->inv_min),
+                          (unsigned long long)~myid);
+                found = (uint32_t)idx;
+                break;
+            }
+            idx = (idx + 1) & t.mask;
+        }
+        if (found == 0xFFFFFFFFu) atomicExch(&t.status[0], 1u);
+        slot_idx[r] = found;
+    }
+}
+
+__global__ void table_lookup_kernel(TableView t, const uint64_t* __restrict__ id,
+                                    const void* rec, const uint32_t* d_n, uint64_t n_host,
+                                    uint64_t cap, const uint32_t* __restrict__ slot_idx,
+                                    uint64_t* __restrict__ first_id, uint8_t* __restrict__ is_dup) {
+    const uint64_t n = record_count(d_n, n_host, cap);
+    for (uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; r < n;
+         r += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t si = slot_idx[r];
+        const uint64_t f = si == 0xFFFFFFFFu ? ~0ull : ~t.slots[si].inv_min;
+        first_id[r] = f;
+        if (is_dup != nullptr) {
+            uint64_t myid = rec != nullptr
+                                ? *reinterpret_cast<const uint64_t*>(
+                                      static_cast<const uint8_t*>(rec) + 32 * r + 24)
+                                : id[r];
+            is_dup[r] = (f != myid) ? 1 : 0;
+        }
+    }
+}
+
+__device__ __forceinline__ uint32_t owner_of(const uint8_t* digest, uint64_t r, uint32_t G) {
+    const uint32_t w = *reinterpret_cast<const uint32_t*>(digest + 20 * r);
+    const uint32_t be = __byte_perm(w, 0, 0x0123);  // BE32(digest[0..3])
+    return (uint32_t)(((uint64_t)be * G) >> 32);
+}
+
+__global__ void route_count_kernel(const uint8_t* __restrict__ digest, const uint32_t* d_n,
+                                   uint64_t cap, uint32_t G, uint32_t* counts) {
+    __shared__ uint32_t h[64];
+    for (int i = threadIdx.x; i < 64; i += blockDim.x) h[i] = 0;
+    __syncthreads();
+    const uint64_t n = min((uint64_t)*d_n, cap);
+    for (uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; r < n;
+         r += (uint64_t)gridDim.x * blockDim.x)
+        atomicAdd(&h[owner_of(digest, r, G)], 1u);
+    __syncthreads();
+    for (uint32_t i = threadIdx.x; i < G; i += blockDim.x)
+        if (h[i]) atomicAdd(&counts[i], h[i]);
+}
+
+__global__ void route_scan_kernel(uint32_t G, uint32_t* counts, uint32_t* send_off) {
+    if (threadIdx.x == 0 && blockIdx.x == 0) {
+        uint32_t acc = 0;
+        for (uint32_t i = 0; i < G; ++i) {
+            const uint32_t c = counts[i];
+            send_off[i] = acc;
+            counts[64 + i] = acc;  // scatter cursor
+            acc += c;
+        }
+        send_off[G] = acc;
+    }
+}
+
+__global__ void route_scatter_kernel(const uint8_t* __restrict__ digest,
+                                     const uint64_t* __restrict__ id, const uint32_t* d_n,
+                                     uint64_t cap, uint32_t G, uint32_t* counts, uint8_t* send,
+                                     uint32_t* __restrict__ send_pos) {
+    const uint64_t n = min((uint64_t)*d_n, cap);
+    for (uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; r < n;
+         r += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t o = owner_of(digest, r, G);
+        const uint32_t pos = atomicAdd(&counts[64 + o], 1u);
+        uint32_t* dst = reinterpret_cast<uint32_t*>(send + 32 * (uint64_t)pos);
+        const uint32_t* src = reinterpret_cast<const uint32_t*>(digest + 20 * r);
+#pragma unroll
+        for (int i = 0; i < 5; ++i) dst[i] = src[i];
+        dst[5] = 0;
+        *reinterpret_cast<uint64_t*>(dst + 6) = id[r];
+        send_pos[r] = pos;
+    }
+}
+
+__global__ void scatter_kernel(const uint64_t* __restrict__ reply,
+                               const uint32_t* __restrict__ send_pos,
+                               const uint64_t* __restrict__ id, const uint32_t* d_n, uint64_t cap,
+                               uint64_t* __restrict__ first_id, uint8_t* __restrict__ is_dup) {
+    const uint64_t n = min((uint64_t)*d_n, cap);
+    for (uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; r < n;
+         r += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t f = reply[send_pos[r]];
+        first_id[r] = f;
+        if (is_dup != nullptr) is_dup[r] = (f != id[r]) ? 1 : 0;
+    }
+}
+
+__global__ void pack_kernel(const uint32_t* __restrict__ n_chunks_p, uint64_t cap,
+                            uint32_t n_items, const uint32_t* __restrict__ chunk_start,
+                            const uint64_t* __restrict__ first_id,
+                            const uint8_t* __restrict__ digest, const uint8_t* __restrict__ is_dup,
+                            const uint32_t* __restrict__ item_first_chunk,
+                            const uint32_t* __restrict__ table_status, HostResultLayout h) {
+    const uint64_t n = min((uint64_t)*n_chunks_p, cap);
+    const uint64_t tid = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    if (tid == 0) {
+        h.header[0] = (uint32_t)*n_chunks_p;
+        h.header[1] = table_status[0];
+    }
+    for (uint64_t r = tid; r < n; r += stride) {
+        h.chunk_start[r] = chunk_start[r];
+        h.first_id[r] = first_id[r];
+        h.is_dup[r] = is_dup[r];
+    }
+    const uint32_t* dw = reinterpret_cast<const uint32_t*>(digest);
+    uint32_t* hw = reinterpret_cast<uint32_t*>(h.digest);
+    for (uint64_t r = tid; r < 5 * n; r += stride) hw[r] = dw[r];
+    for (uint64_t r = tid; r < n_items; r += stride) h.item_first_chunk[r] = item_first_chunk[r];
+}
+
+unsigned grid_for(uint64_t n, int threads, int num_sms, int per_sm) {
+    uint64_t b = (n + threads - 1) / threads;
+    const uint64_t mx = (uint64_t)num_sms * per_sm;
+    if (b > mx) b = mx;
+    if (b == 0) b = 1;
+    return (unsigned)b;
+}
+
+}  // namespace
+
+void launch_table_insert(TableView t, const uint8_t* digest, const uint64_t* id,
+                         const void* rec, const uint32_t* d_n, uint64_t n_host, uint64_t cap,
+                         uint32_t* slot_idx, int num_sms, cudaStream_t s) {
+    const uint64_t n = d_n != nullptr ? cap : n_host;
+    if (n == 0) return;
+    table_insert_kernel<<<grid_for(n, 256, num_sms, 8), 256, 0, s>>>(t, digest, id, rec, d_n,
+                                                                       n_host, cap, slot_idx);
+}
+
+void launch_table_lookup(TableView t, const uint64_t* id, const void* rec,
+                         const uint32_t* d_n, uint64_t n_host, uint64_t cap,
+                         const uint32_t* slot_idx, uint64_t* first_id, uint8_t* is_dup,
+                         int num_sms, cudaStream_t s) {
+    const uint64_t n = d_n != nullptr ? cap : n_host;
+    if (n == 0) return;
+    table_lookup_kernel<<<grid_for(n, 256, num_sms, 8), 256, 0, s>>>(
+        t, id, rec, d_n, n_host, cap, slot_idx, first_id, is_dup);
+}
+
+void launch_route(const uint8_t* digest, const uint64_t* id, const uint32_t* d_n, uint64_t cap,
+                  uint32_t num_owners, void* send, uint32_t* send_off, uint32_t* send_pos,
+                  uint32_t* scratch_counts, int num_sms, cudaStream_t s) {
+    cudaMemsetAsync(scratch_counts, 0, sizeof(uint32_t) * 128, s);
+    const unsigned g = grid_for(cap, 256, num_sms, 4);
+    if (cap) route_count_kernel<<<g, 256, 0, s>>>(digest, d_n, cap, num_owners, scratch_counts);
+    route_scan_kernel<<<1, 32, 0, s>>>(num_owners, scratch_counts, send_off);
+    if (cap)
+        route_scatter_kernel<<<g, 256, 0, s>>>(digest, id, d_n, cap, num_owners, scratch_counts,
+                                               static_cast<uint8_t*>(send), send_pos);
+}
+
+void launch_scatter(const uint64_t* reply, const uint32_t* send_pos, const uint64_t* id,
+                    const uint32_t* d_n, uint64_t cap, uint64_t* first_id, uint8_t* is_dup,
+                    int num_sms, cudaStream_t s) {
+    if (cap == 0) return;
+    scatter_kernel<<<grid_for(cap, 256, num_sms, 8), 256, 0, s>>>(reply, send_pos, id, d_n, cap,
+                                                                  first_id, is_dup);
+}
+
+void launch_pack(const uint32_t* n_chunks, uint64_t cap, uint32_t n_items,
+                 const uint32_t* chunk_start, const uint64_t* first_id, const uint8_t* digest,
+                 const uint8_t* is_dup, const uint32_t* item_first_chunk,
+                 const uint32_t* table_status, HostResultLayout h, int num_sms,
+                 cudaStream_t s) {
+    pack_kernel<<<grid_for(cap * 5 + n_items + 1, 256, num_sms, 4), 256, 0, s>>>(
+        n_chunks, cap, n_items, chunk_start, first_id, digest, is_dup, item_first_chunk,
+        table_status, h);
+}
+
+}  // namespace dd
