@@ -36,7 +36,7 @@ MiB = 1 << 20
 ITEM_BYTES = MiB                 # the paper's fixed 1 MB batches
 BATCH_BYTES = 32 * MiB           # GPU batch (step); C2 batch sweep 1-64 MiB
 BATCH_ITEMS = 64
-SLOTS = 6
+SLOTS = 16
 WORKLOAD = "C2"
 METRIC = "input GB/s & chunks/s (dedup hot path) at 1/2/4/8 B200; % of HBM/INT roofline"
 
@@ -227,7 +227,15 @@ def main():
     ap.add_argument("--impl", default="b200", choices=["b200", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=0, help="0 = min(steps, 120)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--batch-mb", type=int, default=0, help="override the GPU batch size")
+    ap.add_argument("--slots", type=int, default=0, help="override the in-flight batches")
     args = ap.parse_args()
+    global BATCH_BYTES, SLOTS, BATCH_ITEMS
+    if args.batch_mb:
+        BATCH_BYTES = args.batch_mb * MiB
+        BATCH_ITEMS = max(BATCH_ITEMS, BATCH_BYTES // ITEM_BYTES)
+    if args.slots:
+        SLOTS = args.slots
     if args.warmup < 3:
         args.warmup = 3
 

@@ -73,7 +73,7 @@ typedef struct {
     uint32_t min_chunk;      /* GPU v1 requires == window */
     uint32_t max_chunk;      /* 0 = none; GPU v1 requires 0 */
     int32_t device;          /* CUDA device ordinal of this ctx */
-    uint32_t slots;          /* in-flight batches ("memory spaces"), 1..16 */
+    uint32_t slots;          /* in-flight batches ("memory spaces"), 1..64 */
     uint32_t batch_items;    /* max items per GPU batch */
     uint64_t batch_bytes;    /* max bytes per GPU batch (<= 1 GiB) */
     uint64_t table_capacity; /* expected distinct digests per stream (this owner's share) */

@@ -1,20 +1,24 @@
 // api.cpp -- C ABI (include/dedup.h) and the per-GPU streaming engine.
 //
-// Engine (rows A1 + A9 of the hot path): a ring of `slots` batch slots, each
-// with its own CUDA stream, device buffers and a mapped pinned result buffer
-// ("memory spaces" used round-robin).  Per batch,
-// everything is enqueued asynchronously on the slot's stream:
-//   H2D (host-fed only) -> rabin_scan -> select -> chunk_meta -> sha1
-//   -> [wait previous batch's table event] -> table insert -> lookup
+// Engine (rows A1 + A9 of the hot path): a ring of `slots` batch slots used
+// strictly round-robin ("memory spaces").  Each
+// slot owns a CUDA stream, device buffers, a mapped pinned result buffer and
+// ONE CUDA GRAPH holding the whole per-batch launch sequence:
+//   desc + item offsets H2D -> rabin_scan -> select (agg, scan, emit)
+//   -> chunk_meta -> long_list -> sha1 -> [wait: previous slot's table event]
+//   -> table_prepare -> insert -> lookup -> [record table event]
 //   -> pack (kernel stores results straight into pinned host memory)
-// Table work of consecutive batches of one dedup stream is chained with
-// events, so every lookup sees the inserts of all earlier batches (the
-// sequential stream-order answer, reading O12).  No host synchronisation
-// happens between steps; dedup_drain waits on the slot's completion event and
-// hands items out strictly in sequence order.
+// Per-batch parameters live in a device-side BatchDesc copied by the graph
+// from the slot's pinned staging, so a submit is a host memcpy plus one
+// cudaGraphLaunch (+ an event pair for the producer stream or the H2D of
+// host items).  Table work of consecutive batches is chained through the
+// previous slot's table event, so every lookup sees the inserts of all
+// earlier batches (the sequential stream-order answer, reading O12) and a
+// table is only cleared after every earlier batch is done with it.
+// dedup_drain waits on the slot's completion event and hands items out
+// strictly in sequence order.
 #include <cuda_runtime.h>
 
-#include <algorithm>
 #include <chrono>
 #include <cstdio>
 #include <cstring>
@@ -30,35 +34,41 @@ using namespace dd;
 
 namespace {
 
+constexpr int kOpRing = 64;  // descriptors in flight for the dedup_op_* layer
+
 struct Workspace {
-    uint32_t* bitmap = nullptr;   // candidate bitmap, one bit per byte
-    uint64_t* desc = nullptr;     // look-back descriptors
-    uint32_t* counters = nullptr; // [0] tile counter, [1] sha1 work counter, [64..191] route
-    uint32_t* slot_idx = nullptr; // table slot per record
-    uint64_t n_desc_tiles = 0;
-    uint32_t epoch = 0;
+    uint32_t* bitmap = nullptr;      // candidate bitmap, one bit per byte
+    uint32_t* agg = nullptr;         // per-tile transfer functions (32 u32 per tile)
+    uint32_t* tile_entry = nullptr;  // per-tile entry state + cut offset
+    uint32_t* counters = nullptr;    // [0..1] sha1 work/long counters, [64..191] route
+    uint32_t* slot_idx = nullptr;    // table slot per record
+    uint32_t* long_list = nullptr;   // SHA-1 long-chunk list
+    uint64_t max_tiles = 0;
 };
 
 struct Slot {
     cudaStream_t stream = nullptr;
-    cudaEvent_t ev_start = nullptr, ev_h2d = nullptr, ev_scan = nullptr, ev_chunk = nullptr,
-                ev_sha = nullptr, ev_table = nullptr, ev_done = nullptr;
+    cudaEvent_t ev_host = nullptr, ev_start = nullptr, ev_h2d = nullptr, ev_scan = nullptr,
+                ev_chunk = nullptr, ev_sha = nullptr, ev_table = nullptr, ev_done = nullptr;
     cudaEvent_t ev_prod = nullptr;  // producer-stream dependency (no timing)
-    uint8_t* d_bytes = nullptr;  // host-fed input copy
+    cudaGraphExec_t graph = nullptr;
+    BatchDesc* d_desc = nullptr;    // device descriptor (graph copies h_desc into it)
+    BatchDesc* h_desc = nullptr;    // pinned staging
+    uint8_t* d_bytes = nullptr;     // host-fed input copy
     uint64_t* d_item_off = nullptr;
+    uint64_t* h_item_off = nullptr;  // pinned staging of item offsets
     Workspace ws;
     uint32_t* d_cut_pos = nullptr;
     uint32_t* d_chunk_start = nullptr;
     uint32_t* d_item_first = nullptr;
-    uint32_t* d_n_chunks = nullptr;
+    uint32_t* d_small = nullptr;    // [0] n_chunks, [4..5] table status copy
     uint64_t* d_chunk_id = nullptr;
     uint64_t* d_first_id = nullptr;
     uint8_t* d_digest = nullptr;
     uint8_t* d_is_dup = nullptr;
-    uint64_t* h_item_off = nullptr;  // pinned staging of item offsets
-    uint8_t* h_res = nullptr;        // mapped pinned results
-    HostResultLayout hdev{};         // device view of h_res
-    HostResultLayout hhost{};        // host view of h_res
+    uint8_t* h_res = nullptr;       // mapped pinned results
+    HostResultLayout hdev{};        // device view of h_res
+    HostResultLayout hhost{};       // host view of h_res
     // batch in flight
     bool busy = false;
     bool parsed = false;
@@ -75,8 +85,6 @@ struct TableBuf {
     TableSlot* slots = nullptr;
     uint32_t* status = nullptr;
     uint64_t capacity = 0;
-    cudaEvent_t last_use = nullptr;
-    bool used = false;
 };
 
 }  // namespace
@@ -86,20 +94,27 @@ struct dedup_ctx {
     int num_sms = 0;
     uint32_t* d_tab = nullptr;  // R[256] then W256[256]
     std::vector<Slot> slots;
+    uint32_t next_slot = 0;     // round-robin cursor
     TableBuf tables[2];
     int cur_table = 0;
-    bool stream_fresh = true;            // next batch starts a new dedup stream
-    cudaEvent_t chain_ev = nullptr;      // table event of the previous batch of this stream
-    bool chain_valid = false;
-    Workspace op_ws;
-    uint64_t chunk_cap = 0;              // chunks per slot
-    std::deque<int> inflight;            // slot indices in seq order
-    std::vector<int> to_release;         // slots fully handed out by the last drain
+    bool stream_fresh = false;  // next batch starts a new dedup stream
+    uint64_t chunk_cap = 0;     // chunks per slot
+    std::deque<int> inflight;   // slot indices in seq order
+    std::vector<int> to_release;
     uint64_t next_seq = 0;
     uint64_t pending_items = 0;
+    // dedup_op_* layer
+    Workspace op_ws;
+    BatchDesc* op_d_desc = nullptr;  // [kOpRing]
+    BatchDesc* op_h_desc = nullptr;  // [kOpRing] pinned
+    cudaEvent_t op_ev[kOpRing] = {};
+    bool op_ev_used[kOpRing] = {};
+    int op_next = 0;
+    // status
     dedup_status sticky = DEDUP_OK;
     std::string err = "no error";
     uint64_t launches = 0;
+    uint32_t graph_kernels = 0;  // kernels per batch graph
     dedup_stats_t st{};
 };
 
@@ -113,11 +128,17 @@ dedup_status fail(dedup_ctx* c, dedup_status s, const std::string& msg) {
     return s;
 }
 
-#define CU(call)                                                                        \
-    do {                                                                                \
-        cudaError_t e_ = (call);                                                        \
-        if (e_ != cudaSuccess)                                                          \
-            return fail(c, DEDUP_ECUDA, std::string(#call ": ") + cudaGetErrorString(e_)); \
+#define CU(call)                                                                             \
+    do {                                                                                     \
+        cudaError_t e_ = (call);                                                             \
+        if (e_ != cudaSuccess)                                                               \
+            return fail(c, DEDUP_ECUDA, std::string(#call ": ") + cudaGetErrorString(e_));   \
+    } while (0)
+
+#define TRY(x)                         \
+    do {                               \
+        dedup_status s_ = (x);         \
+        if (s_ != DEDUP_OK) return s_; \
     } while (0)
 
 // ---- product-side Rabin tables (independent of the oracle) ----------------
@@ -137,67 +158,125 @@ template <class T>
 dedup_status dalloc(dedup_ctx* c, T** p, uint64_t count) {
     if (count == 0) count = 1;
     cudaError_t e = cudaMalloc(reinterpret_cast<void**>(p), sizeof(T) * count);
-    if (e != cudaSuccess) return fail(c, DEDUP_ENOMEM, std::string("cudaMalloc: ") + cudaGetErrorString(e));
+    if (e != cudaSuccess)
+        return fail(c, DEDUP_ENOMEM, std::string("cudaMalloc: ") + cudaGetErrorString(e));
     return DEDUP_OK;
 }
 
-#define TRY(x)                            \
-    do {                                  \
-        dedup_status s_ = (x);            \
-        if (s_ != DEDUP_OK) return s_;    \
-    } while (0)
+template <class T>
+dedup_status halloc(dedup_ctx* c, T** p, uint64_t count, unsigned flags = cudaHostAllocPortable) {
+    if (count == 0) count = 1;
+    cudaError_t e = cudaHostAlloc(reinterpret_cast<void**>(p), sizeof(T) * count, flags);
+    if (e != cudaSuccess)
+        return fail(c, DEDUP_ENOMEM, std::string("cudaHostAlloc: ") + cudaGetErrorString(e));
+    return DEDUP_OK;
+}
 
 dedup_status ws_alloc(dedup_ctx* c, Workspace& w, uint64_t batch_bytes, uint64_t cap) {
-    w.n_desc_tiles = (batch_bytes + kSelTile - 1) / kSelTile + 1;
+    w.max_tiles = (batch_bytes + kSelTile - 1) / kSelTile + 1;
     TRY(dalloc(c, &w.bitmap, batch_bytes / 32 + 2));
-    TRY(dalloc(c, &w.desc, w.n_desc_tiles * kDescWords));
+    TRY(dalloc(c, &w.agg, w.max_tiles * 32));
+    TRY(dalloc(c, &w.tile_entry, w.max_tiles * 2));
     TRY(dalloc(c, &w.counters, 256));
     TRY(dalloc(c, &w.slot_idx, cap));
-    CU(cudaMemset(w.desc, 0, sizeof(uint64_t) * w.n_desc_tiles * kDescWords));
+    TRY(dalloc(c, &w.long_list, batch_bytes / kMinLongBytes + 2));
     CU(cudaMemset(w.counters, 0, sizeof(uint32_t) * 256));
     return DEDUP_OK;
 }
 
 void ws_free(Workspace& w) {
     cudaFree(w.bitmap);
-    cudaFree(w.desc);
+    cudaFree(w.agg);
+    cudaFree(w.tile_entry);
     cudaFree(w.counters);
     cudaFree(w.slot_idx);
+    cudaFree(w.long_list);
     w = Workspace{};
 }
 
 bool usable(const dedup_ctx* c) { return c != nullptr && c->sticky == DEDUP_OK; }
 
-TableView table_view(dedup_ctx* c) {
-    TableBuf& t = c->tables[c->cur_table];
+// Chunks at least 4x the mean anchor distance are hashed first.
+uint32_t long_bytes(const dedup_ctx* c) {
+    uint64_t v = 4ull * ((uint64_t)c->cfg.anchor_mask + 1);
+    if (v < kMinLongBytes) v = kMinLongBytes;
+    if (v > (1u << 20)) v = 1u << 20;
+    return (uint32_t)v;
+}
+
+TableView table_view(const dedup_ctx* c) {
+    const TableBuf& t = c->tables[c->cur_table];
     return TableView{t.slots, t.capacity - 1, t.status};
 }
 
-// Enqueue rows A2-A3 on stream s (optionally recording `mid` after the scan).
-dedup_status enqueue_chunk(dedup_ctx* c, Workspace& w, cudaStream_t s, const uint8_t* d_bytes,
-                           uint64_t nbytes, const uint64_t* d_item_off, uint32_t n_items,
-                           uint32_t* d_cut_pos, uint64_t cap, uint32_t* d_n,
-                           cudaEvent_t mid = nullptr) {
-    if (++w.epoch == 0) ++w.epoch;
-    launch_rabin_scan(d_bytes, nbytes, c->d_tab, c->cfg.anchor_mask, c->cfg.anchor_value,
-                      w.bitmap, c->num_sms, s);
-    if (mid) CU(cudaEventRecord(mid, s));
-    launch_select(w.bitmap, nbytes, d_item_off, n_items, w.desc, w.counters, w.epoch, d_cut_pos,
-                  cap, d_n, c->num_sms, s);
-    c->launches += nbytes ? 2 : 0;
-    CU(cudaGetLastError());
-    return DEDUP_OK;
+// Kernel sequence of rows A2-A4 for one batch described by *d (device).
+void enqueue_chunk_sha(dedup_ctx* c, Workspace& w, cudaStream_t s, const BatchDesc* d,
+                       uint64_t max_bytes, uint32_t* cut_pos, uint64_t cap, uint32_t* n_chunks,
+                       uint8_t* digest, cudaEvent_t ev_scan, cudaEvent_t ev_chunk,
+                       uint32_t* chunk_start, uint64_t* chunk_id, uint32_t* item_first,
+                       uint32_t max_items) {
+    launch_rabin_scan(d, c->d_tab, c->cfg.anchor_mask, c->cfg.anchor_value, w.bitmap,
+                      c->num_sms, s);
+    if (ev_scan) cudaEventRecordWithFlags(ev_scan, s, cudaEventRecordExternal);
+    launch_select(d, w.bitmap, w.agg, w.tile_entry, (max_bytes + kSelTile - 1) / kSelTile,
+                  cut_pos, cap, n_chunks, c->num_sms, s);
+    if (chunk_start)
+        launch_chunk_meta(d, cut_pos, n_chunks, cap, chunk_start, chunk_id, item_first,
+                          max_items, c->num_sms, s);
+    if (ev_chunk) cudaEventRecordWithFlags(ev_chunk, s, cudaEventRecordExternal);
+    if (digest)
+        launch_sha1(d, max_bytes, cut_pos, n_chunks, cap, long_bytes(c), w.counters,
+                    w.long_list, digest, c->num_sms, s);
 }
 
-dedup_status enqueue_table(dedup_ctx* c, Workspace& w, cudaStream_t s, const uint8_t* d_digest,
-                           const uint64_t* d_id, const uint32_t* d_n, uint64_t cap,
-                           uint64_t* d_first_id, uint8_t* d_is_dup) {
-    TableView tv = table_view(c);
-    launch_table_insert(tv, d_digest, d_id, nullptr, d_n, 0, cap, w.slot_idx, c->num_sms, s);
-    launch_table_lookup(tv, d_id, nullptr, d_n, 0, cap, w.slot_idx, d_first_id, d_is_dup,
-                        c->num_sms, s);
-    c->launches += cap ? 2 : 0;
-    CU(cudaGetLastError());
+// Records the per-batch graph of slot i (capture of the slot's stream).
+dedup_status build_graph(dedup_ctx* c, int i) {
+    Slot& sl = c->slots[i];
+    Slot& prev = c->slots[(i + c->slots.size() - 1) % c->slots.size()];
+    const uint64_t cap = c->chunk_cap;
+    cudaStream_t s = sl.stream;
+    CU(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
+    cudaEventRecordWithFlags(sl.ev_start, s, cudaEventRecordExternal);
+    cudaMemcpyAsync(sl.d_desc, sl.h_desc, sizeof(BatchDesc), cudaMemcpyHostToDevice, s);
+    cudaMemcpyAsync(sl.d_item_off, sl.h_item_off, sizeof(uint64_t) * (c->cfg.batch_items + 1),
+                    cudaMemcpyHostToDevice, s);
+    cudaEventRecordWithFlags(sl.ev_h2d, s, cudaEventRecordExternal);
+    enqueue_chunk_sha(c, sl.ws, s, sl.d_desc, c->cfg.batch_bytes, sl.d_cut_pos, cap,
+                      sl.d_small, sl.d_digest, sl.ev_scan, sl.ev_chunk, sl.d_chunk_start,
+                      sl.d_chunk_id, sl.d_item_first, c->cfg.batch_items);
+    cudaEventRecordWithFlags(sl.ev_sha, s, cudaEventRecordExternal);
+    // table work waits for the previous batch's table work (global chain)
+    cudaStreamWaitEvent(s, prev.ev_table, cudaEventWaitExternal);
+    launch_table_prepare(sl.d_desc, c->tables[0].capacity, c->num_sms, s);
+    const TableView* tv = &sl.d_desc->table;
+    launch_table_insert(tv, sl.d_digest, sl.d_chunk_id, nullptr, sl.d_small, 0, cap,
+                        sl.ws.slot_idx, c->num_sms, s);
+    launch_table_lookup(tv, sl.d_chunk_id, nullptr, sl.d_small, 0, cap, sl.ws.slot_idx,
+                        sl.d_first_id, sl.d_is_dup, sl.d_small + 4, c->num_sms, s);
+    cudaEventRecordWithFlags(sl.ev_table, s, cudaEventRecordExternal);
+    launch_pack(sl.d_desc, sl.d_small, cap, c->cfg.batch_items, sl.d_chunk_start, sl.d_first_id,
+                sl.d_digest, sl.d_is_dup, sl.d_item_first, sl.d_small + 4, sl.hdev, c->num_sms,
+                s);
+    cudaEventRecordWithFlags(sl.ev_done, s, cudaEventRecordExternal);
+    cudaGraph_t g = nullptr;
+    cudaError_t e = cudaStreamEndCapture(s, &g);
+    if (e != cudaSuccess)
+        return fail(c, DEDUP_ECUDA, std::string("graph capture: ") + cudaGetErrorString(e));
+    size_t n_nodes = 0;
+    cudaGraphGetNodes(g, nullptr, &n_nodes);
+    std::vector<cudaGraphNode_t> nodes(n_nodes);
+    cudaGraphGetNodes(g, nodes.data(), &n_nodes);
+    uint32_t kern = 0;
+    for (auto& nd : nodes) {
+        cudaGraphNodeType ty;
+        cudaGraphNodeGetType(nd, &ty);
+        kern += ty == cudaGraphNodeTypeKernel ? 1 : 0;
+    }
+    c->graph_kernels = kern;
+    e = cudaGraphInstantiate(&sl.graph, g, 0);
+    cudaGraphDestroy(g);
+    if (e != cudaSuccess)
+        return fail(c, DEDUP_ECUDA, std::string("graph instantiate: ") + cudaGetErrorString(e));
     return DEDUP_OK;
 }
 
@@ -205,30 +284,31 @@ dedup_status slot_alloc(dedup_ctx* c, Slot& sl) {
     const dedup_config& g = c->cfg;
     const uint64_t cap = c->chunk_cap;
     CU(cudaStreamCreateWithFlags(&sl.stream, cudaStreamNonBlocking));
-    for (cudaEvent_t* e : {&sl.ev_start, &sl.ev_h2d, &sl.ev_scan, &sl.ev_chunk, &sl.ev_sha,
-                           &sl.ev_table, &sl.ev_done})
+    for (cudaEvent_t* e : {&sl.ev_host, &sl.ev_start, &sl.ev_h2d, &sl.ev_scan, &sl.ev_chunk,
+                           &sl.ev_sha, &sl.ev_table, &sl.ev_done})
         CU(cudaEventCreate(e));
     CU(cudaEventCreateWithFlags(&sl.ev_prod, cudaEventDisableTiming));
+    TRY(dalloc(c, &sl.d_desc, 1));
+    TRY(halloc(c, &sl.h_desc, 1));
+    std::memset(sl.h_desc, 0, sizeof(BatchDesc));
     if (g.host_fed) TRY(dalloc(c, &sl.d_bytes, g.batch_bytes + 256));
     TRY(dalloc(c, &sl.d_item_off, (uint64_t)g.batch_items + 1));
+    TRY(halloc(c, &sl.h_item_off, (uint64_t)g.batch_items + 1));
     TRY(ws_alloc(c, sl.ws, g.batch_bytes, cap));
     TRY(dalloc(c, &sl.d_cut_pos, cap));
     TRY(dalloc(c, &sl.d_chunk_start, cap));
     TRY(dalloc(c, &sl.d_item_first, g.batch_items));
-    TRY(dalloc(c, &sl.d_n_chunks, 4));
+    TRY(dalloc(c, &sl.d_small, 16));
     TRY(dalloc(c, &sl.d_chunk_id, cap));
     TRY(dalloc(c, &sl.d_first_id, cap));
     TRY(dalloc(c, &sl.d_digest, cap * 20));
     TRY(dalloc(c, &sl.d_is_dup, cap));
-    CU(cudaHostAlloc(reinterpret_cast<void**>(&sl.h_item_off),
-                     sizeof(uint64_t) * ((uint64_t)g.batch_items + 1), cudaHostAllocPortable));
     // results: header 64 B | chunk_start 4*cap | first_id 8*cap | digest 20*cap | is_dup cap
     //          | item_first 4*items
     const uint64_t o_cs = 64, o_fid = o_cs + ((4 * cap + 63) & ~63ull),
                    o_dg = o_fid + 8 * cap, o_dup = o_dg + 20 * cap,
                    o_if = (o_dup + cap + 63) & ~63ull, total = o_if + 4ull * g.batch_items + 64;
-    CU(cudaHostAlloc(reinterpret_cast<void**>(&sl.h_res), total,
-                     cudaHostAllocMapped | cudaHostAllocPortable));
+    TRY(halloc(c, &sl.h_res, total, cudaHostAllocMapped | cudaHostAllocPortable));
     uint8_t* dres = nullptr;
     CU(cudaHostGetDevicePointer(reinterpret_cast<void**>(&dres), sl.h_res, 0));
     auto lay = [&](uint8_t* b) {
@@ -248,83 +328,47 @@ dedup_status slot_alloc(dedup_ctx* c, Slot& sl) {
 
 void slot_free(Slot& sl) {
     if (sl.stream) cudaStreamSynchronize(sl.stream);
-    for (cudaEvent_t e : {sl.ev_start, sl.ev_h2d, sl.ev_scan, sl.ev_chunk, sl.ev_sha, sl.ev_table,
-                          sl.ev_done, sl.ev_prod})
+    if (sl.graph) cudaGraphExecDestroy(sl.graph);
+    for (cudaEvent_t e : {sl.ev_host, sl.ev_start, sl.ev_h2d, sl.ev_scan, sl.ev_chunk, sl.ev_sha,
+                          sl.ev_table, sl.ev_done, sl.ev_prod})
         if (e) cudaEventDestroy(e);
+    cudaFree(sl.d_desc);
+    if (sl.h_desc) cudaFreeHost(sl.h_desc);
     cudaFree(sl.d_bytes);
     cudaFree(sl.d_item_off);
+    if (sl.h_item_off) cudaFreeHost(sl.h_item_off);
     ws_free(sl.ws);
     cudaFree(sl.d_cut_pos);
     cudaFree(sl.d_chunk_start);
     cudaFree(sl.d_item_first);
-    cudaFree(sl.d_n_chunks);
+    cudaFree(sl.d_small);
     cudaFree(sl.d_chunk_id);
     cudaFree(sl.d_first_id);
     cudaFree(sl.d_digest);
     cudaFree(sl.d_is_dup);
-    if (sl.h_item_off) cudaFreeHost(sl.h_item_off);
     if (sl.h_res) cudaFreeHost(sl.h_res);
     if (sl.stream) cudaStreamDestroy(sl.stream);
     sl = Slot{};
 }
 
-int free_slot_count(const dedup_ctx* c) {
-    int n = 0;
-    for (const Slot& s : c->slots) n += s.busy ? 0 : 1;
-    return n;
-}
-
-int take_free_slot(dedup_ctx* c) {
-    for (size_t i = 0; i < c->slots.size(); ++i)
-        if (!c->slots[i].busy) return (int)i;
-    return -1;
-}
-
-// Enqueue one batch on slot i.  Input is either the slot's own device copy
-// (host-fed, already enqueued) or an external device pointer.
+// Prepare slot i's descriptor for a batch and launch its graph.
 dedup_status launch_batch(dedup_ctx* c, int i, const uint8_t* d_bytes) {
     Slot& sl = c->slots[i];
-    cudaStream_t s = sl.stream;
-    const uint64_t cap = c->chunk_cap;
-    // item offsets -> device (from pinned staging)
-    CU(cudaMemcpyAsync(sl.d_item_off, sl.h_item_off, sizeof(uint64_t) * (sl.n_items + 1),
-                       cudaMemcpyHostToDevice, s));
-    CU(cudaEventRecord(sl.ev_h2d, s));
-    TRY(enqueue_chunk(c, sl.ws, s, d_bytes, sl.nbytes, sl.d_item_off, sl.n_items, sl.d_cut_pos,
-                      cap, sl.d_n_chunks, sl.ev_scan));
-    launch_chunk_meta(sl.d_item_off, sl.n_items, sl.d_cut_pos, sl.d_n_chunks, cap, sl.first_seq,
-                      sl.d_chunk_start, sl.d_chunk_id, sl.d_item_first, c->num_sms, s);
-    c->launches += (cap && sl.n_items) ? 1 : 0;
-    CU(cudaEventRecord(sl.ev_chunk, s));
-    launch_sha1(d_bytes, sl.nbytes, sl.d_cut_pos, sl.d_n_chunks, cap, sl.ws.counters + 1,
-                sl.d_digest, c->num_sms, s);
-    c->launches += 1;
-    CU(cudaEventRecord(sl.ev_sha, s));
-    // table: chain after the previous batch of this dedup stream
-    TableBuf& tb = c->tables[c->cur_table];
-    if (c->stream_fresh) {
-        if (tb.used) CU(cudaStreamWaitEvent(s, tb.last_use, 0));
-        CU(cudaMemsetAsync(tb.slots, 0, sizeof(TableSlot) * tb.capacity, s));
-        CU(cudaMemsetAsync(tb.status, 0, sizeof(uint32_t) * 4, s));
-        c->stream_fresh = false;
-        tb.used = true;
-    } else if (c->chain_valid) {
-        CU(cudaStreamWaitEvent(s, c->chain_ev, 0));
-    }
-    TRY(enqueue_table(c, sl.ws, s, sl.d_digest, sl.d_chunk_id, sl.d_n_chunks, cap,
-                      sl.d_first_id, sl.d_is_dup));
-    CU(cudaEventRecord(sl.ev_table, s));
-    CU(cudaEventRecord(tb.last_use, s));
-    c->chain_ev = sl.ev_table;
-    c->chain_valid = true;
-    launch_pack(sl.d_n_chunks, cap, sl.n_items, sl.d_chunk_start, sl.d_first_id, sl.d_digest,
-                sl.d_is_dup, sl.d_item_first, tb.status, sl.hdev, c->num_sms, s);
-    c->launches += 1;
-    CU(cudaGetLastError());
-    CU(cudaEventRecord(sl.ev_done, s));
+    BatchDesc& d = *sl.h_desc;
+    d.bytes = d_bytes;
+    d.nbytes = sl.nbytes;
+    d.first_seq = sl.first_seq;
+    d.item_off = sl.d_item_off;
+    d.n_items = sl.n_items;
+    d.fresh = c->stream_fresh ? 1u : 0u;
+    d.table = table_view(c);
+    c->stream_fresh = false;
+    CU(cudaGraphLaunch(sl.graph, sl.stream));
+    c->launches += c->graph_kernels;
     sl.busy = true;
     sl.parsed = false;
     sl.next_item = 0;
+    c->next_slot = (uint32_t)((i + 1) % c->slots.size());
     c->inflight.push_back(i);
     c->pending_items += sl.n_items;
     c->st.batches += 1;
@@ -335,7 +379,7 @@ dedup_status check_cfg(const dedup_config* g) {
     if (g == nullptr || g->struct_size != sizeof(dedup_config)) return DEDUP_EINVAL;
     if (g->window == 0 || g->window > 64 || g->min_chunk < g->window) return DEDUP_EINVAL;
     if (g->max_chunk != 0 && g->max_chunk < g->min_chunk) return DEDUP_EINVAL;
-    if (g->slots < 1 || g->slots > 16 || g->batch_items < 1) return DEDUP_EINVAL;
+    if (g->slots < 1 || g->slots > 64 || g->batch_items < 1) return DEDUP_EINVAL;
     if (g->batch_bytes < 1 || g->batch_bytes > (1ull << 30)) return DEDUP_EINVAL;
     if (g->num_owners < 1 || g->num_owners > 64 || g->owner_rank >= g->num_owners)
         return DEDUP_EINVAL;
@@ -354,7 +398,7 @@ dedup_status parse_slot(dedup_ctx* c, Slot& sl) {
     sl.item_n.assign(sl.n_items, 0);
     uint32_t next = n;
     for (int64_t k = (int64_t)sl.n_items - 1; k >= 0; --k) {
-        uint32_t f = sl.hhost.item_first_chunk[k];
+        const uint32_t f = sl.hhost.item_first_chunk[k];
         if (f == 0xFFFFFFFFu) {
             sl.item_first[k] = next;
             sl.item_n[k] = 0;
@@ -364,7 +408,6 @@ dedup_status parse_slot(dedup_ctx* c, Slot& sl) {
             next = f;
         }
     }
-    // stats
     uint64_t dups = 0, dup_bytes = 0, blocks = 0;
     for (uint32_t k = 0; k < sl.n_items; ++k) {
         const uint32_t f = sl.item_first[k], m = sl.item_n[k];
@@ -385,15 +428,31 @@ dedup_status parse_slot(dedup_ctx* c, Slot& sl) {
     c->st.dup_bytes += dup_bytes;
     c->st.items += sl.n_items;
     c->st.bytes += sl.nbytes;
+    c->st.table_used = sl.hhost.header[2];
     float ms = 0;
-    if (sl.host_fed && cudaEventElapsedTime(&ms, sl.ev_start, sl.ev_h2d) == cudaSuccess)
+    if (sl.host_fed && cudaEventElapsedTime(&ms, sl.ev_host, sl.ev_start) == cudaSuccess)
         c->st.ms_h2d += ms;
     if (cudaEventElapsedTime(&ms, sl.ev_h2d, sl.ev_scan) == cudaSuccess) c->st.ms_scan += ms;
     if (cudaEventElapsedTime(&ms, sl.ev_scan, sl.ev_chunk) == cudaSuccess) c->st.ms_select += ms;
     if (cudaEventElapsedTime(&ms, sl.ev_chunk, sl.ev_sha) == cudaSuccess) c->st.ms_sha1 += ms;
     if (cudaEventElapsedTime(&ms, sl.ev_sha, sl.ev_table) == cudaSuccess) c->st.ms_table += ms;
     if (cudaEventElapsedTime(&ms, sl.ev_table, sl.ev_done) == cudaSuccess) c->st.ms_d2h += ms;
+    cudaGetLastError();  // clear a possible error from a timing query
     sl.parsed = true;
+    return DEDUP_OK;
+}
+
+// Descriptor for one dedup_op_* call: next entry of the pinned/device ring.
+dedup_status op_desc(dedup_ctx* c, cudaStream_t s, const BatchDesc& h, const BatchDesc** out) {
+    const int k = c->op_next;
+    c->op_next = (k + 1) % kOpRing;
+    if (c->op_ev_used[k]) CU(cudaEventSynchronize(c->op_ev[k]));
+    c->op_h_desc[k] = h;
+    CU(cudaMemcpyAsync(c->op_d_desc + k, c->op_h_desc + k, sizeof(BatchDesc),
+                       cudaMemcpyHostToDevice, s));
+    CU(cudaEventRecord(c->op_ev[k], s));
+    c->op_ev_used[k] = true;
+    *out = c->op_d_desc + k;
     return DEDUP_OK;
 }
 
@@ -449,16 +508,20 @@ dedup_status dedup_init(const dedup_config* cfg, dedup_ctx** out) {
         if ((s = dalloc(c, &t.slots, t.capacity)) != DEDUP_OK) return bail(s);
         if ((s = dalloc(c, &t.status, 4)) != DEDUP_OK) return bail(s);
         if (cudaMemset(t.slots, 0, sizeof(TableSlot) * t.capacity) != cudaSuccess ||
-            cudaMemset(t.status, 0, 16) != cudaSuccess ||
-            cudaEventCreateWithFlags(&t.last_use, cudaEventDisableTiming) != cudaSuccess)
+            cudaMemset(t.status, 0, 16) != cudaSuccess)
             return bail(DEDUP_ECUDA);
     }
-    c->tables[0].used = true;  // stream 0 starts on table 0 (cleared above)
-    c->stream_fresh = false;
     if ((s = ws_alloc(c, c->op_ws, cfg->batch_bytes, c->chunk_cap)) != DEDUP_OK) return bail(s);
+    if ((s = dalloc(c, &c->op_d_desc, kOpRing)) != DEDUP_OK) return bail(s);
+    if ((s = halloc(c, &c->op_h_desc, kOpRing)) != DEDUP_OK) return bail(s);
+    for (cudaEvent_t& e : c->op_ev)
+        if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
+            return bail(DEDUP_ECUDA);
     c->slots.resize(cfg->slots);
     for (Slot& sl : c->slots)
         if ((s = slot_alloc(c, sl)) != DEDUP_OK) return bail(s);
+    for (size_t i = 0; i < c->slots.size(); ++i)
+        if ((s = build_graph(c, (int)i)) != DEDUP_OK) return bail(s);
     if (cudaDeviceSynchronize() != cudaSuccess) return bail(DEDUP_ECUDA);
     c->st.table_slots = c->tables[0].capacity;
     c->st.num_owners = cfg->num_owners;
@@ -472,10 +535,14 @@ void dedup_destroy(dedup_ctx* c) {
     cudaSetDevice(c->cfg.device);
     for (Slot& sl : c->slots) slot_free(sl);
     ws_free(c->op_ws);
+    cudaDeviceSynchronize();
+    for (cudaEvent_t e : c->op_ev)
+        if (e) cudaEventDestroy(e);
+    cudaFree(c->op_d_desc);
+    if (c->op_h_desc) cudaFreeHost(c->op_h_desc);
     for (TableBuf& t : c->tables) {
         cudaFree(t.slots);
         cudaFree(t.status);
-        if (t.last_use) cudaEventDestroy(t.last_use);
     }
     cudaFree(c->d_tab);
     delete c;
@@ -495,8 +562,8 @@ dedup_status dedup_submit_batch(dedup_ctx* c, uint32_t n_items, const uint8_t* c
     if (n_items > 0 && (item_ptr == nullptr || item_len == nullptr))
         return fail(c, DEDUP_EINVAL, "null item arrays");
     CU(cudaSetDevice(c->cfg.device));
-    // plan batches
-    std::vector<std::pair<uint32_t, uint32_t>> plan;  // [first, last) item ranges
+    // plan batches of whole items
+    std::vector<std::pair<uint32_t, uint32_t>> plan;
     uint32_t b0 = 0;
     uint64_t bytes = 0;
     for (uint32_t k = 0; k < n_items; ++k) {
@@ -512,11 +579,12 @@ dedup_status dedup_submit_batch(dedup_ctx* c, uint32_t n_items, const uint8_t* c
         bytes += L;
     }
     if (n_items > b0) plan.emplace_back(b0, n_items);
-    if ((int)plan.size() > free_slot_count(c))
-        return fail(c, DEDUP_EAGAIN, "no free batch slot");
+    for (size_t j = 0; j < plan.size(); ++j)  // round-robin slots must all be free
+        if (j >= c->slots.size() || c->slots[(c->next_slot + j) % c->slots.size()].busy)
+            return fail(c, DEDUP_EAGAIN, "no free batch slot");
     if (first_seq_out) *first_seq_out = c->next_seq;
     for (auto& r : plan) {
-        const int i = take_free_slot(c);
+        const int i = (int)c->next_slot;
         Slot& sl = c->slots[i];
         sl.host_fed = true;
         sl.first_seq = c->next_seq;
@@ -526,16 +594,17 @@ dedup_status dedup_submit_batch(dedup_ctx* c, uint32_t n_items, const uint8_t* c
         sl.h_item_off[0] = 0;
         for (uint32_t k = 0; k < sl.n_items; ++k) sl.h_item_off[k + 1] = (off += sl.item_len[k]);
         sl.nbytes = off;
-        CU(cudaEventRecord(sl.ev_start, sl.stream));
+        CU(cudaEventRecord(sl.ev_host, sl.stream));
         // H2D of the items (row A1), merging contiguous host ranges
         uint32_t k = 0;
         while (k < sl.n_items) {
             const uint8_t* p = item_ptr[r.first + k];
-            uint64_t dst = sl.h_item_off[k], len = sl.item_len[k];
+            const uint64_t dst = sl.h_item_off[k];
+            uint64_t len = sl.item_len[k];
             uint32_t j = k + 1;
             while (j < sl.n_items && item_ptr[r.first + j] == p + len) len += sl.item_len[j++];
-            if (len) CU(cudaMemcpyAsync(sl.d_bytes + dst, p, len, cudaMemcpyHostToDevice,
-                                        sl.stream));
+            if (len)
+                CU(cudaMemcpyAsync(sl.d_bytes + dst, p, len, cudaMemcpyHostToDevice, sl.stream));
             k = j;
         }
         TRY(launch_batch(c, i, sl.d_bytes));
@@ -561,8 +630,8 @@ dedup_status dedup_submit_device(dedup_ctx* c, const uint8_t* d_bytes, uint64_t 
         return fail(c, DEDUP_EINVAL, "item_off must start at 0 and end at nbytes");
     for (uint32_t k = 0; k < n_items; ++k)
         if (item_off[k + 1] < item_off[k]) return fail(c, DEDUP_EINVAL, "item_off decreasing");
-    const int i = take_free_slot(c);
-    if (i < 0) return fail(c, DEDUP_EAGAIN, "no free batch slot");
+    const int i = (int)c->next_slot;
+    if (c->slots[i].busy) return fail(c, DEDUP_EAGAIN, "no free batch slot");
     CU(cudaSetDevice(c->cfg.device));
     Slot& sl = c->slots[i];
     sl.host_fed = false;
@@ -574,7 +643,6 @@ dedup_status dedup_submit_device(dedup_ctx* c, const uint8_t* d_bytes, uint64_t 
     std::memcpy(sl.h_item_off, item_off, sizeof(uint64_t) * (n_items + 1));
     CU(cudaEventRecord(sl.ev_prod, static_cast<cudaStream_t>(producer)));
     CU(cudaStreamWaitEvent(sl.stream, sl.ev_prod, 0));
-    CU(cudaEventRecord(sl.ev_start, sl.stream));
     if (first_seq_out) *first_seq_out = c->next_seq;
     TRY(launch_batch(c, i, d_bytes));
     c->next_seq += n_items;
@@ -595,7 +663,6 @@ dedup_status dedup_end_stream(dedup_ctx* c) {
     if (!usable(c)) return c->sticky;
     c->cur_table ^= 1;
     c->stream_fresh = true;
-    c->chain_valid = false;
     return DEDUP_OK;
 }
 
@@ -696,8 +763,19 @@ dedup_status dedup_op_chunk(dedup_ctx* c, void* stream, const uint8_t* d_bytes, 
     if (reinterpret_cast<uintptr_t>(d_bytes) & 15)
         return fail(c, DEDUP_EINVAL, "d_bytes must be 16-byte aligned");
     CU(cudaSetDevice(c->cfg.device));
-    return enqueue_chunk(c, c->op_ws, static_cast<cudaStream_t>(stream), d_bytes, nbytes,
-                         d_item_off, n_items, d_cut_pos, cap, d_n_chunks);
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    BatchDesc h{};
+    h.bytes = d_bytes;
+    h.nbytes = nbytes;
+    h.item_off = d_item_off;
+    h.n_items = n_items;
+    const BatchDesc* d = nullptr;
+    TRY(op_desc(c, s, h, &d));
+    enqueue_chunk_sha(c, c->op_ws, s, d, nbytes, d_cut_pos, cap, d_n_chunks, nullptr, nullptr,
+                      nullptr, nullptr, nullptr, nullptr, 0);
+    c->launches += 4;
+    CU(cudaGetLastError());
+    return DEDUP_OK;
 }
 
 dedup_status dedup_op_chunk_meta(dedup_ctx* c, void* stream, const uint64_t* d_item_off,
@@ -708,10 +786,16 @@ dedup_status dedup_op_chunk_meta(dedup_ctx* c, void* stream, const uint64_t* d_i
     if (c == nullptr) return DEDUP_EINVAL;
     if (!usable(c)) return c->sticky;
     CU(cudaSetDevice(c->cfg.device));
-    launch_chunk_meta(d_item_off, n_items, d_cut_pos, d_n_chunks, cap, first_seq, d_chunk_start,
-                      d_chunk_id, d_item_first_chunk, c->num_sms,
-                      static_cast<cudaStream_t>(stream));
-    c->launches += (cap && n_items) ? 1 : 0;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    BatchDesc h{};
+    h.item_off = d_item_off;
+    h.n_items = n_items;
+    h.first_seq = first_seq;
+    const BatchDesc* d = nullptr;
+    TRY(op_desc(c, s, h, &d));
+    launch_chunk_meta(d, d_cut_pos, d_n_chunks, cap, d_chunk_start, d_chunk_id,
+                      d_item_first_chunk, n_items, c->num_sms, s);
+    c->launches += 1;
     CU(cudaGetLastError());
     return DEDUP_OK;
 }
@@ -725,10 +809,17 @@ dedup_status dedup_op_sha1(dedup_ctx* c, void* stream, const uint8_t* d_bytes, u
         return fail(c, DEDUP_EINVAL, "d_bytes must be 16-byte aligned");
     if (reinterpret_cast<uintptr_t>(d_digest) & 3)
         return fail(c, DEDUP_EINVAL, "d_digest must be 4-byte aligned");
+    if (nbytes > c->cfg.batch_bytes) return fail(c, DEDUP_EINVAL, "nbytes > batch_bytes");
     CU(cudaSetDevice(c->cfg.device));
-    launch_sha1(d_bytes, nbytes, d_cut_pos, d_n_chunks, cap, c->op_ws.counters + 1, d_digest,
-                c->num_sms, static_cast<cudaStream_t>(stream));
-    c->launches += 1;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    BatchDesc h{};
+    h.bytes = d_bytes;
+    h.nbytes = nbytes;
+    const BatchDesc* d = nullptr;
+    TRY(op_desc(c, s, h, &d));
+    launch_sha1(d, nbytes, d_cut_pos, d_n_chunks, cap, long_bytes(c), c->op_ws.counters,
+                c->op_ws.long_list, d_digest, c->num_sms, s);
+    c->launches += 2;
     CU(cudaGetLastError());
     return DEDUP_OK;
 }
@@ -740,8 +831,18 @@ dedup_status dedup_op_table_insert_lookup(dedup_ctx* c, void* stream, const uint
     if (!usable(c)) return c->sticky;
     if (cap > c->chunk_cap) return fail(c, DEDUP_EINVAL, "cap larger than the ctx workspace");
     CU(cudaSetDevice(c->cfg.device));
-    return enqueue_table(c, c->op_ws, static_cast<cudaStream_t>(stream), d_digest, d_id, d_n, cap,
-                         d_first_id, d_is_dup);
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    BatchDesc h{};
+    h.table = table_view(c);
+    const BatchDesc* d = nullptr;
+    TRY(op_desc(c, s, h, &d));
+    launch_table_insert(&d->table, d_digest, d_id, nullptr, d_n, 0, cap, c->op_ws.slot_idx,
+                        c->num_sms, s);
+    launch_table_lookup(&d->table, d_id, nullptr, d_n, 0, cap, c->op_ws.slot_idx, d_first_id,
+                        d_is_dup, nullptr, c->num_sms, s);
+    c->launches += cap ? 2 : 1;
+    CU(cudaGetLastError());
+    return DEDUP_OK;
 }
 
 dedup_status dedup_op_table_reset(dedup_ctx* c, void* stream) {
@@ -792,12 +893,17 @@ dedup_status dedup_op_owner(dedup_ctx* c, void* stream, const dedup_record* d_re
     if (n_recv > c->chunk_cap) return fail(c, DEDUP_EINVAL, "n_recv larger than the workspace");
     CU(cudaSetDevice(c->cfg.device));
     cudaStream_t s = static_cast<cudaStream_t>(stream);
-    TableView tv = table_view(c);
-    launch_table_insert(tv, nullptr, nullptr, d_recv, nullptr, n_recv, n_recv,
-                        c->op_ws.slot_idx, c->num_sms, s);
-    launch_table_lookup(tv, nullptr, d_recv, nullptr, n_recv, n_recv, c->op_ws.slot_idx, d_reply,
-                        nullptr, c->num_sms, s);
-    c->launches += n_recv ? 2 : 0;
+    BatchDesc h{};
+    h.table = table_view(c);
+    const BatchDesc* d = nullptr;
+    TRY(op_desc(c, s, h, &d));
+    if (n_recv) {
+        launch_table_insert(&d->table, nullptr, nullptr, d_recv, nullptr, n_recv, n_recv,
+                            c->op_ws.slot_idx, c->num_sms, s);
+        launch_table_lookup(&d->table, nullptr, d_recv, nullptr, n_recv, n_recv,
+                            c->op_ws.slot_idx, d_reply, nullptr, nullptr, c->num_sms, s);
+        c->launches += 2;
+    }
     CU(cudaGetLastError());
     return DEDUP_OK;
 }

@@ -13,14 +13,16 @@
 //                      and emits one candidate bit per byte.  Both tables are
 //                      replicated per lane in shared memory ([x][lane] layout,
 //                      bank = lane, conflict-free), addressed with one PRMT.
-//  select_kernel       greedy cut selection.  With min chunk = window = 32 the
+//  select_*_kernel     greedy cut selection.  With min chunk = window = 32 the
 //                      only state crossing a position is "positions still
 //                      blocked" in [0, 31]; a warp simulates all 32 entry
-//                      states of an 8192-position tile (lane s = state s),
-//                      publishes the 32-entry transfer function, and resolves
-//                      its real entry state with a decoupled look-back that
-//                      composes predecessor functions with warp shuffles.
-//                      Item starts are forced cuts and reset the state.
+//                      states of an 8192-position tile (lane s = state s) and
+//                      stores the tile's 32-entry transfer function (agg); one
+//                      CTA composes the functions in tile order with warp
+//                      shuffles (prefix over an associative operator) giving
+//                      every tile its real entry state and cut offset; a
+//                      replay pass writes the cut positions.  Item starts are
+//                      forced cuts and reset the state.
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -32,15 +34,6 @@ namespace {
 
 constexpr int kScanThreads = 512;
 constexpr int kTabBytes = 256 * 256;  // [x][R|W][lane] u32 = 64 KiB
-
-__device__ __forceinline__ uint64_t ld_relaxed(const uint64_t* p) {
-    uint64_t v;
-    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-    return v;
-}
-__device__ __forceinline__ void st_relaxed(uint64_t* p, uint64_t v) {
-    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
 
 // Rolls the 32 bytes of cur[0..7] (stream bytes, little-endian words) into h,
 // removing the 32 bytes of old[0..7]; returns the 32 candidate bits.
@@ -84,9 +77,18 @@ __device__ __forceinline__ void load32_guard(const uint8_t* base, uint64_t off, 
 }
 
 __global__ void __launch_bounds__(kScanThreads, 2)
-rabin_scan_kernel(const uint8_t* __restrict__ bytes, uint64_t nbytes, uint32_t seg,
-                  uint64_t n_lanes, const uint32_t* __restrict__ gtab, uint32_t mask,
-                  uint32_t value, uint32_t* __restrict__ bitmap) {
+rabin_scan_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ gtab,
+                  uint32_t mask, uint32_t value, uint32_t* __restrict__ bitmap) {
+    const uint8_t* __restrict__ bytes = desc->bytes;
+    const uint64_t nbytes = desc->nbytes;
+    if (nbytes == 0) return;
+    // Segment per lane: long enough that the 32-byte warm-up is cheap, short
+    // enough that the grid's lanes cover the batch in one pass.
+    const uint64_t threads = (uint64_t)gridDim.x * blockDim.x;
+    uint64_t seg = (nbytes + threads - 1) / threads;
+    seg = ((seg + 31) / 32) * 32;
+    if (seg < 256) seg = 256;
+    const uint64_t n_lanes = (nbytes + seg - 1) / seg;
     extern __shared__ __align__(16) uint8_t tab[];
     {
         uint32_t* t32 = reinterpret_cast<uint32_t*>(tab);
@@ -182,134 +184,171 @@ __device__ __forceinline__ uint32_t walk_tile(const SelWarpSmem& sm, uint32_t s,
     return cnt;
 }
 
+constexpr uint32_t kM27 = (1u << 27) - 1;
+
+// Candidate (e-space: cut after byte i <=> e = i + 1) and forced-cut bits of
+// tile t into the warp's shared memory, with one-bit-per-word summaries.
+__device__ __forceinline__ void build_tile(SelWarpSmem& sm, uint64_t t,
+                                           const uint32_t* __restrict__ bitmap, uint64_t nbytes,
+                                           const uint64_t* __restrict__ item_off,
+                                           uint32_t n_items, int lane) {
+    const uint64_t T0 = t * kSelTile;
+    const uint64_t n_words = (nbytes + 31) / 32;
+    uint32_t cw[8], fw[8];
+    const uint64_t E0 = T0 + (uint64_t)lane * 256;  // this lane's e-range
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+        const uint64_t g = T0 / 32 + lane * 8 + j;
+        const uint32_t curw = g < n_words ? bitmap[g] : 0u;
+        const uint32_t prvw = (g >= 1 && g - 1 < n_words) ? bitmap[g - 1] : 0u;
+        uint32_t ew = __funnelshift_l(prvw, curw, 1);
+        const uint64_t e_lo = E0 + 32 * j;
+        if (e_lo >= nbytes) ew = 0;
+        else if (e_lo + 32 > nbytes) ew &= (1u << (uint32_t)(nbytes - e_lo)) - 1u;
+        cw[j] = ew;
+        fw[j] = 0;
+    }
+    // items: no candidate at e in [q, q+32) (window would leave the item),
+    // forced cut at q for non-empty items
+    if (E0 < nbytes && n_items > 0) {
+        const uint64_t key = E0 >= 31 ? E0 - 31 : 0;  // first start > E0 - 32
+        uint32_t lo = 0, hi = n_items;
+        while (lo < hi) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (item_off[mid] < key) lo = mid + 1; else hi = mid;
+        }
+        for (uint32_t it = lo; it < n_items; ++it) {
+            const uint64_t q = item_off[it];
+            if (q >= E0 + 256) break;
+            const bool nonempty = item_off[it + 1] > q;
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+                const int64_t a = (int64_t)q - (int64_t)(E0 + 32 * j);
+                if (a < 32 && a > -32) {
+                    const uint32_t lo_r = a > 0 ? (uint32_t)a : 0u;
+                    const uint32_t hi_r = a < 0 ? (uint32_t)(a + 32) : 32u;
+                    const uint32_t hm = hi_r >= 32 ? 0xFFFFFFFFu : ((1u << hi_r) - 1u);
+                    cw[j] &= ~(hm & ~((1u << lo_r) - 1u));
+                    if (nonempty && a >= 0) fw[j] |= 1u << (uint32_t)a;
+                }
+            }
+        }
+    }
+    uint32_t cm = 0, fm = 0;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+        sm.cand[lane * 8 + j] = cw[j];
+        sm.forced[lane * 8 + j] = fw[j];
+        cm |= (cw[j] ? 1u : 0u) << j;
+        fm |= (fw[j] ? 1u : 0u) << j;
+    }
+    reinterpret_cast<uint8_t*>(sm.csum)[lane] = (uint8_t)cm;
+    reinterpret_cast<uint8_t*>(sm.fsum)[lane] = (uint8_t)fm;
+    __syncwarp();
+}
+
+// Phase 1: the 32-entry transfer function of every tile:
+// agg[32 t + s] = exit_state(s) << 27 | cuts(s).
 __global__ void __launch_bounds__(kSelWarps * 32)
-select_kernel(const uint32_t* __restrict__ bitmap, uint64_t nbytes,
-              const uint64_t* __restrict__ item_off, uint32_t n_items, uint64_t* desc,
-              uint32_t* tile_counter, uint32_t epoch, uint32_t* __restrict__ cut_pos,
-              uint64_t cap, uint32_t* n_chunks) {
+select_agg_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ bitmap,
+                  uint32_t* __restrict__ agg) {
     __shared__ SelWarpSmem smem[kSelWarps];
     const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    SelWarpSmem& sm = smem[wid];
+    const uint64_t nbytes = desc->nbytes;
     const uint64_t n_tiles = (nbytes + kSelTile - 1) / kSelTile;
-    const uint64_t n_words = (nbytes + 31) / 32;
-    const uint64_t M27 = (1u << 27) - 1;
-    while (true) {
-        uint32_t t = 0;
-        if (lane == 0) t = atomicAdd(tile_counter, 1u);
-        t = __shfl_sync(0xFFFFFFFFu, t, 0);
-        if (t >= n_tiles) break;
-        const uint64_t T0 = (uint64_t)t * kSelTile;
-        // -- candidate bits in e-space (cut after byte i <=> e = i + 1) --
-        uint32_t cw[8], fw[8];
-        const uint64_t E0 = T0 + (uint64_t)lane * 256;  // this lane's e-range
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-            uint64_t g = T0 / 32 + lane * 8 + j;
-            uint32_t curw = g < n_words ? bitmap[g] : 0u;
-            uint32_t prvw = (g >= 1 && g - 1 < n_words) ? bitmap[g - 1] : 0u;
-            uint32_t ew = __funnelshift_l(prvw, curw, 1);
-            uint64_t e_lo = E0 + 32 * j;
-            if (e_lo >= nbytes) ew = 0;
-            else if (e_lo + 32 > nbytes) ew &= (1u << (uint32_t)(nbytes - e_lo)) - 1u;
-            cw[j] = ew;
-            fw[j] = 0;
-        }
-        // -- items: mask candidates at e in [q, q+32), forced cut at q --
-        if (E0 < nbytes && n_items > 0) {
-            // first item index with start > E0 - 32
-            uint64_t key = E0 >= 31 ? E0 - 31 : 0;
-            uint32_t lo = 0, hi = n_items;  // search in item_off[0..n_items)
-            while (lo < hi) {
-                uint32_t mid = (lo + hi) >> 1;
-                if (item_off[mid] < key) lo = mid + 1; else hi = mid;
-            }
-            for (uint32_t it = lo; it < n_items; ++it) {
-                const uint64_t q = item_off[it];
-                if (q >= E0 + 256) break;
-                const bool nonempty = item_off[it + 1] > q;
-#pragma unroll
-                for (int j = 0; j < 8; ++j) {
-                    // e in [q, q+32) intersected with this word's [wlo, wlo+32)
-                    const int64_t a = (int64_t)q - (int64_t)(E0 + 32 * j);
-                    if (a < 32 && a > -32) {
-                        const uint32_t lo_r = a > 0 ? (uint32_t)a : 0u;
-                        const uint32_t hi_r = a < 0 ? (uint32_t)(a + 32) : 32u;
-                        const uint32_t hm = hi_r >= 32 ? 0xFFFFFFFFu : ((1u << hi_r) - 1u);
-                        cw[j] &= ~(hm & ~((1u << lo_r) - 1u));
-                        if (nonempty && a >= 0) fw[j] |= 1u << (uint32_t)a;
-                    }
-                }
-            }
-        }
-        uint32_t cm = 0, fm = 0;
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-            sm.cand[lane * 8 + j] = cw[j];
-            sm.forced[lane * 8 + j] = fw[j];
-            cm |= (cw[j] ? 1u : 0u) << j;
-            fm |= (fw[j] ? 1u : 0u) << j;
-        }
-        reinterpret_cast<uint8_t*>(sm.csum)[lane] = (uint8_t)cm;
-        reinterpret_cast<uint8_t*>(sm.fsum)[lane] = (uint8_t)fm;
-        __syncwarp();
-        // -- 32-entry transfer function of this tile --
+    for (uint64_t t = (uint64_t)blockIdx.x * kSelWarps + wid; t < n_tiles;
+         t += (uint64_t)gridDim.x * kSelWarps) {
+        build_tile(smem[wid], t, bitmap, nbytes, desc->item_off, desc->n_items, lane);
         uint32_t ex;
-        const uint32_t cnt = walk_tile(sm, lane, ex, nullptr, 0, 0, T0);
-        uint64_t* d = desc + (uint64_t)t * kDescWords;
-        st_relaxed(d + 1 + lane, ((uint64_t)epoch << 32) | ((uint64_t)ex << 27) | cnt);
-        // -- decoupled look-back --
-        uint32_t in_state = 0, in_cnt = 0;
-        if (t > 0) {
-            uint32_t Gs = lane, Gc = 0;
-            int64_t j = (int64_t)t - 1;
-            while (true) {
-                if (j < 0) {  // tile 0 is entered in state 0 with 0 cuts before it
-                    in_state = __shfl_sync(0xFFFFFFFFu, Gs, 0);
-                    in_cnt = __shfl_sync(0xFFFFFFFFu, Gc, 0);
-                    break;
-                }
-                const uint64_t* dj = desc + (uint64_t)j * kDescWords;
-                uint64_t inc = ld_relaxed(dj);
-                if ((uint32_t)(inc >> 32) == epoch) {
-                    uint32_t st = (uint32_t)(inc >> 27) & 31u;
-                    in_state = __shfl_sync(0xFFFFFFFFu, Gs, st);
-                    in_cnt = (uint32_t)(inc & M27) + __shfl_sync(0xFFFFFFFFu, Gc, st);
-                    break;
-                }
-                uint64_t a = ld_relaxed(dj + 1 + lane);
-                if (!__all_sync(0xFFFFFFFFu, (uint32_t)(a >> 32) == epoch)) {
-                    __nanosleep(64);
-                    continue;
-                }
-                uint32_t as = (uint32_t)(a >> 27) & 31u, ac = (uint32_t)(a & M27);
-                uint32_t ns = __shfl_sync(0xFFFFFFFFu, Gs, as);
-                uint32_t nc = ac + __shfl_sync(0xFFFFFFFFu, Gc, as);
-                Gs = ns;
-                Gc = nc;
-                --j;
-            }
+        const uint32_t cnt = walk_tile(smem[wid], lane, ex, nullptr, 0, 0, 0);
+        agg[32 * t + lane] = (ex << 27) | cnt;
+        __syncwarp();
+    }
+}
+
+// Phase 2 (one CTA of 32 warps): prefix composition of the tile functions.
+// tile_entry[2t] = entry state of tile t, tile_entry[2t+1] = cuts before it.
+__global__ void __launch_bounds__(1024)
+select_scan_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ agg,
+                   uint32_t* __restrict__ tile_entry, uint32_t* __restrict__ n_chunks) {
+    __shared__ uint32_t fs[32][32], fc[32][32], es[32], ec[32];
+    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint64_t n_tiles = (desc->nbytes + kSelTile - 1) / kSelTile;
+    const uint64_t per = (n_tiles + 31) / 32;
+    const uint64_t t0 = w * per, t1 = min(t0 + per, n_tiles);
+    uint32_t Gs = lane, Gc = 0;  // composition of tiles [t0, t): entry lane -> (state, cuts)
+#pragma unroll 4
+    for (uint64_t t = t0; t < t1; ++t) {
+        const uint32_t a = agg[32 * t + lane];
+        const uint32_t ns = __shfl_sync(0xFFFFFFFFu, a >> 27, Gs);
+        const uint32_t nc = Gc + __shfl_sync(0xFFFFFFFFu, a & kM27, Gs);
+        Gs = ns;
+        Gc = nc;
+    }
+    fs[w][lane] = Gs;
+    fc[w][lane] = Gc;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        uint32_t s = 0, c = 0;  // the batch starts with a forced cut: entry state 0
+        for (int r = 0; r < 32; ++r) {
+            es[r] = s;
+            ec[r] = c;
+            c += fc[r][s];
+            s = fs[r][s];
         }
-        const uint32_t real_ex = __shfl_sync(0xFFFFFFFFu, ex, in_state);
-        const uint32_t real_cnt = __shfl_sync(0xFFFFFFFFu, cnt, in_state);
-        if (lane == 0)
-            st_relaxed(d, ((uint64_t)epoch << 32) | ((uint64_t)real_ex << 27) |
-                              (uint64_t)(in_cnt + real_cnt));
-        if (lane == (int)in_state) {
-            uint32_t dummy;
-            walk_tile(sm, in_state, dummy, cut_pos, in_cnt, cap, T0);
-            if (t == n_tiles - 1) *n_chunks = in_cnt + real_cnt;
+        *n_chunks = c;
+    }
+    __syncthreads();
+    const uint32_t e_s = es[w], e_c = ec[w];
+    Gs = lane;
+    Gc = 0;
+#pragma unroll 4
+    for (uint64_t t = t0; t < t1; ++t) {
+        const uint32_t a = agg[32 * t + lane];
+        const uint32_t st = __shfl_sync(0xFFFFFFFFu, Gs, e_s);
+        const uint32_t ct = __shfl_sync(0xFFFFFFFFu, Gc, e_s);
+        if (lane == 0) {
+            tile_entry[2 * t] = st;
+            tile_entry[2 * t + 1] = e_c + ct;
+        }
+        const uint32_t ns = __shfl_sync(0xFFFFFFFFu, a >> 27, Gs);
+        const uint32_t nc = Gc + __shfl_sync(0xFFFFFFFFu, a & kM27, Gs);
+        Gs = ns;
+        Gc = nc;
+    }
+}
+
+// Phase 3: replay every tile from its real entry state, writing cut_pos.
+__global__ void __launch_bounds__(kSelWarps * 32)
+select_emit_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ bitmap,
+                   const uint32_t* __restrict__ tile_entry, uint32_t* __restrict__ cut_pos,
+                   uint64_t cap) {
+    __shared__ SelWarpSmem smem[kSelWarps];
+    const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint64_t nbytes = desc->nbytes;
+    const uint64_t n_tiles = (nbytes + kSelTile - 1) / kSelTile;
+    for (uint64_t t = (uint64_t)blockIdx.x * kSelWarps + wid; t < n_tiles;
+         t += (uint64_t)gridDim.x * kSelWarps) {
+        build_tile(smem[wid], t, bitmap, nbytes, desc->item_off, desc->n_items, lane);
+        const uint32_t st = tile_entry[2 * t], base = tile_entry[2 * t + 1];
+        if (lane == (int)st) {
+            uint32_t ex;
+            walk_tile(smem[wid], st, ex, cut_pos, base, cap, t * kSelTile);
         }
         __syncwarp();
     }
 }
 
-__global__ void chunk_meta_kernel(const uint64_t* __restrict__ item_off, uint32_t n_items,
+__global__ void chunk_meta_kernel(const BatchDesc* __restrict__ desc,
                                   const uint32_t* __restrict__ cut_pos,
                                   const uint32_t* __restrict__ n_chunks_p, uint64_t cap,
-                                  uint64_t first_seq, uint32_t* __restrict__ chunk_start,
+                                  uint32_t* __restrict__ chunk_start,
                                   uint64_t* __restrict__ chunk_id,
                                   uint32_t* __restrict__ item_first_chunk) {
     const uint64_t n = min((uint64_t)*n_chunks_p, cap);
+    const uint64_t* __restrict__ item_off = desc->item_off;
+    const uint32_t n_items = desc->n_items;
+    const uint64_t first_seq = desc->first_seq;
     for (uint64_t k = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; k < n;
          k += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t e = cut_pos[k];
@@ -340,60 +379,42 @@ __global__ void chunk_meta_kernel(const uint64_t* __restrict__ item_off, uint32_
 
 }  // namespace
 
-void launch_rabin_scan(const uint8_t* bytes, uint64_t nbytes, const uint32_t* d_tab,
-                       uint32_t mask, uint32_t value, uint32_t* bitmap, int num_sms,
-                       cudaStream_t s) {
-    if (nbytes == 0) return;
+void launch_rabin_scan(const BatchDesc* d, const uint32_t* d_tab, uint32_t mask, uint32_t value,
+                       uint32_t* bitmap, int num_sms, cudaStream_t s) {
     static bool attr_set = false;
     if (!attr_set) {
         cudaFuncSetAttribute(rabin_scan_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              kTabBytes);
         attr_set = true;
     }
-    const uint64_t resident = (uint64_t)num_sms * 2 * kScanThreads;
-    // Segment length per lane: long enough that the 32-byte warm-up is cheap,
-    // short enough that the grid fills every SM (multiple of 32 bytes).
-    uint64_t seg = (nbytes + resident - 1) / resident;
-    seg = ((seg + 31) / 32) * 32;
-    if (seg < 256) seg = 256;
-    if (seg > 4096) seg = 4096;
-    const uint64_t n_lanes = (nbytes + seg - 1) / seg;
-    uint64_t blocks = (n_lanes + kScanThreads - 1) / kScanThreads;
-    const uint64_t max_blocks = (uint64_t)num_sms * 2;
-    if (blocks > max_blocks) blocks = max_blocks;
-    rabin_scan_kernel<<<(unsigned)blocks, kScanThreads, kTabBytes, s>>>(
-        bytes, nbytes, (uint32_t)seg, n_lanes, d_tab, mask, value, bitmap);
+    rabin_scan_kernel<<<(unsigned)(num_sms * 2), kScanThreads, kTabBytes, s>>>(d, d_tab, mask,
+                                                                               value, bitmap);
 }
 
-void launch_select(const uint32_t* bitmap, uint64_t nbytes, const uint64_t* item_off,
-                   uint32_t n_items, uint64_t* desc, uint32_t* tile_counter, uint32_t epoch,
-                   uint32_t* cut_pos, uint64_t cap, uint32_t* n_chunks, int num_sms,
-                   cudaStream_t s) {
-    cudaMemsetAsync(tile_counter, 0, sizeof(uint32_t), s);
-    if (nbytes == 0) {
-        cudaMemsetAsync(n_chunks, 0, sizeof(uint32_t), s);
-        return;
-    }
-    const uint64_t n_tiles = (nbytes + kSelTile - 1) / kSelTile;
-    uint64_t blocks = (n_tiles + kSelWarps - 1) / kSelWarps;
+void launch_select(const BatchDesc* d, const uint32_t* bitmap, uint32_t* agg,
+                   uint32_t* tile_entry, uint64_t max_tiles, uint32_t* cut_pos, uint64_t cap,
+                   uint32_t* n_chunks, int num_sms, cudaStream_t s) {
+    uint64_t blocks = (max_tiles + kSelWarps - 1) / kSelWarps;
     const uint64_t max_blocks = (uint64_t)num_sms * 8;
     if (blocks > max_blocks) blocks = max_blocks;
-    select_kernel<<<(unsigned)blocks, kSelWarps * 32, 0, s>>>(
-        bitmap, nbytes, item_off, n_items, desc, tile_counter, epoch, cut_pos, cap, n_chunks);
+    if (blocks < 1) blocks = 1;
+    select_agg_kernel<<<(unsigned)blocks, kSelWarps * 32, 0, s>>>(d, bitmap, agg);
+    select_scan_kernel<<<1, 1024, 0, s>>>(d, agg, tile_entry, n_chunks);
+    select_emit_kernel<<<(unsigned)blocks, kSelWarps * 32, 0, s>>>(d, bitmap, tile_entry, cut_pos,
+                                                                   cap);
 }
 
-void launch_chunk_meta(const uint64_t* item_off, uint32_t n_items, const uint32_t* cut_pos,
-                       const uint32_t* n_chunks, uint64_t cap, uint64_t first_seq,
-                       uint32_t* chunk_start, uint64_t* chunk_id, uint32_t* item_first_chunk,
-                       int num_sms, cudaStream_t s) {
-    if (n_items) cudaMemsetAsync(item_first_chunk, 0xFF, sizeof(uint32_t) * n_items, s);
-    if (cap == 0 || n_items == 0) return;
+void launch_chunk_meta(const BatchDesc* d, const uint32_t* cut_pos, const uint32_t* n_chunks,
+                       uint64_t cap, uint32_t* chunk_start, uint64_t* chunk_id,
+                       uint32_t* item_first_chunk, uint32_t max_items, int num_sms,
+                       cudaStream_t s) {
+    if (max_items) cudaMemsetAsync(item_first_chunk, 0xFF, sizeof(uint32_t) * max_items, s);
     uint64_t blocks = (cap + 255) / 256;
-    const uint64_t max_blocks = (uint64_t)num_sms * 8;
+    const uint64_t max_blocks = (uint64_t)num_sms * 4;
     if (blocks > max_blocks) blocks = max_blocks;
-    chunk_meta_kernel<<<(unsigned)blocks, 256, 0, s>>>(item_off, n_items, cut_pos, n_chunks, cap,
-                                                       first_seq, chunk_start, chunk_id,
-                                                       item_first_chunk);
+    if (blocks < 1) blocks = 1;
+    chunk_meta_kernel<<<(unsigned)blocks, 256, 0, s>>>(d, cut_pos, n_chunks, cap, chunk_start,
+                                                       chunk_id, item_first_chunk);
 }
 
 }  // namespace dd

@@ -28,7 +28,10 @@ constexpr uint32_t kFull = 0xFFFFFFFFu;
 
 __device__ __forceinline__ uint32_t rotl(uint32_t x, int s) { return __funnelshift_l(x, x, s); }
 
-__device__ __forceinline__ void sha1_compress(uint32_t H[5], uint32_t W[16]) {
+// `one` is a runtime 1 (kernel argument): w * one + K compiles to an IMAD on
+// the FMA pipe that ptxas cannot fold back onto the a -> a' dependency chain,
+// leaving LEA.HI (rotl(a,5) + x) as the only op on it.
+__device__ __forceinline__ void sha1_compress(uint32_t H[5], uint32_t W[16], uint32_t one) {
     uint32_t a = H[0], b = H[1], c = H[2], d = H[3], e = H[4];
 #pragma unroll
     for (int t = 0; t < 80; ++t) {
@@ -53,7 +56,9 @@ __device__ __forceinline__ void sha1_compress(uint32_t H[5], uint32_t W[16]) {
             f = b ^ c ^ d;
             K = 0xCA62C1D6u;
         }
-        const uint32_t T = rotl(a, 5) + f + e + K + w;
+        // keep only rotl(a,5) + x on the a -> a' dependency chain
+        const uint32_t x = (f + e) + (w * one + K);
+        const uint32_t T = rotl(a, 5) + x;
         e = d;
         d = c;
         c = rotl(b, 30);
@@ -67,20 +72,18 @@ __device__ __forceinline__ void sha1_compress(uint32_t H[5], uint32_t W[16]) {
     H[4] += e;
 }
 
-// 64 message bytes starting at byte offset p (any alignment) as 16
-// big-endian words.  Reads the 16-byte-aligned window [p & ~15, +80); with
-// guard, vectors at or beyond lim16 read as zero.
+// Raw 16-byte-aligned window [p & ~15, +80) holding the 64 message bytes at
+// byte offset p.  With kGuard, vectors at or beyond lim16 read as zero.
 template <bool kGuard>
-__device__ __forceinline__ void load_block(const uint8_t* __restrict__ bytes, uint64_t p,
-                                           uint64_t lim16, uint32_t M[16]) {
+__device__ __forceinline__ void load_raw(const uint8_t* __restrict__ bytes, uint64_t p,
+                                         uint64_t lim16, uint32_t v[20]) {
     const uint64_t base = p & ~uint64_t(15);
-    const uint32_t o = (uint32_t)(p & 15);
-    uint32_t v[20];
+    const bool need5 = (p & 15) != 0;
 #pragma unroll
     for (int i = 0; i < 5; ++i) {
         uint4 x = make_uint4(0, 0, 0, 0);
         const uint64_t a = base + 16 * i;
-        bool ok = (i < 4) || (o != 0);
+        bool ok = (i < 4) || need5;
         if (kGuard) ok = ok && (a < lim16);
         if (ok) x = __ldg(reinterpret_cast<const uint4*>(bytes + a));
         v[4 * i] = x.x;
@@ -88,58 +91,90 @@ __device__ __forceinline__ void load_block(const uint8_t* __restrict__ bytes, ui
         v[4 * i + 2] = x.z;
         v[4 * i + 3] = x.w;
     }
+}
+
+// Realign the raw window to byte offset (p & 15) and byte-swap to 16
+// big-endian message words: two select stages for the word offset, one PRMT
+// per word for the byte offset + endianness.
+__device__ __forceinline__ void realign(uint32_t v[20], uint32_t o, uint32_t M[16]) {
     const uint32_t wsh = o >> 2;
-    if (wsh & 2) {
 #pragma unroll
-        for (int i = 0; i < 18; ++i) v[i] = v[i + 2];
-    }
-    if (wsh & 1) {
+    for (int i = 0; i < 18; ++i) v[i] = (wsh & 2) ? v[i + 2] : v[i];
 #pragma unroll
-        for (int i = 0; i < 17; ++i) v[i] = v[i + 1];
-    }
+    for (int i = 0; i < 17; ++i) v[i] = (wsh & 1) ? v[i + 1] : v[i];
     const uint32_t sel = 0x0123u + (o & 3) * 0x1111u;
 #pragma unroll
     for (int j = 0; j < 16; ++j) M[j] = __byte_perm(v[j], v[j + 1], sel);
 }
 
-__global__ void __launch_bounds__(kShaThreads, 8)
-sha1_kernel(const uint8_t* __restrict__ bytes, uint64_t nbytes,
-            const uint32_t* __restrict__ cut_pos, const uint32_t* __restrict__ n_chunks_p,
-            uint64_t cap, uint32_t* work_counter, uint8_t* __restrict__ digest) {
+// Chunks of at least `long_bytes` are listed so that the SHA-1 kernel starts
+// them first (longest-processing-time-first: a batch's latency is bounded by
+// its longest chunk, a sequential chain of 64-byte compressions).
+__global__ void long_list_kernel(const BatchDesc* __restrict__ desc,
+                                 const uint32_t* __restrict__ cut_pos,
+                                 const uint32_t* __restrict__ n_chunks_p, uint64_t cap,
+                                 uint32_t long_bytes, uint32_t* counters,
+                                 uint32_t* __restrict__ long_list) {
     const uint32_t n = (uint32_t)min((uint64_t)*n_chunks_p, cap);
+    const uint64_t nbytes = desc->nbytes;
+    for (uint32_t k = blockIdx.x * blockDim.x + threadIdx.x; k < n; k += gridDim.x * blockDim.x) {
+        const uint64_t e = (k + 1 < n) ? (uint64_t)cut_pos[k + 1] : nbytes;
+        if (e - cut_pos[k] >= long_bytes) long_list[atomicAdd(&counters[1], 1u)] = k;
+    }
+}
+
+// counters[0]: work counter, counters[1]: number of long chunks.
+__global__ void __launch_bounds__(kShaThreads, 6)
+sha1_kernel(const BatchDesc* __restrict__ desc,
+            const uint32_t* __restrict__ cut_pos, const uint32_t* __restrict__ n_chunks_p,
+            uint64_t cap, uint32_t long_bytes, uint32_t* counters,
+            const uint32_t* __restrict__ long_list, uint8_t* __restrict__ digest, uint32_t one) {
+    const uint8_t* __restrict__ bytes = desc->bytes;
+    const uint64_t nbytes = desc->nbytes;
+    const uint32_t n = (uint32_t)min((uint64_t)*n_chunks_p, cap);
+    const uint32_t n_long = *((volatile uint32_t*)&counters[1]);
+    const uint32_t total = n + n_long;
     const uint32_t lane = threadIdx.x & 31;
     const uint64_t lim16 = (nbytes + 15) & ~uint64_t(15);
     int64_t k = -1;      // chunk owned by this lane
-    uint64_t p = 0;      // next byte of the chunk to consume
+    uint64_t p = 0;      // byte offset of the next block's data
     uint32_t rem = 0;    // chunk bytes not yet consumed
     uint32_t len = 0;    // chunk length
     uint32_t phase = 0;  // 1: only the length block is left
     bool done = false;
     uint32_t H[5] = {0, 0, 0, 0, 0};
+    uint32_t raw[20];    // prefetched data window of the next block
     while (true) {
-        const bool need = !done && k < 0;
-        const uint32_t m = __ballot_sync(kFull, need);
-        if (m) {
+        // ---- pull work: long chunks first, then all others in order ----
+        while (true) {
+            const bool need = !done && k < 0;
+            const uint32_t m = __ballot_sync(kFull, need);
+            if (!m) break;
             const int leader = __ffs(m) - 1;
             uint32_t base = 0;
-            if ((int)lane == leader) base = atomicAdd(work_counter, (uint32_t)__popc(m));
+            if ((int)lane == leader) base = atomicAdd(&counters[0], (uint32_t)__popc(m));
             base = __shfl_sync(kFull, base, leader);
             if (need) {
-                const uint32_t idx = base + __popc(m & ((1u << lane) - 1u));
-                if (idx < n) {
-                    k = idx;
+                const uint32_t w = base + __popc(m & ((1u << lane) - 1u));
+                if (w >= total) {
+                    done = true;
+                } else {
+                    const uint32_t idx = w < n_long ? long_list[w] : w - n_long;
                     const uint32_t s = cut_pos[idx];
                     const uint64_t e = (idx + 1 < n) ? (uint64_t)cut_pos[idx + 1] : nbytes;
-                    p = s;
-                    rem = len = (uint32_t)(e - s);
-                    phase = 0;
-                    H[0] = 0x67452301u;
-                    H[1] = 0xEFCDAB89u;
-                    H[2] = 0x98BADCFEu;
-                    H[3] = 0x10325476u;
-                    H[4] = 0xC3D2E1F0u;
-                } else {
-                    done = true;
+                    const uint32_t L = (uint32_t)(e - s);
+                    if (w < n_long || L < long_bytes) {  // else: already taken as long
+                        k = idx;
+                        p = s;
+                        rem = len = L;
+                        phase = 0;
+                        H[0] = 0x67452301u;
+                        H[1] = 0xEFCDAB89u;
+                        H[2] = 0x98BADCFEu;
+                        H[3] = 0x10325476u;
+                        H[4] = 0xC3D2E1F0u;
+                        load_raw<true>(bytes, p, lim16, raw);
+                    }
                 }
             }
         }
@@ -147,35 +182,40 @@ sha1_kernel(const uint8_t* __restrict__ bytes, uint64_t nbytes,
         if (!done) {
             uint32_t M[16];
             bool fin = false;
-            if (phase == 0 && rem >= 64) {
-                load_block<false>(bytes, p, lim16, M);
-                p += 64;
-                rem -= 64;
-            } else if (phase == 0) {
-                // final data block: rem (0..63) bytes, 0x80, zeros [, length]
-                load_block<true>(bytes, p, lim16, M);
+            if (phase == 0) {
+                realign(raw, (uint32_t)(p & 15), M);
+                if (rem < 64) {
+                    // final data block: rem (0..63) bytes, 0x80, zeros [, length]
 #pragma unroll
-                for (int j = 0; j < 16; ++j) {
-                    const int nv = (int)rem - 4 * j;
-                    uint32_t w = M[j];
-                    if (nv < 4) {
-                        if (nv >= 0) {
-                            const uint32_t keep = nv == 0 ? 0u : (0xFFFFFFFFu << (32 - 8 * nv));
-                            w = (w & keep) | (0x80u << (24 - 8 * nv));
-                        } else {
-                            w = 0;
+                    for (int j = 0; j < 16; ++j) {
+                        const int nv = (int)rem - 4 * j;
+                        uint32_t w = M[j];
+                        if (nv < 4) {
+                            if (nv >= 0) {
+                                const uint32_t keep =
+                                    nv == 0 ? 0u : (0xFFFFFFFFu << (32 - 8 * nv));
+                                w = (w & keep) | (0x80u << (24 - 8 * nv));
+                            } else {
+                                w = 0;
+                            }
                         }
+                        M[j] = w;
                     }
-                    M[j] = w;
-                }
-                if (rem <= 55) {
-                    M[14] = len >> 29;
-                    M[15] = len << 3;
-                    fin = true;
+                    if (rem <= 55) {
+                        M[14] = len >> 29;
+                        M[15] = len << 3;
+                        fin = true;
+                    } else {
+                        phase = 1;
+                    }
+                    rem = 0;
                 } else {
-                    phase = 1;
+                    p += 64;
+                    rem -= 64;
+                    // prefetch the next block's window while this one compresses
+                    if (rem >= 64) load_raw<false>(bytes, p, lim16, raw);
+                    else if (rem > 0) load_raw<true>(bytes, p, lim16, raw);
                 }
-                rem = 0;
             } else {
 #pragma unroll
                 for (int j = 0; j < 14; ++j) M[j] = 0;
@@ -183,7 +223,7 @@ sha1_kernel(const uint8_t* __restrict__ bytes, uint64_t nbytes,
                 M[15] = len << 3;
                 fin = true;
             }
-            sha1_compress(H, M);
+            sha1_compress(H, M, one);
             if (fin) {
                 uint32_t* out = reinterpret_cast<uint32_t*>(digest + 20 * (uint64_t)k);
 #pragma unroll
@@ -196,16 +236,26 @@ sha1_kernel(const uint8_t* __restrict__ bytes, uint64_t nbytes,
 
 }  // namespace
 
-void launch_sha1(const uint8_t* bytes, uint64_t nbytes, const uint32_t* cut_pos,
-                 const uint32_t* n_chunks, uint64_t cap, uint32_t* work_counter,
-                 uint8_t* digest, int num_sms, cudaStream_t s) {
-    cudaMemsetAsync(work_counter, 0, sizeof(uint32_t), s);
-    if (cap == 0) return;
-    uint64_t blocks = (cap + kShaThreads - 1) / kShaThreads;
-    const uint64_t max_blocks = (uint64_t)num_sms * 8;
-    if (blocks > max_blocks) blocks = max_blocks;
-    sha1_kernel<<<(unsigned)blocks, kShaThreads, 0, s>>>(bytes, nbytes, cut_pos, n_chunks, cap,
-                                                         work_counter, digest);
+void launch_sha1(const BatchDesc* d, uint64_t max_bytes, const uint32_t* cut_pos,
+                 const uint32_t* n_chunks, uint64_t cap, uint32_t long_bytes, uint32_t* counters,
+                 uint32_t* long_list, uint8_t* digest, int num_sms, cudaStream_t s) {
+    cudaMemsetAsync(counters, 0, 2 * sizeof(uint32_t), s);
+    // Persistent lanes pull chunks dynamically, so the grid only needs enough
+    // lanes to finish the batch's bulk within its longest chunk's latency:
+    // one lane per kShaLaneBytes of input keeps the per-batch footprint small
+    // and leaves the SMs to the other in-flight batches.
+    const uint64_t kShaLaneBytes = 8192;
+    uint64_t lanes = max_bytes / kShaLaneBytes;
+    if (lanes < 1024) lanes = 1024;
+    uint64_t blocks = (lanes + kShaThreads - 1) / kShaThreads;
+    if (blocks > (uint64_t)num_sms * 6) blocks = (uint64_t)num_sms * 6;
+    uint64_t lb = (cap + 255) / 256;
+    if (lb > (uint64_t)num_sms * 2) lb = (uint64_t)num_sms * 2;
+    if (lb < 1) lb = 1;
+    long_list_kernel<<<(unsigned)lb, 256, 0, s>>>(d, cut_pos, n_chunks, cap, long_bytes, counters,
+                                                  long_list);
+    sha1_kernel<<<(unsigned)blocks, kShaThreads, 0, s>>>(d, cut_pos, n_chunks, cap, long_bytes,
+                                                         counters, long_list, digest, 1u);
 }
 
 }  // namespace dd

@@ -47,10 +47,23 @@ __device__ __forceinline__ uint64_t record_count(const uint32_t* d_n, uint64_t n
     return d_n != nullptr ? min((uint64_t)*d_n, cap) : n_host;
 }
 
-__global__ void table_insert_kernel(TableView t, const uint8_t* __restrict__ digest,
+__global__ void table_prepare_kernel(const BatchDesc* __restrict__ desc) {
+    if (!desc->fresh) return;
+    const TableView t = desc->table;
+    uint4* p = reinterpret_cast<uint4*>(t.slots);
+    const uint64_t n = 2 * (t.mask + 1);  // two uint4 per 32-byte slot
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n;
+         i += (uint64_t)gridDim.x * blockDim.x)
+        p[i] = make_uint4(0, 0, 0, 0);
+    if (blockIdx.x == 0 && threadIdx.x < 4) t.status[threadIdx.x] = 0;
+}
+
+__global__ void table_insert_kernel(const TableView* __restrict__ tv,
+                                    const uint8_t* __restrict__ digest,
                                     const uint64_t* __restrict__ id, const void* rec,
                                     const uint32_t* d_n, uint64_t n_host, uint64_t cap,
                                     uint32_t* __restrict__ slot_idx) {
+    const TableView t = *tv;
     const uint64_t n = record_count(d_n, n_host, cap);
     for (uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; r < n;
          r += (uint64_t)gridDim.x * blockDim.x) {
@@ -95,11 +108,16 @@ __global__ void table_insert_kernel(TableView t, const uint8_t* __restrict__ dig
     }
 }
 
-__global__ void table_lookup_kernel(TableView t, const uint64_t* __restrict__ id,
+__global__ void table_lookup_kernel(const TableView* __restrict__ tv,
+                                    const uint64_t* __restrict__ id,
                                     const void* rec, const uint32_t* d_n, uint64_t n_host,
                                     uint64_t cap, const uint32_t* __restrict__ slot_idx,
-                                    uint64_t* __restrict__ first_id, uint8_t* __restrict__ is_dup) {
+                                    uint64_t* __restrict__ first_id, uint8_t* __restrict__ is_dup,
+                                    uint32_t* __restrict__ status_out) {
+    const TableView t = *tv;
     const uint64_t n = record_count(d_n, n_host, cap);
+    if (status_out != nullptr && blockIdx.x == 0 && threadIdx.x < 2)
+        status_out[threadIdx.x] = t.status[threadIdx.x];  // overflow flag, used slots
     for (uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; r < n;
          r += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t si = slot_idx[r];
@@ -180,18 +198,21 @@ __global__ void scatter_kernel(const uint64_t* __restrict__ reply,
     }
 }
 
-__global__ void pack_kernel(const uint32_t* __restrict__ n_chunks_p, uint64_t cap,
-                            uint32_t n_items, const uint32_t* __restrict__ chunk_start,
+__global__ void pack_kernel(const BatchDesc* __restrict__ desc,
+                            const uint32_t* __restrict__ n_chunks_p, uint64_t cap,
+                            const uint32_t* __restrict__ chunk_start,
                             const uint64_t* __restrict__ first_id,
                             const uint8_t* __restrict__ digest, const uint8_t* __restrict__ is_dup,
                             const uint32_t* __restrict__ item_first_chunk,
                             const uint32_t* __restrict__ table_status, HostResultLayout h) {
     const uint64_t n = min((uint64_t)*n_chunks_p, cap);
+    const uint32_t n_items = desc->n_items;
     const uint64_t tid = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
     if (tid == 0) {
         h.header[0] = (uint32_t)*n_chunks_p;
-        h.header[1] = table_status[0];
+        h.header[1] = table_status[0];  // overflow flag (copied by the lookup)
+        h.header[2] = table_status[1];  // used table slots
     }
     for (uint64_t r = tid; r < n; r += stride) {
         h.chunk_start[r] = chunk_start[r];
@@ -214,7 +235,11 @@ unsigned grid_for(uint64_t n, int threads, int num_sms, int per_sm) {
 
 }  // namespace
 
-void launch_table_insert(TableView t, const uint8_t* digest, const uint64_t* id,
+void launch_table_prepare(const BatchDesc* d, uint64_t max_slots, int num_sms, cudaStream_t s) {
+    table_prepare_kernel<<<grid_for(2 * max_slots, 256, num_sms, 4), 256, 0, s>>>(d);
+}
+
+void launch_table_insert(const TableView* t, const uint8_t* digest, const uint64_t* id,
                          const void* rec, const uint32_t* d_n, uint64_t n_host, uint64_t cap,
                          uint32_t* slot_idx, int num_sms, cudaStream_t s) {
     const uint64_t n = d_n != nullptr ? cap : n_host;
@@ -223,14 +248,13 @@ void launch_table_insert(TableView t, const uint8_t* digest, const uint64_t* id,
                                                                        n_host, cap, slot_idx);
 }
 
-void launch_table_lookup(TableView t, const uint64_t* id, const void* rec,
+void launch_table_lookup(const TableView* t, const uint64_t* id, const void* rec,
                          const uint32_t* d_n, uint64_t n_host, uint64_t cap,
                          const uint32_t* slot_idx, uint64_t* first_id, uint8_t* is_dup,
-                         int num_sms, cudaStream_t s) {
+                         uint32_t* status_out, int num_sms, cudaStream_t s) {
     const uint64_t n = d_n != nullptr ? cap : n_host;
-    if (n == 0) return;
     table_lookup_kernel<<<grid_for(n, 256, num_sms, 8), 256, 0, s>>>(
-        t, id, rec, d_n, n_host, cap, slot_idx, first_id, is_dup);
+        t, id, rec, d_n, n_host, cap, slot_idx, first_id, is_dup, status_out);
 }
 
 void launch_route(const uint8_t* digest, const uint64_t* id, const uint32_t* d_n, uint64_t cap,
@@ -253,14 +277,14 @@ void launch_scatter(const uint64_t* reply, const uint32_t* send_pos, const uint6
                                                                   first_id, is_dup);
 }
 
-void launch_pack(const uint32_t* n_chunks, uint64_t cap, uint32_t n_items,
+void launch_pack(const BatchDesc* d, const uint32_t* n_chunks, uint64_t cap, uint32_t max_items,
                  const uint32_t* chunk_start, const uint64_t* first_id, const uint8_t* digest,
                  const uint8_t* is_dup, const uint32_t* item_first_chunk,
                  const uint32_t* table_status, HostResultLayout h, int num_sms,
                  cudaStream_t s) {
-    pack_kernel<<<grid_for(cap * 5 + n_items + 1, 256, num_sms, 4), 256, 0, s>>>(
-        n_chunks, cap, n_items, chunk_start, first_id, digest, is_dup, item_first_chunk,
-        table_status, h);
+    pack_kernel<<<grid_for(cap / 4 + max_items + 1, 256, num_sms, 2), 256, 0, s>>>(
+        d, n_chunks, cap, chunk_start, first_id, digest, is_dup, item_first_chunk, table_status,
+        h);
 }
 
 }  // namespace dd

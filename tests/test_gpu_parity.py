@@ -253,6 +253,25 @@ def test_adversarial_streams(cuda, kind):
         assert all(g.n_chunks == 1 for g in got)
 
 
+def test_table_chain_orders_batches(cuda):
+    """Batch 0 = one 1 MiB no-anchor item (a long sequential SHA-1 chain) +
+    small item B; batch 1 = a copy of B, submitted right behind it.  Batch 1's
+    lookup must wait for batch 0's inserts: B' is a duplicate of B."""
+    long_item = A.constructed_no_hit(1 << 20, 77)
+    b = np.random.default_rng(8).integers(0, 256, 100, dtype=np.uint8)
+    d0 = torch.from_numpy(np.concatenate([long_item, b, np.zeros(12, np.uint8)])).to(cuda)
+    d1 = torch.from_numpy(np.concatenate([b, np.zeros(12, np.uint8)])).to(cuda)
+    with make_ctx(batch_bytes=2 << 20, slots=4) as d:
+        for rep in range(4):
+            s0 = d.submit_device(d0, np.array([0, 1 << 20, (1 << 20) + 100], np.uint64))
+            d.submit_device(d1, np.array([0, 100], np.uint64))
+            got = d.drain_all()
+            assert [g.seq for g in got] == [s0, s0 + 1, s0 + 2]
+            assert got[2].is_dup[0] == 1 and int(got[2].first_id[0]) == ((s0 + 1) << 32)
+            assert got[0].n_chunks == 1 and got[0].is_dup[0] == 0
+            d.end_stream()
+
+
 def test_end_stream_fresh_table(cuda):
     data = U.stream(6 << 20, seed=31, dup_frac=0.6)
     off = synthgen.split_items(data)
