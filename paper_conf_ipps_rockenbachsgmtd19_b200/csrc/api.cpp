@@ -39,7 +39,8 @@ constexpr int kOpRing = 64;  // descriptors in flight for the dedup_op_* layer
 struct Workspace {
     uint32_t* bitmap = nullptr;      // candidate bitmap, one bit per byte
     uint32_t* agg = nullptr;         // per-tile transfer functions (32 u32 per tile)
-    uint32_t* tile_entry = nullptr;  // per-tile entry state + cut offset
+    uint32_t* gagg = nullptr;        // per-group transfer functions (32 u32 per group)
+    uint32_t* gentry = nullptr;      // per-group entry state + cut offset
     uint32_t* counters = nullptr;    // [0..1] sha1 work/long counters, [64..191] route
     uint32_t* slot_idx = nullptr;    // table slot per record
     uint32_t* long_list = nullptr;   // SHA-1 long-chunk list
@@ -176,7 +177,8 @@ dedup_status ws_alloc(dedup_ctx* c, Workspace& w, uint64_t batch_bytes, uint64_t
     w.max_tiles = (batch_bytes + kSelTile - 1) / kSelTile + 1;
     TRY(dalloc(c, &w.bitmap, batch_bytes / 32 + 2));
     TRY(dalloc(c, &w.agg, w.max_tiles * 32));
-    TRY(dalloc(c, &w.tile_entry, w.max_tiles * 2));
+    TRY(dalloc(c, &w.gagg, (select_groups(w.max_tiles) + 1) * 32));
+    TRY(dalloc(c, &w.gentry, (select_groups(w.max_tiles) + 1) * 2));
     TRY(dalloc(c, &w.counters, 256));
     TRY(dalloc(c, &w.slot_idx, cap));
     TRY(dalloc(c, &w.long_list, batch_bytes / kMinLongBytes + 2));
@@ -187,7 +189,8 @@ dedup_status ws_alloc(dedup_ctx* c, Workspace& w, uint64_t batch_bytes, uint64_t
 void ws_free(Workspace& w) {
     cudaFree(w.bitmap);
     cudaFree(w.agg);
-    cudaFree(w.tile_entry);
+    cudaFree(w.gagg);
+    cudaFree(w.gentry);
     cudaFree(w.counters);
     cudaFree(w.slot_idx);
     cudaFree(w.long_list);
@@ -218,7 +221,7 @@ void enqueue_chunk_sha(dedup_ctx* c, Workspace& w, cudaStream_t s, const BatchDe
     launch_rabin_scan(d, c->d_tab, c->cfg.anchor_mask, c->cfg.anchor_value, w.bitmap,
                       c->num_sms, s);
     if (ev_scan) cudaEventRecordWithFlags(ev_scan, s, cudaEventRecordExternal);
-    launch_select(d, w.bitmap, w.agg, w.tile_entry, (max_bytes + kSelTile - 1) / kSelTile,
+    launch_select(d, w.bitmap, w.agg, w.gagg, w.gentry, (max_bytes + kSelTile - 1) / kSelTile,
                   cut_pos, cap, n_chunks, c->num_sms, s);
     if (chunk_start)
         launch_chunk_meta(d, cut_pos, n_chunks, cap, chunk_start, chunk_id, item_first,
@@ -277,6 +280,7 @@ dedup_status build_graph(dedup_ctx* c, int i) {
     cudaGraphDestroy(g);
     if (e != cudaSuccess)
         return fail(c, DEDUP_ECUDA, std::string("graph instantiate: ") + cudaGetErrorString(e));
+    CU(cudaGraphUpload(sl.graph, s));  // keep the first launch off the critical path
     return DEDUP_OK;
 }
 

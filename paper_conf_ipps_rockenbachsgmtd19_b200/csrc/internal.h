@@ -42,12 +42,13 @@ constexpr uint32_t kSelTileWords = kSelTile / 32;
 void launch_rabin_scan(const BatchDesc* d, const uint32_t* d_tab, uint32_t mask, uint32_t value,
                        uint32_t* bitmap, int num_sms, cudaStream_t s);
 
-// Greedy cut selection over kSelTile-position tiles in three phases:
-// per-tile 32-entry transfer functions (agg), one-CTA prefix composition
-// (tile_entry = entry state | cut offset), per-tile replay writing cut_pos.
-// agg: 32 u32 per tile; tile_entry: 2 u32 per tile; max_tiles from batch_bytes.
-void launch_select(const BatchDesc* d, const uint32_t* bitmap, uint32_t* agg,
-                   uint32_t* tile_entry, uint64_t max_tiles, uint32_t* cut_pos, uint64_t cap,
+// Greedy cut selection over kSelTile-position tiles: per-tile 32-entry
+// transfer functions (agg, 32 u32 per tile) composed per group of 32 tiles
+// (gagg, 32 u32 per group), a one-CTA prefix over the groups (gentry, 2 u32
+// per group: entry state, cut offset) and a replay writing cut_pos.
+uint64_t select_groups(uint64_t max_tiles);
+void launch_select(const BatchDesc* d, const uint32_t* bitmap, uint32_t* agg, uint32_t* gagg,
+                   uint32_t* gentry, uint64_t max_tiles, uint32_t* cut_pos, uint64_t cap,
                    uint32_t* n_chunks, int num_sms, cudaStream_t s);
 
 void launch_chunk_meta(const BatchDesc* d, const uint32_t* cut_pos, const uint32_t* n_chunks,
