@@ -26,6 +26,10 @@ import time
 
 import numpy as np
 
+# Up to 32 hardware work queues, so that the engine's per-slot streams run
+# concurrently (must be set before CUDA is initialised).
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
+
 ROOT = os.path.dirname(os.path.abspath(__file__))
 if ROOT not in sys.path:
     sys.path.insert(0, ROOT)

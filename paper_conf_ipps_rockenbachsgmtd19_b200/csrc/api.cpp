@@ -21,6 +21,7 @@
 
 #include <chrono>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <deque>
 #include <string>
@@ -41,6 +42,7 @@ struct Workspace {
     uint32_t* agg = nullptr;         // per-tile transfer functions (32 u32 per tile)
     uint32_t* gagg = nullptr;        // per-group transfer functions (32 u32 per group)
     uint32_t* gentry = nullptr;      // per-group entry state + cut offset
+    uint32_t* scan_ctr = nullptr;    // scan tile counter + per-group arrival counters
     uint32_t* counters = nullptr;    // [0..1] sha1 work/long counters, [64..191] route
     uint32_t* slot_idx = nullptr;    // table slot per record
     uint32_t* long_list = nullptr;   // SHA-1 long-chunk list
@@ -117,6 +119,8 @@ struct dedup_ctx {
     uint64_t launches = 0;
     uint32_t graph_kernels = 0;  // kernels per batch graph
     dedup_stats_t st{};
+    bool trace = false;           // DEDUP_TRACE environment variable
+    cudaEvent_t ev_ref = nullptr;  // time origin of the trace
 };
 
 namespace {
@@ -179,6 +183,7 @@ dedup_status ws_alloc(dedup_ctx* c, Workspace& w, uint64_t batch_bytes, uint64_t
     TRY(dalloc(c, &w.agg, w.max_tiles * 32));
     TRY(dalloc(c, &w.gagg, (select_groups(w.max_tiles) + 1) * 32));
     TRY(dalloc(c, &w.gentry, (select_groups(w.max_tiles) + 1) * 2));
+    TRY(dalloc(c, &w.scan_ctr, select_groups(w.max_tiles) + 2));
     TRY(dalloc(c, &w.counters, 256));
     TRY(dalloc(c, &w.slot_idx, cap));
     TRY(dalloc(c, &w.long_list, batch_bytes / kMinLongBytes + 2));
@@ -191,6 +196,7 @@ void ws_free(Workspace& w) {
     cudaFree(w.agg);
     cudaFree(w.gagg);
     cudaFree(w.gentry);
+    cudaFree(w.scan_ctr);
     cudaFree(w.counters);
     cudaFree(w.slot_idx);
     cudaFree(w.long_list);
@@ -218,11 +224,9 @@ void enqueue_chunk_sha(dedup_ctx* c, Workspace& w, cudaStream_t s, const BatchDe
                        uint8_t* digest, cudaEvent_t ev_scan, cudaEvent_t ev_chunk,
                        uint32_t* chunk_start, uint64_t* chunk_id, uint32_t* item_first,
                        uint32_t max_items) {
-    launch_rabin_scan(d, c->d_tab, c->cfg.anchor_mask, c->cfg.anchor_value, w.bitmap,
-                      c->num_sms, s);
-    if (ev_scan) cudaEventRecordWithFlags(ev_scan, s, cudaEventRecordExternal);
-    launch_select(d, w.bitmap, w.agg, w.gagg, w.gentry, (max_bytes + kSelTile - 1) / kSelTile,
-                  cut_pos, cap, n_chunks, c->num_sms, s);
+    launch_chunk_select(d, c->d_tab, c->cfg.anchor_mask, c->cfg.anchor_value, w.bitmap, w.agg,
+                        w.gagg, w.gentry, w.scan_ctr, (max_bytes + kSelTile - 1) / kSelTile,
+                        cut_pos, cap, n_chunks, c->num_sms, s, ev_scan);
     if (chunk_start)
         launch_chunk_meta(d, cut_pos, n_chunks, cap, chunk_start, chunk_id, item_first,
                           max_items, c->num_sms, s);
@@ -441,6 +445,17 @@ dedup_status parse_slot(dedup_ctx* c, Slot& sl) {
     if (cudaEventElapsedTime(&ms, sl.ev_chunk, sl.ev_sha) == cudaSuccess) c->st.ms_sha1 += ms;
     if (cudaEventElapsedTime(&ms, sl.ev_sha, sl.ev_table) == cudaSuccess) c->st.ms_table += ms;
     if (cudaEventElapsedTime(&ms, sl.ev_table, sl.ev_done) == cudaSuccess) c->st.ms_d2h += ms;
+    if (c->trace) {  // DEDUP_TRACE=1: per-batch event timeline (ms since ctx init)
+        float t[7] = {0, 0, 0, 0, 0, 0, 0};
+        const cudaEvent_t ev[7] = {sl.ev_start, sl.ev_h2d, sl.ev_scan, sl.ev_chunk,
+                                   sl.ev_sha, sl.ev_table, sl.ev_done};
+        for (int k = 0; k < 7; ++k) cudaEventElapsedTime(&t[k], c->ev_ref, ev[k]);
+        std::fprintf(stderr,
+                     "trace seq=%llu bytes=%llu start=%.3f h2d=%.3f scan=%.3f chunk=%.3f "
+                     "sha=%.3f table=%.3f done=%.3f\n",
+                     (unsigned long long)sl.first_seq, (unsigned long long)sl.nbytes, t[0], t[1],
+                     t[2], t[3], t[4], t[5], t[6]);
+    }
     cudaGetLastError();  // clear a possible error from a timing query
     sl.parsed = true;
     return DEDUP_OK;
@@ -530,6 +545,9 @@ dedup_status dedup_init(const dedup_config* cfg, dedup_ctx** out) {
     c->st.table_slots = c->tables[0].capacity;
     c->st.num_owners = cfg->num_owners;
     c->st.owner_rank = cfg->owner_rank;
+    c->trace = std::getenv("DEDUP_TRACE") != nullptr;
+    if (cudaEventCreate(&c->ev_ref) != cudaSuccess || cudaEventRecord(c->ev_ref, 0) != cudaSuccess)
+        return bail(DEDUP_ECUDA);
     *out = c;
     return DEDUP_OK;
 }
@@ -549,6 +567,7 @@ void dedup_destroy(dedup_ctx* c) {
         cudaFree(t.status);
     }
     cudaFree(c->d_tab);
+    if (c->ev_ref) cudaEventDestroy(c->ev_ref);
     delete c;
 }
 

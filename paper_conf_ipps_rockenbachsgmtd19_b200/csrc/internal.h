@@ -37,19 +37,19 @@ struct BatchDesc {
 constexpr uint32_t kSelTile = 8192;
 constexpr uint32_t kSelTileWords = kSelTile / 32;
 
-// Bitmap bit i (i < nbytes) set iff (fp(bytes[i-31..i]) & mask) == value.
-// Grid: fixed (2 CTAs per SM); sized from desc->nbytes inside the kernel.
-void launch_rabin_scan(const BatchDesc* d, const uint32_t* d_tab, uint32_t mask, uint32_t value,
-                       uint32_t* bitmap, int num_sms, cudaStream_t s);
-
-// Greedy cut selection over kSelTile-position tiles: per-tile 32-entry
-// transfer functions (agg, 32 u32 per tile) composed per group of 32 tiles
-// (gagg, 32 u32 per group), a one-CTA prefix over the groups (gentry, 2 u32
-// per group: entry state, cut offset) and a replay writing cut_pos.
+// Rows A2 + A3: Rabin scan fused with the per-tile 32-entry transfer
+// functions of the greedy cut selection (agg, 32 u32 per kSelTile tile) and
+// their per-group composition (gagg, 32 u32 per group of 32 tiles); a one-CTA
+// prefix over the groups (gentry, 2 u32 per group: entry state, cut offset);
+// a replay writing cut_pos.  bitmap: e-space candidate words (nbytes/32 + 1);
+// scan_ctr: select_groups(max_tiles) + 2 words, zeroed by the launcher.
+// after_scan (optional) is recorded between the scan and the selection.
 uint64_t select_groups(uint64_t max_tiles);
-void launch_select(const BatchDesc* d, const uint32_t* bitmap, uint32_t* agg, uint32_t* gagg,
-                   uint32_t* gentry, uint64_t max_tiles, uint32_t* cut_pos, uint64_t cap,
-                   uint32_t* n_chunks, int num_sms, cudaStream_t s);
+void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mask,
+                         uint32_t value, uint32_t* bitmap, uint32_t* agg, uint32_t* gagg,
+                         uint32_t* gentry, uint32_t* scan_ctr, uint64_t max_tiles,
+                         uint32_t* cut_pos, uint64_t cap, uint32_t* n_chunks, int num_sms,
+                         cudaStream_t s, cudaEvent_t after_scan);
 
 void launch_chunk_meta(const BatchDesc* d, const uint32_t* cut_pos, const uint32_t* n_chunks,
                        uint64_t cap, uint32_t* chunk_start, uint64_t* chunk_id,

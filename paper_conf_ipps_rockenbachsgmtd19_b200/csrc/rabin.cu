@@ -3,27 +3,30 @@
 // fragmentation of fixed batches, "saved all the indexes where the algorithm
 // would fragment the data"), P:199 / Fig. 2 (startPos).
 //
-// The paper ran this on the CPU; here it is a set of sm_100a kernels:
+// The paper ran this on the CPU; here it is three sm_100a kernels:
 //
-//  rabin_scan_kernel   every lane owns a contiguous segment of the batch,
-//                      re-derives the 32-byte window hash over the 32 bytes
-//                      before its segment (warm-up), then rolls byte by byte
-//                      with the post-shift recurrence
-//                        h' = ((h << 8) | in) ^ R[h >> 24] ^ W256[out]
-//                      and emits one candidate bit per byte.  Both tables are
-//                      replicated per lane in shared memory ([x][lane] layout,
-//                      bank = lane, conflict-free), addressed with one PRMT.
-//  select_*_kernel     greedy cut selection.  With min chunk = window = 32 the
-//                      only state crossing a position is "positions still
-//                      blocked" in [0, 31]; a warp simulates all 32 entry
-//                      states of an 8192-position tile (lane s = state s)
-//                      giving the tile's 32-entry transfer function; a CTA of
-//                      32 warps composes its 32 tiles into a group function;
-//                      one CTA composes the group functions in order (a prefix
-//                      over an associative operator, warp shuffles); a replay
-//                      pass walks every tile from its real entry state and
-//                      writes the cut positions.  Item starts are forced cuts
-//                      and reset the state.
+//  rabin_scan_agg_kernel  persistent, one CTA of 32 warps per SM.  A warp
+//      takes an 8 KiB tile (dynamic counter); each lane rolls the 32-byte
+//      window hash over its 256 bytes (after a 32-byte warm-up) with the
+//      post-shift recurrence
+//          h' = ((h << 8) | in) ^ R[h >> 24] ^ W256[out]
+//      and records one candidate bit per byte.  R and W256 are replicated per
+//      lane in shared memory ([x][lane] layout: bank = lane, conflict-free);
+//      the table sits on a 64 KiB boundary of the shared window so that one
+//      PRMT builds the whole LDS address.  Greedy cut selection is then a
+//      32-state machine (with min chunk = window = 32 the only state crossing
+//      a position is "positions still blocked", 0..31): the warp simulates all
+//      32 entry states over its tile (lane s = state s) and stores the tile's
+//      transfer function; the last warp to finish a group of 32 tiles composes
+//      them into the group function (warp shuffles).
+//  select_scan_kernel     one CTA composes the group functions in order (a
+//      prefix over an associative operator) -> entry state and cut offset of
+//      every group, and the batch's chunk count.
+//  select_emit_kernel     one CTA per group derives its tiles' entry states
+//      and every warp replays its tile from the real entry state, writing the
+//      cut positions (the paper's startPos).
+// Item starts are forced cuts and reset the state; a candidate is valid only
+// if its 32-byte window lies inside one item.
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -33,30 +36,61 @@ namespace dd {
 
 namespace {
 
-constexpr int kScanThreads = 512;
+constexpr int kScanThreads = 1024;  // 32 warps = one group of 32 tiles
 constexpr int kTabBytes = 256 * 256;  // [x][R|W][lane] u32 = 64 KiB
+constexpr uint32_t kLaneBytes = kSelTile / 32;  // 256 bytes per lane per tile
 constexpr uint32_t kFull = 0xFFFFFFFFu;
+constexpr uint32_t kInf = 0xFFFFFFFFu;
+constexpr uint32_t kM27 = (1u << 27) - 1;
+constexpr int kGroup = 32;        // tiles per group
+constexpr int kItemCache = 2048;  // item offsets cached in shared memory
+
+struct SelWarpSmem {
+    uint32_t cand[kSelTileWords];
+    uint32_t forced[kSelTileWords];
+    uint32_t csum[8];
+    uint32_t fsum[8];
+};
+
+// scan: [pad to a 64 KiB shared-window boundary][table][SelWarpSmem x 32][items]
+constexpr int kScanSmem =
+    65536 + kTabBytes + kGroup * (int)sizeof(SelWarpSmem) + kItemCache * 8;
+
+struct EmitSmem {
+    SelWarpSmem w[kGroup];
+    uint32_t fun[kGroup][32];
+    uint32_t te_state[kGroup], te_cnt[kGroup];
+    uint64_t items[kItemCache];
+};
+
+__device__ __forceinline__ uint32_t lds(uint32_t addr) {
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(addr));
+    return v;
+}
 
 // Rolls the 32 bytes of cur[0..7] (stream bytes, little-endian words) into h,
-// removing the 32 bytes of old[0..7]; returns the 32 candidate bits.
+// removing the 32 bytes of old[0..7]; returns the 32 candidate bits
+// (bit b <=> the window ending at byte b of this step).
+// laneR / laneW = table base (64 KiB aligned) | lane*4 (+128 for W256).
 template <bool kZeroValue>
 __device__ __forceinline__ uint32_t roll32(uint32_t& h, const uint32_t cur[8],
-                                           const uint32_t old[8], const uint8_t* tab,
-                                           uint32_t laneoff, uint32_t mask, uint32_t value) {
+                                           const uint32_t old[8], uint32_t laneR, uint32_t laneW,
+                                           uint32_t mask, uint32_t value) {
     uint32_t bits = 0;
 #pragma unroll
     for (int w = 0; w < 8; ++w) {
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
-            // R[x] at x*256 + lane*4, W256[o] at o*256 + 128 + lane*4.
-            const uint32_t aR = __byte_perm(h, laneoff, 0x6534);
-            const uint32_t aW = __byte_perm(old[w], laneoff, 0x6504 | (k << 4));
+            // R[x] at base + x*256 + lane*4, W256[o] at base + o*256 + 128 + lane*4.
+            const uint32_t aR = __byte_perm(h, laneR, 0x7634);
+            const uint32_t aW = __byte_perm(old[w], laneW, 0x7604 | (k << 4));
             const uint32_t hs = __byte_perm(cur[w], h, 0x6540 | k);  // (h << 8) | in
-            const uint32_t r = *reinterpret_cast<const uint32_t*>(tab + aR);
-            const uint32_t o = *reinterpret_cast<const uint32_t*>(tab + 128 + aW);
-            h = hs ^ r ^ o;
-            const bool hit = kZeroValue ? (h & mask) == 0 : (h & mask) == value;
-            if (hit) bits |= 1u << (4 * w + k);
+            h = hs ^ lds(aR) ^ lds(aW);
+            const uint32_t t = kZeroValue ? (h & mask) : ((h & mask) ^ value);
+            asm("{\n\t.reg .pred p;\n\tsetp.eq.u32 p, %1, 0;\n\t@p or.b32 %0, %0, %2;\n\t}"
+                : "+r"(bits)
+                : "r"(t), "r"(1u << (4 * w + k)));
         }
     }
     return bits;
@@ -69,100 +103,20 @@ __device__ __forceinline__ void load32(const uint8_t* p, uint32_t v[8]) {
     v[4] = b.x; v[5] = b.y; v[6] = b.z; v[7] = b.w;
 }
 
-// Guarded version: 16-byte vectors at or beyond lim16 (nbytes rounded up to
+// 32 bytes at off; 16-byte vectors at or beyond lim16 (nbytes rounded up to
 // 16) read as zero.
-__device__ __forceinline__ void load32_guard(const uint8_t* base, uint64_t off, uint64_t lim16,
-                                             uint32_t v[8]) {
+__device__ __forceinline__ void load32_any(const uint8_t* base, uint64_t off, uint64_t nbytes,
+                                           uint64_t lim16, uint32_t v[8]) {
+    if (off + 32 <= nbytes) {
+        load32(base + off, v);
+        return;
+    }
     uint4 a = make_uint4(0, 0, 0, 0), b = make_uint4(0, 0, 0, 0);
     if (off < lim16) a = __ldg(reinterpret_cast<const uint4*>(base + off));
     if (off + 16 < lim16) b = __ldg(reinterpret_cast<const uint4*>(base + off + 16));
     v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
     v[4] = b.x; v[5] = b.y; v[6] = b.z; v[7] = b.w;
 }
-
-__device__ __forceinline__ void load32_any(const uint8_t* base, uint64_t off, uint64_t nbytes,
-                                           uint64_t lim16, uint32_t v[8]) {
-    if (off + 32 <= nbytes) load32(base + off, v);
-    else load32_guard(base, off, lim16, v);
-}
-
-template <bool kZeroValue>
-__global__ void __launch_bounds__(kScanThreads, 2)
-rabin_scan_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ gtab,
-                  uint32_t mask, uint32_t value, uint32_t* __restrict__ bitmap) {
-    extern __shared__ __align__(16) uint8_t tab[];
-    __shared__ uint32_t src[512];
-    const uint8_t* __restrict__ bytes = desc->bytes;
-    const uint64_t nbytes = desc->nbytes;
-    if (threadIdx.x < 512) src[threadIdx.x] = gtab[threadIdx.x];
-    __syncthreads();
-    {   // replicate R / W256 per lane: word idx = x*64 + half*32 + lane
-        uint32_t* t32 = reinterpret_cast<uint32_t*>(tab);
-        for (int idx = threadIdx.x; idx < kTabBytes / 4; idx += blockDim.x)
-            t32[idx] = src[((idx >> 5) & 1) * 256 + (idx >> 6)];
-    }
-    __syncthreads();
-    if (nbytes == 0) return;
-    // Segment per lane: long enough that the 32-byte warm-up is cheap, short
-    // enough that the grid's lanes cover the batch in one pass.
-    const uint64_t threads = (uint64_t)gridDim.x * blockDim.x;
-    uint64_t seg = (nbytes + threads - 1) / threads;
-    seg = ((seg + 31) / 32) * 32;
-    if (seg < 256) seg = 256;
-    const uint64_t n_lanes = (nbytes + seg - 1) / seg;
-    const uint32_t laneoff = (threadIdx.x & 31) * 4;
-    const uint64_t lim16 = (nbytes + 15) & ~uint64_t(15);
-    for (uint64_t L = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; L < n_lanes;
-         L += threads) {
-        const uint64_t q = L * seg;
-        const uint64_t end = min(q + seg, nbytes);
-        uint32_t h = 0;
-        uint32_t prev[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-        uint32_t cur[8];
-        // issue the warm-up and the first step's loads together
-        if (q >= 32) load32(bytes + q - 32, prev);
-        load32_any(bytes, q, nbytes, lim16, cur);
-        if (q >= 32) {  // warm-up: hash of the window ending at q-1
-            const uint32_t zero[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-            (void)roll32<kZeroValue>(h, prev, zero, tab, laneoff, mask, value);
-        }
-        for (uint64_t base = q; base < end; base += 32) {
-            uint32_t nxt[8];
-            const uint64_t nb = base + 32;
-            if (nb < end) load32_any(bytes, nb, nbytes, lim16, nxt);  // prefetch
-            uint32_t bits = roll32<kZeroValue>(h, cur, prev, tab, laneoff, mask, value);
-            if (base + 32 > nbytes) bits &= (1u << (uint32_t)(nbytes - base)) - 1u;
-            bitmap[base >> 5] = bits;
-#pragma unroll
-            for (int i = 0; i < 8; ++i) {
-                prev[i] = cur[i];
-                cur[i] = nxt[i];
-            }
-        }
-    }
-}
-
-// ---------------------------------------------------------------------------
-// Cut selection.
-// ---------------------------------------------------------------------------
-constexpr uint32_t kInf = 0xFFFFFFFFu;
-constexpr uint32_t kM27 = (1u << 27) - 1;
-constexpr int kGroup = 32;        // tiles per CTA (one per warp)
-constexpr int kItemCache = 2048;  // item offsets cached in shared memory
-
-struct SelWarpSmem {
-    uint32_t cand[kSelTileWords];
-    uint32_t forced[kSelTileWords];
-    uint32_t csum[8];
-    uint32_t fsum[8];
-};
-
-struct SelSmem {
-    SelWarpSmem w[kGroup];
-    uint32_t fun[kGroup][32];  // tile transfer functions of the group
-    uint32_t te_state[kGroup], te_cnt[kGroup];
-    uint64_t items[kItemCache];
-};
 
 // First set bit at tile-relative position >= from, or kInf.
 __device__ __forceinline__ uint32_t next_set(const uint32_t* words, const uint32_t* summary,
@@ -204,39 +158,26 @@ __device__ __forceinline__ uint32_t walk_tile(const SelWarpSmem& sm, uint32_t s,
 }
 
 // Item offsets: cached in shared memory when they fit.
-__device__ __forceinline__ const uint64_t* cache_items(SelSmem& sm, const BatchDesc* desc) {
+__device__ __forceinline__ const uint64_t* cache_items(uint64_t* cache, const BatchDesc* desc) {
     const uint32_t n = desc->n_items + 1;
     if (n > kItemCache) return desc->item_off;
-    for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) sm.items[i] = desc->item_off[i];
-    return sm.items;
+    for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) cache[i] = desc->item_off[i];
+    return cache;
 }
 
-// Candidate (e-space: cut after byte i <=> e = i + 1) and forced-cut bits of
-// tile t into the warp's shared memory, with one-bit-per-word summaries.
-__device__ __forceinline__ void build_tile(SelWarpSmem& sm, uint64_t t,
-                                           const uint32_t* __restrict__ bitmap, uint64_t nbytes,
-                                           const uint64_t* item_off, uint32_t n_items, int lane) {
-    const uint64_t T0 = t * kSelTile;
-    const uint64_t n_words = (nbytes + 31) / 32;
-    uint32_t cw[8], fw[8], raw[9];
-    const uint64_t E0 = T0 + (uint64_t)lane * 256;  // this lane's e-range
-    const uint64_t g0 = T0 / 32 + lane * 8;
-#pragma unroll
-    for (int j = 0; j < 9; ++j) {  // bitmap words g0-1 .. g0+7
-        const uint64_t g = g0 + j - 1;
-        raw[j] = (g0 + j >= 1 && g < n_words) ? bitmap[g] : 0u;
-    }
+// Lane's 8 e-space candidate words (already in sm.cand) get the item rules:
+// no candidate at e in [q, q+32) (the window would leave the item), a forced
+// cut at q for every non-empty item; then the summaries.  Ends with syncwarp.
+__device__ __forceinline__ void apply_items(SelWarpSmem& sm, uint64_t T0, uint64_t nbytes,
+                                            const uint64_t* item_off, uint32_t n_items,
+                                            int lane) {
+    uint32_t cw[8], fw[8];
 #pragma unroll
     for (int j = 0; j < 8; ++j) {
-        uint32_t ew = __funnelshift_l(raw[j], raw[j + 1], 1);
-        const uint64_t e_lo = E0 + 32 * j;
-        if (e_lo >= nbytes) ew = 0;
-        else if (e_lo + 32 > nbytes) ew &= (1u << (uint32_t)(nbytes - e_lo)) - 1u;
-        cw[j] = ew;
+        cw[j] = sm.cand[lane * 8 + j];
         fw[j] = 0;
     }
-    // items: no candidate at e in [q, q+32) (window would leave the item),
-    // forced cut at q for non-empty items
+    const uint64_t E0 = T0 + (uint64_t)lane * kLaneBytes;  // this lane's e-range
     if (E0 < nbytes && n_items > 0) {
         const uint64_t key = E0 >= 31 ? E0 - 31 : 0;  // first start > E0 - 32
         uint32_t lo = 0, hi = n_items;
@@ -246,7 +187,7 @@ __device__ __forceinline__ void build_tile(SelWarpSmem& sm, uint64_t t,
         }
         for (uint32_t it = lo; it < n_items; ++it) {
             const uint64_t q = item_off[it];
-            if (q >= E0 + 256) break;
+            if (q >= E0 + kLaneBytes) break;
             const bool nonempty = item_off[it + 1] > q;
 #pragma unroll
             for (int j = 0; j < 8; ++j) {
@@ -274,50 +215,119 @@ __device__ __forceinline__ void build_tile(SelWarpSmem& sm, uint64_t t,
     __syncwarp();
 }
 
-// Phase 1 (CTA = 32 warps = one group of 32 tiles): every warp derives its
-// tile's 32-entry transfer function agg[32 t + s] = exit(s) << 27 | cuts(s);
-// warp 0 composes the 32 functions into the group function gagg[32 g + s].
-__global__ void __launch_bounds__(1024)
-select_agg_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ bitmap,
-                  uint32_t* __restrict__ agg, uint32_t* __restrict__ gagg) {
-    extern __shared__ __align__(16) uint8_t smraw[];
-    SelSmem& sm = *reinterpret_cast<SelSmem*>(smraw);
-    const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+// Scan + per-tile transfer functions + per-group composition.
+// bitmap: e-space candidate words (bit e%32 of word e/32 <=> a window ends at
+// byte e-1), before the item rules.  agg[32 t + s] = exit(s) << 27 | cuts(s).
+// ctr[0] = tile counter, ctr[1 + g] = arrivals of group g (zeroed per batch).
+template <bool kZeroValue>
+__global__ void __launch_bounds__(kScanThreads, 1)
+rabin_scan_agg_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ gtab,
+                      uint32_t mask, uint32_t value, uint32_t* __restrict__ bitmap,
+                      uint32_t* __restrict__ agg, uint32_t* __restrict__ gagg,
+                      uint32_t* __restrict__ ctr) {
+    extern __shared__ __align__(16) uint8_t smem[];
+    __shared__ uint32_t src[512];
+    const uint8_t* __restrict__ bytes = desc->bytes;
     const uint64_t nbytes = desc->nbytes;
-    const uint64_t n_tiles = (nbytes + kSelTile - 1) / kSelTile;
-    const uint64_t n_groups = (n_tiles + kGroup - 1) / kGroup;
-    const uint64_t* items = cache_items(sm, desc);
+    const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    // the table starts at the first 64 KiB boundary of the shared window
+    const uint32_t win = (uint32_t)__cvta_generic_to_shared(smem);
+    const uint32_t pad = (0x10000u - (win & 0xFFFFu)) & 0xFFFFu;
+    const uint32_t base = win + pad;
+    SelWarpSmem* wsm = reinterpret_cast<SelWarpSmem*>(smem + pad + kTabBytes);
+    uint64_t* icache = reinterpret_cast<uint64_t*>(wsm + kGroup);
+    SelWarpSmem& sm = wsm[wid];
+    if (threadIdx.x < 512) src[threadIdx.x] = gtab[threadIdx.x];
+    const uint64_t* items = cache_items(icache, desc);
     const uint32_t n_items = desc->n_items;
     __syncthreads();
-    for (uint64_t g = blockIdx.x; g < n_groups; g += gridDim.x) {
-        const uint64_t t = g * kGroup + wid;
-        uint32_t f = (uint32_t)lane << 27;  // identity beyond the last tile
-        if (t < n_tiles) {
-            build_tile(sm.w[wid], t, bitmap, nbytes, items, n_items, lane);
-            uint32_t ex;
-            const uint32_t cnt = walk_tile(sm.w[wid], lane, ex, nullptr, 0, 0, 0);
-            f = (ex << 27) | cnt;
-            agg[32 * t + lane] = f;
+    {   // replicate R / W256 per lane: word idx = x*64 + half*32 + lane
+        uint32_t* t32 = reinterpret_cast<uint32_t*>(smem + pad);
+        for (int idx = threadIdx.x; idx < kTabBytes / 4; idx += blockDim.x)
+            t32[idx] = src[((idx >> 5) & 1) * 256 + (idx >> 6)];
+    }
+    __syncthreads();
+    if (nbytes == 0) return;
+    const uint64_t n_tiles = (nbytes + kSelTile - 1) / kSelTile;
+    const uint32_t laneR = base | (lane * 4);
+    const uint32_t laneW = laneR + 128;
+    const uint64_t lim16 = (nbytes + 15) & ~uint64_t(15);
+    while (true) {
+        uint32_t t = 0;
+        if (lane == 0) t = atomicAdd(&ctr[0], 1u);
+        t = __shfl_sync(kFull, t, 0);
+        if (t >= n_tiles) break;
+        const uint64_t T0 = (uint64_t)t * kSelTile;
+        const uint64_t q = T0 + (uint64_t)lane * kLaneBytes;
+        // ---- scan: 8 steps of 32 bytes, bits written in e-space ----
+        uint32_t h = 0, prev_bits = 0;
+        uint32_t prev[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+        uint32_t cur[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+        if (q >= 32) load32(bytes + q - 32, prev);
+        if (q < nbytes) load32_any(bytes, q, nbytes, lim16, cur);
+        if (q >= 32) {  // warm-up: the window ending at q-1 -> bit for e = q
+            const uint32_t zero[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+            prev_bits = roll32<kZeroValue>(h, prev, zero, laneR, laneW, mask, value);
         }
-        sm.fun[wid][lane] = f;
-        __syncthreads();
-        if (wid == 0) {
+#pragma unroll 1
+        for (int j = 0; j < 8; ++j) {
+            const uint64_t b0 = q + 32 * j;
+            uint32_t bits = 0, nxt[8];
+            if (j < 7 && b0 + 32 < nbytes) load32_any(bytes, b0 + 32, nbytes, lim16, nxt);
+            if (b0 < nbytes) {
+                bits = roll32<kZeroValue>(h, cur, prev, laneR, laneW, mask, value);
+                if (b0 + 32 > nbytes) bits &= (1u << (uint32_t)(nbytes - b0)) - 1u;
+            }
+            uint32_t ew = __funnelshift_l(prev_bits, bits, 1);  // e = i + 1
+            if (b0 >= nbytes) ew = 0;
+            else if (b0 + 32 > nbytes) ew &= (1u << (uint32_t)(nbytes - b0)) - 1u;
+            sm.cand[lane * 8 + j] = ew;
+            bitmap[T0 / 32 + lane * 8 + j] = ew;
+            prev_bits = bits;
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                prev[i] = cur[i];
+                cur[i] = nxt[i];
+            }
+        }
+        // ---- the tile's 32-entry transfer function ----
+        apply_items(sm, T0, nbytes, items, n_items, lane);
+        uint32_t ex;
+        const uint32_t cnt = walk_tile(sm, lane, ex, nullptr, 0, 0, 0);
+        agg[32 * (uint64_t)t + lane] = (ex << 27) | cnt;
+        __syncwarp();
+        // ---- the last tile of a group to finish composes the group ----
+        const uint64_t g = t / kGroup;
+        const uint64_t left = n_tiles - g * kGroup;
+        const uint32_t expected = left < (uint64_t)kGroup ? (uint32_t)left : (uint32_t)kGroup;
+        __threadfence();
+        uint32_t arrived = 0;
+        if (lane == 0) arrived = atomicAdd(&ctr[1 + g], 1u) + 1;
+        arrived = __shfl_sync(kFull, arrived, 0);
+        if (arrived == expected) {
+            __threadfence();
             uint32_t Gs = lane, Gc = 0;
-#pragma unroll 8
-            for (int j = 0; j < kGroup; ++j) {
-                const uint32_t a = sm.fun[j][lane];
-                const uint32_t ns = __shfl_sync(kFull, a >> 27, Gs);
-                const uint32_t nc = Gc + __shfl_sync(kFull, a & kM27, Gs);
-                Gs = ns;
-                Gc = nc;
+            for (uint32_t jb = 0; jb < expected; jb += 16) {
+                uint32_t a[16];
+#pragma unroll
+                for (int j = 0; j < 16; ++j)
+                    a[j] = jb + j < expected
+                               ? __ldcg(&agg[32 * (g * kGroup + jb + j) + lane])
+                               : ((uint32_t)lane << 27);
+#pragma unroll
+                for (int j = 0; j < 16; ++j) {
+                    const uint32_t ns = __shfl_sync(kFull, a[j] >> 27, Gs);
+                    const uint32_t nc = Gc + __shfl_sync(kFull, a[j] & kM27, Gs);
+                    Gs = ns;
+                    Gc = nc;
+                }
             }
             gagg[32 * g + lane] = (Gs << 27) | Gc;
         }
-        __syncthreads();
     }
 }
 
-// Phase 2 (one CTA of 32 warps): prefix composition of the group functions.
+// Prefix composition of the group functions (one CTA of 32 warps).
 // gentry[2g] = entry state of group g, gentry[2g+1] = cuts before it.
 __global__ void __launch_bounds__(1024)
 select_scan_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ gagg,
@@ -380,25 +390,28 @@ select_scan_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restric
     }
 }
 
-// Phase 3 (CTA = one group): entry states of the group's tiles from the group
-// entry, then every warp replays its tile from its real entry state, writing
-// cut_pos.
+// One CTA per group: entry states of the group's tiles from the group entry,
+// then every warp replays its tile from its real entry state, writing cut_pos.
 __global__ void __launch_bounds__(1024)
 select_emit_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ bitmap,
                    const uint32_t* __restrict__ agg, const uint32_t* __restrict__ gentry,
                    uint32_t* __restrict__ cut_pos, uint64_t cap) {
     extern __shared__ __align__(16) uint8_t smraw[];
-    SelSmem& sm = *reinterpret_cast<SelSmem*>(smraw);
+    EmitSmem& sm = *reinterpret_cast<EmitSmem*>(smraw);
     const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint64_t nbytes = desc->nbytes;
     const uint64_t n_tiles = (nbytes + kSelTile - 1) / kSelTile;
     const uint64_t n_groups = (n_tiles + kGroup - 1) / kGroup;
-    const uint64_t* items = cache_items(sm, desc);
+    const uint64_t* items = cache_items(sm.items, desc);
     const uint32_t n_items = desc->n_items;
     __syncthreads();
     for (uint64_t g = blockIdx.x; g < n_groups; g += gridDim.x) {
         const uint64_t t = g * kGroup + wid;
         sm.fun[wid][lane] = t < n_tiles ? agg[32 * t + lane] : ((uint32_t)lane << 27);
+        if (t < n_tiles) {
+#pragma unroll
+            for (int j = 0; j < 8; ++j) sm.w[wid].cand[lane * 8 + j] = bitmap[t * kSelTileWords + lane * 8 + j];
+        }
         __syncthreads();
         if (threadIdx.x == 0) {
             uint32_t s = gentry[2 * g], c = gentry[2 * g + 1];
@@ -412,7 +425,7 @@ select_emit_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restric
         }
         __syncthreads();
         if (t < n_tiles) {
-            build_tile(sm.w[wid], t, bitmap, nbytes, items, n_items, lane);
+            apply_items(sm.w[wid], t * kSelTile, nbytes, items, n_items, lane);
             const uint32_t st = sm.te_state[wid];
             if (lane == (int)st) {
                 uint32_t ex;
@@ -463,44 +476,38 @@ __global__ void chunk_meta_kernel(const BatchDesc* __restrict__ desc,
 
 }  // namespace
 
-void launch_rabin_scan(const BatchDesc* d, const uint32_t* d_tab, uint32_t mask, uint32_t value,
-                       uint32_t* bitmap, int num_sms, cudaStream_t s) {
-    static bool attr_set = false;
-    if (!attr_set) {
-        cudaFuncSetAttribute(rabin_scan_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             kTabBytes);
-        cudaFuncSetAttribute(rabin_scan_kernel<false>,
-                             cudaFuncAttributeMaxDynamicSharedMemorySize, kTabBytes);
-        attr_set = true;
-    }
-    const unsigned grid = (unsigned)(num_sms * 2);
-    if (value == 0)
-        rabin_scan_kernel<true><<<grid, kScanThreads, kTabBytes, s>>>(d, d_tab, mask, value, bitmap);
-    else
-        rabin_scan_kernel<false><<<grid, kScanThreads, kTabBytes, s>>>(d, d_tab, mask, value,
-                                                                       bitmap);
-}
-
 uint64_t select_groups(uint64_t max_tiles) { return (max_tiles + kGroup - 1) / kGroup; }
 
-void launch_select(const BatchDesc* d, const uint32_t* bitmap, uint32_t* agg, uint32_t* gagg,
-                   uint32_t* gentry, uint64_t max_tiles, uint32_t* cut_pos, uint64_t cap,
-                   uint32_t* n_chunks, int num_sms, cudaStream_t s) {
+void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mask,
+                         uint32_t value, uint32_t* bitmap, uint32_t* agg, uint32_t* gagg,
+                         uint32_t* gentry, uint32_t* scan_ctr, uint64_t max_tiles,
+                         uint32_t* cut_pos, uint64_t cap, uint32_t* n_chunks, int num_sms,
+                         cudaStream_t s, cudaEvent_t after_scan) {
     static bool attr_set = false;
     if (!attr_set) {
-        cudaFuncSetAttribute(select_agg_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)sizeof(SelSmem));
+        cudaFuncSetAttribute(rabin_scan_agg_kernel<true>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
+        cudaFuncSetAttribute(rabin_scan_agg_kernel<false>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
         cudaFuncSetAttribute(select_emit_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)sizeof(SelSmem));
+                             (int)sizeof(EmitSmem));
         attr_set = true;
     }
-    uint64_t blocks = select_groups(max_tiles);
-    const uint64_t max_blocks = (uint64_t)num_sms * 2;
-    if (blocks > max_blocks) blocks = max_blocks;
-    if (blocks < 1) blocks = 1;
-    select_agg_kernel<<<(unsigned)blocks, 1024, sizeof(SelSmem), s>>>(d, bitmap, agg, gagg);
+    const uint64_t groups = select_groups(max_tiles);
+    cudaMemsetAsync(scan_ctr, 0, sizeof(uint32_t) * (groups + 2), s);
+    const unsigned grid = (unsigned)num_sms;
+    if (value == 0)
+        rabin_scan_agg_kernel<true><<<grid, kScanThreads, kScanSmem, s>>>(
+            d, d_tab, mask, value, bitmap, agg, gagg, scan_ctr);
+    else
+        rabin_scan_agg_kernel<false><<<grid, kScanThreads, kScanSmem, s>>>(
+            d, d_tab, mask, value, bitmap, agg, gagg, scan_ctr);
+    if (after_scan) cudaEventRecordWithFlags(after_scan, s, cudaEventRecordExternal);
     select_scan_kernel<<<1, 1024, 0, s>>>(d, gagg, gentry, n_chunks);
-    select_emit_kernel<<<(unsigned)blocks, 1024, sizeof(SelSmem), s>>>(d, bitmap, agg, gentry,
+    uint64_t blocks = groups;
+    if (blocks > (uint64_t)num_sms * 2) blocks = (uint64_t)num_sms * 2;
+    if (blocks < 1) blocks = 1;
+    select_emit_kernel<<<(unsigned)blocks, 1024, sizeof(EmitSmem), s>>>(d, bitmap, agg, gentry,
                                                                        cut_pos, cap);
 }
 
