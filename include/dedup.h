@@ -167,7 +167,12 @@ typedef struct {
      * input, Rabin scan kernel, cut selection + chunk metadata, SHA-1 kernel,
      * table insert + lookup, pack of results into pinned host memory */
     double ms_h2d, ms_scan, ms_select, ms_sha1, ms_table, ms_d2h;
+    double ms_host_launch, ms_host_parse; /* host time in cudaGraphLaunch / result parsing */
     uint64_t sha1_blocks; /* 64-byte SHA-1 compressions over drained batches */
+    /* the ms_* stage times cover only the sampled batches (every
+     * DEDUP_TIME_EVERY-th drained batch, default 1; none if
+     * DEDUP_STAGE_EVENTS=0): their count, bytes and SHA-1 blocks */
+    uint64_t timed_batches, timed_bytes, timed_sha1_blocks;
 } dedup_stats_t;
 
 /* Counters over all drained batches of the ctx (all streams). */

@@ -64,7 +64,9 @@ class Stats(ctypes.Structure):
         "batches", "table_used", "table_slots", "kernel_launches")] + [
         ("num_owners", ctypes.c_uint32), ("owner_rank", ctypes.c_uint32)] + [
         (n, ctypes.c_double) for n in ("ms_h2d", "ms_scan", "ms_select", "ms_sha1", "ms_table",
-                                       "ms_d2h")] + [("sha1_blocks", ctypes.c_uint64)]
+                                       "ms_d2h", "ms_host_launch", "ms_host_parse")] + [
+        ("sha1_blocks", ctypes.c_uint64), ("timed_batches", ctypes.c_uint64),
+        ("timed_bytes", ctypes.c_uint64), ("timed_sha1_blocks", ctypes.c_uint64)]
 
 
 class Record(ctypes.Structure):
@@ -94,7 +96,7 @@ def lib():
         "dedup_destroy": (None, [vp]),
         "dedup_last_error": (ctypes.c_char_p, [vp]),
         "dedup_submit_batch": (st, [vp, u32, P(vp), P(u64), P(u64)]),
-        "dedup_submit_device": (st, [vp, vp, u64, P(u64), u32, vp, P(u64)]),
+        "dedup_submit_device": (st, [vp, vp, u64, vp, u32, vp, P(u64)]),
         "dedup_join": (st, [vp, vp]),
         "dedup_end_stream": (st, [vp]),
         "dedup_drain": (st, [vp, u32, i32, P(ItemResult), P(u32)]),

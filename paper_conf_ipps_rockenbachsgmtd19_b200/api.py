@@ -93,6 +93,7 @@ class Dedup:
         self._borrowed = collections.deque()  # (last_seq_exclusive, objects)
         self._next_out = 0
         self._pinned = []
+        self._seq = _u64()
 
     # -- lifetime --------------------------------------------------------
     @property
@@ -157,12 +158,15 @@ class Dedup:
         """Submit ONE GPU batch already resident in device memory: ``data`` is
         a CUDA uint8 tensor (or device pointer int + nbytes via item_off[-1]);
         the batch waits for ``producer`` (default: torch's current stream)."""
-        off = np.ascontiguousarray(item_off, np.uint64)
+        off = item_off
+        if not (isinstance(off, np.ndarray) and off.dtype == np.uint64
+                and off.flags.c_contiguous):
+            off = np.ascontiguousarray(off, np.uint64)
         n = len(off) - 1
-        seq = _u64()
+        seq = self._seq
         self._check(N.lib().dedup_submit_device(
-            self._ctx, _ptr(data), int(off[-1]), off.ctypes.data_as(ctypes.POINTER(_u64)), n,
-            _stream(producer), ctypes.byref(seq)))
+            self._ctx, _ptr(data), int(off[-1]), off.ctypes.data, n, _stream(producer),
+            ctypes.byref(seq)))
         self._borrowed.append((seq.value + n, data))
         return seq.value
 

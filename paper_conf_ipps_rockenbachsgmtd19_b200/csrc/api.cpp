@@ -120,6 +120,9 @@ struct dedup_ctx {
     uint32_t graph_kernels = 0;  // kernels per batch graph
     dedup_stats_t st{};
     bool trace = false;           // DEDUP_TRACE environment variable
+    bool stage_events = true;     // per-stage timing events in the batch graphs
+    uint32_t time_every = 1;      // query stage times of every n-th batch (DEDUP_TIME_EVERY)
+    uint64_t parsed_batches = 0;
     cudaEvent_t ev_ref = nullptr;  // time origin of the trace
 };
 
@@ -242,16 +245,19 @@ dedup_status build_graph(dedup_ctx* c, int i) {
     Slot& prev = c->slots[(i + c->slots.size() - 1) % c->slots.size()];
     const uint64_t cap = c->chunk_cap;
     cudaStream_t s = sl.stream;
+    const bool se = c->stage_events;  // per-stage timing events (DEDUP_STAGE_EVENTS=0: off)
     CU(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
-    cudaEventRecordWithFlags(sl.ev_start, s, cudaEventRecordExternal);
+    if (se) cudaEventRecordWithFlags(sl.ev_start, s, cudaEventRecordExternal);
     cudaMemcpyAsync(sl.d_desc, sl.h_desc, sizeof(BatchDesc), cudaMemcpyHostToDevice, s);
     cudaMemcpyAsync(sl.d_item_off, sl.h_item_off, sizeof(uint64_t) * (c->cfg.batch_items + 1),
                     cudaMemcpyHostToDevice, s);
-    cudaEventRecordWithFlags(sl.ev_h2d, s, cudaEventRecordExternal);
+    cudaMemsetAsync(sl.d_small, 0, sizeof(uint32_t) * 16, s);  // counts + batch statistics
+    if (se) cudaEventRecordWithFlags(sl.ev_h2d, s, cudaEventRecordExternal);
     enqueue_chunk_sha(c, sl.ws, s, sl.d_desc, c->cfg.batch_bytes, sl.d_cut_pos, cap,
-                      sl.d_small, sl.d_digest, sl.ev_scan, sl.ev_chunk, sl.d_chunk_start,
-                      sl.d_chunk_id, sl.d_item_first, c->cfg.batch_items);
-    cudaEventRecordWithFlags(sl.ev_sha, s, cudaEventRecordExternal);
+                      sl.d_small, sl.d_digest, se ? sl.ev_scan : nullptr,
+                      se ? sl.ev_chunk : nullptr, sl.d_chunk_start, sl.d_chunk_id,
+                      sl.d_item_first, c->cfg.batch_items);
+    if (se) cudaEventRecordWithFlags(sl.ev_sha, s, cudaEventRecordExternal);
     // table work waits for the previous batch's table work (global chain)
     cudaStreamWaitEvent(s, prev.ev_table, cudaEventWaitExternal);
     launch_table_prepare(sl.d_desc, c->tables[0].capacity, c->num_sms, s);
@@ -259,7 +265,8 @@ dedup_status build_graph(dedup_ctx* c, int i) {
     launch_table_insert(tv, sl.d_digest, sl.d_chunk_id, nullptr, sl.d_small, 0, cap,
                         sl.ws.slot_idx, c->num_sms, s);
     launch_table_lookup(tv, sl.d_chunk_id, nullptr, sl.d_small, 0, cap, sl.ws.slot_idx,
-                        sl.d_first_id, sl.d_is_dup, sl.d_small + 4, c->num_sms, s);
+                        sl.d_first_id, sl.d_is_dup, sl.d_small + 4, sl.d_cut_pos, sl.d_desc,
+                        c->num_sms, s);
     cudaEventRecordWithFlags(sl.ev_table, s, cudaEventRecordExternal);
     launch_pack(sl.d_desc, sl.d_small, cap, c->cfg.batch_items, sl.d_chunk_start, sl.d_first_id,
                 sl.d_digest, sl.d_is_dup, sl.d_item_first, sl.d_small + 4, sl.hdev, c->num_sms,
@@ -371,7 +378,10 @@ dedup_status launch_batch(dedup_ctx* c, int i, const uint8_t* d_bytes) {
     d.fresh = c->stream_fresh ? 1u : 0u;
     d.table = table_view(c);
     c->stream_fresh = false;
+    const auto t0 = std::chrono::steady_clock::now();
     CU(cudaGraphLaunch(sl.graph, sl.stream));
+    c->st.ms_host_launch +=
+        std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     c->launches += c->graph_kernels;
     sl.busy = true;
     sl.parsed = false;
@@ -398,6 +408,7 @@ dedup_status check_cfg(const dedup_config* g) {
 
 // Turn a completed slot's host results into per-item views + stats.
 dedup_status parse_slot(dedup_ctx* c, Slot& sl) {
+    const auto t_parse = std::chrono::steady_clock::now();
     const uint32_t n = sl.hhost.header[0];
     if (sl.hhost.header[1] != 0)
         return fail(c, DEDUP_ETABLEFULL, "digest table overflow: raise table_capacity");
@@ -416,20 +427,9 @@ dedup_status parse_slot(dedup_ctx* c, Slot& sl) {
             next = f;
         }
     }
-    uint64_t dups = 0, dup_bytes = 0, blocks = 0;
-    for (uint32_t k = 0; k < sl.n_items; ++k) {
-        const uint32_t f = sl.item_first[k], m = sl.item_n[k];
-        for (uint32_t j = 0; j < m; ++j) {
-            const uint64_t s0 = sl.hhost.chunk_start[f + j];
-            const uint64_t s1 = j + 1 < m ? sl.hhost.chunk_start[f + j + 1] : sl.item_len[k];
-            blocks += (s1 - s0 + 9 + 63) / 64;
-            if (sl.hhost.is_dup[f + j]) {
-                ++dups;
-                dup_bytes += s1 - s0;
-            }
-        }
-    }
-    c->st.sha1_blocks += blocks;
+    // batch statistics reduced on the device by the lookup kernel
+    const uint64_t dups = sl.hhost.header[3], dup_bytes = sl.hhost.header[4];
+    c->st.sha1_blocks += sl.hhost.header[5];
     c->st.chunks += n;
     c->st.dup_chunks += dups;
     c->st.unique_chunks += n - dups;
@@ -437,15 +437,24 @@ dedup_status parse_slot(dedup_ctx* c, Slot& sl) {
     c->st.items += sl.n_items;
     c->st.bytes += sl.nbytes;
     c->st.table_used = sl.hhost.header[2];
-    float ms = 0;
-    if (sl.host_fed && cudaEventElapsedTime(&ms, sl.ev_host, sl.ev_start) == cudaSuccess)
-        c->st.ms_h2d += ms;
-    if (cudaEventElapsedTime(&ms, sl.ev_h2d, sl.ev_scan) == cudaSuccess) c->st.ms_scan += ms;
-    if (cudaEventElapsedTime(&ms, sl.ev_scan, sl.ev_chunk) == cudaSuccess) c->st.ms_select += ms;
-    if (cudaEventElapsedTime(&ms, sl.ev_chunk, sl.ev_sha) == cudaSuccess) c->st.ms_sha1 += ms;
-    if (cudaEventElapsedTime(&ms, sl.ev_sha, sl.ev_table) == cudaSuccess) c->st.ms_table += ms;
-    if (cudaEventElapsedTime(&ms, sl.ev_table, sl.ev_done) == cudaSuccess) c->st.ms_d2h += ms;
-    if (c->trace) {  // DEDUP_TRACE=1: per-batch event timeline (ms since ctx init)
+    // CUDA-event stage times of every time_every-th batch (event queries cost
+    // host time, so they are sampled; timed_batches counts the samples)
+    if (c->stage_events && c->parsed_batches++ % c->time_every == 0) {
+        float ms = 0;
+        c->st.timed_batches += 1;
+        c->st.timed_bytes += sl.nbytes;
+        if (sl.host_fed && cudaEventElapsedTime(&ms, sl.ev_host, sl.ev_start) == cudaSuccess)
+            c->st.ms_h2d += ms;
+        if (cudaEventElapsedTime(&ms, sl.ev_h2d, sl.ev_scan) == cudaSuccess) c->st.ms_scan += ms;
+        if (cudaEventElapsedTime(&ms, sl.ev_scan, sl.ev_chunk) == cudaSuccess)
+            c->st.ms_select += ms;
+        if (cudaEventElapsedTime(&ms, sl.ev_chunk, sl.ev_sha) == cudaSuccess) c->st.ms_sha1 += ms;
+        if (cudaEventElapsedTime(&ms, sl.ev_sha, sl.ev_table) == cudaSuccess)
+            c->st.ms_table += ms;
+        if (cudaEventElapsedTime(&ms, sl.ev_table, sl.ev_done) == cudaSuccess) c->st.ms_d2h += ms;
+        c->st.timed_sha1_blocks += sl.hhost.header[5];
+    }
+    if (c->trace && c->stage_events) {  // DEDUP_TRACE=1: per-batch event timeline (ms)
         float t[7] = {0, 0, 0, 0, 0, 0, 0};
         const cudaEvent_t ev[7] = {sl.ev_start, sl.ev_h2d, sl.ev_scan, sl.ev_chunk,
                                    sl.ev_sha, sl.ev_table, sl.ev_done};
@@ -458,6 +467,9 @@ dedup_status parse_slot(dedup_ctx* c, Slot& sl) {
     }
     cudaGetLastError();  // clear a possible error from a timing query
     sl.parsed = true;
+    c->st.ms_host_parse +=
+        std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_parse)
+            .count();
     return DEDUP_OK;
 }
 
@@ -536,6 +548,9 @@ dedup_status dedup_init(const dedup_config* cfg, dedup_ctx** out) {
     for (cudaEvent_t& e : c->op_ev)
         if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
             return bail(DEDUP_ECUDA);
+    if (const char* v = std::getenv("DEDUP_STAGE_EVENTS")) c->stage_events = std::atoi(v) != 0;
+    if (const char* v = std::getenv("DEDUP_TIME_EVERY"))
+        c->time_every = std::atoi(v) > 0 ? (uint32_t)std::atoi(v) : 1u;
     c->slots.resize(cfg->slots);
     for (Slot& sl : c->slots)
         if ((s = slot_alloc(c, sl)) != DEDUP_OK) return bail(s);
@@ -862,7 +877,7 @@ dedup_status dedup_op_table_insert_lookup(dedup_ctx* c, void* stream, const uint
     launch_table_insert(&d->table, d_digest, d_id, nullptr, d_n, 0, cap, c->op_ws.slot_idx,
                         c->num_sms, s);
     launch_table_lookup(&d->table, d_id, nullptr, d_n, 0, cap, c->op_ws.slot_idx, d_first_id,
-                        d_is_dup, nullptr, c->num_sms, s);
+                        d_is_dup, nullptr, nullptr, nullptr, c->num_sms, s);
     c->launches += cap ? 2 : 1;
     CU(cudaGetLastError());
     return DEDUP_OK;
@@ -924,7 +939,8 @@ dedup_status dedup_op_owner(dedup_ctx* c, void* stream, const dedup_record* d_re
         launch_table_insert(&d->table, nullptr, nullptr, d_recv, nullptr, n_recv, n_recv,
                             c->op_ws.slot_idx, c->num_sms, s);
         launch_table_lookup(&d->table, nullptr, d_recv, nullptr, n_recv, n_recv,
-                            c->op_ws.slot_idx, d_reply, nullptr, nullptr, c->num_sms, s);
+                            c->op_ws.slot_idx, d_reply, nullptr, nullptr, nullptr, nullptr,
+                            c->num_sms, s);
         c->launches += 2;
     }
     CU(cudaGetLastError());

@@ -76,7 +76,8 @@ void launch_table_insert(const TableView* tv, const uint8_t* digest, const uint6
 void launch_table_lookup(const TableView* tv, const uint64_t* id, const void* rec,
                          const uint32_t* d_n, uint64_t n_host, uint64_t cap,
                          const uint32_t* slot_idx, uint64_t* first_id, uint8_t* is_dup,
-                         uint32_t* status_out, int num_sms, cudaStream_t s);
+                         uint32_t* status_out, const uint32_t* cut_pos,
+                         const BatchDesc* desc, int num_sms, cudaStream_t s);
 
 void launch_route(const uint8_t* digest, const uint64_t* id, const uint32_t* d_n, uint64_t cap,
                   uint32_t num_owners, void* send, uint32_t* send_off, uint32_t* send_pos,

@@ -113,11 +113,17 @@ __global__ void table_lookup_kernel(const TableView* __restrict__ tv,
                                     const void* rec, const uint32_t* d_n, uint64_t n_host,
                                     uint64_t cap, const uint32_t* __restrict__ slot_idx,
                                     uint64_t* __restrict__ first_id, uint8_t* __restrict__ is_dup,
-                                    uint32_t* __restrict__ status_out) {
+                                    uint32_t* __restrict__ status_out,
+                                    const uint32_t* __restrict__ cut_pos,
+                                    const BatchDesc* __restrict__ desc) {
     const TableView t = *tv;
     const uint64_t n = record_count(d_n, n_host, cap);
     if (status_out != nullptr && blockIdx.x == 0 && threadIdx.x < 2)
         status_out[threadIdx.x] = t.status[threadIdx.x];  // overflow flag, used slots
+    // batch statistics (status_out[2..4], zeroed by the caller): duplicate
+    // chunks, duplicate bytes, 64-byte SHA-1 blocks
+    uint32_t s_dup = 0, s_dup_bytes = 0, s_blocks = 0;
+    const uint64_t nbytes = cut_pos != nullptr ? desc->nbytes : 0;
     for (uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; r < n;
          r += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t si = slot_idx[r];
@@ -128,7 +134,27 @@ __global__ void table_lookup_kernel(const TableView* __restrict__ tv,
                                 ? *reinterpret_cast<const uint64_t*>(
                                       static_cast<const uint8_t*>(rec) + 32 * r + 24)
                                 : id[r];
-            is_dup[r] = (f != myid) ? 1 : 0;
+            const bool dup = f != myid;
+            is_dup[r] = dup ? 1 : 0;
+            if (cut_pos != nullptr) {
+                const uint64_t e = r + 1 < n ? (uint64_t)cut_pos[r + 1] : nbytes;
+                const uint32_t len = (uint32_t)(e - cut_pos[r]);
+                s_blocks += (len + 9 + 63) / 64;
+                if (dup) {
+                    ++s_dup;
+                    s_dup_bytes += len;
+                }
+            }
+        }
+    }
+    if (cut_pos != nullptr) {
+        s_dup = __reduce_add_sync(0xFFFFFFFFu, s_dup);
+        s_dup_bytes = __reduce_add_sync(0xFFFFFFFFu, s_dup_bytes);
+        s_blocks = __reduce_add_sync(0xFFFFFFFFu, s_blocks);
+        if ((threadIdx.x & 31) == 0 && (s_dup | s_dup_bytes | s_blocks)) {
+            atomicAdd(&status_out[2], s_dup);
+            atomicAdd(&status_out[3], s_dup_bytes);
+            atomicAdd(&status_out[4], s_blocks);
         }
     }
 }
@@ -213,6 +239,9 @@ __global__ void pack_kernel(const BatchDesc* __restrict__ desc,
         h.header[0] = (uint32_t)*n_chunks_p;
         h.header[1] = table_status[0];  // overflow flag (copied by the lookup)
         h.header[2] = table_status[1];  // used table slots
+        h.header[3] = table_status[2];  // duplicate chunks
+        h.header[4] = table_status[3];  // duplicate bytes
+        h.header[5] = table_status[4];  // SHA-1 blocks
     }
     for (uint64_t r = tid; r < n; r += stride) {
         h.chunk_start[r] = chunk_start[r];
@@ -236,7 +265,9 @@ unsigned grid_for(uint64_t n, int threads, int num_sms, int per_sm) {
 }  // namespace
 
 void launch_table_prepare(const BatchDesc* d, uint64_t max_slots, int num_sms, cudaStream_t s) {
-    table_prepare_kernel<<<grid_for(2 * max_slots, 256, num_sms, 4), 256, 0, s>>>(d);
+    // small grids (grid-stride loops) so that the kernels of other in-flight
+    // batches keep their SMs
+    table_prepare_kernel<<<grid_for(2 * max_slots, 256, 32, 1), 256, 0, s>>>(d);
 }
 
 void launch_table_insert(const TableView* t, const uint8_t* digest, const uint64_t* id,
@@ -244,17 +275,18 @@ void launch_table_insert(const TableView* t, const uint8_t* digest, const uint64
                          uint32_t* slot_idx, int num_sms, cudaStream_t s) {
     const uint64_t n = d_n != nullptr ? cap : n_host;
     if (n == 0) return;
-    table_insert_kernel<<<grid_for(n, 256, num_sms, 8), 256, 0, s>>>(t, digest, id, rec, d_n,
+    table_insert_kernel<<<grid_for(n, 256, num_sms, 1), 256, 0, s>>>(t, digest, id, rec, d_n,
                                                                        n_host, cap, slot_idx);
 }
 
 void launch_table_lookup(const TableView* t, const uint64_t* id, const void* rec,
                          const uint32_t* d_n, uint64_t n_host, uint64_t cap,
                          const uint32_t* slot_idx, uint64_t* first_id, uint8_t* is_dup,
-                         uint32_t* status_out, int num_sms, cudaStream_t s) {
+                         uint32_t* status_out, const uint32_t* cut_pos,
+                         const BatchDesc* desc, int num_sms, cudaStream_t s) {
     const uint64_t n = d_n != nullptr ? cap : n_host;
-    table_lookup_kernel<<<grid_for(n, 256, num_sms, 8), 256, 0, s>>>(
-        t, id, rec, d_n, n_host, cap, slot_idx, first_id, is_dup, status_out);
+    table_lookup_kernel<<<grid_for(n, 256, num_sms, 1), 256, 0, s>>>(
+        t, id, rec, d_n, n_host, cap, slot_idx, first_id, is_dup, status_out, cut_pos, desc);
 }
 
 void launch_route(const uint8_t* digest, const uint64_t* id, const uint32_t* d_n, uint64_t cap,
@@ -282,7 +314,7 @@ void launch_pack(const BatchDesc* d, const uint32_t* n_chunks, uint64_t cap, uin
                  const uint8_t* is_dup, const uint32_t* item_first_chunk,
                  const uint32_t* table_status, HostResultLayout h, int num_sms,
                  cudaStream_t s) {
-    pack_kernel<<<grid_for(cap / 4 + max_items + 1, 256, num_sms, 2), 256, 0, s>>>(
+    pack_kernel<<<grid_for(cap / 4 + max_items + 1, 256, 64, 1), 256, 0, s>>>(
         d, n_chunks, cap, chunk_start, first_id, digest, is_dup, item_first_chunk, table_status,
         h);
 }

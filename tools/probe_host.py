@@ -14,7 +14,7 @@ from paper_conf_ipps_rockenbachsgmtd19_b200 import _native as N  # noqa: E402
 MiB = 1 << 20
 x = torch.zeros(32 * MiB, dtype=torch.uint8, device="cuda")
 off = (np.arange(33, dtype=np.uint64) * MiB)
-d = Dedup(0, batch_bytes=32 * MiB, batch_items=64, slots=8, table_capacity=1 << 17)
+d = Dedup(0, batch_bytes=32 * MiB, batch_items=64, slots=40, table_capacity=1 << 17)
 L = N.lib()
 torch.cuda.synchronize()
 # python wrapper
@@ -30,7 +30,10 @@ seq = ctypes.c_uint64()
 ptr = x.data_ptr()
 t2 = time.perf_counter()
 for i in range(32):
-    L.dedup_submit_device(d.ctx, ptr, 32 * MiB, offp, 32, st, ctypes.byref(seq))
+    L.dedup_submit_device(d.ctx, ptr, 32 * MiB, off.ctypes.data, 32, st, ctypes.byref(seq))
 t3 = time.perf_counter()
 d.drain_all()
 print(f"python submit {1e6 * (t1 - t0) / 32:.1f} us, raw C submit {1e6 * (t3 - t2) / 32:.1f} us")
+s = d.stats()
+print(f"per batch: host graph launch {1e3 * s['ms_host_launch'] / s['batches']:.1f} us, "
+      f"host parse {1e3 * s['ms_host_parse'] / s['batches']:.1f} us over {s['batches']} batches")
