@@ -1,0 +1,239 @@
+"""Multi-GPU orchestration of the dedup hot path (rows A5-A8).
+
+Batches (whole items) are processed in WAVES: in wave w every rank r runs
+its own batch through the device ops of include/dedup.h, then the digests are
+routed to their owner GPU, owner(d) = floor(BE32(d[0..3]) * G / 2^32)
+(row A5, kernel ``dedup_op_route``), exchanged with an all-to-all (row A6),
+inserted + looked up in the owner's table shard (row A7, ``dedup_op_owner``),
+and the first-occurrence ids are sent back and scattered to chunk order
+(row A8, ``dedup_op_scatter``).  Owners insert every record of a wave before
+looking any of them up, and waves are processed in order, so the result is
+the sequential stream-order answer (reading O12) whatever the GPU
+count.  The paper itself has no inter-GPU step (GPUs take batches
+round-robin); the exchange is needed because the
+duplicate check is global (reading O11).
+
+The per-rank work is split in three phases so that the same code runs
+  * with ``TorchDistExchange``: one process per GPU, torch.distributed
+    all_to_all_single (NCCL over NVLink on B200, gloo in the CPU tests), and
+  * with ``LoopbackExchange``: G logical ranks on ONE GPU in one process (the
+    GPU parity test of the routing).
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+import numpy as np
+
+REC_WORDS = 4  # a dedup_record is 32 bytes = 4 int64 words
+
+
+@dataclass
+class WaveOut:
+    """Per-rank output of one wave (host numpy arrays, chunk order)."""
+    first_seq: int
+    item_len: np.ndarray      # u64 [n_items]
+    item_first: np.ndarray    # u32 [n_items] (0xFFFFFFFF = empty item)
+    chunk_start: np.ndarray   # u32 [n]
+    digest: np.ndarray        # u8 [n, 20]
+    first_id: np.ndarray      # u64 [n]
+    is_dup: np.ndarray        # u8 [n]
+
+    def items(self):
+        """Per-item (seq, chunk_start, digest, is_dup, first_id) tuples."""
+        n = len(self.chunk_start)
+        nxt = n
+        bounds = [None] * len(self.item_len)
+        for k in range(len(self.item_len) - 1, -1, -1):
+            f = int(self.item_first[k])
+            if f == 0xFFFFFFFF:
+                bounds[k] = (nxt, nxt)
+            else:
+                bounds[k] = (f, nxt)
+                nxt = f
+        for k, (a, b) in enumerate(bounds):
+            yield (self.first_seq + k, self.chunk_start[a:b], self.digest[a:b],
+                   self.is_dup[a:b], self.first_id[a:b])
+
+
+class TorchDistExchange:
+    """All-to-all of variable-size segments with torch.distributed.
+
+    ``send`` is a 2-D tensor [n, w] whose rows are grouped by destination
+    rank (``counts[r]`` rows for rank r); returns the received rows grouped
+    by source rank and the per-source counts.  Counts are exchanged first
+    (one small all-to-all), then the payload.
+    """
+
+    def __init__(self, group=None):
+        import torch.distributed as dist
+        self.dist = dist
+        self.group = group
+        self.rank = dist.get_rank(group)
+        self.world = dist.get_world_size(group)
+
+    def counts(self, send_counts):
+        import torch
+        sc = torch.as_tensor(send_counts, dtype=torch.int64)
+        dev = self._device()
+        sc = sc.to(dev)
+        rc = torch.empty_like(sc)
+        self.dist.all_to_all_single(rc, sc, group=self.group)
+        return rc.cpu().tolist()
+
+    def payload(self, send, send_counts, recv_counts):
+        import torch
+        recv = torch.empty((int(sum(recv_counts)),) + tuple(send.shape[1:]), dtype=send.dtype,
+                           device=send.device)
+        self.dist.all_to_all_single(recv, send.contiguous(),
+                                    output_split_sizes=[int(x) for x in recv_counts],
+                                    input_split_sizes=[int(x) for x in send_counts],
+                                    group=self.group)
+        return recv
+
+    def _device(self):
+        import torch
+        backend = self.dist.get_backend(self.group)
+        return torch.device("cuda", torch.cuda.current_device()) if backend == "nccl" else \
+            torch.device("cpu")
+
+
+def loopback_all_to_all(sends, counts):
+    """In-process all-to-all for G logical ranks: sends[s] rows grouped by
+    destination with counts[s][d] rows each; returns (recvs, recv_counts)."""
+    import torch
+    G = len(sends)
+    offs = [np.concatenate([[0], np.cumsum(c)]).astype(np.int64) for c in counts]
+    recvs, rcounts = [], []
+    for d in range(G):
+        parts = [sends[s][int(offs[s][d]):int(offs[s][d + 1])] for s in range(G)]
+        recvs.append(torch.cat(parts, 0) if parts else sends[d][:0])
+        rcounts.append([int(counts[s][d]) for s in range(G)])
+    return recvs, rcounts
+
+
+class RankState:
+    """Device buffers + ctx of one rank (owner of one table shard)."""
+
+    def __init__(self, dedup, batch_bytes: int, batch_items: int, device, num_owners: int):
+        import torch
+        self.d = dedup
+        self.G = num_owners
+        self.dev = device
+        cap = batch_bytes // 32 + batch_items + 2
+        self.cap = cap
+        i32 = dict(dtype=torch.int32, device=device)
+        i64 = dict(dtype=torch.int64, device=device)
+        self.cut = torch.zeros(cap, **i32)
+        self.n = torch.zeros(1, **i32)
+        self.chunk_start = torch.zeros(cap, **i32)
+        self.chunk_id = torch.zeros(cap, **i64)
+        self.item_first = torch.zeros(batch_items + 1, **i32)
+        self.digest = torch.zeros(cap * 20, dtype=torch.uint8, device=device)
+        self.send = torch.zeros((cap, REC_WORDS), **i64)
+        self.send_off = torch.zeros(self.G + 1, **i32)
+        self.send_pos = torch.zeros(cap, **i32)
+        self.first_id = torch.zeros(cap, **i64)
+        self.is_dup = torch.zeros(cap, dtype=torch.uint8, device=device)
+        self.item_off_dev = torch.zeros(batch_items + 1, **i64)
+
+    # phase 1: rows A2-A5 on this rank's batch
+    def local(self, data, item_off: np.ndarray, first_seq: int):
+        import torch
+        self.first_seq = first_seq
+        self.item_off = np.asarray(item_off, np.uint64)
+        n_items = len(self.item_off) - 1
+        nbytes = int(self.item_off[-1])
+        self.item_off_dev[:n_items + 1].copy_(torch.from_numpy(self.item_off.view(np.int64)))
+        d = self.d
+        d.op_chunk(data, nbytes, self.item_off_dev, n_items, self.cut, self.cap, self.n)
+        d.op_chunk_meta(self.item_off_dev, n_items, self.cut, self.n, self.cap, first_seq,
+                        self.chunk_start, self.chunk_id, self.item_first)
+        d.op_sha1(data, nbytes, self.cut, self.n, self.cap, self.digest)
+        d.op_route(self.digest, self.chunk_id, self.n, self.cap, self.G, self.send,
+                   self.send_off, self.send_pos)
+        off = self.send_off.cpu().numpy().astype(np.int64)   # host sync (counts)
+        self.n_host = int(off[-1])
+        self.send_counts = np.diff(off).tolist()
+        return self.send[:self.n_host], self.send_counts
+
+    # phase 2: row A7 on the records this rank owns
+    def owner(self, recv):
+        import torch
+        reply = torch.zeros(len(recv), dtype=torch.int64, device=self.dev)
+        if len(recv):
+            self.d.op_owner(recv, len(recv), reply)
+        return reply
+
+    # phase 3: row A8 + read-back of this rank's results
+    def finish(self, reply_back) -> WaveOut:
+        n = self.n_host
+        if n:
+            self.d.op_scatter(reply_back, self.send_pos, self.chunk_id, self.n, self.cap,
+                              self.first_id, self.is_dup)
+        n_items = len(self.item_off) - 1
+        return WaveOut(
+            first_seq=self.first_seq,
+            item_len=np.diff(self.item_off),
+            item_first=self.item_first[:n_items].cpu().numpy().view(np.uint32).copy(),
+            chunk_start=self.chunk_start[:n].cpu().numpy().view(np.uint32).copy(),
+            digest=self.digest[:20 * n].cpu().numpy().reshape(n, 20).copy(),
+            first_id=self.first_id[:n].cpu().numpy().view(np.uint64).copy(),
+            is_dup=self.is_dup[:n].cpu().numpy().copy())
+
+
+def run_wave(x, state, data, item_off, first_seq: int) -> WaveOut:
+    """One wave on one rank: local rows A2-A5, record all-to-all (A6), owner
+    insert + lookup (A7), reply all-to-all and scatter (A8).  Every rank of
+    the group must call it for the same wave."""
+    send, send_counts = state.local(data, item_off, first_seq)
+    recv_counts = x.counts(send_counts)
+    recv = x.payload(send, send_counts, recv_counts)
+    reply = state.owner(recv)
+    reply_back = x.payload(reply, recv_counts, send_counts)
+    return state.finish(reply_back)
+
+
+class DistDedup:
+    """One rank of the multi-GPU dedup (one process per GPU)."""
+
+    def __init__(self, exchange: TorchDistExchange, device_index: int, batch_bytes: int,
+                 batch_items: int, table_capacity: int, **cfg):
+        import torch
+
+        from .api import Dedup
+        self.x = exchange
+        self.G = exchange.world
+        self.dedup = Dedup(device_index, batch_bytes=batch_bytes, batch_items=batch_items,
+                           slots=1, table_capacity=table_capacity, host_fed=False,
+                           owner_rank=exchange.rank, num_owners=self.G, **cfg)
+        self.state = RankState(self.dedup, batch_bytes, batch_items,
+                               torch.device("cuda", device_index), self.G)
+
+    def wave(self, data, item_off, first_seq: int) -> WaveOut:
+        return run_wave(self.x, self.state, data, item_off, first_seq)
+
+    def end_stream(self):
+        self.dedup.op_table_reset()
+
+    def close(self):
+        self.dedup.close()
+
+
+def loopback_waves(states, batches):
+    """Run one wave on G logical ranks sharing one GPU.
+
+    states: list of RankState (rank r owns shard r); batches: list of
+    (data_tensor, item_off, first_seq) per rank.  Returns a WaveOut per rank.
+    """
+    sends, counts = [], []
+    for st, (data, off, seq) in zip(states, batches):
+        s, c = st.local(data, off, seq)
+        sends.append(s)
+        counts.append(c)
+    recvs, rcounts = loopback_all_to_all(sends, counts)
+    replies = [st.owner(r) for st, r in zip(states, recvs)]
+    # reverse: owner d's reply rows are grouped by source rank s
+    back_counts = [[rcounts[d][s] for s in range(len(states))] for d in range(len(states))]
+    backs, _ = loopback_all_to_all(replies, back_counts)
+    return [st.finish(b) for st, b in zip(states, backs)]
