@@ -324,8 +324,10 @@ def main():
     kd = kernels[dom]
     traffic = None
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    if os.path.exists(tp):
-        traffic = json.load(open(tp)).get(dom)
+    if os.path.exists(tp):  # DRAM bytes per launch from the committed ncu capture,
+        tj = json.load(open(tp))  # scaled from its batch size to this run's mean batch
+        if dom in tj:
+            traffic = tj[dom] / tj["capture_batch_bytes"] * (bytes_timed / args.steps)
     roofline = {"kernel": dom, "bound": kd["bound"], "achieved": kd["achieved"],
                 "peak": kd["peak"], "unit": kd["unit"], "frac": kd["frac"], "traffic": traffic,
                 "peak_source": f"{src} (MEASURED_PEAKS.json)" if kd["bound"] == "hbm" else
