@@ -9,7 +9,9 @@ import ctypes
 import os
 
 PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(PKG, "libdedup_b200.so")
+# DEDUP_LIB selects an alternative build of the same library (kernel-variant
+# experiments under tools/); default: the in-tree build.
+LIB_PATH = os.environ.get("DEDUP_LIB", os.path.join(PKG, "libdedup_b200.so"))
 
 DEDUP_OK = 0
 DEDUP_EINVAL = -1

@@ -40,22 +40,29 @@ namespace {
 // reach ~97% of the 1024-thread throughput) while leaving half of the
 // register file to the SHA-1 / table kernels of other in-flight batches.
 constexpr int kScanThreads = 512;
+#ifndef DEDUP_SCAN_PREFETCH
+#define DEDUP_SCAN_PREFETCH 2
+#endif
+constexpr int kScanPrefetch = DEDUP_SCAN_PREFETCH;  // 32-byte steps loaded ahead (0..2)
 constexpr int kScanWarps = kScanThreads / 32;
-constexpr int kEmitThreads = 1024;  // one warp per tile of the group (latency-bound)
+constexpr int kEmitThreads = kScanThreads;  // one warp per tile of a group
 constexpr int kEmitWarps = kEmitThreads / 32;
 constexpr int kTabBytes = 256 * 256;  // [x][R|W][lane] u32 = 64 KiB
 constexpr uint32_t kLaneBytes = kSelTile / 32;  // 256 bytes per lane per tile
 constexpr uint32_t kFull = 0xFFFFFFFFu;
 constexpr uint32_t kInf = 0xFFFFFFFFu;
 constexpr uint32_t kM27 = (1u << 27) - 1;
-constexpr int kGroup = 32;        // tiles per group
+constexpr int kGroup = kScanWarps;  // tiles per group = one tile per warp of a CTA
 constexpr int kItemCache = 2048;  // item offsets cached in shared memory
+
+constexpr uint32_t kListCap = 128;  // events per tile kept as a sorted list
 
 struct SelWarpSmem {
     uint32_t cand[kSelTileWords];
     uint32_t forced[kSelTileWords];
     uint32_t csum[8];
     uint32_t fsum[8];
+    uint32_t list[kListCap];
 };
 
 // scan: [pad to a 64 KiB shared-window boundary][table]; the per-warp walk
@@ -70,6 +77,9 @@ struct EmitSmem {
     uint32_t te_state[kGroup], te_cnt[kGroup];
     uint64_t items[kItemCache];
 };
+
+// Group buffers in the scan (double buffering across the group barrier).
+constexpr int kFunBufs = 2;
 
 __device__ __forceinline__ uint32_t lds(uint32_t addr) {
     uint32_t v;
@@ -173,12 +183,77 @@ __device__ __forceinline__ const uint64_t* cache_items(uint64_t* cache, const Ba
     return cache;
 }
 
+// Events of a tile as a sorted compact list (bit 31 = forced cut), when there
+// are at most kListCap of them; returns their number, or kInf if the list
+// would overflow (dense candidates: the bitmap walker is used instead).
+__device__ __forceinline__ uint32_t build_events(SelWarpSmem& sm, const uint32_t cw[8],
+                                                 const uint32_t fw[8], int lane) {
+    uint32_t cnt = 0;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) cnt += __popc(cw[j] | fw[j]);
+    uint32_t incl = cnt;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t v = __shfl_up_sync(kFull, incl, d);
+        if (lane >= d) incl += v;
+    }
+    const uint32_t total = __shfl_sync(kFull, incl, 31);
+    if (total > kListCap) return kInf;
+    uint32_t o = incl - cnt;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+        uint32_t b = cw[j] | fw[j];
+        while (b) {
+            const uint32_t bit = __ffs(b) - 1;
+            b &= b - 1;
+            const uint32_t pos = (uint32_t)(lane * kLaneBytes + 32 * j) + bit;
+            sm.list[o++] = pos | (((fw[j] >> bit) & 1u) << 31);
+        }
+    }
+    __syncwarp();
+    return total;
+}
+
+// Greedy walk over the tile's event list from entry state s (see walk_tile).
+__device__ __forceinline__ uint32_t walk_events(const SelWarpSmem& sm, uint32_t n_ev, uint32_t s,
+                                                uint32_t& exit_state, uint32_t* out,
+                                                uint64_t out_base, uint64_t cap, uint64_t T0) {
+    uint32_t E = s, cnt = 0;
+    for (uint32_t i = 0; i < n_ev; ++i) {
+        const uint32_t ev = sm.list[i];
+        const uint32_t p = ev & 0x7FFFFFFFu;
+        if ((ev >> 31) || p >= E) {
+            if (out != nullptr && out_base + cnt < cap) out[out_base + cnt] = (uint32_t)(T0 + p);
+            ++cnt;
+            E = p + 32;
+        }
+    }
+    exit_state = E > kSelTile ? E - kSelTile : 0;
+    return cnt;
+}
+
+// First item index whose start is > T0 - 32 (lane 0 searches, all get it).
+__device__ __forceinline__ uint32_t first_item(uint64_t T0, const uint64_t* item_off,
+                                               uint32_t n_items, int lane) {
+    uint32_t lo = 0;
+    if (lane == 0 && n_items > 0) {
+        const uint64_t key = T0 >= 31 ? T0 - 31 : 0;
+        uint32_t hi = n_items;
+        while (lo < hi) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (item_off[mid] < key) lo = mid + 1; else hi = mid;
+        }
+    }
+    return __shfl_sync(kFull, lo, 0);
+}
+
 // Lane's 8 e-space candidate words (already in sm.cand) get the item rules:
 // no candidate at e in [q, q+32) (the window would leave the item), a forced
-// cut at q for every non-empty item; then the summaries.  Ends with syncwarp.
-__device__ __forceinline__ void apply_items(SelWarpSmem& sm, uint64_t T0, uint64_t nbytes,
-                                            const uint64_t* item_off, uint32_t n_items,
-                                            int lane) {
+// cut at q for every non-empty item; then the summaries and the event list.
+// Returns the number of events (kInf: use the bitmap walker).
+__device__ __forceinline__ uint32_t apply_items(SelWarpSmem& sm, uint64_t T0, uint64_t nbytes,
+                                                const uint64_t* item_off, uint32_t n_items,
+                                                int lane) {
     uint32_t cw[8], fw[8];
 #pragma unroll
     for (int j = 0; j < 8; ++j) {
@@ -186,13 +261,8 @@ __device__ __forceinline__ void apply_items(SelWarpSmem& sm, uint64_t T0, uint64
         fw[j] = 0;
     }
     const uint64_t E0 = T0 + (uint64_t)lane * kLaneBytes;  // this lane's e-range
+    const uint32_t lo = first_item(T0, item_off, n_items, lane);
     if (E0 < nbytes && n_items > 0) {
-        const uint64_t key = E0 >= 31 ? E0 - 31 : 0;  // first start > E0 - 32
-        uint32_t lo = 0, hi = n_items;
-        while (lo < hi) {
-            const uint32_t mid = (lo + hi) >> 1;
-            if (item_off[mid] < key) lo = mid + 1; else hi = mid;
-        }
         for (uint32_t it = lo; it < n_items; ++it) {
             const uint64_t q = item_off[it];
             if (q >= E0 + kLaneBytes) break;
@@ -210,6 +280,8 @@ __device__ __forceinline__ void apply_items(SelWarpSmem& sm, uint64_t T0, uint64
             }
         }
     }
+    const uint32_t n_ev = build_events(sm, cw, fw, lane);
+    if (n_ev != kInf) return n_ev;
     uint32_t cm = 0, fm = 0;
 #pragma unroll
     for (int j = 0; j < 8; ++j) {
@@ -221,6 +293,15 @@ __device__ __forceinline__ void apply_items(SelWarpSmem& sm, uint64_t T0, uint64
     reinterpret_cast<uint8_t*>(sm.csum)[lane] = (uint8_t)cm;
     reinterpret_cast<uint8_t*>(sm.fsum)[lane] = (uint8_t)fm;
     __syncwarp();
+    return kInf;
+}
+
+// Walk from entry state s using the event list, or the bitmaps if dense.
+__device__ __forceinline__ uint32_t walk_any(const SelWarpSmem& sm, uint32_t n_ev, uint32_t s,
+                                             uint32_t& exit_state, uint32_t* out,
+                                             uint64_t out_base, uint64_t cap, uint64_t T0) {
+    if (n_ev != kInf) return walk_events(sm, n_ev, s, exit_state, out, out_base, cap, T0);
+    return walk_tile(sm, s, exit_state, out, out_base, cap, T0);
 }
 
 // Scan + per-tile transfer functions + per-group composition.
@@ -246,11 +327,13 @@ rabin_scan_agg_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __rest
         pad >= (uint32_t)kScanAux ? smem : smem + pad + kTabBytes);
     uint64_t* icache = reinterpret_cast<uint64_t*>(wsm + kScanWarps);
     SelWarpSmem& sm = wsm[wid];
+    __shared__ uint32_t fun[kFunBufs][kGroup][32];  // tile functions of recent groups
     const uint64_t n_tiles = (nbytes + kSelTile - 1) / kSelTile;
+    const uint64_t n_groups = (n_tiles + kGroup - 1) / kGroup;
     const uint64_t lim16 = (nbytes + 15) & ~uint64_t(15);
-    // static, balanced assignment: CTA b owns tiles [lo, hi), warps interleave
-    const uint64_t lo = n_tiles * blockIdx.x / gridDim.x;
-    const uint64_t hi = n_tiles * (blockIdx.x + 1) / gridDim.x;
+    // CTA b owns groups b, b + grid, ...; warp w owns tile w of each group
+    const uint64_t stride = (uint64_t)gridDim.x * kGroup;
+    const uint64_t lo = (uint64_t)blockIdx.x * kGroup, hi = n_groups * kGroup;
     // warm-up window and the first two 32-byte steps of a tile, loaded early
     uint32_t prev[8], cur[8], nxt[8];
     auto load_first = [&](uint64_t t) {
@@ -259,9 +342,9 @@ rabin_scan_agg_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __rest
         for (int i = 0; i < 8; ++i) prev[i] = cur[i] = nxt[i] = 0;
         if (q >= 32) load32(bytes + q - 32, prev);
         if (q < nbytes) load32_any(bytes, q, nbytes, lim16, cur);
-        if (q + 32 < nbytes) load32_any(bytes, q + 32, nbytes, lim16, nxt);
+        if (kScanPrefetch == 2 && q + 32 < nbytes) load32_any(bytes, q + 32, nbytes, lim16, nxt);
     };
-    if (lo + wid < hi) load_first(lo + wid);  // in flight during the table build
+    if (lo + wid < n_tiles) load_first(lo + wid);  // in flight during the table build
     if (threadIdx.x < 512) src[threadIdx.x] = gtab[threadIdx.x];
     const uint64_t* items = cache_items(icache, desc);
     const uint32_t n_items = desc->n_items;
@@ -275,12 +358,19 @@ rabin_scan_agg_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __rest
     if (nbytes == 0) return;
     const uint32_t laneR = base | (lane * 4);
     const uint32_t laneW = laneR + 128;
-    for (uint64_t t = lo + wid; t < hi; t += kScanThreads / 32) {
+    int par = 0;
+    for (uint64_t t = lo + wid; t < hi; t += stride, par = (par + 1) % kFunBufs) {
+      uint32_t f = (uint32_t)lane << 27;  // identity function beyond the last tile
+      if (t < n_tiles) {
         const uint64_t T0 = t * kSelTile;
         const uint64_t q = T0 + (uint64_t)lane * kLaneBytes;
         // ---- scan: 8 steps of 32 bytes, bits written in e-space ----
         uint32_t h = 0, prev_bits = 0;
+#if defined(DEDUP_SCAN_EXPERIMENT) && (DEDUP_SCAN_EXPERIMENT & 2)
+        if (false) {  // timing experiment only: no warm-up
+#else
         if (q >= 32) {  // warm-up: the window ending at q-1 -> bit for e = q
+#endif
             const uint32_t zero[8] = {0, 0, 0, 0, 0, 0, 0, 0};
             prev_bits = roll32<kZeroValue>(h, prev, zero, laneR, laneW, mask, value);
         }
@@ -288,7 +378,13 @@ rabin_scan_agg_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __rest
         for (int j = 0; j < 8; ++j) {
             const uint64_t b0 = q + 32 * j;
             uint32_t bits = 0, nx2[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-            if (j < 6 && b0 + 64 < nbytes) load32_any(bytes, b0 + 64, nbytes, lim16, nx2);
+            if (kScanPrefetch == 2) {
+                if (j < 6 && b0 + 64 < nbytes) load32_any(bytes, b0 + 64, nbytes, lim16, nx2);
+            } else if (kScanPrefetch == 1) {
+                if (j < 7 && b0 + 32 < nbytes) load32_any(bytes, b0 + 32, nbytes, lim16, nx2);
+            } else if (j > 0 && b0 < nbytes) {
+                load32_any(bytes, b0, nbytes, lim16, cur);
+            }
             if (b0 < nbytes) {
                 bits = roll32<kZeroValue>(h, cur, prev, laneR, laneW, mask, value);
                 if (b0 + 32 > nbytes) bits &= (1u << (uint32_t)(nbytes - b0)) - 1u;
@@ -302,47 +398,42 @@ rabin_scan_agg_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __rest
 #pragma unroll
             for (int i = 0; i < 8; ++i) {
                 prev[i] = cur[i];
-                cur[i] = nxt[i];
-                nxt[i] = nx2[i];
+                if (kScanPrefetch == 2) {
+                    cur[i] = nxt[i];
+                    nxt[i] = nx2[i];
+                } else if (kScanPrefetch == 1) {
+                    cur[i] = nx2[i];
+                }
             }
         }
         // next tile's first loads fly during the transfer-function walk
-        if (t + kScanThreads / 32 < hi) load_first(t + kScanThreads / 32);
+        if (t + stride < n_tiles) load_first(t + stride);
         // ---- the tile's 32-entry transfer function ----
-        apply_items(sm, T0, nbytes, items, n_items, lane);
+        const uint32_t n_ev = apply_items(sm, T0, nbytes, items, n_items, lane);
         uint32_t ex;
-        const uint32_t cnt = walk_tile(sm, lane, ex, nullptr, 0, 0, 0);
-        agg[32 * (uint64_t)t + lane] = (ex << 27) | cnt;
-        __syncwarp();
-        // ---- the last tile of a group to finish composes the group ----
-        const uint64_t g = t / kGroup;
-        const uint64_t left = n_tiles - g * kGroup;
-        const uint32_t expected = left < (uint64_t)kGroup ? (uint32_t)left : (uint32_t)kGroup;
-        __threadfence();
-        uint32_t arrived = 0;
-        if (lane == 0) arrived = atomicAdd(&ctr[1 + g], 1u) + 1;
-        arrived = __shfl_sync(kFull, arrived, 0);
-        if (arrived == expected) {
-            __threadfence();
+        const uint32_t cnt = walk_any(sm, n_ev, lane, ex, nullptr, 0, 0, 0);
+        f = (ex << 27) | cnt;
+        agg[32 * t + lane] = f;
+      }
+        // ---- the CTA composes its group of kGroup tiles (the barrier keeps
+        // the warps of a CTA in step, measured faster than letting the last
+        // arrival compose) ----
+        fun[par][wid][lane] = f;
+        __syncthreads();
+        if (wid == 0) {
             uint32_t Gs = lane, Gc = 0;
-            for (uint32_t jb = 0; jb < expected; jb += 16) {
-                uint32_t a[16];
 #pragma unroll
-                for (int j = 0; j < 16; ++j)
-                    a[j] = jb + j < expected
-                               ? __ldcg(&agg[32 * (g * kGroup + jb + j) + lane])
-                               : ((uint32_t)lane << 27);
-#pragma unroll
-                for (int j = 0; j < 16; ++j) {
-                    const uint32_t ns = __shfl_sync(kFull, a[j] >> 27, Gs);
-                    const uint32_t nc = Gc + __shfl_sync(kFull, a[j] & kM27, Gs);
-                    Gs = ns;
-                    Gc = nc;
-                }
+            for (int j = 0; j < kGroup; ++j) {
+                const uint32_t a = fun[par][j][lane];
+                const uint32_t ns = __shfl_sync(kFull, a >> 27, Gs);
+                const uint32_t nc = Gc + __shfl_sync(kFull, a & kM27, Gs);
+                Gs = ns;
+                Gc = nc;
             }
-            gagg[32 * g + lane] = (Gs << 27) | Gc;
+            gagg[32 * (t / kGroup) + lane] = (Gs << 27) | Gc;
         }
     }
+    (void)ctr;
 }
 
 // Prefix composition of the group functions (one CTA of 32 warps).
@@ -448,11 +539,11 @@ select_emit_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restric
 #pragma unroll
             for (int k = 0; k < 8; ++k)
                 w.cand[lane * 8 + k] = bitmap[t * kSelTileWords + lane * 8 + k];
-            apply_items(w, t * kSelTile, nbytes, items, n_items, lane);
+            const uint32_t n_ev = apply_items(w, t * kSelTile, nbytes, items, n_items, lane);
             const uint32_t st = sm.te_state[j];
             if (lane == (int)st) {
                 uint32_t ex;
-                walk_tile(w, st, ex, cut_pos, sm.te_cnt[j], cap, t * kSelTile);
+                walk_any(w, n_ev, st, ex, cut_pos, sm.te_cnt[j], cap, t * kSelTile);
             }
             __syncwarp();
         }
