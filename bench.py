@@ -144,7 +144,10 @@ def run_steps(d, submit, n_batches, steps, first_step):
             except Exception as e:
                 if "EAGAIN" not in str(e):
                     raise
-                d.drain_raw(wait_ms=-1)
+                # a non-blocking drain first releases the slots handed out by
+                # the previous drain; block only if nothing has completed
+                if d.drain_raw(wait_ms=0) == 0:
+                    d.drain_raw(wait_ms=-1)
     while d.pending():
         d.drain_raw(wait_ms=-1)
 

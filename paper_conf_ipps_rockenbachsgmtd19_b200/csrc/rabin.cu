@@ -52,8 +52,12 @@ constexpr uint32_t kLaneBytes = kSelTile / 32;  // 256 bytes per lane per tile
 constexpr uint32_t kFull = 0xFFFFFFFFu;
 constexpr uint32_t kInf = 0xFFFFFFFFu;
 constexpr uint32_t kM27 = (1u << 27) - 1;
-constexpr int kGroup = kScanWarps;  // tiles per group = one tile per warp of a CTA
-constexpr int kItemCache = 2048;  // item offsets cached in shared memory
+#ifndef DEDUP_SCAN_ILP
+#define DEDUP_SCAN_ILP 2
+#endif
+constexpr int kScanIlp = DEDUP_SCAN_ILP;  // tiles rolled together per warp (1 or 2)
+constexpr int kGroup = kScanWarps * kScanIlp;  // tiles per group = one CTA round
+constexpr int kItemCache = 1024;  // item offsets cached in shared memory
 
 constexpr uint32_t kListCap = 128;  // events per tile kept as a sorted list
 
@@ -68,8 +72,12 @@ struct SelWarpSmem {
 // scan: [pad to a 64 KiB shared-window boundary][table]; the per-warp walk
 // buffers and the item cache (aux) live in the pad when it is large enough,
 // else after the table.
+// The aux data must fit the pad, so that a scan CTA needs only 128 KiB of
+// dynamic shared memory and other batches' kernels can share the SM; the
+// kernel traps if the runtime layout ever leaves a smaller pad.
 constexpr int kScanAux = kScanWarps * (int)sizeof(SelWarpSmem) + kItemCache * 8;
-constexpr int kScanSmem = 65536 + kTabBytes + kScanAux;
+constexpr int kScanSmem = 65536 + kTabBytes;
+static_assert(kScanAux <= 65536 - 1024 - 8192, "scan aux data must fit the alignment pad");
 
 struct EmitSmem {
     SelWarpSmem w[kEmitWarps];
@@ -324,7 +332,8 @@ rabin_scan_agg_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __rest
     const uint32_t pad = (0x10000u - (win & 0xFFFFu)) & 0xFFFFu;
     const uint32_t base = win + pad;
     SelWarpSmem* wsm = reinterpret_cast<SelWarpSmem*>(
-        pad >= (uint32_t)kScanAux ? smem : smem + pad + kTabBytes);
+        smem);
+    if (pad < (uint32_t)kScanAux) __trap();  // layout assumption (see kScanSmem)
     uint64_t* icache = reinterpret_cast<uint64_t*>(wsm + kScanWarps);
     SelWarpSmem& sm = wsm[wid];
     __shared__ uint32_t fun[kFunBufs][kGroup][32];  // tile functions of recent groups
@@ -434,6 +443,164 @@ rabin_scan_agg_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __rest
         }
     }
     (void)ctr;
+}
+
+// Two independent rolling chains per lane (ILP 2): the LDS -> LOP3 -> PRMT
+// dependency of one chain overlaps with the other's.
+template <bool kZeroValue>
+__device__ __forceinline__ void roll32x2(uint32_t& hA, const uint32_t curA[8],
+                                         const uint32_t oldA[8], uint32_t& bitsA, uint32_t& hB,
+                                         const uint32_t curB[8], const uint32_t oldB[8],
+                                         uint32_t& bitsB, uint32_t laneR, uint32_t laneW,
+                                         uint32_t mask, uint32_t value) {
+    bitsA = bitsB = 0;
+#pragma unroll
+    for (int w = 0; w < 8; ++w) {
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            const uint32_t aRA = __byte_perm(hA, laneR, 0x7634);
+            const uint32_t aRB = __byte_perm(hB, laneR, 0x7634);
+            const uint32_t aWA = __byte_perm(oldA[w], laneW, 0x7604 | (k << 4));
+            const uint32_t aWB = __byte_perm(oldB[w], laneW, 0x7604 | (k << 4));
+            const uint32_t hsA = __byte_perm(curA[w], hA, 0x6540 | k);
+            const uint32_t hsB = __byte_perm(curB[w], hB, 0x6540 | k);
+            hA = hsA ^ lds(aRA) ^ lds(aWA);
+            hB = hsB ^ lds(aRB) ^ lds(aWB);
+            const uint32_t tA = kZeroValue ? (hA & mask) : ((hA & mask) ^ value);
+            const uint32_t tB = kZeroValue ? (hB & mask) : ((hB & mask) ^ value);
+            asm("{\n\t.reg .pred p;\n\tsetp.eq.u32 p, %1, 0;\n\t@p or.b32 %0, %0, %2;\n\t}"
+                : "+r"(bitsA)
+                : "r"(tA), "r"(1u << (4 * w + k)));
+            asm("{\n\t.reg .pred p;\n\tsetp.eq.u32 p, %1, 0;\n\t@p or.b32 %0, %0, %2;\n\t}"
+                : "+r"(bitsB)
+                : "r"(tB), "r"(1u << (4 * w + k)));
+        }
+    }
+}
+
+// ILP-2 scan: a CTA of kScanWarps warps takes groups of 2 x kScanWarps tiles;
+// warp w rolls tiles w and w + kScanWarps of the group together.
+template <bool kZeroValue>
+__global__ void __launch_bounds__(kScanThreads, 2)
+rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ gtab,
+                       uint32_t mask, uint32_t value, uint32_t* __restrict__ bitmap,
+                       uint32_t* __restrict__ agg, uint32_t* __restrict__ gagg) {
+    extern __shared__ __align__(16) uint8_t smem[];
+    __shared__ uint32_t src[512];
+    __shared__ uint32_t fun[kFunBufs][kGroup][32];
+    const uint8_t* __restrict__ bytes = desc->bytes;
+    const uint64_t nbytes = desc->nbytes;
+    const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t win = (uint32_t)__cvta_generic_to_shared(smem);
+    const uint32_t pad = (0x10000u - (win & 0xFFFFu)) & 0xFFFFu;
+    const uint32_t base = win + pad;
+    SelWarpSmem* wsm = reinterpret_cast<SelWarpSmem*>(smem);
+    if (pad < (uint32_t)kScanAux) __trap();  // layout assumption (see kScanSmem)
+    uint64_t* icache = reinterpret_cast<uint64_t*>(wsm + kScanWarps);
+    SelWarpSmem& sm = wsm[wid];
+    if (threadIdx.x < 512) src[threadIdx.x] = gtab[threadIdx.x];
+    const uint64_t* items = cache_items(icache, desc);
+    const uint32_t n_items = desc->n_items;
+    __syncthreads();
+    {
+        uint32_t* t32 = reinterpret_cast<uint32_t*>(smem + pad);
+        for (int idx = threadIdx.x; idx < kTabBytes / 4; idx += blockDim.x)
+            t32[idx] = src[((idx >> 5) & 1) * 256 + (idx >> 6)];
+    }
+    __syncthreads();
+    if (nbytes == 0) return;
+    const uint64_t n_tiles = (nbytes + kSelTile - 1) / kSelTile;
+    const uint64_t n_groups = (n_tiles + kGroup - 1) / kGroup;
+    const uint64_t lim16 = (nbytes + 15) & ~uint64_t(15);
+    const uint32_t laneR = base | (lane * 4);
+    const uint32_t laneW = laneR + 128;
+    int par = 0;
+    for (uint64_t g = blockIdx.x; g < n_groups; g += gridDim.x, par ^= 1) {
+        const uint64_t tA = g * kGroup + wid, tB = tA + kScanWarps;
+        const uint64_t qA = tA * kSelTile + (uint64_t)lane * kLaneBytes;
+        const uint64_t qB = tB * kSelTile + (uint64_t)lane * kLaneBytes;
+        uint32_t prevA[8], curA[8], prevB[8], curB[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) prevA[i] = curA[i] = prevB[i] = curB[i] = 0;
+        if (qA >= 32 && qA < nbytes) load32(bytes + qA - 32, prevA);
+        if (qB >= 32 && qB < nbytes) load32(bytes + qB - 32, prevB);
+        if (qA < nbytes) load32_any(bytes, qA, nbytes, lim16, curA);
+        if (qB < nbytes) load32_any(bytes, qB, nbytes, lim16, curB);
+        uint32_t hA = 0, hB = 0, pbA = 0, pbB = 0;
+        {   // warm-up of both chains: the windows ending at q-1
+            const uint32_t zero[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+            uint32_t bA, bB;
+            roll32x2<kZeroValue>(hA, prevA, zero, bA, hB, prevB, zero, bB, laneR, laneW, mask,
+                                 value);
+            pbA = qA >= 32 ? bA : 0;
+            pbB = qB >= 32 ? bB : 0;
+            if (qA < 32) hA = 0;
+            if (qB < 32) hB = 0;
+        }
+#pragma unroll 1
+        for (int j = 0; j < 8; ++j) {
+            const uint64_t bA0 = qA + 32 * j, bB0 = qB + 32 * j;
+            if (j > 0) {
+                if (bA0 < nbytes) load32_any(bytes, bA0, nbytes, lim16, curA);
+                if (bB0 < nbytes) load32_any(bytes, bB0, nbytes, lim16, curB);
+            }
+            uint32_t bitsA, bitsB;
+            roll32x2<kZeroValue>(hA, curA, prevA, bitsA, hB, curB, prevB, bitsB, laneR, laneW,
+                                 mask, value);
+            uint32_t ewA = __funnelshift_l(pbA, bitsA, 1), ewB = __funnelshift_l(pbB, bitsB, 1);
+            if (bA0 >= nbytes) ewA = 0;
+            else if (bA0 + 32 > nbytes) ewA &= (1u << (uint32_t)(nbytes - bA0)) - 1u;
+            if (bB0 >= nbytes) ewB = 0;
+            else if (bB0 + 32 > nbytes) ewB &= (1u << (uint32_t)(nbytes - bB0)) - 1u;
+            if (bA0 + 32 > nbytes) bitsA &= bA0 < nbytes ? (1u << (uint32_t)(nbytes - bA0)) - 1u : 0u;
+            if (bB0 + 32 > nbytes) bitsB &= bB0 < nbytes ? (1u << (uint32_t)(nbytes - bB0)) - 1u : 0u;
+            sm.cand[lane * 8 + j] = ewA;
+            if (tA < n_tiles) bitmap[tA * kSelTileWords + lane * 8 + j] = ewA;
+            if (tB < n_tiles) bitmap[tB * kSelTileWords + lane * 8 + j] = ewB;
+            pbA = bitsA;
+            pbB = bitsB;
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                prevA[i] = curA[i];
+                prevB[i] = curB[i];
+            }
+        }
+        // transfer functions of tile A (candidate words already in smem), then B
+        uint32_t fA = (uint32_t)lane << 27, fB = fA;
+        if (tA < n_tiles) {
+            const uint32_t n_ev = apply_items(sm, tA * kSelTile, nbytes, items, n_items, lane);
+            uint32_t ex;
+            const uint32_t cnt = walk_any(sm, n_ev, lane, ex, nullptr, 0, 0, 0);
+            fA = (ex << 27) | cnt;
+            agg[32 * tA + lane] = fA;
+        }
+        __syncwarp();
+        if (tB < n_tiles) {
+#pragma unroll
+            for (int k = 0; k < 8; ++k)
+                sm.cand[lane * 8 + k] = bitmap[tB * kSelTileWords + lane * 8 + k];
+            const uint32_t n_ev = apply_items(sm, tB * kSelTile, nbytes, items, n_items, lane);
+            uint32_t ex;
+            const uint32_t cnt = walk_any(sm, n_ev, lane, ex, nullptr, 0, 0, 0);
+            fB = (ex << 27) | cnt;
+            agg[32 * tB + lane] = fB;
+        }
+        fun[par][wid][lane] = fA;
+        fun[par][wid + kScanWarps][lane] = fB;
+        __syncthreads();
+        if (wid == 0) {
+            uint32_t Gs = lane, Gc = 0;
+#pragma unroll
+            for (int j = 0; j < kGroup; ++j) {
+                const uint32_t a = fun[par][j][lane];
+                const uint32_t ns = __shfl_sync(kFull, a >> 27, Gs);
+                const uint32_t nc = Gc + __shfl_sync(kFull, a & kM27, Gs);
+                Gs = ns;
+                Gc = nc;
+            }
+            gagg[32 * g + lane] = (Gs << 27) | Gc;
+        }
+    }
 }
 
 // Prefix composition of the group functions (one CTA of 32 warps).
@@ -599,24 +766,36 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
                          uint32_t* cut_pos, uint64_t cap, uint32_t* n_chunks, int num_sms,
                          cudaStream_t s, cudaEvent_t after_scan) {
     static bool attr_set = false;
+    auto kT = kScanIlp == 2 ? rabin_scan_agg2_kernel<true> : nullptr;
+    auto kF = kScanIlp == 2 ? rabin_scan_agg2_kernel<false> : nullptr;
     if (!attr_set) {
-        cudaFuncSetAttribute(rabin_scan_agg_kernel<true>,
-                             cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
-        cudaFuncSetAttribute(rabin_scan_agg_kernel<false>,
-                             cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
+        if (kScanIlp == 2) {
+            cudaFuncSetAttribute(kT, cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
+            cudaFuncSetAttribute(kF, cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
+        } else {
+            cudaFuncSetAttribute(rabin_scan_agg_kernel<true>,
+                                 cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
+            cudaFuncSetAttribute(rabin_scan_agg_kernel<false>,
+                                 cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
+        }
         cudaFuncSetAttribute(select_emit_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)sizeof(EmitSmem));
         attr_set = true;
     }
     const uint64_t groups = select_groups(max_tiles);
-    cudaMemsetAsync(scan_ctr, 0, sizeof(uint32_t) * (groups + 2), s);
     const unsigned grid = (unsigned)num_sms;
-    if (value == 0)
-        rabin_scan_agg_kernel<true><<<grid, kScanThreads, kScanSmem, s>>>(
-            d, d_tab, mask, value, bitmap, agg, gagg, scan_ctr);
-    else
-        rabin_scan_agg_kernel<false><<<grid, kScanThreads, kScanSmem, s>>>(
-            d, d_tab, mask, value, bitmap, agg, gagg, scan_ctr);
+    if (kScanIlp == 2) {
+        (value == 0 ? kT : kF)<<<grid, kScanThreads, kScanSmem, s>>>(d, d_tab, mask, value,
+                                                                     bitmap, agg, gagg);
+    } else {
+        cudaMemsetAsync(scan_ctr, 0, sizeof(uint32_t) * (groups + 2), s);
+        if (value == 0)
+            rabin_scan_agg_kernel<true><<<grid, kScanThreads, kScanSmem, s>>>(
+                d, d_tab, mask, value, bitmap, agg, gagg, scan_ctr);
+        else
+            rabin_scan_agg_kernel<false><<<grid, kScanThreads, kScanSmem, s>>>(
+                d, d_tab, mask, value, bitmap, agg, gagg, scan_ctr);
+    }
     if (after_scan) cudaEventRecordWithFlags(after_scan, s, cudaEventRecordExternal);
     select_scan_kernel<<<1, 1024, 0, s>>>(d, gagg, gentry, n_chunks);
     uint64_t blocks = groups;

@@ -27,6 +27,7 @@ for b in range(n):
         except Exception as e:
             if "EAGAIN" not in str(e):
                 raise
-            d.drain_raw(wait_ms=-1)
+            if d.drain_raw(wait_ms=0) == 0:
+                d.drain_raw(wait_ms=-1)
 d.drain_all()
 torch.cuda.synchronize()
