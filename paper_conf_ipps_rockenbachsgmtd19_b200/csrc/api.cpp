@@ -208,6 +208,13 @@ void ws_free(Workspace& w) {
 
 bool usable(const dedup_ctx* c) { return c != nullptr && c->sticky == DEDUP_OK; }
 
+// Attribution builds (tools/attrib.sh) only: 1 = omit the SHA-1 kernels,
+// 2 = omit the table kernels, 4 = omit chunk selection.  Results are invalid;
+// the product build has 0.
+#ifndef DEDUP_ATTRIB_SKIP
+#define DEDUP_ATTRIB_SKIP 0
+#endif
+
 // Chunks at least 4x the mean anchor distance are hashed first.
 uint32_t long_bytes(const dedup_ctx* c) {
     uint64_t v = 4ull * ((uint64_t)c->cfg.anchor_mask + 1);
@@ -227,14 +234,16 @@ void enqueue_chunk_sha(dedup_ctx* c, Workspace& w, cudaStream_t s, const BatchDe
                        uint8_t* digest, cudaEvent_t ev_scan, cudaEvent_t ev_chunk,
                        uint32_t* chunk_start, uint64_t* chunk_id, uint32_t* item_first,
                        uint32_t max_items) {
-    launch_chunk_select(d, c->d_tab, c->cfg.anchor_mask, c->cfg.anchor_value, w.bitmap, w.agg,
-                        w.gagg, w.gentry, w.scan_ctr, (max_bytes + kSelTile - 1) / kSelTile,
-                        cut_pos, cap, n_chunks, c->num_sms, s, ev_scan);
+    if (!(DEDUP_ATTRIB_SKIP & 4))
+        launch_chunk_select(d, c->d_tab, c->cfg.anchor_mask, c->cfg.anchor_value, w.bitmap,
+                            w.agg, w.gagg, w.gentry, w.scan_ctr,
+                            (max_bytes + kSelTile - 1) / kSelTile, cut_pos, cap, n_chunks,
+                            c->num_sms, s, ev_scan);
     if (chunk_start)
         launch_chunk_meta(d, cut_pos, n_chunks, cap, chunk_start, chunk_id, item_first,
                           max_items, c->num_sms, s);
     if (ev_chunk) cudaEventRecordWithFlags(ev_chunk, s, cudaEventRecordExternal);
-    if (digest)
+    if (digest && !(DEDUP_ATTRIB_SKIP & 1))
         launch_sha1(d, max_bytes, cut_pos, n_chunks, cap, long_bytes(c), w.counters,
                     w.long_list, digest, c->num_sms, s);
 }
@@ -260,11 +269,13 @@ dedup_status build_graph(dedup_ctx* c, int i) {
     if (se) cudaEventRecordWithFlags(sl.ev_sha, s, cudaEventRecordExternal);
     // table work waits for the previous batch's table work (global chain)
     cudaStreamWaitEvent(s, prev.ev_table, cudaEventWaitExternal);
-    launch_table_prepare(sl.d_desc, c->tables[0].capacity, c->num_sms, s);
     const TableView* tv = &sl.d_desc->table;
-    launch_table_insert(tv, sl.d_digest, sl.d_chunk_id, nullptr, sl.d_small, 0, cap,
-                        sl.ws.slot_idx, c->num_sms, s);
-    launch_table_lookup(tv, sl.d_chunk_id, nullptr, sl.d_small, 0, cap, sl.ws.slot_idx,
+    if (!(DEDUP_ATTRIB_SKIP & 2)) {
+        launch_table_prepare(sl.d_desc, c->tables[0].capacity, c->num_sms, s);
+        launch_table_insert(tv, sl.d_digest, sl.d_chunk_id, nullptr, sl.d_small, 0, cap,
+                            sl.ws.slot_idx, c->num_sms, s);
+    }
+    if (!(DEDUP_ATTRIB_SKIP & 2)) launch_table_lookup(tv, sl.d_chunk_id, nullptr, sl.d_small, 0, cap, sl.ws.slot_idx,
                         sl.d_first_id, sl.d_is_dup, sl.d_small + 4, sl.d_cut_pos, sl.d_desc,
                         c->num_sms, s);
     cudaEventRecordWithFlags(sl.ev_table, s, cudaEventRecordExternal);
@@ -525,6 +536,13 @@ dedup_status dedup_init(const dedup_config* cfg, dedup_ctx** out) {
     if (cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, cfg->device) !=
         cudaSuccess)
         return bail(DEDUP_ECUDA);
+    for (const char* bad : {chunk_unlaunchable(), sha1_unlaunchable()}) {
+        if (bad) {
+            std::fprintf(stderr, "dedup_init: %s cannot launch on device %d\n", bad,
+                         cfg->device);
+            return bail(DEDUP_ECUDA);
+        }
+    }
     c->chunk_cap = cfg->batch_bytes / 32 + cfg->batch_items + 2;
     uint32_t tab[512];
     for (uint32_t b = 0; b < 256; ++b) {

@@ -45,6 +45,19 @@ constexpr uint32_t kSelTileWords = kSelTile / 32;
 // scan_ctr: select_groups(max_tiles) + 2 words, zeroed by the launcher.
 // after_scan (optional) is recorded between the scan and the selection.
 uint64_t select_groups(uint64_t max_tiles);
+
+// Launch-configuration check (dedup_init fails with DEDUP_ECUDA instead of
+// losing a launch inside a graph): true iff one CTA of fn fits on an SM.
+inline bool fits(const void* fn, int threads, size_t dyn_smem) {
+    int n = 0;
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, threads, dyn_smem) ==
+               cudaSuccess &&
+           n >= 1;
+}
+// Name of a kernel of rabin.cu / sha1.cu that cannot launch with its
+// configuration, or nullptr.
+const char* chunk_unlaunchable();
+const char* sha1_unlaunchable();
 void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mask,
                          uint32_t value, uint32_t* bitmap, uint32_t* agg, uint32_t* gagg,
                          uint32_t* gentry, uint32_t* scan_ctr, uint64_t max_tiles,

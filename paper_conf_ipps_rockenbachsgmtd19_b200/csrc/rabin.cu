@@ -760,28 +760,44 @@ __global__ void chunk_meta_kernel(const BatchDesc* __restrict__ desc,
 
 uint64_t select_groups(uint64_t max_tiles) { return (max_tiles + kGroup - 1) / kGroup; }
 
+namespace {
+void chunk_set_attrs() {
+    static bool attr_set = false;
+    if (attr_set) return;
+    for (const void* f : {(const void*)rabin_scan_agg2_kernel<true>,
+                          (const void*)rabin_scan_agg2_kernel<false>,
+                          (const void*)rabin_scan_agg_kernel<true>,
+                          (const void*)rabin_scan_agg_kernel<false>})
+        cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
+    cudaFuncSetAttribute(select_emit_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)sizeof(EmitSmem));
+    attr_set = true;
+}
+}  // namespace
+
+const char* chunk_unlaunchable() {
+    chunk_set_attrs();
+    const void* kT = kScanIlp == 2 ? (const void*)rabin_scan_agg2_kernel<true>
+                                   : (const void*)rabin_scan_agg_kernel<true>;
+    const void* kF = kScanIlp == 2 ? (const void*)rabin_scan_agg2_kernel<false>
+                                   : (const void*)rabin_scan_agg_kernel<false>;
+    if (!fits(kT, kScanThreads, kScanSmem) || !fits(kF, kScanThreads, kScanSmem))
+        return "rabin_scan_agg_kernel";
+    if (!fits((const void*)select_scan_kernel, 1024, 0)) return "select_scan_kernel";
+    if (!fits((const void*)select_emit_kernel, kEmitThreads, sizeof(EmitSmem)))
+        return "select_emit_kernel";
+    if (!fits((const void*)chunk_meta_kernel, 256, 0)) return "chunk_meta_kernel";
+    return nullptr;
+}
+
 void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mask,
                          uint32_t value, uint32_t* bitmap, uint32_t* agg, uint32_t* gagg,
                          uint32_t* gentry, uint32_t* scan_ctr, uint64_t max_tiles,
                          uint32_t* cut_pos, uint64_t cap, uint32_t* n_chunks, int num_sms,
                          cudaStream_t s, cudaEvent_t after_scan) {
-    static bool attr_set = false;
+    chunk_set_attrs();
     auto kT = kScanIlp == 2 ? rabin_scan_agg2_kernel<true> : nullptr;
     auto kF = kScanIlp == 2 ? rabin_scan_agg2_kernel<false> : nullptr;
-    if (!attr_set) {
-        if (kScanIlp == 2) {
-            cudaFuncSetAttribute(kT, cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
-            cudaFuncSetAttribute(kF, cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
-        } else {
-            cudaFuncSetAttribute(rabin_scan_agg_kernel<true>,
-                                 cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
-            cudaFuncSetAttribute(rabin_scan_agg_kernel<false>,
-                                 cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
-        }
-        cudaFuncSetAttribute(select_emit_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)sizeof(EmitSmem));
-        attr_set = true;
-    }
     const uint64_t groups = select_groups(max_tiles);
     const unsigned grid = (unsigned)num_sms;
     if (kScanIlp == 2) {

@@ -23,7 +23,21 @@ namespace dd {
 
 namespace {
 
-constexpr int kShaThreads = 128;
+#ifndef DEDUP_SHA_THREADS
+#define DEDUP_SHA_THREADS 512
+#endif
+constexpr int kShaThreads = DEDUP_SHA_THREADS;
+constexpr int kShaWarps = kShaThreads / 32;
+#ifndef DEDUP_SHA_MINB
+#define DEDUP_SHA_MINB (kShaThreads >= 768 ? 1 : 768 / kShaThreads)
+#endif
+constexpr int kShaMinBlocks = DEDUP_SHA_MINB;
+constexpr int kShaStateWords = 11;
+#ifndef DEDUP_SHA_COMPACT_EVERY
+#define DEDUP_SHA_COMPACT_EVERY 8
+#endif
+// iterations (64-byte blocks) between compaction points
+constexpr uint32_t kCompactEvery = DEDUP_SHA_COMPACT_EVERY;
 constexpr uint32_t kFull = 0xFFFFFFFFu;
 
 __device__ __forceinline__ uint32_t rotl(uint32_t x, int s) { return __funnelshift_l(x, x, s); }
@@ -124,27 +138,40 @@ __global__ void long_list_kernel(const BatchDesc* __restrict__ desc,
 }
 
 // counters[0]: work counter, counters[1]: number of long chunks.
-__global__ void __launch_bounds__(kShaThreads, 6)
+//
+// Tail compaction: once the work list is exhausted, lanes whose chunks are done
+// idle while their warp keeps issuing for the lanes still hashing (long chunks
+// outlive the bulk of a batch by up to ~4x).  Every kCompactEvery iterations
+// the live warps of the CTA meet at a named barrier; if the list is exhausted,
+// the active lanes' states (H, position, lengths) are packed through shared
+// memory into the first ceil(active/32) warps and the other warps exit, so
+// the issue slots of the tail go to lanes that do work.
+__global__ void __launch_bounds__(kShaThreads, kShaMinBlocks)
 sha1_kernel(const BatchDesc* __restrict__ desc,
             const uint32_t* __restrict__ cut_pos, const uint32_t* __restrict__ n_chunks_p,
             uint64_t cap, uint32_t long_bytes, uint32_t* counters,
             const uint32_t* __restrict__ long_list, uint8_t* __restrict__ digest, uint32_t one) {
+    __shared__ uint32_t s_state[kShaStateWords][kShaThreads];
+    __shared__ uint32_t s_warp_active[kShaWarps];
+    __shared__ uint32_t s_exhausted;
     const uint8_t* __restrict__ bytes = desc->bytes;
     const uint64_t nbytes = desc->nbytes;
     const uint32_t n = (uint32_t)min((uint64_t)*n_chunks_p, cap);
     const uint32_t n_long = *((volatile uint32_t*)&counters[1]);
     const uint32_t total = n + n_long;
     const uint32_t lane = threadIdx.x & 31;
+    uint32_t wid = threadIdx.x >> 5;
+    uint32_t live = blockDim.x >> 5;  // warps of this CTA still running (CTA-uniform)
     const uint64_t lim16 = (nbytes + 15) & ~uint64_t(15);
     int64_t k = -1;      // chunk owned by this lane
     uint64_t p = 0;      // byte offset of the next block's data
     uint32_t rem = 0;    // chunk bytes not yet consumed
     uint32_t len = 0;    // chunk length
     uint32_t phase = 0;  // 1: only the length block is left
-    bool done = false;
+    bool done = false;   // the work list is exhausted for this lane
     uint32_t H[5] = {0, 0, 0, 0, 0};
     uint32_t raw[20];    // prefetched data window of the next block
-    while (true) {
+    for (uint32_t iter = 1;; ++iter) {
         // ---- pull work: long chunks first, then all others in order ----
         while (true) {
             const bool need = !done && k < 0;
@@ -178,8 +205,66 @@ sha1_kernel(const BatchDesc* __restrict__ desc,
                 }
             }
         }
-        if (__all_sync(kFull, done)) break;
-        if (!done) {
+        if (iter % kCompactEvery == 0 && live > 1) {
+            // ---- CTA compaction point (all live warps arrive here together:
+            // every warp runs exactly one iteration per step) ----
+            const uint32_t act = __ballot_sync(kFull, k >= 0);
+            const uint32_t nthr = live * 32;
+            if (lane == 0) s_warp_active[wid] = __popc(act);
+            // one read of the (monotone) work counter makes the decision
+            // CTA-uniform: once it has passed the end, no lane can get new work
+            if (threadIdx.x == 0)
+                s_exhausted = *((volatile uint32_t*)&counters[0]) >= total ? 1u : 0u;
+            asm volatile("bar.sync 1, %0;" ::"r"(nthr) : "memory");
+            uint32_t before = 0, tot = 0;
+            for (uint32_t i = 0; i < live; ++i) {
+                const uint32_t c = s_warp_active[i];
+                before += i < wid ? c : 0;
+                tot += c;
+            }
+            const bool exhausted = s_exhausted != 0;
+            const uint32_t new_live = (tot + 31) / 32;
+            if (exhausted && new_live < live) {
+                if (k >= 0) {
+                    const uint32_t slot = before + __popc(act & ((1u << lane) - 1u));
+#pragma unroll
+                    for (int i = 0; i < 5; ++i) s_state[i][slot] = H[i];
+                    s_state[5][slot] = (uint32_t)k;
+                    s_state[6][slot] = (uint32_t)p;
+                    s_state[7][slot] = (uint32_t)(p >> 32);
+                    s_state[8][slot] = rem;
+                    s_state[9][slot] = len;
+                    s_state[10][slot] = phase;
+                }
+                asm volatile("bar.sync 1, %0;" ::"r"(nthr) : "memory");
+                if (wid >= new_live) return;  // CTA-uniform per warp
+                const uint32_t slot = wid * 32 + lane;
+                if (slot < tot) {
+#pragma unroll
+                    for (int i = 0; i < 5; ++i) H[i] = s_state[i][slot];
+                    k = s_state[5][slot];
+                    p = (uint64_t)s_state[6][slot] | ((uint64_t)s_state[7][slot] << 32);
+                    rem = s_state[8][slot];
+                    len = s_state[9][slot];
+                    phase = s_state[10][slot];
+                    if (phase == 0 && rem > 0) load_raw<true>(bytes, p, lim16, raw);
+                } else {
+                    k = -1;
+                }
+                done = true;
+                live = new_live;
+                // the slots are reused at the next compaction point only after
+                // every remaining warp has read its state
+                asm volatile("bar.sync 1, %0;" ::"r"(new_live * 32) : "memory");
+            } else {
+                // keep s_warp_active stable until everyone has read it
+                asm volatile("bar.sync 1, %0;" ::"r"(nthr) : "memory");
+            }
+            if (tot == 0 && exhausted) return;
+        } else if (live == 1 && __all_sync(kFull, done && k < 0)) {
+            return;
+        }
+        if (k >= 0) {
             uint32_t M[16];
             bool fin = false;
             if (phase == 0) {
@@ -236,6 +321,12 @@ sha1_kernel(const BatchDesc* __restrict__ desc,
 
 }  // namespace
 
+const char* sha1_unlaunchable() {
+    if (!fits((const void*)long_list_kernel, 256, 0)) return "long_list_kernel";
+    if (!fits((const void*)sha1_kernel, kShaThreads, 0)) return "sha1_kernel";
+    return nullptr;
+}
+
 void launch_sha1(const BatchDesc* d, uint64_t max_bytes, const uint32_t* cut_pos,
                  const uint32_t* n_chunks, uint64_t cap, uint32_t long_bytes, uint32_t* counters,
                  uint32_t* long_list, uint8_t* digest, int num_sms, cudaStream_t s) {
@@ -248,7 +339,7 @@ void launch_sha1(const BatchDesc* d, uint64_t max_bytes, const uint32_t* cut_pos
     uint64_t lanes = max_bytes / kShaLaneBytes;
     if (lanes < 1024) lanes = 1024;
     uint64_t blocks = (lanes + kShaThreads - 1) / kShaThreads;
-    if (blocks > (uint64_t)num_sms * 6) blocks = (uint64_t)num_sms * 6;
+    if (blocks > (uint64_t)num_sms * kShaMinBlocks) blocks = (uint64_t)num_sms * kShaMinBlocks;
     uint64_t lb = (cap + 255) / 256;
     if (lb > (uint64_t)num_sms * 2) lb = (uint64_t)num_sms * 2;
     if (lb < 1) lb = 1;
