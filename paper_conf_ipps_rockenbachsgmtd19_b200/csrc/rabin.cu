@@ -122,7 +122,17 @@ __device__ __forceinline__ uint32_t roll32(uint32_t& h, const uint32_t cur[8],
     return bits;
 }
 
+#ifndef DEDUP_SCAN_EXPERIMENT
+#define DEDUP_SCAN_EXPERIMENT 0  // timing experiments only (results invalid): 4 = no
+                                 // global loads in the scan, 8 = no per-tile epilogue
+#endif
+
 __device__ __forceinline__ void load32(const uint8_t* p, uint32_t v[8]) {
+    if (DEDUP_SCAN_EXPERIMENT & 4) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) v[i] = (uint32_t)(uintptr_t)p * 2654435761u + i;
+        return;
+    }
     const uint4 a = __ldg(reinterpret_cast<const uint4*>(p));
     const uint4 b = __ldg(reinterpret_cast<const uint4*>(p + 16));
     v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
@@ -133,8 +143,56 @@ __device__ __forceinline__ void load32(const uint8_t* p, uint32_t v[8]) {
 // 16) read as zero.
 __device__ __forceinline__ void load32_any(const uint8_t* base, uint64_t off, uint64_t nbytes,
                                            uint64_t lim16, uint32_t v[8]) {
-    if (off + 32 <= nbytes) {
+    if (off + 32 <= nbytes || (DEDUP_SCAN_EXPERIMENT & 4)) {
         load32(base + off, v);
+        return;
+    }
+    uint4 a = make_uint4(0, 0, 0, 0), b = make_uint4(0, 0, 0, 0);
+    if (off < lim16) a = __ldg(reinterpret_cast<const uint4*>(base + off));
+    if (off + 16 < lim16) b = __ldg(reinterpret_cast<const uint4*>(base + off + 16));
+    v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
+    v[4] = b.x; v[5] = b.y; v[6] = b.z; v[7] = b.w;
+}
+
+// 16 bytes at off (16-byte aligned); vectors at or beyond lim16 read as zero.
+__device__ __forceinline__ void load16_any(const uint8_t* base, uint64_t off, uint64_t lim16,
+                                           uint32_t v[4]) {
+    if (DEDUP_SCAN_EXPERIMENT & 4) {
+#pragma unroll
+        for (int i = 0; i < 4; ++i) v[i] = (uint32_t)off * 2654435761u + i;
+        return;
+    }
+    uint4 a = make_uint4(0, 0, 0, 0);
+    if (off < lim16) a = __ldg(reinterpret_cast<const uint4*>(base + off));
+    v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
+}
+
+// 32 bytes at off with one 256-bit load (LDG.E.256, sm_100) when the address
+// is 32-byte aligned (a32) and the whole vector lies below lim16, else as
+// 16-byte vectors (at or beyond lim16: zero).  One request per lane-sector
+// instead of two halves the L1 tag work of the lane-strided scan loads.
+__device__ __forceinline__ void load32_v8(const uint8_t* base, uint32_t off, uint32_t lim16,
+                                          bool a32, uint32_t v[8]) {
+    if (DEDUP_SCAN_EXPERIMENT & 4) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) v[i] = off * 2654435761u + i;
+        return;
+    }
+    if (a32 && off + 32 <= lim16) {
+#ifndef DEDUP_SCAN_LDHINT
+#define DEDUP_SCAN_LDHINT 0  // 1: L1::no_allocate, 2: L2::256B prefetch (timing knobs)
+#endif
+#if DEDUP_SCAN_LDHINT == 1
+#define DEDUP_LDV8 "ld.global.nc.L1::no_allocate.v8.u32"
+#elif DEDUP_SCAN_LDHINT == 2
+#define DEDUP_LDV8 "ld.global.nc.L2::256B.v8.u32"
+#else
+#define DEDUP_LDV8 "ld.global.nc.v8.u32"
+#endif
+        asm(DEDUP_LDV8 " {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+            : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]),
+              "=r"(v[6]), "=r"(v[7])
+            : "l"(base + off));
         return;
     }
     uint4 a = make_uint4(0, 0, 0, 0), b = make_uint4(0, 0, 0, 0);
@@ -375,7 +433,7 @@ rabin_scan_agg_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __rest
         const uint64_t q = T0 + (uint64_t)lane * kLaneBytes;
         // ---- scan: 8 steps of 32 bytes, bits written in e-space ----
         uint32_t h = 0, prev_bits = 0;
-#if defined(DEDUP_SCAN_EXPERIMENT) && (DEDUP_SCAN_EXPERIMENT & 2)
+#if DEDUP_SCAN_EXPERIMENT & 2
         if (false) {  // timing experiment only: no warm-up
 #else
         if (q >= 32) {  // warm-up: the window ending at q-1 -> bit for e = q
@@ -447,19 +505,41 @@ rabin_scan_agg_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __rest
 
 // Two independent rolling chains per lane (ILP 2): the LDS -> LOP3 -> PRMT
 // dependency of one chain overlaps with the other's.
-template <bool kZeroValue>
+// Words [W0, W1) of the 32-byte step; bits accumulate into bitsA / bitsB.
+#ifndef DEDUP_SCAN_FMA_AR
+#define DEDUP_SCAN_FMA_AR 0
+#endif
+__device__ __forceinline__ uint32_t mad_hi_u32(uint32_t a, uint32_t b, uint32_t c) {
+    uint32_t d;
+    asm("mad.hi.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
+    return d;
+}
+__device__ __forceinline__ uint32_t mad_lo_u32(uint32_t a, uint32_t b, uint32_t c) {
+    uint32_t d;
+    asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
+    return d;
+}
+// LDS address of R[h >> 24] for this lane.  PRMT (ALU pipe), or with
+// DEDUP_SCAN_FMA_AR two FMA-pipe ops (c256 = 256 at run time, so that ptxas
+// keeps the IMADs): (h >> 24) = mad.hi(h, 256), then * 256 + laneR.
+__device__ __forceinline__ uint32_t addr_r(uint32_t h, uint32_t laneR, uint32_t c256) {
+    if (DEDUP_SCAN_FMA_AR) return mad_lo_u32(mad_hi_u32(h, c256, 0u), c256, laneR);
+    return __byte_perm(h, laneR, 0x7634);
+}
+
+template <bool kZeroValue, int W0 = 0, int W1 = 8>
 __device__ __forceinline__ void roll32x2(uint32_t& hA, const uint32_t curA[8],
                                          const uint32_t oldA[8], uint32_t& bitsA, uint32_t& hB,
                                          const uint32_t curB[8], const uint32_t oldB[8],
                                          uint32_t& bitsB, uint32_t laneR, uint32_t laneW,
-                                         uint32_t mask, uint32_t value) {
-    bitsA = bitsB = 0;
+                                         uint32_t mask, uint32_t value, uint32_t c256) {
+    if (W0 == 0) bitsA = bitsB = 0;
 #pragma unroll
-    for (int w = 0; w < 8; ++w) {
+    for (int w = W0; w < W1; ++w) {
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
-            const uint32_t aRA = __byte_perm(hA, laneR, 0x7634);
-            const uint32_t aRB = __byte_perm(hB, laneR, 0x7634);
+            const uint32_t aRA = addr_r(hA, laneR, c256);
+            const uint32_t aRB = addr_r(hB, laneR, c256);
             const uint32_t aWA = __byte_perm(oldA[w], laneW, 0x7604 | (k << 4));
             const uint32_t aWB = __byte_perm(oldB[w], laneW, 0x7604 | (k << 4));
             const uint32_t hsA = __byte_perm(curA[w], hA, 0x6540 | k);
@@ -478,18 +558,48 @@ __device__ __forceinline__ void roll32x2(uint32_t& hA, const uint32_t curA[8],
     }
 }
 
+// L2 prefetch of tile t's bytes (and the 32 warm-up bytes before it) by the
+// TMA unit: one bulk request per tile, no registers, issued a whole group
+// ahead so that the per-step loads of the roll hit L2 instead of HBM.
+__device__ __forceinline__ void prefetch_tile_l2(const uint8_t* bytes, uint64_t t,
+                                                 uint64_t lim16) {
+    uint64_t a = t * kSelTile;
+    if (a >= lim16) return;
+    a = a >= 32 ? a - 32 : 0;
+    uint64_t n = kSelTile + 32;
+    if (a + n > lim16) n = lim16 - a;
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(bytes + a), "r"((uint32_t)n)
+                 : "memory");
+}
+
+// Measured (isolated chunk stage, 256 MiB): no prefetch 938 GB/s, register
+// prefetch 949, L2 bulk prefetch 899, both 890 -- the scan is not load-latency
+// bound at 16 warps x 2 chains per SM.
+#ifndef DEDUP_SCAN_L2PF
+#define DEDUP_SCAN_L2PF 0
+#endif
+#ifndef DEDUP_SCAN_REGPF
+#define DEDUP_SCAN_REGPF 1
+#endif
+// 1: the next step's 32 bytes come with one 256-bit load at the end of a step
+// (instead of two 128-bit loads at the halves); needs DEDUP_SCAN_REGPF.
+#ifndef DEDUP_SCAN_V8
+#define DEDUP_SCAN_V8 1
+#endif
+
 // ILP-2 scan: a CTA of kScanWarps warps takes groups of 2 x kScanWarps tiles;
 // warp w rolls tiles w and w + kScanWarps of the group together.
 template <bool kZeroValue>
 __global__ void __launch_bounds__(kScanThreads, 2)
 rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ gtab,
                        uint32_t mask, uint32_t value, uint32_t* __restrict__ bitmap,
-                       uint32_t* __restrict__ agg, uint32_t* __restrict__ gagg) {
+                       uint32_t* __restrict__ agg, uint32_t* __restrict__ gagg,
+                       uint32_t c256) {
     extern __shared__ __align__(16) uint8_t smem[];
     __shared__ uint32_t src[512];
     __shared__ uint32_t fun[kFunBufs][kGroup][32];
     const uint8_t* __restrict__ bytes = desc->bytes;
-    const uint64_t nbytes = desc->nbytes;
+    const uint32_t nbytes = (uint32_t)desc->nbytes;  // <= 2^30 (check_cfg)
     const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t win = (uint32_t)__cvta_generic_to_shared(smem);
     const uint32_t pad = (0x10000u - (win & 0xFFFFu)) & 0xFFFFu;
@@ -498,6 +608,13 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
     if (pad < (uint32_t)kScanAux) __trap();  // layout assumption (see kScanSmem)
     uint64_t* icache = reinterpret_cast<uint64_t*>(wsm + kScanWarps);
     SelWarpSmem& sm = wsm[wid];
+    const uint32_t n_tiles = (nbytes + kSelTile - 1) / kSelTile;
+    const uint32_t n_groups = (n_tiles + kGroup - 1) / kGroup;
+    const uint32_t lim16 = (nbytes + 15) & ~15u;
+    if (DEDUP_SCAN_L2PF && lane == 0 && blockIdx.x < n_groups) {  // first group, during the table build
+        prefetch_tile_l2(bytes, (uint64_t)blockIdx.x * kGroup + wid, lim16);
+        prefetch_tile_l2(bytes, (uint64_t)blockIdx.x * kGroup + wid + kScanWarps, lim16);
+    }
     if (threadIdx.x < 512) src[threadIdx.x] = gtab[threadIdx.x];
     const uint64_t* items = cache_items(icache, desc);
     const uint32_t n_items = desc->n_items;
@@ -509,44 +626,81 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
     }
     __syncthreads();
     if (nbytes == 0) return;
-    const uint64_t n_tiles = (nbytes + kSelTile - 1) / kSelTile;
-    const uint64_t n_groups = (n_tiles + kGroup - 1) / kGroup;
-    const uint64_t lim16 = (nbytes + 15) & ~uint64_t(15);
     const uint32_t laneR = base | (lane * 4);
     const uint32_t laneW = laneR + 128;
+    const bool a32 = (reinterpret_cast<uintptr_t>(bytes) & 31) == 0;
     int par = 0;
-    for (uint64_t g = blockIdx.x; g < n_groups; g += gridDim.x, par ^= 1) {
-        const uint64_t tA = g * kGroup + wid, tB = tA + kScanWarps;
-        const uint64_t qA = tA * kSelTile + (uint64_t)lane * kLaneBytes;
-        const uint64_t qB = tB * kSelTile + (uint64_t)lane * kLaneBytes;
+    for (uint32_t g = blockIdx.x; g < n_groups; g += gridDim.x, par ^= 1) {
+        const uint32_t tA = g * kGroup + wid, tB = tA + kScanWarps;
+        if (DEDUP_SCAN_L2PF && lane == 0 && g + gridDim.x < n_groups) {  // next group
+            prefetch_tile_l2(bytes, tA + gridDim.x * kGroup, lim16);
+            prefetch_tile_l2(bytes, tB + gridDim.x * kGroup, lim16);
+        }
+        const uint32_t qA = tA * kSelTile + lane * kLaneBytes;
+        const uint32_t qB = tB * kSelTile + lane * kLaneBytes;
         uint32_t prevA[8], curA[8], prevB[8], curB[8];
 #pragma unroll
         for (int i = 0; i < 8; ++i) prevA[i] = curA[i] = prevB[i] = curB[i] = 0;
-        if (qA >= 32 && qA < nbytes) load32(bytes + qA - 32, prevA);
-        if (qB >= 32 && qB < nbytes) load32(bytes + qB - 32, prevB);
-        if (qA < nbytes) load32_any(bytes, qA, nbytes, lim16, curA);
-        if (qB < nbytes) load32_any(bytes, qB, nbytes, lim16, curB);
+        if (DEDUP_SCAN_V8) {
+            if (qA >= 32 && qA < nbytes) load32_v8(bytes, qA - 32, lim16, a32, prevA);
+            if (qB >= 32 && qB < nbytes) load32_v8(bytes, qB - 32, lim16, a32, prevB);
+            if (qA < nbytes) load32_v8(bytes, qA, lim16, a32, curA);
+            if (qB < nbytes) load32_v8(bytes, qB, lim16, a32, curB);
+        } else {
+            if (qA >= 32 && qA < nbytes) load32(bytes + qA - 32, prevA);
+            if (qB >= 32 && qB < nbytes) load32(bytes + qB - 32, prevB);
+            if (qA < nbytes) load32_any(bytes, qA, nbytes, lim16, curA);
+            if (qB < nbytes) load32_any(bytes, qB, nbytes, lim16, curB);
+        }
         uint32_t hA = 0, hB = 0, pbA = 0, pbB = 0;
         {   // warm-up of both chains: the windows ending at q-1
             const uint32_t zero[8] = {0, 0, 0, 0, 0, 0, 0, 0};
             uint32_t bA, bB;
             roll32x2<kZeroValue>(hA, prevA, zero, bA, hB, prevB, zero, bB, laneR, laneW, mask,
-                                 value);
+                                 value, c256);
             pbA = qA >= 32 ? bA : 0;
             pbB = qB >= 32 ? bB : 0;
             if (qA < 32) hA = 0;
             if (qB < 32) hB = 0;
         }
-#pragma unroll 1
-        for (int j = 0; j < 8; ++j) {
-            const uint64_t bA0 = qA + 32 * j, bB0 = qB + 32 * j;
+        // One 32-byte step of both chains: roll `in` against `old`, then the
+        // bits in e-space.  With DEDUP_SCAN_REGPF the registers of `old` are
+        // recycled: once a half (16 bytes) of `old` has been rolled out, the
+        // same four registers receive the NEXT step's bytes of that half, so
+        // the loads fly for a whole step with no extra registers; `in` and
+        // `old` swap roles every step (the loop body holds two steps).
+        auto step = [&](int j, uint32_t (&inA)[8], uint32_t (&oldA)[8], uint32_t (&inB)[8],
+                        uint32_t (&oldB)[8]) {
+            const uint32_t bA0 = qA + 32 * j, bB0 = qB + 32 * j;
+#if !DEDUP_SCAN_REGPF
             if (j > 0) {
-                if (bA0 < nbytes) load32_any(bytes, bA0, nbytes, lim16, curA);
-                if (bB0 < nbytes) load32_any(bytes, bB0, nbytes, lim16, curB);
+                if (bA0 < nbytes) load32_any(bytes, bA0, nbytes, lim16, inA);
+                if (bB0 < nbytes) load32_any(bytes, bB0, nbytes, lim16, inB);
             }
+#endif
             uint32_t bitsA, bitsB;
-            roll32x2<kZeroValue>(hA, curA, prevA, bitsA, hB, curB, prevB, bitsB, laneR, laneW,
-                                 mask, value);
+            roll32x2<kZeroValue, 0, 4>(hA, inA, oldA, bitsA, hB, inB, oldB, bitsB, laneR, laneW,
+                                       mask, value, c256);
+#if DEDUP_SCAN_REGPF && !DEDUP_SCAN_V8
+            if (j < 7) {
+                load16_any(bytes, bA0 + 32, lim16, oldA);
+                load16_any(bytes, bB0 + 32, lim16, oldB);
+            }
+#endif
+            roll32x2<kZeroValue, 4, 8>(hA, inA, oldA, bitsA, hB, inB, oldB, bitsB, laneR, laneW,
+                                       mask, value, c256);
+#if DEDUP_SCAN_REGPF && !DEDUP_SCAN_V8
+            if (j < 7) {
+                load16_any(bytes, bA0 + 48, lim16, oldA + 4);
+                load16_any(bytes, bB0 + 48, lim16, oldB + 4);
+            }
+#endif
+#if DEDUP_SCAN_REGPF && DEDUP_SCAN_V8
+            if (j < 7) {
+                load32_v8(bytes, bA0 + 32, lim16, a32, oldA);
+                load32_v8(bytes, bB0 + 32, lim16, a32, oldB);
+            }
+#endif
             uint32_t ewA = __funnelshift_l(pbA, bitsA, 1), ewB = __funnelshift_l(pbB, bitsB, 1);
             if (bA0 >= nbytes) ewA = 0;
             else if (bA0 + 32 > nbytes) ewA &= (1u << (uint32_t)(nbytes - bA0)) - 1u;
@@ -559,15 +713,27 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
             if (tB < n_tiles) bitmap[tB * kSelTileWords + lane * 8 + j] = ewB;
             pbA = bitsA;
             pbB = bitsB;
+        };
+#if DEDUP_SCAN_REGPF
+#pragma unroll 1
+        for (int j = 0; j < 8; j += 2) {
+            step(j, curA, prevA, curB, prevB);      // prev now holds step j+1's bytes
+            step(j + 1, prevA, curA, prevB, curB);  // cur now holds step j+2's bytes
+        }
+#else
+#pragma unroll 1
+        for (int j = 0; j < 8; ++j) {
+            step(j, curA, prevA, curB, prevB);
 #pragma unroll
             for (int i = 0; i < 8; ++i) {
                 prevA[i] = curA[i];
                 prevB[i] = curB[i];
             }
         }
+#endif
         // transfer functions of tile A (candidate words already in smem), then B
         uint32_t fA = (uint32_t)lane << 27, fB = fA;
-        if (tA < n_tiles) {
+        if (tA < n_tiles && !(DEDUP_SCAN_EXPERIMENT & 8)) {
             const uint32_t n_ev = apply_items(sm, tA * kSelTile, nbytes, items, n_items, lane);
             uint32_t ex;
             const uint32_t cnt = walk_any(sm, n_ev, lane, ex, nullptr, 0, 0, 0);
@@ -575,7 +741,7 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
             agg[32 * tA + lane] = fA;
         }
         __syncwarp();
-        if (tB < n_tiles) {
+        if (tB < n_tiles && !(DEDUP_SCAN_EXPERIMENT & 8)) {
 #pragma unroll
             for (int k = 0; k < 8; ++k)
                 sm.cand[lane * 8 + k] = bitmap[tB * kSelTileWords + lane * 8 + k];
@@ -802,7 +968,7 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
     const unsigned grid = (unsigned)num_sms;
     if (kScanIlp == 2) {
         (value == 0 ? kT : kF)<<<grid, kScanThreads, kScanSmem, s>>>(d, d_tab, mask, value,
-                                                                     bitmap, agg, gagg);
+                                                                     bitmap, agg, gagg, 256u);
     } else {
         cudaMemsetAsync(scan_ctr, 0, sizeof(uint32_t) * (groups + 2), s);
         if (value == 0)

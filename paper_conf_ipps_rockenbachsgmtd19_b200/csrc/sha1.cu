@@ -42,10 +42,48 @@ constexpr uint32_t kFull = 0xFFFFFFFFu;
 
 __device__ __forceinline__ uint32_t rotl(uint32_t x, int s) { return __funnelshift_l(x, x, s); }
 
+#ifndef DEDUP_SHA_FMA
+#define DEDUP_SHA_FMA 0
+#endif
+
+// Pipe balancing.  LOP3/SHF/LEA issue to the ALU pipe and IMAD/VIADD to the
+// FMA pipe, each at half a warp instruction per clock per SMSP
+// (B300_MICROARCH.md "Pipe rates").  As compiled, a round is LOP3 (f), LEA.HI
+// (rotl5 + x), SHF (rotl30) on the ALU pipe and IMAD.IADD, IMAD (w + ...),
+// VIADD (K) on the FMA pipe, and the schedule is 2 LOP3 + 1 SHF: ~432 ALU vs
+// ~240 FMA ops per block (ncu: ALU 51 %, FMA-heavy ~1.6x less busy), so the
+// block is ALU-bound.  A rotate by s is x * 2^s + (x >> (32 - s)) (the parts
+// do not overlap), i.e. mad.lo(x, 2^s, mad.hi(x, 2^s, 0)): two FMA-pipe ops
+// for one ALU op.  DEDUP_SHA_FMA bit 0 moves the 64 schedule rotl1 (-> ~368
+// on each pipe), bit 1 the 80 rotl30.  The multipliers are kernel arguments
+// (runtime values) so that ptxas cannot turn them back into shifts.
+// Measured (1 GiB of 4 KiB chunks, B200): 0 -> 1750 GB/s, 1 -> 1626, 3 -> 1254:
+// the kernel is issue/latency-bound, not ALU-pipe-bound, so extra instructions
+// cost more than the pipe balance gains.  Default 0.
+struct ShaMul {
+    uint32_t one, two, p30;  // 1, 2, 2^30 at run time
+};
+
+__device__ __forceinline__ uint32_t mad_hi(uint32_t a, uint32_t b, uint32_t c) {
+    uint32_t d;
+    asm("mad.hi.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
+    return d;
+}
+__device__ __forceinline__ uint32_t mad_lo(uint32_t a, uint32_t b, uint32_t c) {
+    uint32_t d;
+    asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
+    return d;
+}
+// rotl(x, s) on the FMA pipe, m = 2^s (runtime)
+__device__ __forceinline__ uint32_t rotl_fma(uint32_t x, uint32_t m) {
+    return mad_lo(x, m, mad_hi(x, m, 0u));
+}
+
 // `one` is a runtime 1 (kernel argument): w * one + K compiles to an IMAD on
 // the FMA pipe that ptxas cannot fold back onto the a -> a' dependency chain,
 // leaving LEA.HI (rotl(a,5) + x) as the only op on it.
-__device__ __forceinline__ void sha1_compress(uint32_t H[5], uint32_t W[16], uint32_t one) {
+__device__ __forceinline__ void sha1_compress(uint32_t H[5], uint32_t W[16], ShaMul m) {
+    const uint32_t one = m.one;
     uint32_t a = H[0], b = H[1], c = H[2], d = H[3], e = H[4];
 #pragma unroll
     for (int t = 0; t < 80; ++t) {
@@ -53,7 +91,8 @@ __device__ __forceinline__ void sha1_compress(uint32_t H[5], uint32_t W[16], uin
         if (t < 16) {
             w = W[t];
         } else {
-            w = rotl(W[(t - 3) & 15] ^ W[(t - 8) & 15] ^ W[(t - 14) & 15] ^ W[t & 15], 1);
+            const uint32_t x = W[(t - 3) & 15] ^ W[(t - 8) & 15] ^ W[(t - 14) & 15] ^ W[t & 15];
+            w = (DEDUP_SHA_FMA & 1) ? rotl_fma(x, m.two) : rotl(x, 1);
             W[t & 15] = w;
         }
         uint32_t f, K;
@@ -75,7 +114,7 @@ __device__ __forceinline__ void sha1_compress(uint32_t H[5], uint32_t W[16], uin
         const uint32_t T = rotl(a, 5) + x;
         e = d;
         d = c;
-        c = rotl(b, 30);
+        c = (DEDUP_SHA_FMA & 2) ? rotl_fma(b, m.p30) : rotl(b, 30);
         b = a;
         a = T;
     }
@@ -150,7 +189,7 @@ __global__ void __launch_bounds__(kShaThreads, kShaMinBlocks)
 sha1_kernel(const BatchDesc* __restrict__ desc,
             const uint32_t* __restrict__ cut_pos, const uint32_t* __restrict__ n_chunks_p,
             uint64_t cap, uint32_t long_bytes, uint32_t* counters,
-            const uint32_t* __restrict__ long_list, uint8_t* __restrict__ digest, uint32_t one) {
+            const uint32_t* __restrict__ long_list, uint8_t* __restrict__ digest, ShaMul mul) {
     __shared__ uint32_t s_state[kShaStateWords][kShaThreads];
     __shared__ uint32_t s_warp_active[kShaWarps];
     __shared__ uint32_t s_exhausted;
@@ -308,7 +347,7 @@ sha1_kernel(const BatchDesc* __restrict__ desc,
                 M[15] = len << 3;
                 fin = true;
             }
-            sha1_compress(H, M, one);
+            sha1_compress(H, M, mul);
             if (fin) {
                 uint32_t* out = reinterpret_cast<uint32_t*>(digest + 20 * (uint64_t)k);
 #pragma unroll
@@ -346,7 +385,8 @@ void launch_sha1(const BatchDesc* d, uint64_t max_bytes, const uint32_t* cut_pos
     long_list_kernel<<<(unsigned)lb, 256, 0, s>>>(d, cut_pos, n_chunks, cap, long_bytes, counters,
                                                   long_list);
     sha1_kernel<<<(unsigned)blocks, kShaThreads, 0, s>>>(d, cut_pos, n_chunks, cap, long_bytes,
-                                                         counters, long_list, digest, 1u);
+                                                         counters, long_list, digest,
+                                                         ShaMul{1u, 2u, 1u << 30});
 }
 
 }  // namespace dd
