@@ -51,8 +51,13 @@ METRIC = "input GB/s & chunks/s (dedup hot path) at 1/2/4/8 B200; % of HBM/INT r
 # counting a 3-input logic/add as one op and a rotate as one op):
 #   80 rounds x (f 1 + rotl5 1 + adds 2 + rotl30 1) + 64 x schedule 3 + 5.
 SHA1_OPS_PER_BLOCK = 80 * 5 + 64 * 3 + 5
-# alu-pipe peak (LOP3/SHF/IADD3/PRMT): 148 SM x 4 SMSP x 16 lanes/clk
-ALU_LANES_PER_SM_CLK = 64
+# Rabin rolling step per input byte: 2 table lookups, shift-in,
+# 2 address formations, 1 3-way XOR, test + bit = 8 ops.
+SCAN_OPS_PER_BYTE = 8
+# Integer-op peak = instruction issue: 148 SM x 4 SMSP x 1 warp-instr/clk x 32
+# lanes (B300_MICROARCH.md: 4 SMSPs, ALU and FMA pipes 16 lanes/clk each per
+# SMSP, so a mix of ALU-pipe and IMAD ops can fill every issue slot).
+INT_LANES_PER_SM_CLK = 128
 
 
 def engine_kwargs(stream_bytes: int) -> dict:
@@ -229,6 +234,73 @@ def reference_arm(args, data, off):
     print(json.dumps(line), flush=True)
 
 
+def isolated_kernels(dd, off, int_peak, copies=4, reps=3, streams=4):
+    """Live per-kernel throughput with the GPU filled by one kernel type.
+
+    chunk stage: one op_chunk call (scan + select) over the C2 stream tiled
+    `copies` times (a full-GPU grid).  SHA-1: one launch's duration is floored
+    by the longest chunk's serial chain of 64-byte compressions (latency, not
+    throughput), so `streams` contexts launch the same SHA-1 work concurrently
+    on their own streams and the throughput is all their blocks over the
+    joint elapsed time.  CUDA events on torch's current stream bracket both."""
+    import torch
+
+    from paper_conf_ipps_rockenbachsgmtd19_b200 import Dedup
+    nb1 = int(off[-1])
+    data = dd.repeat(copies)
+    nb = nb1 * copies
+    n_items = (len(off) - 1) * copies
+    offs = np.concatenate([off[:-1] + k * nb1 for k in range(copies)] + [np.array([nb], off.dtype)])
+    item_off = torch.from_numpy(offs.astype(np.int64)).cuda()
+    cap = nb // 32 + n_items + 2
+    ctxs = [Dedup(0, batch_bytes=nb, batch_items=n_items + 1, slots=1, table_capacity=1 << 12,
+                  host_fed=False) for _ in range(streams)]
+    try:
+        cut = torch.zeros(cap, dtype=torch.int32, device="cuda")
+        n = torch.zeros(1, dtype=torch.int32, device="cuda")
+        digs = [torch.zeros(cap * 20, dtype=torch.uint8, device="cuda") for _ in range(streams)]
+        sts = [torch.cuda.Stream() for _ in range(streams)]
+        ev = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
+        ctxs[0].op_chunk(data, nb, item_off, n_items, cut, cap, n)   # warm-up
+        ctxs[0].op_sha1(data, nb, cut, n, cap, digs[0])
+        torch.cuda.synchronize()
+        ev[0].record()
+        for _ in range(reps):
+            ctxs[0].op_chunk(data, nb, item_off, n_items, cut, cap, n)
+        ev[1].record()
+        for k in range(streams):
+            sts[k].wait_event(ev[1])
+            for _ in range(reps):
+                ctxs[k].op_sha1(data, nb, cut, n, cap, digs[k], stream=sts[k].cuda_stream)
+            torch.cuda.current_stream().wait_stream(sts[k])
+        ev[2].record()
+        ev[2].synchronize()
+        chunk_us = ev[0].elapsed_time(ev[1]) * 1e3 / reps
+        sha_us = ev[1].elapsed_time(ev[2]) * 1e3 / (reps * streams)  # per launch's worth
+        k = int(n.item())
+        cp = cut[:k].cpu().numpy().astype(np.int64)
+    finally:
+        for c in ctxs:
+            c.close()
+    lens = np.diff(np.append(cp, nb))
+    blocks = int(((lens + 9 + 63) // 64).sum())
+    sha_ops = blocks * SHA1_OPS_PER_BLOCK / (sha_us * 1e-6) / 1e12
+    scan_ops = nb * SCAN_OPS_PER_BYTE / (chunk_us * 1e-6) / 1e12
+    return {
+        "sha1": {"bound": "alu", "achieved": sha_ops, "peak": int_peak, "unit": "Tops/s",
+                 "frac": sha_ops / int_peak, "launch_us": sha_us, "launch_bytes": nb,
+                 "input_gbs": nb / (sha_us * 1e-6) / 1e9, "blocks": blocks,
+                 "note": f"{streams} concurrent streams x {reps} launches; launch_us = "
+                         "joint elapsed / launches"},
+        "chunk_stage": {"bound": "alu", "achieved": scan_ops, "peak": int_peak, "unit": "Tops/s",
+                        "frac": scan_ops / int_peak, "launch_us": chunk_us,
+                        "input_gbs": nb / (chunk_us * 1e-6) / 1e9,
+                        "note": "scan + select_scan + select_emit, one op_chunk call; "
+                                "HBM: reads 1 B/B -> "
+                                f"{nb / (chunk_us * 1e-6) / 1e9 / 6462.1:.3f} of the copy peak"},
+    }
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -301,40 +373,49 @@ def main():
     value = bytes_timed / (ms / 1e3) / 1e9
     chunks_per_s = ds["chunks"] / (ms / 1e3)
 
-    # ---- roofline of the dominant kernel (live CUDA-event stage times) ----
+    # ---- rooflines ----
     pk, src = peaks()
     clocks = clk.summary()
     sm_mhz = pk.get("sm_max_mhz", 1965.0)
-    alu_peak = 148 * ALU_LANES_PER_SM_CLK * sm_mhz * 1e6 / 1e12      # Tops/s
-    # stage times are CUDA events of every DEDUP_TIME_EVERY-th batch (sampled)
+    int_peak = 148 * INT_LANES_PER_SM_CLK * sm_mhz * 1e6 / 1e12      # Tops/s
+    peak_source = (f"derived: 148 SM x 4 SMSP x 32 lanes (1 warp-instr/clk/SMSP) x "
+                   f"{sm_mhz:.0f} MHz ({src} max SM clock); B200_PROFILING.md has no "
+                   "integer peak")
+    # pipeline stage latencies: CUDA events of every DEDUP_TIME_EVERY-th batch on
+    # the slot's own stream (the stages of ~SLOTS batches overlap, so these are
+    # latencies, not costs)
     nt = max(ds["timed_batches"], 1)
-    sha_achieved = ds["timed_sha1_blocks"] * SHA1_OPS_PER_BLOCK / max(ds["ms_sha1"] / 1e3,
-                                                                     1e-12) / 1e12
-    scan_achieved = ds["timed_bytes"] * (1 + 1 / 8) / max(ds["ms_scan"] / 1e3, 1e-12) / 1e9
     kernels = {
-        "sha1": {"ms_per_batch": ds["ms_sha1"] / nt, "bound": "alu",
-                 "achieved": sha_achieved, "peak": alu_peak, "unit": "Tops/s",
-                 "frac": sha_achieved / alu_peak},
-        "rabin_scan": {"ms_per_batch": ds["ms_scan"] / nt, "bound": "hbm",
-                       "achieved": scan_achieved, "peak": pk["hbm_gbs"], "unit": "GB/s",
-                       "frac": scan_achieved / pk["hbm_gbs"]},
-        "select+meta": {"ms_per_batch": ds["ms_select"] / nt},
-        "table": {"ms_per_batch": ds["ms_table"] / nt},
-        "pack_d2h": {"ms_per_batch": ds["ms_d2h"] / nt},
+        "stage_latency_ms_per_batch": {
+            "rabin_scan": ds["ms_scan"] / nt, "select+meta": ds["ms_select"] / nt,
+            "sha1": ds["ms_sha1"] / nt, "table": ds["ms_table"] / nt,
+            "pack_d2h": ds["ms_d2h"] / nt},
         "timed_batches": ds["timed_batches"],
     }
-    dom = "sha1" if ds["ms_sha1"] >= ds["ms_scan"] else "rabin_scan"
-    kd = kernels[dom]
+    iso = isolated_kernels(dd, off, int_peak)
+    kernels.update(iso)
+    sha_blocks_per_byte = ds["sha1_blocks"] / max(ds["bytes"], 1)
+    path_ops = value * 1e9 * (SCAN_OPS_PER_BYTE + sha_blocks_per_byte * SHA1_OPS_PER_BLOCK) / 1e12
+    kernels["path"] = {"bound": "alu", "achieved": path_ops, "peak": int_peak, "unit": "Tops/s",
+                       "frac": path_ops / int_peak,
+                       "ops_per_byte": SCAN_OPS_PER_BYTE + sha_blocks_per_byte * SHA1_OPS_PER_BLOCK,
+                       "note": "whole step: algorithmic scan + SHA-1 int ops at `value`"}
+    # dominant kernel: SHA-1 (largest marginal cost per batch in the pipeline,
+    # DESIGN.md section 8); achieved = its algorithmic ops per launch / launch
+    # duration of an isolated full-GPU launch on the C2 data
+    kd = kernels["sha1"]
     traffic = None
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tp):  # DRAM bytes per launch from the committed ncu capture,
-        tj = json.load(open(tp))  # scaled from its batch size to this run's mean batch
-        if dom in tj:
-            traffic = tj[dom] / tj["capture_batch_bytes"] * (bytes_timed / args.steps)
-    roofline = {"kernel": dom, "bound": kd["bound"], "achieved": kd["achieved"],
-                "peak": kd["peak"], "unit": kd["unit"], "frac": kd["frac"], "traffic": traffic,
-                "peak_source": f"{src} (MEASURED_PEAKS.json)" if kd["bound"] == "hbm" else
-                f"derived: 148 SM x 64 alu lanes/clk x {sm_mhz:.0f} MHz ({src} max clock)"}
+        tj = json.load(open(tp))  # scaled from its batch size to this launch's bytes
+        if "sha1" in tj:
+            traffic = tj["sha1"] / tj["capture_batch_bytes"] * kd["launch_bytes"]
+    roofline = {"kernel": "sha1_kernel", "bound": "alu", "achieved": kd["achieved"],
+                "peak": int_peak, "unit": "Tops/s", "frac": kd["achieved"] / int_peak,
+                "traffic": traffic, "peak_source": peak_source,
+                "launch": f"{kd['launch_bytes'] / MiB:.0f} MiB of C2 chunks per launch, "
+                          f"{kd['launch_us']:.0f} us per launch (CUDA events, "
+                          "4 concurrent streams)"}
 
     # ---- end-to-end through the host-fed C ABI ----
     e2e_steps = args.e2e_steps or min(args.steps, 120)

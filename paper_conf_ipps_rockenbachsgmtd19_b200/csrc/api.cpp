@@ -42,7 +42,7 @@ struct Workspace {
     uint32_t* agg = nullptr;         // per-tile transfer functions (32 u32 per tile)
     uint32_t* gagg = nullptr;        // per-group transfer functions (32 u32 per group)
     uint32_t* gentry = nullptr;      // per-group entry state + cut offset
-    uint32_t* scan_ctr = nullptr;    // scan tile counter + per-group arrival counters
+    uint32_t* evbuf = nullptr;       // per-tile event lists (scan -> cut emission)
     uint32_t* counters = nullptr;    // [0..1] sha1 work/long counters, [64..191] route
     uint32_t* slot_idx = nullptr;    // table slot per record
     uint32_t* long_list = nullptr;   // SHA-1 long-chunk list
@@ -186,7 +186,7 @@ dedup_status ws_alloc(dedup_ctx* c, Workspace& w, uint64_t batch_bytes, uint64_t
     TRY(dalloc(c, &w.agg, w.max_tiles * 32));
     TRY(dalloc(c, &w.gagg, (select_groups(w.max_tiles) + 1) * 32));
     TRY(dalloc(c, &w.gentry, (select_groups(w.max_tiles) + 1) * 2));
-    TRY(dalloc(c, &w.scan_ctr, select_groups(w.max_tiles) + 2));
+    TRY(dalloc(c, &w.evbuf, event_words(w.max_tiles)));
     TRY(dalloc(c, &w.counters, 256));
     TRY(dalloc(c, &w.slot_idx, cap));
     TRY(dalloc(c, &w.long_list, batch_bytes / kMinLongBytes + 2));
@@ -199,7 +199,7 @@ void ws_free(Workspace& w) {
     cudaFree(w.agg);
     cudaFree(w.gagg);
     cudaFree(w.gentry);
-    cudaFree(w.scan_ctr);
+    cudaFree(w.evbuf);
     cudaFree(w.counters);
     cudaFree(w.slot_idx);
     cudaFree(w.long_list);
@@ -236,7 +236,7 @@ void enqueue_chunk_sha(dedup_ctx* c, Workspace& w, cudaStream_t s, const BatchDe
                        uint32_t max_items) {
     if (!(DEDUP_ATTRIB_SKIP & 4))
         launch_chunk_select(d, c->d_tab, c->cfg.anchor_mask, c->cfg.anchor_value, w.bitmap,
-                            w.agg, w.gagg, w.gentry, w.scan_ctr,
+                            w.agg, w.gagg, w.gentry, w.evbuf,
                             (max_bytes + kSelTile - 1) / kSelTile, cut_pos, cap, n_chunks,
                             c->num_sms, s, ev_scan);
     if (chunk_start)
@@ -390,6 +390,7 @@ dedup_status launch_batch(dedup_ctx* c, int i, const uint8_t* d_bytes) {
     d.table = table_view(c);
     c->stream_fresh = false;
     const auto t0 = std::chrono::steady_clock::now();
+    encode_scan_tmap(d);  // TMA view for the scan (tma_rows = 0: LDG path)
     CU(cudaGraphLaunch(sl.graph, sl.stream));
     c->st.ms_host_launch +=
         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
@@ -825,6 +826,7 @@ dedup_status dedup_op_chunk(dedup_ctx* c, void* stream, const uint8_t* d_bytes, 
     h.nbytes = nbytes;
     h.item_off = d_item_off;
     h.n_items = n_items;
+    encode_scan_tmap(h);
     const BatchDesc* d = nullptr;
     TRY(op_desc(c, s, h, &d));
     enqueue_chunk_sha(c, c->op_ws, s, d, nbytes, d_cut_pos, cap, d_n_chunks, nullptr, nullptr,

@@ -22,7 +22,7 @@ struct TableView {
 
 // Per-batch parameters, read by the kernels from device memory so that the
 // launch sequence of a batch slot is a fixed CUDA graph.
-struct BatchDesc {
+struct alignas(64) BatchDesc {
     const uint8_t* bytes;      // batch bytes (16-byte aligned)
     uint64_t nbytes;
     uint64_t first_seq;        // seq of the batch's first item
@@ -30,7 +30,17 @@ struct BatchDesc {
     uint32_t n_items;
     uint32_t fresh;            // 1: clear the table before inserting
     TableView table;
+    // TMA view of the batch for the scan (encode_scan_tmap): bytes as a 2-D
+    // tensor of tma_rows rows x 256 B (the lane segments), 32 x 32 B boxes.
+    // tma_rows = 0: no tensor map, the scan loads with LDG.
+    uint32_t tma_rows;
+    uint32_t pad_[7];
+    alignas(64) unsigned char tmap[128];
 };
+
+// Fills d.tmap / d.tma_rows from d.bytes, d.nbytes (host; false and
+// tma_rows = 0 if the driver cannot encode it, the scan then uses LDG).
+bool encode_scan_tmap(BatchDesc& d);
 
 // ---- chunking (rabin.cu) --------------------------------------------------
 // Positions per cut-selection tile (e-space), words of the candidate bitmap.
@@ -42,9 +52,11 @@ constexpr uint32_t kSelTileWords = kSelTile / 32;
 // their per-group composition (gagg, 32 u32 per group of 32 tiles); a one-CTA
 // prefix over the groups (gentry, 2 u32 per group: entry state, cut offset);
 // a replay writing cut_pos.  bitmap: e-space candidate words (nbytes/32 + 1);
-// scan_ctr: select_groups(max_tiles) + 2 words, zeroed by the launcher.
+// evbuf: event_words(max_tiles) words.
 // after_scan (optional) is recorded between the scan and the selection.
 uint64_t select_groups(uint64_t max_tiles);
+// Per-tile event slots (evbuf) written by the scan for the cut emission.
+uint64_t event_words(uint64_t max_tiles);
 
 // Launch-configuration check (dedup_init fails with DEDUP_ECUDA instead of
 // losing a launch inside a graph): true iff one CTA of fn fits on an SM.
@@ -60,7 +72,7 @@ const char* chunk_unlaunchable();
 const char* sha1_unlaunchable();
 void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mask,
                          uint32_t value, uint32_t* bitmap, uint32_t* agg, uint32_t* gagg,
-                         uint32_t* gentry, uint32_t* scan_ctr, uint64_t max_tiles,
+                         uint32_t* gentry, uint32_t* evbuf, uint64_t max_tiles,
                          uint32_t* cut_pos, uint64_t cap, uint32_t* n_chunks, int num_sms,
                          cudaStream_t s, cudaEvent_t after_scan);
 

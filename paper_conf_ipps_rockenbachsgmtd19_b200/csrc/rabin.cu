@@ -27,6 +27,7 @@
 //      cut positions (the paper's startPos).
 // Item starts are forced cuts and reset the state; a candidate is valid only
 // if its 32-byte window lies inside one item.
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -40,10 +41,6 @@ namespace {
 // reach ~97% of the 1024-thread throughput) while leaving half of the
 // register file to the SHA-1 / table kernels of other in-flight batches.
 constexpr int kScanThreads = 512;
-#ifndef DEDUP_SCAN_PREFETCH
-#define DEDUP_SCAN_PREFETCH 2
-#endif
-constexpr int kScanPrefetch = DEDUP_SCAN_PREFETCH;  // 32-byte steps loaded ahead (0..2)
 constexpr int kScanWarps = kScanThreads / 32;
 constexpr int kEmitThreads = kScanThreads;  // one warp per tile of a group
 constexpr int kEmitWarps = kEmitThreads / 32;
@@ -52,11 +49,7 @@ constexpr uint32_t kLaneBytes = kSelTile / 32;  // 256 bytes per lane per tile
 constexpr uint32_t kFull = 0xFFFFFFFFu;
 constexpr uint32_t kInf = 0xFFFFFFFFu;
 constexpr uint32_t kM27 = (1u << 27) - 1;
-#ifndef DEDUP_SCAN_ILP
-#define DEDUP_SCAN_ILP 2
-#endif
-constexpr int kScanIlp = DEDUP_SCAN_ILP;  // tiles rolled together per warp (1 or 2)
-constexpr int kGroup = kScanWarps * kScanIlp;  // tiles per group = one CTA round
+constexpr int kGroup = kScanWarps * 2;  // tiles per group = one CTA round (2 per warp)
 constexpr int kItemCache = 1024;  // item offsets cached in shared memory
 
 constexpr uint32_t kListCap = 128;  // events per tile kept as a sorted list
@@ -95,77 +88,10 @@ __device__ __forceinline__ uint32_t lds(uint32_t addr) {
     return v;
 }
 
-// Rolls the 32 bytes of cur[0..7] (stream bytes, little-endian words) into h,
-// removing the 32 bytes of old[0..7]; returns the 32 candidate bits
-// (bit b <=> the window ending at byte b of this step).
-// laneR / laneW = table base (64 KiB aligned) | lane*4 (+128 for W256).
-template <bool kZeroValue>
-__device__ __forceinline__ uint32_t roll32(uint32_t& h, const uint32_t cur[8],
-                                           const uint32_t old[8], uint32_t laneR, uint32_t laneW,
-                                           uint32_t mask, uint32_t value) {
-    uint32_t bits = 0;
-#pragma unroll
-    for (int w = 0; w < 8; ++w) {
-#pragma unroll
-        for (int k = 0; k < 4; ++k) {
-            // R[x] at base + x*256 + lane*4, W256[o] at base + o*256 + 128 + lane*4.
-            const uint32_t aR = __byte_perm(h, laneR, 0x7634);
-            const uint32_t aW = __byte_perm(old[w], laneW, 0x7604 | (k << 4));
-            const uint32_t hs = __byte_perm(cur[w], h, 0x6540 | k);  // (h << 8) | in
-            h = hs ^ lds(aR) ^ lds(aW);
-            const uint32_t t = kZeroValue ? (h & mask) : ((h & mask) ^ value);
-            asm("{\n\t.reg .pred p;\n\tsetp.eq.u32 p, %1, 0;\n\t@p or.b32 %0, %0, %2;\n\t}"
-                : "+r"(bits)
-                : "r"(t), "r"(1u << (4 * w + k)));
-        }
-    }
-    return bits;
-}
-
 #ifndef DEDUP_SCAN_EXPERIMENT
 #define DEDUP_SCAN_EXPERIMENT 0  // timing experiments only (results invalid): 4 = no
                                  // global loads in the scan, 8 = no per-tile epilogue
 #endif
-
-__device__ __forceinline__ void load32(const uint8_t* p, uint32_t v[8]) {
-    if (DEDUP_SCAN_EXPERIMENT & 4) {
-#pragma unroll
-        for (int i = 0; i < 8; ++i) v[i] = (uint32_t)(uintptr_t)p * 2654435761u + i;
-        return;
-    }
-    const uint4 a = __ldg(reinterpret_cast<const uint4*>(p));
-    const uint4 b = __ldg(reinterpret_cast<const uint4*>(p + 16));
-    v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
-    v[4] = b.x; v[5] = b.y; v[6] = b.z; v[7] = b.w;
-}
-
-// 32 bytes at off; 16-byte vectors at or beyond lim16 (nbytes rounded up to
-// 16) read as zero.
-__device__ __forceinline__ void load32_any(const uint8_t* base, uint64_t off, uint64_t nbytes,
-                                           uint64_t lim16, uint32_t v[8]) {
-    if (off + 32 <= nbytes || (DEDUP_SCAN_EXPERIMENT & 4)) {
-        load32(base + off, v);
-        return;
-    }
-    uint4 a = make_uint4(0, 0, 0, 0), b = make_uint4(0, 0, 0, 0);
-    if (off < lim16) a = __ldg(reinterpret_cast<const uint4*>(base + off));
-    if (off + 16 < lim16) b = __ldg(reinterpret_cast<const uint4*>(base + off + 16));
-    v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
-    v[4] = b.x; v[5] = b.y; v[6] = b.z; v[7] = b.w;
-}
-
-// 16 bytes at off (16-byte aligned); vectors at or beyond lim16 read as zero.
-__device__ __forceinline__ void load16_any(const uint8_t* base, uint64_t off, uint64_t lim16,
-                                           uint32_t v[4]) {
-    if (DEDUP_SCAN_EXPERIMENT & 4) {
-#pragma unroll
-        for (int i = 0; i < 4; ++i) v[i] = (uint32_t)off * 2654435761u + i;
-        return;
-    }
-    uint4 a = make_uint4(0, 0, 0, 0);
-    if (off < lim16) a = __ldg(reinterpret_cast<const uint4*>(base + off));
-    v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
-}
 
 // 32 bytes at off with one 256-bit load (LDG.E.256, sm_100) when the address
 // is 32-byte aligned (a32) and the whole vector lies below lim16, else as
@@ -180,7 +106,7 @@ __device__ __forceinline__ void load32_v8(const uint8_t* base, uint32_t off, uin
     }
     if (a32 && off + 32 <= lim16) {
 #ifndef DEDUP_SCAN_LDHINT
-#define DEDUP_SCAN_LDHINT 0  // 1: L1::no_allocate, 2: L2::256B prefetch (timing knobs)
+#define DEDUP_SCAN_LDHINT 1  // 1: L1::no_allocate (measured +10 %), 2: L2::256B (no gain)
 #endif
 #if DEDUP_SCAN_LDHINT == 1
 #define DEDUP_LDV8 "ld.global.nc.L1::no_allocate.v8.u32"
@@ -362,6 +288,17 @@ __device__ __forceinline__ uint32_t apply_items(SelWarpSmem& sm, uint64_t T0, ui
     return kInf;
 }
 
+// Per-tile event slot for the emit kernel: word 0 = number of events (kInf:
+// more than kEvSlot, the emit kernel rebuilds the tile), words 1.. = events.
+constexpr uint32_t kEvSlot = 15;
+constexpr uint32_t kEvWords = kEvSlot + 1;
+__device__ __forceinline__ void store_events(const SelWarpSmem& sm, uint32_t n_ev,
+                                             uint32_t* __restrict__ slot, int lane) {
+    const uint32_t n = n_ev <= kEvSlot ? n_ev : kInf;
+    if (lane == 0) slot[0] = n;
+    if (n != kInf && (uint32_t)lane < n) slot[1 + lane] = sm.list[lane];
+}
+
 // Walk from entry state s using the event list, or the bitmaps if dense.
 __device__ __forceinline__ uint32_t walk_any(const SelWarpSmem& sm, uint32_t n_ev, uint32_t s,
                                              uint32_t& exit_state, uint32_t* out,
@@ -370,176 +307,22 @@ __device__ __forceinline__ uint32_t walk_any(const SelWarpSmem& sm, uint32_t n_e
     return walk_tile(sm, s, exit_state, out, out_base, cap, T0);
 }
 
-// Scan + per-tile transfer functions + per-group composition.
-// bitmap: e-space candidate words (bit e%32 of word e/32 <=> a window ends at
-// byte e-1), before the item rules.  agg[32 t + s] = exit(s) << 27 | cuts(s).
-// ctr[0] = tile counter, ctr[1 + g] = arrivals of group g (zeroed per batch).
-template <bool kZeroValue>
-__global__ void __launch_bounds__(kScanThreads, 2)  // <= 64 registers: half the RF
-rabin_scan_agg_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ gtab,
-                      uint32_t mask, uint32_t value, uint32_t* __restrict__ bitmap,
-                      uint32_t* __restrict__ agg, uint32_t* __restrict__ gagg,
-                      uint32_t* __restrict__ ctr) {
-    extern __shared__ __align__(16) uint8_t smem[];
-    __shared__ uint32_t src[512];
-    const uint8_t* __restrict__ bytes = desc->bytes;
-    const uint64_t nbytes = desc->nbytes;
-    const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    // the table starts at the first 64 KiB boundary of the shared window
-    const uint32_t win = (uint32_t)__cvta_generic_to_shared(smem);
-    const uint32_t pad = (0x10000u - (win & 0xFFFFu)) & 0xFFFFu;
-    const uint32_t base = win + pad;
-    SelWarpSmem* wsm = reinterpret_cast<SelWarpSmem*>(
-        smem);
-    if (pad < (uint32_t)kScanAux) __trap();  // layout assumption (see kScanSmem)
-    uint64_t* icache = reinterpret_cast<uint64_t*>(wsm + kScanWarps);
-    SelWarpSmem& sm = wsm[wid];
-    __shared__ uint32_t fun[kFunBufs][kGroup][32];  // tile functions of recent groups
-    const uint64_t n_tiles = (nbytes + kSelTile - 1) / kSelTile;
-    const uint64_t n_groups = (n_tiles + kGroup - 1) / kGroup;
-    const uint64_t lim16 = (nbytes + 15) & ~uint64_t(15);
-    // CTA b owns groups b, b + grid, ...; warp w owns tile w of each group
-    const uint64_t stride = (uint64_t)gridDim.x * kGroup;
-    const uint64_t lo = (uint64_t)blockIdx.x * kGroup, hi = n_groups * kGroup;
-    // warm-up window and the first two 32-byte steps of a tile, loaded early
-    uint32_t prev[8], cur[8], nxt[8];
-    auto load_first = [&](uint64_t t) {
-        const uint64_t q = t * kSelTile + (uint64_t)lane * kLaneBytes;
-#pragma unroll
-        for (int i = 0; i < 8; ++i) prev[i] = cur[i] = nxt[i] = 0;
-        if (q >= 32) load32(bytes + q - 32, prev);
-        if (q < nbytes) load32_any(bytes, q, nbytes, lim16, cur);
-        if (kScanPrefetch == 2 && q + 32 < nbytes) load32_any(bytes, q + 32, nbytes, lim16, nxt);
-    };
-    if (lo + wid < n_tiles) load_first(lo + wid);  // in flight during the table build
-    if (threadIdx.x < 512) src[threadIdx.x] = gtab[threadIdx.x];
-    const uint64_t* items = cache_items(icache, desc);
-    const uint32_t n_items = desc->n_items;
-    __syncthreads();
-    {   // replicate R / W256 per lane: word idx = x*64 + half*32 + lane
-        uint32_t* t32 = reinterpret_cast<uint32_t*>(smem + pad);
-        for (int idx = threadIdx.x; idx < kTabBytes / 4; idx += blockDim.x)
-            t32[idx] = src[((idx >> 5) & 1) * 256 + (idx >> 6)];
-    }
-    __syncthreads();
-    if (nbytes == 0) return;
-    const uint32_t laneR = base | (lane * 4);
-    const uint32_t laneW = laneR + 128;
-    int par = 0;
-    for (uint64_t t = lo + wid; t < hi; t += stride, par = (par + 1) % kFunBufs) {
-      uint32_t f = (uint32_t)lane << 27;  // identity function beyond the last tile
-      if (t < n_tiles) {
-        const uint64_t T0 = t * kSelTile;
-        const uint64_t q = T0 + (uint64_t)lane * kLaneBytes;
-        // ---- scan: 8 steps of 32 bytes, bits written in e-space ----
-        uint32_t h = 0, prev_bits = 0;
-#if DEDUP_SCAN_EXPERIMENT & 2
-        if (false) {  // timing experiment only: no warm-up
-#else
-        if (q >= 32) {  // warm-up: the window ending at q-1 -> bit for e = q
-#endif
-            const uint32_t zero[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-            prev_bits = roll32<kZeroValue>(h, prev, zero, laneR, laneW, mask, value);
-        }
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-            const uint64_t b0 = q + 32 * j;
-            uint32_t bits = 0, nx2[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-            if (kScanPrefetch == 2) {
-                if (j < 6 && b0 + 64 < nbytes) load32_any(bytes, b0 + 64, nbytes, lim16, nx2);
-            } else if (kScanPrefetch == 1) {
-                if (j < 7 && b0 + 32 < nbytes) load32_any(bytes, b0 + 32, nbytes, lim16, nx2);
-            } else if (j > 0 && b0 < nbytes) {
-                load32_any(bytes, b0, nbytes, lim16, cur);
-            }
-            if (b0 < nbytes) {
-                bits = roll32<kZeroValue>(h, cur, prev, laneR, laneW, mask, value);
-                if (b0 + 32 > nbytes) bits &= (1u << (uint32_t)(nbytes - b0)) - 1u;
-            }
-            uint32_t ew = __funnelshift_l(prev_bits, bits, 1);  // e = i + 1
-            if (b0 >= nbytes) ew = 0;
-            else if (b0 + 32 > nbytes) ew &= (1u << (uint32_t)(nbytes - b0)) - 1u;
-            sm.cand[lane * 8 + j] = ew;
-            bitmap[T0 / 32 + lane * 8 + j] = ew;
-            prev_bits = bits;
-#pragma unroll
-            for (int i = 0; i < 8; ++i) {
-                prev[i] = cur[i];
-                if (kScanPrefetch == 2) {
-                    cur[i] = nxt[i];
-                    nxt[i] = nx2[i];
-                } else if (kScanPrefetch == 1) {
-                    cur[i] = nx2[i];
-                }
-            }
-        }
-        // next tile's first loads fly during the transfer-function walk
-        if (t + stride < n_tiles) load_first(t + stride);
-        // ---- the tile's 32-entry transfer function ----
-        const uint32_t n_ev = apply_items(sm, T0, nbytes, items, n_items, lane);
-        uint32_t ex;
-        const uint32_t cnt = walk_any(sm, n_ev, lane, ex, nullptr, 0, 0, 0);
-        f = (ex << 27) | cnt;
-        agg[32 * t + lane] = f;
-      }
-        // ---- the CTA composes its group of kGroup tiles (the barrier keeps
-        // the warps of a CTA in step, measured faster than letting the last
-        // arrival compose) ----
-        fun[par][wid][lane] = f;
-        __syncthreads();
-        if (wid == 0) {
-            uint32_t Gs = lane, Gc = 0;
-#pragma unroll
-            for (int j = 0; j < kGroup; ++j) {
-                const uint32_t a = fun[par][j][lane];
-                const uint32_t ns = __shfl_sync(kFull, a >> 27, Gs);
-                const uint32_t nc = Gc + __shfl_sync(kFull, a & kM27, Gs);
-                Gs = ns;
-                Gc = nc;
-            }
-            gagg[32 * (t / kGroup) + lane] = (Gs << 27) | Gc;
-        }
-    }
-    (void)ctr;
-}
-
 // Two independent rolling chains per lane (ILP 2): the LDS -> LOP3 -> PRMT
 // dependency of one chain overlaps with the other's.
 // Words [W0, W1) of the 32-byte step; bits accumulate into bitsA / bitsB.
-#ifndef DEDUP_SCAN_FMA_AR
-#define DEDUP_SCAN_FMA_AR 0
-#endif
-__device__ __forceinline__ uint32_t mad_hi_u32(uint32_t a, uint32_t b, uint32_t c) {
-    uint32_t d;
-    asm("mad.hi.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
-    return d;
-}
-__device__ __forceinline__ uint32_t mad_lo_u32(uint32_t a, uint32_t b, uint32_t c) {
-    uint32_t d;
-    asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
-    return d;
-}
-// LDS address of R[h >> 24] for this lane.  PRMT (ALU pipe), or with
-// DEDUP_SCAN_FMA_AR two FMA-pipe ops (c256 = 256 at run time, so that ptxas
-// keeps the IMADs): (h >> 24) = mad.hi(h, 256), then * 256 + laneR.
-__device__ __forceinline__ uint32_t addr_r(uint32_t h, uint32_t laneR, uint32_t c256) {
-    if (DEDUP_SCAN_FMA_AR) return mad_lo_u32(mad_hi_u32(h, c256, 0u), c256, laneR);
-    return __byte_perm(h, laneR, 0x7634);
-}
-
 template <bool kZeroValue, int W0 = 0, int W1 = 8>
 __device__ __forceinline__ void roll32x2(uint32_t& hA, const uint32_t curA[8],
                                          const uint32_t oldA[8], uint32_t& bitsA, uint32_t& hB,
                                          const uint32_t curB[8], const uint32_t oldB[8],
                                          uint32_t& bitsB, uint32_t laneR, uint32_t laneW,
-                                         uint32_t mask, uint32_t value, uint32_t c256) {
+                                         uint32_t mask, uint32_t value) {
     if (W0 == 0) bitsA = bitsB = 0;
 #pragma unroll
     for (int w = W0; w < W1; ++w) {
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
-            const uint32_t aRA = addr_r(hA, laneR, c256);
-            const uint32_t aRB = addr_r(hB, laneR, c256);
+            const uint32_t aRA = __byte_perm(hA, laneR, 0x7634);
+            const uint32_t aRB = __byte_perm(hB, laneR, 0x7634);
             const uint32_t aWA = __byte_perm(oldA[w], laneW, 0x7604 | (k << 4));
             const uint32_t aWB = __byte_perm(oldB[w], laneW, 0x7604 | (k << 4));
             const uint32_t hsA = __byte_perm(curA[w], hA, 0x6540 | k);
@@ -572,29 +355,88 @@ __device__ __forceinline__ void prefetch_tile_l2(const uint8_t* bytes, uint64_t 
                  : "memory");
 }
 
-// Measured (isolated chunk stage, 256 MiB): no prefetch 938 GB/s, register
-// prefetch 949, L2 bulk prefetch 899, both 890 -- the scan is not load-latency
-// bound at 16 warps x 2 chains per SM.
+// Measured (isolated chunk stage, 256 MiB of C2-like data): next-step loads
+// issued one step ahead into the recycled registers 949 GB/s (none: 938);
+// one LDG.E.256 per step instead of two LDG.128: 996; an L2 bulk prefetch of
+// the next group's tiles: slightly slower (899 / 938), off.
 #ifndef DEDUP_SCAN_L2PF
 #define DEDUP_SCAN_L2PF 0
 #endif
-#ifndef DEDUP_SCAN_REGPF
-#define DEDUP_SCAN_REGPF 1
+
+// ---- TMA staging of the scan's input (kTma) ----------------------------------
+// The lane-strided LDGs of the scan (32 lanes x 32 B at a 256 B stride per
+// step) cost 32 L1 tag lookups per warp instruction and contend with the
+// table LDS in the L1/shared pipeline (ncu: short-scoreboard stalls 0.4 -> 2.9
+// per issue when the loads are present; the scan without loads is 39 %
+// faster).  With kTma one lane per warp asks the TMA unit for the next steps'
+// 32 rows x 32 B boxes (2-D tensor map: rows = lane segments of 256 B) into a
+// per-warp ring of kScanStages shared-memory stages, and the lanes read their
+// rows with two conflict-free LDS.128 (SWIZZLE_32B: the 16-byte halves of row
+// r are swapped when bit 2 of r is set, so 8 consecutive lanes cover all 32
+// banks).  Tiles whose rows are not all inside the tensor (the batch's ragged
+// end) keep the LDG path.
+#ifndef DEDUP_SCAN_TMA
+#define DEDUP_SCAN_TMA 0
 #endif
-// 1: the next step's 32 bytes come with one 256-bit load at the end of a step
-// (instead of two 128-bit loads at the halves); needs DEDUP_SCAN_REGPF.
-#ifndef DEDUP_SCAN_V8
-#define DEDUP_SCAN_V8 1
+#ifndef DEDUP_SCAN_STAGES
+#define DEDUP_SCAN_STAGES 3
 #endif
+constexpr int kScanStages = DEDUP_SCAN_STAGES;
+constexpr int kBoxBytes = 32 * 32;                 // one step of 32 lane rows
+constexpr int kUnitsPerTile = 1 + kLaneBytes / 32;  // warm-up box + 8 steps
+constexpr int kRingBytes = kScanWarps * kScanStages * 2 * kBoxBytes;
+// dynamic smem: [pad to the 64 KiB boundary (aux)][table 64 KiB][ring].  The
+// pad is 64 KiB minus the static smem (~10.4 KiB), so 10 KiB less than the
+// worst case is requested (the kernel traps if the runtime layout disagrees).
+constexpr int kScanSmemTma = 2 * 65536 - 10240 + kRingBytes;
+
+__device__ __forceinline__ void mbar_init(uint32_t mbar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(mbar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_tx(uint32_t mbar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mbar), "r"(bytes)
+                 : "memory");
+}
+// Bounded wait: a lost transfer traps (the context fails) instead of hanging.
+__device__ __forceinline__ void mbar_wait(uint32_t mbar, uint32_t parity) {
+    uint32_t done = 0;
+    for (uint32_t spin = 0;; ++spin) {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}"
+            : "=r"(done)
+            : "r"(mbar), "r"(parity)
+            : "memory");
+        if (done) return;
+        if (spin > (1u << 24)) __trap();
+    }
+}
+__device__ __forceinline__ void tma_box(uint32_t dst, const void* tmap, int x, int y,
+                                        uint32_t mbar) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%2, %3}], [%4];" ::"r"(dst),
+        "l"(tmap), "r"(x), "r"(y), "r"(mbar)
+        : "memory");
+}
+// Row `lane` of a 32 x 32 B box (SWIZZLE_32B) -> v[0..7].
+__device__ __forceinline__ void lds_row(uint32_t box, int lane, uint32_t v[8]) {
+    const uint32_t sw = ((uint32_t)lane >> 2) & 1u;
+    const uint32_t a0 = box + lane * 32 + 16 * sw, a1 = box + lane * 32 + 16 * (sw ^ 1u);
+    asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]) : "r"(a0));
+    asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]) : "r"(a1));
+}
 
 // ILP-2 scan: a CTA of kScanWarps warps takes groups of 2 x kScanWarps tiles;
 // warp w rolls tiles w and w + kScanWarps of the group together.
-template <bool kZeroValue>
-__global__ void __launch_bounds__(kScanThreads, 2)
+template <bool kZeroValue, bool kTma>
+__global__ void __launch_bounds__(kScanThreads, 2)  // <= 64 registers
 rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ gtab,
                        uint32_t mask, uint32_t value, uint32_t* __restrict__ bitmap,
                        uint32_t* __restrict__ agg, uint32_t* __restrict__ gagg,
-                       uint32_t c256) {
+                       uint32_t* __restrict__ evbuf) {
     extern __shared__ __align__(16) uint8_t smem[];
     __shared__ uint32_t src[512];
     __shared__ uint32_t fun[kFunBufs][kGroup][32];
@@ -624,11 +466,66 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
         for (int idx = threadIdx.x; idx < kTabBytes / 4; idx += blockDim.x)
             t32[idx] = src[((idx >> 5) & 1) * 256 + (idx >> 6)];
     }
+    // TMA ring: per warp kScanStages stages x 2 chains x 1 KiB after the table
+    __shared__ __align__(8) uint64_t mbar_s[kScanWarps][kScanStages];
+    const uint32_t ring = base + kTabBytes + (uint32_t)wid * (kScanStages * 2 * kBoxBytes);
+    if (kTma && base + kTabBytes + kRingBytes > win + (uint32_t)kScanSmemTma) __trap();
+    const uint32_t mbar0 = (uint32_t)__cvta_generic_to_shared(&mbar_s[wid][0]);
+    const uint32_t tma_rows = kTma ? desc->tma_rows : 0u;
+    const void* tmap = desc->tmap;
+    if (kTma && lane == 0) {
+        for (int i = 0; i < kScanStages; ++i) mbar_init(mbar0 + 8 * i, 1);
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        asm volatile("fence.proxy.tensormap::generic.acquire.gpu [%0], 128;" ::"l"(tmap)
+                     : "memory");
+    }
     __syncthreads();
     if (nbytes == 0) return;
     const uint32_t laneR = base | (lane * 4);
     const uint32_t laneW = laneR + 128;
     const bool a32 = (reinterpret_cast<uintptr_t>(bytes) & 31) == 0;
+    // Unit v of this warp = box s = v % 9 (0: warm-up, 1..8: steps) of the
+    // k = v / 9-th group of the CTA.  Unit v lives in stage v % kScanStages,
+    // phase (v / kScanStages) & 1.  Lane 0 issues unit v + kScanStages - 1
+    // when the lanes start reading unit v (its stage was read and released by
+    // the __syncwarp that ended unit v - 1).
+    auto tile_tma = [&](uint32_t t) { return (t + 1) * 32u <= tma_rows; };
+    auto issue = [&](uint32_t v) {
+        const uint32_t k = v / kUnitsPerTile, sidx = v % kUnitsPerTile;
+        const uint32_t g = blockIdx.x + k * gridDim.x;
+        if (g >= n_groups) return;
+        const uint32_t st = v % kScanStages, mb = mbar0 + 8 * st;
+        const uint32_t t0 = g * kGroup + wid, t1 = t0 + kScanWarps;
+        const bool c0 = tile_tma(t0), c1 = tile_tma(t1);
+        mbar_arrive_tx(mb, (c0 ? kBoxBytes : 0) + (c1 ? kBoxBytes : 0));
+        const int x = sidx == 0 ? (int)(kLaneBytes - 32) : 32 * (int)(sidx - 1);
+        const int dy = sidx == 0 ? -1 : 0;
+        const uint32_t dst = ring + st * 2 * kBoxBytes;
+        if (c0) tma_box(dst, tmap, x, (int)(t0 * 32) + dy, mb);
+        if (c1) tma_box(dst + kBoxBytes, tmap, x, (int)(t1 * 32) + dy, mb);
+    };
+    if (kTma && lane == 0)
+        for (uint32_t v = 0; v + 1 < (uint32_t)kScanStages; ++v) issue(v);
+    uint32_t unit = 0;  // next unit to read (kTma)
+    // The bytes of unit `unit` for both chains (TMA ring or LDG fallback).
+    auto fetch = [&](uint32_t offA, uint32_t offB, bool okA, bool okB, bool tA_tma,
+                     bool tB_tma, uint32_t (&vA)[8], uint32_t (&vB)[8]) {
+        if (kTma) {
+            if (lane == 0) issue(unit + kScanStages - 1);
+            const uint32_t st = unit % kScanStages;
+            if (tA_tma || tB_tma) mbar_wait(mbar0 + 8 * st, (unit / kScanStages) & 1u);
+            const uint32_t box = ring + st * 2 * kBoxBytes;
+            if (tA_tma) lds_row(box, lane, vA);
+            else if (okA) load32_v8(bytes, offA, lim16, a32, vA);
+            if (tB_tma) lds_row(box + kBoxBytes, lane, vB);
+            else if (okB) load32_v8(bytes, offB, lim16, a32, vB);
+            __syncwarp();
+            ++unit;
+        } else {
+            if (okA) load32_v8(bytes, offA, lim16, a32, vA);
+            if (okB) load32_v8(bytes, offB, lim16, a32, vB);
+        }
+    };
     int par = 0;
     for (uint32_t g = blockIdx.x; g < n_groups; g += gridDim.x, par ^= 1) {
         const uint32_t tA = g * kGroup + wid, tB = tA + kScanWarps;
@@ -641,66 +538,40 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
         uint32_t prevA[8], curA[8], prevB[8], curB[8];
 #pragma unroll
         for (int i = 0; i < 8; ++i) prevA[i] = curA[i] = prevB[i] = curB[i] = 0;
-        if (DEDUP_SCAN_V8) {
-            if (qA >= 32 && qA < nbytes) load32_v8(bytes, qA - 32, lim16, a32, prevA);
-            if (qB >= 32 && qB < nbytes) load32_v8(bytes, qB - 32, lim16, a32, prevB);
-            if (qA < nbytes) load32_v8(bytes, qA, lim16, a32, curA);
-            if (qB < nbytes) load32_v8(bytes, qB, lim16, a32, curB);
-        } else {
-            if (qA >= 32 && qA < nbytes) load32(bytes + qA - 32, prevA);
-            if (qB >= 32 && qB < nbytes) load32(bytes + qB - 32, prevB);
-            if (qA < nbytes) load32_any(bytes, qA, nbytes, lim16, curA);
-            if (qB < nbytes) load32_any(bytes, qB, nbytes, lim16, curB);
-        }
+        const bool tmaA = kTma && tile_tma(tA), tmaB = kTma && tile_tma(tB);
+        fetch(qA - 32, qB - 32, qA >= 32 && qA < nbytes, qB >= 32 && qB < nbytes, tmaA, tmaB,
+              prevA, prevB);
+        fetch(qA, qB, qA < nbytes, qB < nbytes, tmaA, tmaB, curA, curB);
         uint32_t hA = 0, hB = 0, pbA = 0, pbB = 0;
         {   // warm-up of both chains: the windows ending at q-1
             const uint32_t zero[8] = {0, 0, 0, 0, 0, 0, 0, 0};
             uint32_t bA, bB;
             roll32x2<kZeroValue>(hA, prevA, zero, bA, hB, prevB, zero, bB, laneR, laneW, mask,
-                                 value, c256);
+                                 value);
             pbA = qA >= 32 ? bA : 0;
             pbB = qB >= 32 ? bB : 0;
             if (qA < 32) hA = 0;
             if (qB < 32) hB = 0;
         }
         // One 32-byte step of both chains: roll `in` against `old`, then the
-        // bits in e-space.  With DEDUP_SCAN_REGPF the registers of `old` are
-        // recycled: once a half (16 bytes) of `old` has been rolled out, the
-        // same four registers receive the NEXT step's bytes of that half, so
-        // the loads fly for a whole step with no extra registers; `in` and
-        // `old` swap roles every step (the loop body holds two steps).
+        // bits in e-space.  Once `old` has been rolled out, its registers
+        // receive the NEXT step's bytes (TMA ring or LDG), so `in` and `old`
+        // swap roles every step (the loop body holds two steps) and no extra
+        // registers are needed.
         auto step = [&](int j, uint32_t (&inA)[8], uint32_t (&oldA)[8], uint32_t (&inB)[8],
                         uint32_t (&oldB)[8]) {
             const uint32_t bA0 = qA + 32 * j, bB0 = qB + 32 * j;
-#if !DEDUP_SCAN_REGPF
-            if (j > 0) {
-                if (bA0 < nbytes) load32_any(bytes, bA0, nbytes, lim16, inA);
-                if (bB0 < nbytes) load32_any(bytes, bB0, nbytes, lim16, inB);
-            }
-#endif
             uint32_t bitsA, bitsB;
             roll32x2<kZeroValue, 0, 4>(hA, inA, oldA, bitsA, hB, inB, oldB, bitsB, laneR, laneW,
-                                       mask, value, c256);
-#if DEDUP_SCAN_REGPF && !DEDUP_SCAN_V8
-            if (j < 7) {
-                load16_any(bytes, bA0 + 32, lim16, oldA);
-                load16_any(bytes, bB0 + 32, lim16, oldB);
-            }
-#endif
+                                       mask, value);
             roll32x2<kZeroValue, 4, 8>(hA, inA, oldA, bitsA, hB, inB, oldB, bitsB, laneR, laneW,
-                                       mask, value, c256);
-#if DEDUP_SCAN_REGPF && !DEDUP_SCAN_V8
-            if (j < 7) {
-                load16_any(bytes, bA0 + 48, lim16, oldA + 4);
-                load16_any(bytes, bB0 + 48, lim16, oldB + 4);
+                                       mask, value);
+            if (j < 7) {  // the next step's bytes into the registers `old` just freed
+#pragma unroll
+                for (int i = 0; i < 8; ++i) oldA[i] = oldB[i] = 0;
+                fetch(bA0 + 32, bB0 + 32, bA0 + 32 < nbytes, bB0 + 32 < nbytes, tmaA, tmaB, oldA,
+                      oldB);
             }
-#endif
-#if DEDUP_SCAN_REGPF && DEDUP_SCAN_V8
-            if (j < 7) {
-                load32_v8(bytes, bA0 + 32, lim16, a32, oldA);
-                load32_v8(bytes, bB0 + 32, lim16, a32, oldB);
-            }
-#endif
             uint32_t ewA = __funnelshift_l(pbA, bitsA, 1), ewB = __funnelshift_l(pbB, bitsB, 1);
             if (bA0 >= nbytes) ewA = 0;
             else if (bA0 + 32 > nbytes) ewA &= (1u << (uint32_t)(nbytes - bA0)) - 1u;
@@ -714,27 +585,16 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
             pbA = bitsA;
             pbB = bitsB;
         };
-#if DEDUP_SCAN_REGPF
 #pragma unroll 1
         for (int j = 0; j < 8; j += 2) {
             step(j, curA, prevA, curB, prevB);      // prev now holds step j+1's bytes
             step(j + 1, prevA, curA, prevB, curB);  // cur now holds step j+2's bytes
         }
-#else
-#pragma unroll 1
-        for (int j = 0; j < 8; ++j) {
-            step(j, curA, prevA, curB, prevB);
-#pragma unroll
-            for (int i = 0; i < 8; ++i) {
-                prevA[i] = curA[i];
-                prevB[i] = curB[i];
-            }
-        }
-#endif
         // transfer functions of tile A (candidate words already in smem), then B
         uint32_t fA = (uint32_t)lane << 27, fB = fA;
         if (tA < n_tiles && !(DEDUP_SCAN_EXPERIMENT & 8)) {
             const uint32_t n_ev = apply_items(sm, tA * kSelTile, nbytes, items, n_items, lane);
+            store_events(sm, n_ev, evbuf + (size_t)tA * kEvWords, lane);
             uint32_t ex;
             const uint32_t cnt = walk_any(sm, n_ev, lane, ex, nullptr, 0, 0, 0);
             fA = (ex << 27) | cnt;
@@ -746,6 +606,7 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
             for (int k = 0; k < 8; ++k)
                 sm.cand[lane * 8 + k] = bitmap[tB * kSelTileWords + lane * 8 + k];
             const uint32_t n_ev = apply_items(sm, tB * kSelTile, nbytes, items, n_items, lane);
+            store_events(sm, n_ev, evbuf + (size_t)tB * kEvWords, lane);
             uint32_t ex;
             const uint32_t cnt = walk_any(sm, n_ev, lane, ex, nullptr, 0, 0, 0);
             fB = (ex << 27) | cnt;
@@ -884,6 +745,102 @@ select_emit_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restric
     }
 }
 
+// Cut emission from the scan's per-tile event lists: one warp per group.
+// Lane 0 derives the group's tile entry states from the group entry (gentry)
+// and the tiles' transfer functions; lane j then walks tile j's stored event
+// list (<= kEvSlot events: the common case, ~2 per 8 KiB tile) from its real
+// entry state and writes its cut positions.  Tiles with more events (dense
+// candidates) are rebuilt cooperatively from the bitmap as in the scan.
+constexpr int kEmitEvWarps = 4;
+struct EmitEvSmem {
+    uint32_t fun[kEmitEvWarps][kGroup][33];
+    uint32_t te_state[kEmitEvWarps][kGroup], te_cnt[kEmitEvWarps][kGroup];
+    SelWarpSmem w[kEmitEvWarps];
+};
+
+__global__ void __launch_bounds__(kEmitEvWarps * 32)
+select_emit_ev_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ bitmap,
+                      const uint32_t* __restrict__ agg, const uint32_t* __restrict__ gentry,
+                      const uint32_t* __restrict__ evbuf, uint32_t* __restrict__ cut_pos,
+                      uint64_t cap) {
+    extern __shared__ __align__(16) uint8_t smraw[];
+    EmitEvSmem& sm = *reinterpret_cast<EmitEvSmem*>(smraw);
+    const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint64_t nbytes = desc->nbytes;
+    const uint32_t n_tiles = (uint32_t)((nbytes + kSelTile - 1) / kSelTile);
+    const uint32_t n_groups = (n_tiles + kGroup - 1) / kGroup;
+    const uint64_t* items = desc->item_off;
+    const uint32_t n_items = desc->n_items;
+    for (uint32_t g = blockIdx.x * kEmitEvWarps + wid; g < n_groups;
+         g += gridDim.x * kEmitEvWarps) {
+#pragma unroll 4
+        for (int j = 0; j < kGroup; ++j) {
+            const uint32_t t = g * kGroup + j;
+            sm.fun[wid][j][lane] = t < n_tiles ? agg[32 * t + lane] : ((uint32_t)lane << 27);
+        }
+        // this lane's event slot (64 B) flies during the entry-state chain
+        const uint32_t t = g * kGroup + lane;
+        uint32_t ev[kEvWords];
+        {
+            const uint4* sl = reinterpret_cast<const uint4*>(evbuf + (size_t)t * kEvWords);
+#pragma unroll
+            for (int i = 0; i < (int)kEvWords / 4; ++i) {
+                const uint4 v = t < n_tiles ? sl[i] : make_uint4(0, 0, 0, 0);
+                ev[4 * i] = v.x; ev[4 * i + 1] = v.y; ev[4 * i + 2] = v.z; ev[4 * i + 3] = v.w;
+            }
+        }
+        __syncwarp();
+        if (lane == 0) {
+            uint32_t st = gentry[2 * g], c = gentry[2 * g + 1];
+            for (int j = 0; j < kGroup; ++j) {
+                sm.te_state[wid][j] = st;
+                sm.te_cnt[wid][j] = c;
+                const uint32_t a = sm.fun[wid][j][st];
+                c += a & kM27;
+                st = a >> 27;
+            }
+        }
+        __syncwarp();
+        const bool dense = t < n_tiles && ev[0] > kEvSlot;
+        if (t < n_tiles && !dense) {
+            uint32_t E = sm.te_state[wid][lane];
+            uint64_t o = sm.te_cnt[wid][lane];
+            const uint32_t T0 = t * kSelTile;
+#pragma unroll
+            for (uint32_t i = 0; i < kEvSlot; ++i) {
+                if (i < ev[0]) {
+                    const uint32_t e = ev[1 + i], p = e & 0x7FFFFFFFu;
+                    if ((e >> 31) || p >= E) {
+                        if (o < cap) cut_pos[o] = T0 + p;
+                        ++o;
+                        E = p + 32;
+                    }
+                }
+            }
+        }
+        uint32_t dm = __ballot_sync(kFull, dense);
+        while (dm) {  // dense tiles: rebuild the candidate words and walk the bitmap
+            const int j = __ffs(dm) - 1;
+            dm &= dm - 1;
+            const uint32_t td = g * kGroup + j;
+            SelWarpSmem& w = sm.w[wid];
+#pragma unroll
+            for (int k = 0; k < 8; ++k)
+                w.cand[lane * 8 + k] = bitmap[(size_t)td * kSelTileWords + lane * 8 + k];
+            const uint32_t n_ev = apply_items(w, (uint64_t)td * kSelTile, nbytes, items,
+                                              n_items, lane);
+            const uint32_t st = sm.te_state[wid][j];
+            if (lane == (int)st) {
+                uint32_t ex;
+                walk_any(w, n_ev, st, ex, cut_pos, sm.te_cnt[wid][j], cap,
+                         (uint64_t)td * kSelTile);
+            }
+            __syncwarp();
+        }
+        __syncwarp();
+    }
+}
+
 __global__ void chunk_meta_kernel(const BatchDesc* __restrict__ desc,
                                   const uint32_t* __restrict__ cut_pos,
                                   const uint32_t* __restrict__ n_chunks_p, uint64_t cap,
@@ -925,61 +882,110 @@ __global__ void chunk_meta_kernel(const BatchDesc* __restrict__ desc,
 }  // namespace
 
 uint64_t select_groups(uint64_t max_tiles) { return (max_tiles + kGroup - 1) / kGroup; }
+uint64_t event_words(uint64_t max_tiles) { return max_tiles * kEvWords; }
 
 namespace {
 void chunk_set_attrs() {
     static bool attr_set = false;
     if (attr_set) return;
-    for (const void* f : {(const void*)rabin_scan_agg2_kernel<true>,
-                          (const void*)rabin_scan_agg2_kernel<false>,
-                          (const void*)rabin_scan_agg_kernel<true>,
-                          (const void*)rabin_scan_agg_kernel<false>})
+    for (const void* f : {(const void*)rabin_scan_agg2_kernel<true, false>,
+                          (const void*)rabin_scan_agg2_kernel<false, false>})
         cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
+    for (const void* f : {(const void*)rabin_scan_agg2_kernel<true, true>,
+                          (const void*)rabin_scan_agg2_kernel<false, true>})
+        cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmemTma);
     cudaFuncSetAttribute(select_emit_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)sizeof(EmitSmem));
+    cudaFuncSetAttribute(select_emit_ev_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)sizeof(EmitEvSmem));
     attr_set = true;
 }
 }  // namespace
 
 const char* chunk_unlaunchable() {
     chunk_set_attrs();
-    const void* kT = kScanIlp == 2 ? (const void*)rabin_scan_agg2_kernel<true>
-                                   : (const void*)rabin_scan_agg_kernel<true>;
-    const void* kF = kScanIlp == 2 ? (const void*)rabin_scan_agg2_kernel<false>
-                                   : (const void*)rabin_scan_agg_kernel<false>;
-    if (!fits(kT, kScanThreads, kScanSmem) || !fits(kF, kScanThreads, kScanSmem))
-        return "rabin_scan_agg_kernel";
+    for (const void* f : {(const void*)rabin_scan_agg2_kernel<true, false>,
+                          (const void*)rabin_scan_agg2_kernel<false, false>})
+        if (!fits(f, kScanThreads, kScanSmem)) return "rabin_scan_agg2_kernel";
+    if (DEDUP_SCAN_TMA)
+        for (const void* f : {(const void*)rabin_scan_agg2_kernel<true, true>,
+                              (const void*)rabin_scan_agg2_kernel<false, true>})
+            if (!fits(f, kScanThreads, kScanSmemTma)) return "rabin_scan_agg2_kernel (TMA)";
     if (!fits((const void*)select_scan_kernel, 1024, 0)) return "select_scan_kernel";
     if (!fits((const void*)select_emit_kernel, kEmitThreads, sizeof(EmitSmem)))
         return "select_emit_kernel";
+    if (!fits((const void*)select_emit_ev_kernel, kEmitEvWarps * 32, sizeof(EmitEvSmem)))
+        return "select_emit_ev_kernel";
     if (!fits((const void*)chunk_meta_kernel, 256, 0)) return "chunk_meta_kernel";
     return nullptr;
 }
 
+// Host side of the TMA view (internal.h).  The driver's tensor-map encoder is
+// resolved once through the runtime's entry-point query (no libcuda link).
+bool encode_scan_tmap(BatchDesc& d) {
+    d.tma_rows = 0;
+    if (!DEDUP_SCAN_TMA) return false;
+    using EncodeFn = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
+                                  const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
+                                  const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                  CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+    static EncodeFn enc = [] {
+        void* fn = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) !=
+                cudaSuccess ||
+            q != cudaDriverEntryPointSuccess)
+            fn = nullptr;
+        cudaGetLastError();
+        return reinterpret_cast<EncodeFn>(fn);
+    }();
+    const uint64_t rows = d.nbytes / kLaneBytes;
+    if (enc == nullptr || rows < 32 || (reinterpret_cast<uintptr_t>(d.bytes) & 15)) return false;
+    const cuuint64_t dims[2] = {kLaneBytes, rows};
+    const cuuint64_t strides[1] = {kLaneBytes};
+    const cuuint32_t box[2] = {32, 32};
+    const cuuint32_t estr[2] = {1, 1};
+    CUtensorMap* m = reinterpret_cast<CUtensorMap*>(d.tmap);
+    const CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<uint8_t*>(d.bytes),
+                           dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                           CU_TENSOR_MAP_SWIZZLE_32B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return false;
+    d.tma_rows = (uint32_t)rows;
+    return true;
+}
+
+#ifndef DEDUP_EMIT_EV
+#define DEDUP_EMIT_EV 1  // cut emission from stored event lists (0: rebuild every tile)
+#endif
+
 void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mask,
                          uint32_t value, uint32_t* bitmap, uint32_t* agg, uint32_t* gagg,
-                         uint32_t* gentry, uint32_t* scan_ctr, uint64_t max_tiles,
+                         uint32_t* gentry, uint32_t* evbuf, uint64_t max_tiles,
                          uint32_t* cut_pos, uint64_t cap, uint32_t* n_chunks, int num_sms,
                          cudaStream_t s, cudaEvent_t after_scan) {
     chunk_set_attrs();
-    auto kT = kScanIlp == 2 ? rabin_scan_agg2_kernel<true> : nullptr;
-    auto kF = kScanIlp == 2 ? rabin_scan_agg2_kernel<false> : nullptr;
     const uint64_t groups = select_groups(max_tiles);
     const unsigned grid = (unsigned)num_sms;
-    if (kScanIlp == 2) {
-        (value == 0 ? kT : kF)<<<grid, kScanThreads, kScanSmem, s>>>(d, d_tab, mask, value,
-                                                                     bitmap, agg, gagg, 256u);
+    // the kernel reads d->tma_rows at run time: 0 -> every tile on the LDG path
+    if (DEDUP_SCAN_TMA) {
+        auto k = value == 0 ? rabin_scan_agg2_kernel<true, true> : rabin_scan_agg2_kernel<false, true>;
+        k<<<grid, kScanThreads, kScanSmemTma, s>>>(d, d_tab, mask, value, bitmap, agg, gagg, evbuf);
     } else {
-        cudaMemsetAsync(scan_ctr, 0, sizeof(uint32_t) * (groups + 2), s);
-        if (value == 0)
-            rabin_scan_agg_kernel<true><<<grid, kScanThreads, kScanSmem, s>>>(
-                d, d_tab, mask, value, bitmap, agg, gagg, scan_ctr);
-        else
-            rabin_scan_agg_kernel<false><<<grid, kScanThreads, kScanSmem, s>>>(
-                d, d_tab, mask, value, bitmap, agg, gagg, scan_ctr);
+        auto k = value == 0 ? rabin_scan_agg2_kernel<true, false>
+                            : rabin_scan_agg2_kernel<false, false>;
+        k<<<grid, kScanThreads, kScanSmem, s>>>(d, d_tab, mask, value, bitmap, agg, gagg, evbuf);
     }
     if (after_scan) cudaEventRecordWithFlags(after_scan, s, cudaEventRecordExternal);
     select_scan_kernel<<<1, 1024, 0, s>>>(d, gagg, gentry, n_chunks);
+    if (DEDUP_EMIT_EV) {
+        uint64_t blocks = (groups + kEmitEvWarps - 1) / kEmitEvWarps;
+        if (blocks > (uint64_t)num_sms * 4) blocks = (uint64_t)num_sms * 4;
+        if (blocks < 1) blocks = 1;
+        select_emit_ev_kernel<<<(unsigned)blocks, kEmitEvWarps * 32, sizeof(EmitEvSmem), s>>>(
+            d, bitmap, agg, gentry, evbuf, cut_pos, cap);
+        return;
+    }
     uint64_t blocks = groups;
     if (blocks > (uint64_t)num_sms) blocks = (uint64_t)num_sms;
     if (blocks < 1) blocks = 1;
