@@ -249,27 +249,42 @@ typedef struct {
     uint64_t id;
 } dedup_record;
 
+/* Row A5, local combine ("per batch: collapse equal digests to
+ * their min id"): for the *d_n (<= cap <= this ctx's chunk capacity) digests
+ * of one batch (d_digest, 20 B each, chunk order), writes d_rep[r] = the
+ * smallest index r' with digest r' == digest r (r itself for a first
+ * occurrence).  Only representatives (d_rep[r] == r) need to travel to their
+ * owner: the batch's chunks are in stream order, so the representative holds
+ * the smallest id of its digest in the batch and the owner's minimum over
+ * representatives is the global first occurrence (reading O12).  Uses a
+ * ctx-owned local digest table (allocated on the first call, 2 x the ctx's
+ * chunk capacity slots) that is left empty again. */
+dedup_status dedup_op_local_combine(dedup_ctx* c, void* stream, const uint8_t* d_digest,
+                                    const uint32_t* d_n, uint64_t cap, uint32_t* d_rep);
+
 /* Row A5: owner(r) = floor(BE32(digest[0..3]) * num_owners / 2^32).
  * Writes records grouped by owner into d_send (capacity cap records):
  * owner o's records occupy d_send[d_send_off[o] .. d_send_off[o+1]) (u32
  * exclusive offsets, num_owners + 1 entries); d_send_pos[r] = slot of record r
- * in d_send.  num_owners <= 64. */
+ * in d_send.  d_rep (optional, from dedup_op_local_combine): only records with
+ * d_rep[r] == r are routed (d_send_pos of the others is not written).
+ * num_owners <= 64. */
 dedup_status dedup_op_route(dedup_ctx* c, void* stream, const uint8_t* d_digest,
                             const uint64_t* d_id, const uint32_t* d_n, uint64_t cap,
-                            uint32_t num_owners, dedup_record* d_send, uint32_t* d_send_off,
-                            uint32_t* d_send_pos);
+                            const uint32_t* d_rep, uint32_t num_owners, dedup_record* d_send,
+                            uint32_t* d_send_off, uint32_t* d_send_pos);
 
 /* Row A7 on the owner: insert all n_recv (host count) received records into
  * this ctx's table shard, then write d_reply[i] = first id of record i. */
 dedup_status dedup_op_owner(dedup_ctx* c, void* stream, const dedup_record* d_recv,
                             uint64_t n_recv, uint64_t* d_reply);
 
-/* Row A8: d_first_id[r] = d_reply_back[d_send_pos[r]],
- * d_is_dup[r] = (d_first_id[r] != d_id[r]). */
+/* Row A8: d_first_id[r] = d_reply_back[d_send_pos[q]] with q = d_rep[r] (or
+ * q = r when d_rep is NULL), d_is_dup[r] = (d_first_id[r] != d_id[r]). */
 dedup_status dedup_op_scatter(dedup_ctx* c, void* stream, const uint64_t* d_reply_back,
-                              const uint32_t* d_send_pos, const uint64_t* d_id,
-                              const uint32_t* d_n, uint64_t cap, uint64_t* d_first_id,
-                              uint8_t* d_is_dup);
+                              const uint32_t* d_send_pos, const uint32_t* d_rep,
+                              const uint64_t* d_id, const uint32_t* d_n, uint64_t cap,
+                              uint64_t* d_first_id, uint8_t* d_is_dup);
 
 /* Number of kernels this ctx has launched so far (all layers). */
 uint64_t dedup_kernel_launches(const dedup_ctx* c);

@@ -31,7 +31,8 @@ EXPORTS = [
     "dedup_submit_batch", "dedup_submit_device", "dedup_join", "dedup_end_stream", "dedup_drain",
     "dedup_pending", "dedup_stats", "dedup_host_alloc", "dedup_host_free",
     "dedup_op_chunk", "dedup_op_chunk_meta", "dedup_op_sha1", "dedup_op_table_insert_lookup",
-    "dedup_op_table_reset", "dedup_op_table_status", "dedup_op_route", "dedup_op_owner",
+    "dedup_op_table_reset", "dedup_op_table_status", "dedup_op_local_combine",
+    "dedup_op_route", "dedup_op_owner",
     "dedup_op_scatter", "dedup_kernel_launches",
 ]
 
@@ -112,9 +113,10 @@ def lib():
         "dedup_op_table_insert_lookup": (st, [vp, vp, vp, vp, vp, u64, vp, vp]),
         "dedup_op_table_reset": (st, [vp, vp]),
         "dedup_op_table_status": (st, [vp, vp, P(u64), P(u64), P(i32)]),
-        "dedup_op_route": (st, [vp, vp, vp, vp, vp, u64, u32, vp, vp, vp]),
+        "dedup_op_local_combine": (st, [vp, vp, vp, vp, u64, vp]),
+        "dedup_op_route": (st, [vp, vp, vp, vp, vp, u64, vp, u32, vp, vp, vp]),
         "dedup_op_owner": (st, [vp, vp, vp, u64, vp]),
-        "dedup_op_scatter": (st, [vp, vp, vp, vp, vp, vp, u64, vp, vp]),
+        "dedup_op_scatter": (st, [vp, vp, vp, vp, vp, vp, vp, u64, vp, vp]),
         "dedup_kernel_launches": (u64, [vp]),
     }
     for name, (res, args) in sig.items():

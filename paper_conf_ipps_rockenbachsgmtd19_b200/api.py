@@ -253,16 +253,22 @@ class Dedup:
                                                   ctypes.byref(slots), ctypes.byref(ovf)))
         return used.value, slots.value, ovf.value
 
-    def op_route(self, digest, ids, n, cap, num_owners, send, send_off, send_pos, stream=None):
+    def op_local_combine(self, digest, n, cap, rep, stream=None):
+        self._check(N.lib().dedup_op_local_combine(self._ctx, _stream(stream), _ptr(digest),
+                                                   _ptr(n), cap, _ptr(rep)))
+
+    def op_route(self, digest, ids, n, cap, num_owners, send, send_off, send_pos, rep=None,
+                 stream=None):
         self._check(N.lib().dedup_op_route(self._ctx, _stream(stream), _ptr(digest), _ptr(ids),
-                                           _ptr(n), cap, num_owners, _ptr(send), _ptr(send_off),
-                                           _ptr(send_pos)))
+                                           _ptr(n), cap, _ptr(rep), num_owners, _ptr(send),
+                                           _ptr(send_off), _ptr(send_pos)))
 
     def op_owner(self, recv, n_recv, reply, stream=None):
         self._check(N.lib().dedup_op_owner(self._ctx, _stream(stream), _ptr(recv), n_recv,
                                            _ptr(reply)))
 
-    def op_scatter(self, reply_back, send_pos, ids, n, cap, first_id, is_dup=None, stream=None):
+    def op_scatter(self, reply_back, send_pos, ids, n, cap, first_id, is_dup=None, rep=None,
+                   stream=None):
         self._check(N.lib().dedup_op_scatter(self._ctx, _stream(stream), _ptr(reply_back),
-                                             _ptr(send_pos), _ptr(ids), _ptr(n), cap,
+                                             _ptr(send_pos), _ptr(rep), _ptr(ids), _ptr(n), cap,
                                              _ptr(first_id), _ptr(is_dup)))

@@ -100,6 +100,8 @@ struct dedup_ctx {
     uint32_t next_slot = 0;     // round-robin cursor
     TableBuf tables[2];
     int cur_table = 0;
+    TableBuf local;                   // local-combine table (dedup_op_local_combine)
+    TableView* d_local_view = nullptr;
     bool stream_fresh = false;  // next batch starts a new dedup stream
     uint64_t chunk_cap = 0;     // chunks per slot
     std::deque<int> inflight;   // slot indices in seq order
@@ -600,6 +602,9 @@ void dedup_destroy(dedup_ctx* c) {
         cudaFree(t.slots);
         cudaFree(t.status);
     }
+    cudaFree(c->local.slots);
+    cudaFree(c->local.status);
+    cudaFree(c->d_local_view);
     cudaFree(c->d_tab);
     if (c->ev_ref) cudaEventDestroy(c->ev_ref);
     delete c;
@@ -929,15 +934,42 @@ dedup_status dedup_op_table_status(dedup_ctx* c, void* stream, uint64_t* used, u
     return DEDUP_OK;
 }
 
+dedup_status dedup_op_local_combine(dedup_ctx* c, void* stream, const uint8_t* d_digest,
+                                    const uint32_t* d_n, uint64_t cap, uint32_t* d_rep) {
+    if (c == nullptr) return DEDUP_EINVAL;
+    if (!usable(c)) return c->sticky;
+    if (cap > c->chunk_cap) return fail(c, DEDUP_EINVAL, "cap larger than the ctx workspace");
+    if (d_rep == nullptr || (cap > 0 && (d_digest == nullptr || d_n == nullptr)))
+        return fail(c, DEDUP_EINVAL, "null argument");
+    CU(cudaSetDevice(c->cfg.device));
+    if (c->local.slots == nullptr) {  // first call: an empty local table
+        TableBuf& t = c->local;
+        t.capacity = next_pow2(2 * c->chunk_cap);
+        TRY(dalloc(c, &t.slots, t.capacity));
+        TRY(dalloc(c, &t.status, 4));
+        TRY(dalloc(c, &c->d_local_view, 1));
+        CU(cudaMemset(t.slots, 0, sizeof(TableSlot) * t.capacity));
+        CU(cudaMemset(t.status, 0, 16));
+        const TableView v{t.slots, t.capacity - 1, t.status};
+        CU(cudaMemcpy(c->d_local_view, &v, sizeof(v), cudaMemcpyHostToDevice));
+    }
+    const TableView v{c->local.slots, c->local.capacity - 1, c->local.status};
+    launch_local_combine(v, d_digest, d_n, cap, c->op_ws.slot_idx, d_rep, c->num_sms,
+                         static_cast<cudaStream_t>(stream), c->d_local_view);
+    c->launches += cap ? 3 : 0;
+    CU(cudaGetLastError());
+    return DEDUP_OK;
+}
+
 dedup_status dedup_op_route(dedup_ctx* c, void* stream, const uint8_t* d_digest,
                             const uint64_t* d_id, const uint32_t* d_n, uint64_t cap,
-                            uint32_t num_owners, dedup_record* d_send, uint32_t* d_send_off,
-                            uint32_t* d_send_pos) {
+                            const uint32_t* d_rep, uint32_t num_owners, dedup_record* d_send,
+                            uint32_t* d_send_off, uint32_t* d_send_pos) {
     if (c == nullptr) return DEDUP_EINVAL;
     if (!usable(c)) return c->sticky;
     if (num_owners < 1 || num_owners > 64) return fail(c, DEDUP_EINVAL, "num_owners in 1..64");
     CU(cudaSetDevice(c->cfg.device));
-    launch_route(d_digest, d_id, d_n, cap, num_owners, d_send, d_send_off, d_send_pos,
+    launch_route(d_digest, d_id, d_n, cap, d_rep, num_owners, d_send, d_send_off, d_send_pos,
                  c->op_ws.counters + 64, c->num_sms, static_cast<cudaStream_t>(stream));
     c->launches += cap ? 3 : 1;
     CU(cudaGetLastError());
@@ -968,14 +1000,14 @@ dedup_status dedup_op_owner(dedup_ctx* c, void* stream, const dedup_record* d_re
 }
 
 dedup_status dedup_op_scatter(dedup_ctx* c, void* stream, const uint64_t* d_reply_back,
-                              const uint32_t* d_send_pos, const uint64_t* d_id,
-                              const uint32_t* d_n, uint64_t cap, uint64_t* d_first_id,
-                              uint8_t* d_is_dup) {
+                              const uint32_t* d_send_pos, const uint32_t* d_rep,
+                              const uint64_t* d_id, const uint32_t* d_n, uint64_t cap,
+                              uint64_t* d_first_id, uint8_t* d_is_dup) {
     if (c == nullptr) return DEDUP_EINVAL;
     if (!usable(c)) return c->sticky;
     CU(cudaSetDevice(c->cfg.device));
-    launch_scatter(d_reply_back, d_send_pos, d_id, d_n, cap, d_first_id, d_is_dup, c->num_sms,
-                   static_cast<cudaStream_t>(stream));
+    launch_scatter(d_reply_back, d_send_pos, d_rep, d_id, d_n, cap, d_first_id, d_is_dup,
+                   c->num_sms, static_cast<cudaStream_t>(stream));
     c->launches += cap ? 1 : 0;
     CU(cudaGetLastError());
     return DEDUP_OK;

@@ -104,12 +104,20 @@ void launch_table_lookup(const TableView* tv, const uint64_t* id, const void* re
                          uint32_t* status_out, const uint32_t* cut_pos,
                          const BatchDesc* desc, int num_sms, cudaStream_t s);
 
+// rep (optional): local-combine representatives; only records with
+// rep[r] == r are routed, and scatter gives chunk r the reply of rep[r].
 void launch_route(const uint8_t* digest, const uint64_t* id, const uint32_t* d_n, uint64_t cap,
-                  uint32_t num_owners, void* send, uint32_t* send_off, uint32_t* send_pos,
-                  uint32_t* scratch_counts, int num_sms, cudaStream_t s);
-void launch_scatter(const uint64_t* reply, const uint32_t* send_pos, const uint64_t* id,
-                    const uint32_t* d_n, uint64_t cap, uint64_t* first_id, uint8_t* is_dup,
-                    int num_sms, cudaStream_t s);
+                  const uint32_t* rep, uint32_t num_owners, void* send, uint32_t* send_off,
+                  uint32_t* send_pos, uint32_t* scratch_counts, int num_sms, cudaStream_t s);
+void launch_scatter(const uint64_t* reply, const uint32_t* send_pos, const uint32_t* rep,
+                    const uint64_t* id, const uint32_t* d_n, uint64_t cap, uint64_t* first_id,
+                    uint8_t* is_dup, int num_sms, cudaStream_t s);
+// Row A5 local combine: rep[r] = smallest record index with digest r's digest,
+// through the (empty) local table `local` (*d_local: the same view in device
+// memory); the used slots are cleared again afterwards.
+void launch_local_combine(TableView local, const uint8_t* digest, const uint32_t* d_n,
+                          uint64_t cap, uint32_t* slot_idx, uint32_t* rep, int num_sms,
+                          cudaStream_t s, const TableView* d_local);
 
 // Results of one batch written straight into mapped pinned host memory.
 struct HostResultLayout {

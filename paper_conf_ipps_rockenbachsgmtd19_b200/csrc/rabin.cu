@@ -5,10 +5,11 @@
 //
 // The paper ran this on the CPU; here it is three sm_100a kernels:
 //
-//  rabin_scan_agg_kernel  persistent, one CTA of 32 warps per SM.  A warp
-//      takes an 8 KiB tile (dynamic counter); each lane rolls the 32-byte
-//      window hash over its 256 bytes (after a 32-byte warm-up) with the
-//      post-shift recurrence
+//  rabin_scan_agg2_kernel  persistent, one CTA of 16 warps per SM.  A CTA
+//      takes groups of 32 tiles of 8 KiB; warp w rolls tiles w and w + 16 of
+//      the group together (two independent chains per lane, ILP 2); each lane
+//      rolls the 32-byte window hash over its 256 bytes (after a 32-byte
+//      warm-up) with the post-shift recurrence
 //          h' = ((h << 8) | in) ^ R[h >> 24] ^ W256[out]
 //      and records one candidate bit per byte.  R and W256 are replicated per
 //      lane in shared memory ([x][lane] layout: bank = lane, conflict-free);
@@ -17,14 +18,14 @@
 //      32-state machine (with min chunk = window = 32 the only state crossing
 //      a position is "positions still blocked", 0..31): the warp simulates all
 //      32 entry states over its tile (lane s = state s) and stores the tile's
-//      transfer function; the last warp to finish a group of 32 tiles composes
-//      them into the group function (warp shuffles).
+//      transfer function and its sorted event list (candidates + forced
+//      cuts); the CTA composes each group's 32 functions (warp shuffles).
 //  select_scan_kernel     one CTA composes the group functions in order (a
 //      prefix over an associative operator) -> entry state and cut offset of
 //      every group, and the batch's chunk count.
-//  select_emit_kernel     one CTA per group derives its tiles' entry states
-//      and every warp replays its tile from the real entry state, writing the
-//      cut positions (the paper's startPos).
+//  select_emit_ev_kernel  one warp per group derives its tiles' entry states;
+//      lane j walks tile j's stored event list from its real entry state,
+//      writing the cut positions (the paper's startPos).
 // Item starts are forced cuts and reset the state; a candidate is valid only
 // if its 32-byte window lies inside one item.
 #include <cuda.h>
@@ -37,19 +38,28 @@ namespace dd {
 
 namespace {
 
-// 16 warps per SM: enough to saturate the roll (measured: 512 threads/SM
-// reach ~97% of the 1024-thread throughput) while leaving half of the
-// register file to the SHA-1 / table kernels of other in-flight batches.
-constexpr int kScanThreads = 512;
-constexpr int kScanWarps = kScanThreads / 32;
-constexpr int kEmitThreads = kScanThreads;  // one warp per tile of a group
-constexpr int kEmitWarps = kEmitThreads / 32;
+// Scan CTA: DEDUP_SCAN_CTA_WARPS warps (64 registers each).  A select group
+// is 32 tiles rolled by 16 warps (2 tiles per warp, ILP 2); a 32-warp CTA
+// runs two groups at once (its two halves share the 64 KiB table).  Measured:
+// the 32-warp CTA scans faster alone (736 MiB chunk stage 1647 vs 1527 GB/s:
+// 16 warps x 2 chains leave the roll latency-bound) but it takes a whole SM
+// (64K registers, 220 KiB smem), and the pipelined bench is faster with 16
+// warps (590 vs 576 GB/s): other batches' SHA-1 / table / emit CTAs share the
+// SM with a 16-warp scan CTA.
+#ifndef DEDUP_SCAN_CTA_WARPS
+#define DEDUP_SCAN_CTA_WARPS 16
+#endif
+constexpr int kScanWarps = DEDUP_SCAN_CTA_WARPS;
+constexpr int kScanThreads = kScanWarps * 32;
+constexpr int kGroupWarps = 16;                    // warps per select group
+constexpr int kHalves = kScanWarps / kGroupWarps;  // groups in flight per CTA
+static_assert(kHalves == 1 || kHalves == 2, "16 or 32 warps per scan CTA");
 constexpr int kTabBytes = 256 * 256;  // [x][R|W][lane] u32 = 64 KiB
 constexpr uint32_t kLaneBytes = kSelTile / 32;  // 256 bytes per lane per tile
 constexpr uint32_t kFull = 0xFFFFFFFFu;
 constexpr uint32_t kInf = 0xFFFFFFFFu;
 constexpr uint32_t kM27 = (1u << 27) - 1;
-constexpr int kGroup = kScanWarps * 2;  // tiles per group = one CTA round (2 per warp)
+constexpr int kGroup = kGroupWarps * 2;  // tiles per select group (2 per warp)
 constexpr int kItemCache = 1024;  // item offsets cached in shared memory
 
 constexpr uint32_t kListCap = 128;  // events per tile kept as a sorted list
@@ -62,22 +72,17 @@ struct SelWarpSmem {
     uint32_t list[kListCap];
 };
 
-// scan: [pad to a 64 KiB shared-window boundary][table]; the per-warp walk
-// buffers and the item cache (aux) live in the pad when it is large enough,
-// else after the table.
-// The aux data must fit the pad, so that a scan CTA needs only 128 KiB of
-// dynamic shared memory and other batches' kernels can share the SM; the
-// kernel traps if the runtime layout ever leaves a smaller pad.
+// scan: [pad to a 64 KiB shared-window boundary][table][aux?]; the per-warp
+// walk buffers and the item cache (aux) live in the pad when it is large
+// enough (16-warp CTA: the CTA then needs only 128 KiB of dynamic shared
+// memory and other batches' kernels can share the SM), else after the table
+// (32-warp CTA).  The pad is 64 KiB minus the static smem, so the request
+// assumes at least kStaticMin bytes of static smem; the kernel traps if the
+// runtime layout disagrees.
 constexpr int kScanAux = kScanWarps * (int)sizeof(SelWarpSmem) + kItemCache * 8;
-constexpr int kScanSmem = 65536 + kTabBytes;
-static_assert(kScanAux <= 65536 - 1024 - 8192, "scan aux data must fit the alignment pad");
-
-struct EmitSmem {
-    SelWarpSmem w[kEmitWarps];
-    uint32_t fun[kGroup][32];
-    uint32_t te_state[kGroup], te_cnt[kGroup];
-    uint64_t items[kItemCache];
-};
+constexpr int kStaticMin = kHalves == 1 ? 8192 : 16384;
+constexpr bool kAuxInPad = kScanAux <= 65536 - 1024 - 10752;
+constexpr int kScanSmem = kAuxInPad ? 65536 + kTabBytes : 2 * 65536 - kStaticMin + kScanAux;
 
 // Group buffers in the scan (double buffering across the group barrier).
 constexpr int kFunBufs = 2;
@@ -93,18 +98,6 @@ __device__ __forceinline__ uint32_t lds(uint32_t addr) {
                                  // global loads in the scan, 8 = no per-tile epilogue
 #endif
 
-// 32 bytes at off with one 256-bit load (LDG.E.256, sm_100) when the address
-// is 32-byte aligned (a32) and the whole vector lies below lim16, else as
-// 16-byte vectors (at or beyond lim16: zero).  One request per lane-sector
-// instead of two halves the L1 tag work of the lane-strided scan loads.
-__device__ __forceinline__ void load32_v8(const uint8_t* base, uint32_t off, uint32_t lim16,
-                                          bool a32, uint32_t v[8]) {
-    if (DEDUP_SCAN_EXPERIMENT & 4) {
-#pragma unroll
-        for (int i = 0; i < 8; ++i) v[i] = off * 2654435761u + i;
-        return;
-    }
-    if (a32 && off + 32 <= lim16) {
 #ifndef DEDUP_SCAN_LDHINT
 #define DEDUP_SCAN_LDHINT 1  // 1: L1::no_allocate (measured +10 %), 2: L2::256B (no gain)
 #endif
@@ -115,10 +108,29 @@ __device__ __forceinline__ void load32_v8(const uint8_t* base, uint32_t off, uin
 #else
 #define DEDUP_LDV8 "ld.global.nc.v8.u32"
 #endif
-        asm(DEDUP_LDV8 " {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-            : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]),
-              "=r"(v[6]), "=r"(v[7])
-            : "l"(base + off));
+
+// One 256-bit load (LDG.E.256, sm_100) of 32 bytes at a 32-byte aligned p.
+// One request per lane-sector instead of two halves the L1 tag work of the
+// lane-strided scan loads; L1::no_allocate keeps the streamed bytes out of
+// the L1 that the table lookups share.
+__device__ __forceinline__ void ldg_v8(const uint8_t* p, uint32_t v[8]) {
+    if (DEDUP_SCAN_EXPERIMENT & 4) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) v[i] = (uint32_t)(uintptr_t)p * 2654435761u + i;
+        return;
+    }
+    asm(DEDUP_LDV8 " {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]),
+          "=r"(v[7])
+        : "l"(p));
+}
+
+// 32 bytes at off: ldg_v8 when 32-byte aligned (a32) and the vector lies below
+// lim16, else as 16-byte vectors (at or beyond lim16: zero).
+__device__ __forceinline__ void load32_v8(const uint8_t* base, uint32_t off, uint32_t lim16,
+                                          bool a32, uint32_t v[8]) {
+    if (a32 && off + 32 <= lim16) {
+        ldg_v8(base + off, v);
         return;
     }
     uint4 a = make_uint4(0, 0, 0, 0), b = make_uint4(0, 0, 0, 0);
@@ -378,6 +390,9 @@ __device__ __forceinline__ void prefetch_tile_l2(const uint8_t* bytes, uint64_t 
 #ifndef DEDUP_SCAN_TMA
 #define DEDUP_SCAN_TMA 0
 #endif
+#if DEDUP_SCAN_TMA && DEDUP_SCAN_CTA_WARPS != 16
+#error "the TMA ring fits the shared memory of a 16-warp scan CTA only"
+#endif
 #ifndef DEDUP_SCAN_STAGES
 #define DEDUP_SCAN_STAGES 3
 #endif
@@ -432,30 +447,36 @@ __device__ __forceinline__ void lds_row(uint32_t box, int lane, uint32_t v[8]) {
 // ILP-2 scan: a CTA of kScanWarps warps takes groups of 2 x kScanWarps tiles;
 // warp w rolls tiles w and w + kScanWarps of the group together.
 template <bool kZeroValue, bool kTma>
-__global__ void __launch_bounds__(kScanThreads, 2)  // <= 64 registers
+__global__ void __launch_bounds__(kScanThreads, 1024 / kScanThreads)  // <= 64 registers
 rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ gtab,
                        uint32_t mask, uint32_t value, uint32_t* __restrict__ bitmap,
                        uint32_t* __restrict__ agg, uint32_t* __restrict__ gagg,
                        uint32_t* __restrict__ evbuf) {
     extern __shared__ __align__(16) uint8_t smem[];
     __shared__ uint32_t src[512];
-    __shared__ uint32_t fun[kFunBufs][kGroup][32];
+    __shared__ uint32_t fun[kFunBufs][kHalves][kGroup][32];
     const uint8_t* __restrict__ bytes = desc->bytes;
     const uint32_t nbytes = (uint32_t)desc->nbytes;  // <= 2^30 (check_cfg)
     const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int half = wid / kGroupWarps, hw = wid % kGroupWarps;  // group slot, warp in group
     const uint32_t win = (uint32_t)__cvta_generic_to_shared(smem);
     const uint32_t pad = (0x10000u - (win & 0xFFFFu)) & 0xFFFFu;
     const uint32_t base = win + pad;
-    SelWarpSmem* wsm = reinterpret_cast<SelWarpSmem*>(smem);
-    if (pad < (uint32_t)kScanAux) __trap();  // layout assumption (see kScanSmem)
+    // layout assumptions (see kScanSmem)
+    if (kAuxInPad ? pad < (uint32_t)kScanAux
+                  : base + kTabBytes + kScanAux > win + (uint32_t)kScanSmem)
+        __trap();
+    SelWarpSmem* wsm = reinterpret_cast<SelWarpSmem*>(kAuxInPad ? smem : smem + pad + kTabBytes);
     uint64_t* icache = reinterpret_cast<uint64_t*>(wsm + kScanWarps);
     SelWarpSmem& sm = wsm[wid];
     const uint32_t n_tiles = (nbytes + kSelTile - 1) / kSelTile;
     const uint32_t n_groups = (n_tiles + kGroup - 1) / kGroup;
     const uint32_t lim16 = (nbytes + 15) & ~15u;
-    if (DEDUP_SCAN_L2PF && lane == 0 && blockIdx.x < n_groups) {  // first group, during the table build
-        prefetch_tile_l2(bytes, (uint64_t)blockIdx.x * kGroup + wid, lim16);
-        prefetch_tile_l2(bytes, (uint64_t)blockIdx.x * kGroup + wid + kScanWarps, lim16);
+    // CTA b, half h takes groups b * kHalves + h + k * gridDim.x * kHalves
+    const uint32_t g0 = blockIdx.x * kHalves + half, gstride = gridDim.x * kHalves;
+    if (DEDUP_SCAN_L2PF && lane == 0 && g0 < n_groups) {  // first group, during the table build
+        prefetch_tile_l2(bytes, (uint64_t)g0 * kGroup + hw, lim16);
+        prefetch_tile_l2(bytes, (uint64_t)g0 * kGroup + hw + kGroupWarps, lim16);
     }
     if (threadIdx.x < 512) src[threadIdx.x] = gtab[threadIdx.x];
     const uint64_t* items = cache_items(icache, desc);
@@ -492,10 +513,10 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
     auto tile_tma = [&](uint32_t t) { return (t + 1) * 32u <= tma_rows; };
     auto issue = [&](uint32_t v) {
         const uint32_t k = v / kUnitsPerTile, sidx = v % kUnitsPerTile;
-        const uint32_t g = blockIdx.x + k * gridDim.x;
+        const uint32_t g = g0 + k * gstride;
         if (g >= n_groups) return;
         const uint32_t st = v % kScanStages, mb = mbar0 + 8 * st;
-        const uint32_t t0 = g * kGroup + wid, t1 = t0 + kScanWarps;
+        const uint32_t t0 = g * kGroup + hw, t1 = t0 + kGroupWarps;
         const bool c0 = tile_tma(t0), c1 = tile_tma(t1);
         mbar_arrive_tx(mb, (c0 ? kBoxBytes : 0) + (c1 ? kBoxBytes : 0));
         const int x = sidx == 0 ? (int)(kLaneBytes - 32) : 32 * (int)(sidx - 1);
@@ -527,11 +548,11 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
         }
     };
     int par = 0;
-    for (uint32_t g = blockIdx.x; g < n_groups; g += gridDim.x, par ^= 1) {
-        const uint32_t tA = g * kGroup + wid, tB = tA + kScanWarps;
-        if (DEDUP_SCAN_L2PF && lane == 0 && g + gridDim.x < n_groups) {  // next group
-            prefetch_tile_l2(bytes, tA + gridDim.x * kGroup, lim16);
-            prefetch_tile_l2(bytes, tB + gridDim.x * kGroup, lim16);
+    for (uint32_t g = g0; g < n_groups; g += gstride, par ^= 1) {
+        const uint32_t tA = g * kGroup + hw, tB = tA + kGroupWarps;
+        if (DEDUP_SCAN_L2PF && lane == 0 && g + gstride < n_groups) {  // next group
+            prefetch_tile_l2(bytes, tA + gstride * kGroup, lim16);
+            prefetch_tile_l2(bytes, tB + gstride * kGroup, lim16);
         }
         const uint32_t qA = tA * kSelTile + lane * kLaneBytes;
         const uint32_t qB = tB * kSelTile + lane * kLaneBytes;
@@ -539,6 +560,8 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
 #pragma unroll
         for (int i = 0; i < 8; ++i) prevA[i] = curA[i] = prevB[i] = curB[i] = 0;
         const bool tmaA = kTma && tile_tma(tA), tmaB = kTma && tile_tma(tB);
+        // both tiles inside the batch and 32-byte aligned loads: no guards
+        const bool full = !kTma && a32 && (tB + 1) * kSelTile <= nbytes;
         fetch(qA - 32, qB - 32, qA >= 32 && qA < nbytes, qB >= 32 && qB < nbytes, tmaA, tmaB,
               prevA, prevB);
         fetch(qA, qB, qA < nbytes, qB < nbytes, tmaA, tmaB, curA, curB);
@@ -567,21 +590,30 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
             roll32x2<kZeroValue, 4, 8>(hA, inA, oldA, bitsA, hB, inB, oldB, bitsB, laneR, laneW,
                                        mask, value);
             if (j < 7) {  // the next step's bytes into the registers `old` just freed
+                if (full) {
+                    ldg_v8(bytes + bA0 + 32, oldA);
+                    ldg_v8(bytes + bB0 + 32, oldB);
+                } else {
 #pragma unroll
-                for (int i = 0; i < 8; ++i) oldA[i] = oldB[i] = 0;
-                fetch(bA0 + 32, bB0 + 32, bA0 + 32 < nbytes, bB0 + 32 < nbytes, tmaA, tmaB, oldA,
-                      oldB);
+                    for (int i = 0; i < 8; ++i) oldA[i] = oldB[i] = 0;
+                    fetch(bA0 + 32, bB0 + 32, bA0 + 32 < nbytes, bB0 + 32 < nbytes, tmaA, tmaB,
+                          oldA, oldB);
+                }
             }
             uint32_t ewA = __funnelshift_l(pbA, bitsA, 1), ewB = __funnelshift_l(pbB, bitsB, 1);
-            if (bA0 >= nbytes) ewA = 0;
-            else if (bA0 + 32 > nbytes) ewA &= (1u << (uint32_t)(nbytes - bA0)) - 1u;
-            if (bB0 >= nbytes) ewB = 0;
-            else if (bB0 + 32 > nbytes) ewB &= (1u << (uint32_t)(nbytes - bB0)) - 1u;
-            if (bA0 + 32 > nbytes) bitsA &= bA0 < nbytes ? (1u << (uint32_t)(nbytes - bA0)) - 1u : 0u;
-            if (bB0 + 32 > nbytes) bitsB &= bB0 < nbytes ? (1u << (uint32_t)(nbytes - bB0)) - 1u : 0u;
+            if (!full) {  // the batch's ragged end
+                if (bA0 >= nbytes) ewA = 0;
+                else if (bA0 + 32 > nbytes) ewA &= (1u << (uint32_t)(nbytes - bA0)) - 1u;
+                if (bB0 >= nbytes) ewB = 0;
+                else if (bB0 + 32 > nbytes) ewB &= (1u << (uint32_t)(nbytes - bB0)) - 1u;
+                if (bA0 + 32 > nbytes)
+                    bitsA &= bA0 < nbytes ? (1u << (uint32_t)(nbytes - bA0)) - 1u : 0u;
+                if (bB0 + 32 > nbytes)
+                    bitsB &= bB0 < nbytes ? (1u << (uint32_t)(nbytes - bB0)) - 1u : 0u;
+            }
             sm.cand[lane * 8 + j] = ewA;
-            if (tA < n_tiles) bitmap[tA * kSelTileWords + lane * 8 + j] = ewA;
-            if (tB < n_tiles) bitmap[tB * kSelTileWords + lane * 8 + j] = ewB;
+            if (full || tA < n_tiles) bitmap[tA * kSelTileWords + lane * 8 + j] = ewA;
+            if (full || tB < n_tiles) bitmap[tB * kSelTileWords + lane * 8 + j] = ewB;
             pbA = bitsA;
             pbB = bitsB;
         };
@@ -612,14 +644,15 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
             fB = (ex << 27) | cnt;
             agg[32 * tB + lane] = fB;
         }
-        fun[par][wid][lane] = fA;
-        fun[par][wid + kScanWarps][lane] = fB;
-        __syncthreads();
-        if (wid == 0) {
+        fun[par][half][hw][lane] = fA;
+        fun[par][half][hw + kGroupWarps][lane] = fB;
+        if (kHalves == 1) __syncthreads();
+        else asm volatile("bar.sync %0, %1;" ::"r"(1 + half), "r"(kGroupWarps * 32) : "memory");
+        if (hw == 0) {
             uint32_t Gs = lane, Gc = 0;
 #pragma unroll
             for (int j = 0; j < kGroup; ++j) {
-                const uint32_t a = fun[par][j][lane];
+                const uint32_t a = fun[par][half][j][lane];
                 const uint32_t ns = __shfl_sync(kFull, a >> 27, Gs);
                 const uint32_t nc = Gc + __shfl_sync(kFull, a & kM27, Gs);
                 Gs = ns;
@@ -690,58 +723,6 @@ select_scan_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restric
             Gs = ns;
             Gc = nc;
         }
-    }
-}
-
-// One CTA per group: entry states of the group's tiles from the group entry,
-// then the warps replay the group's tiles from their real entry states,
-// writing cut_pos.
-__global__ void __launch_bounds__(kEmitThreads)
-select_emit_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ bitmap,
-                   const uint32_t* __restrict__ agg, const uint32_t* __restrict__ gentry,
-                   uint32_t* __restrict__ cut_pos, uint64_t cap) {
-    extern __shared__ __align__(16) uint8_t smraw[];
-    EmitSmem& sm = *reinterpret_cast<EmitSmem*>(smraw);
-    const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const uint64_t nbytes = desc->nbytes;
-    const uint64_t n_tiles = (nbytes + kSelTile - 1) / kSelTile;
-    const uint64_t n_groups = (n_tiles + kGroup - 1) / kGroup;
-    const uint64_t* items = cache_items(sm.items, desc);
-    const uint32_t n_items = desc->n_items;
-    __syncthreads();
-    for (uint64_t g = blockIdx.x; g < n_groups; g += gridDim.x) {
-        for (int j = wid; j < kGroup; j += kEmitWarps) {
-            const uint64_t t = g * kGroup + j;
-            sm.fun[j][lane] = t < n_tiles ? agg[32 * t + lane] : ((uint32_t)lane << 27);
-        }
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            uint32_t s = gentry[2 * g], c = gentry[2 * g + 1];
-            for (int j = 0; j < kGroup; ++j) {
-                sm.te_state[j] = s;
-                sm.te_cnt[j] = c;
-                const uint32_t a = sm.fun[j][s];
-                c += a & kM27;
-                s = a >> 27;
-            }
-        }
-        __syncthreads();
-        for (int j = wid; j < kGroup; j += kEmitWarps) {
-            const uint64_t t = g * kGroup + j;
-            if (t >= n_tiles) break;
-            SelWarpSmem& w = sm.w[wid];
-#pragma unroll
-            for (int k = 0; k < 8; ++k)
-                w.cand[lane * 8 + k] = bitmap[t * kSelTileWords + lane * 8 + k];
-            const uint32_t n_ev = apply_items(w, t * kSelTile, nbytes, items, n_items, lane);
-            const uint32_t st = sm.te_state[j];
-            if (lane == (int)st) {
-                uint32_t ex;
-                walk_any(w, n_ev, st, ex, cut_pos, sm.te_cnt[j], cap, t * kSelTile);
-            }
-            __syncwarp();
-        }
-        __syncthreads();
     }
 }
 
@@ -891,11 +872,10 @@ void chunk_set_attrs() {
     for (const void* f : {(const void*)rabin_scan_agg2_kernel<true, false>,
                           (const void*)rabin_scan_agg2_kernel<false, false>})
         cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
-    for (const void* f : {(const void*)rabin_scan_agg2_kernel<true, true>,
-                          (const void*)rabin_scan_agg2_kernel<false, true>})
-        cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmemTma);
-    cudaFuncSetAttribute(select_emit_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)sizeof(EmitSmem));
+    if (DEDUP_SCAN_TMA)
+        for (const void* f : {(const void*)rabin_scan_agg2_kernel<true, true>,
+                              (const void*)rabin_scan_agg2_kernel<false, true>})
+            cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmemTma);
     cudaFuncSetAttribute(select_emit_ev_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)sizeof(EmitEvSmem));
     attr_set = true;
@@ -912,8 +892,6 @@ const char* chunk_unlaunchable() {
                               (const void*)rabin_scan_agg2_kernel<false, true>})
             if (!fits(f, kScanThreads, kScanSmemTma)) return "rabin_scan_agg2_kernel (TMA)";
     if (!fits((const void*)select_scan_kernel, 1024, 0)) return "select_scan_kernel";
-    if (!fits((const void*)select_emit_kernel, kEmitThreads, sizeof(EmitSmem)))
-        return "select_emit_kernel";
     if (!fits((const void*)select_emit_ev_kernel, kEmitEvWarps * 32, sizeof(EmitEvSmem)))
         return "select_emit_ev_kernel";
     if (!fits((const void*)chunk_meta_kernel, 256, 0)) return "chunk_meta_kernel";
@@ -955,10 +933,6 @@ bool encode_scan_tmap(BatchDesc& d) {
     return true;
 }
 
-#ifndef DEDUP_EMIT_EV
-#define DEDUP_EMIT_EV 1  // cut emission from stored event lists (0: rebuild every tile)
-#endif
-
 void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mask,
                          uint32_t value, uint32_t* bitmap, uint32_t* agg, uint32_t* gagg,
                          uint32_t* gentry, uint32_t* evbuf, uint64_t max_tiles,
@@ -966,7 +940,8 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
                          cudaStream_t s, cudaEvent_t after_scan) {
     chunk_set_attrs();
     const uint64_t groups = select_groups(max_tiles);
-    const unsigned grid = (unsigned)num_sms;
+    uint64_t gneed = (groups + kHalves - 1) / kHalves;
+    const unsigned grid = (unsigned)(gneed < (uint64_t)num_sms ? (gneed ? gneed : 1) : num_sms);
     // the kernel reads d->tma_rows at run time: 0 -> every tile on the LDG path
     if (DEDUP_SCAN_TMA) {
         auto k = value == 0 ? rabin_scan_agg2_kernel<true, true> : rabin_scan_agg2_kernel<false, true>;
@@ -978,19 +953,11 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
     }
     if (after_scan) cudaEventRecordWithFlags(after_scan, s, cudaEventRecordExternal);
     select_scan_kernel<<<1, 1024, 0, s>>>(d, gagg, gentry, n_chunks);
-    if (DEDUP_EMIT_EV) {
-        uint64_t blocks = (groups + kEmitEvWarps - 1) / kEmitEvWarps;
-        if (blocks > (uint64_t)num_sms * 4) blocks = (uint64_t)num_sms * 4;
-        if (blocks < 1) blocks = 1;
-        select_emit_ev_kernel<<<(unsigned)blocks, kEmitEvWarps * 32, sizeof(EmitEvSmem), s>>>(
-            d, bitmap, agg, gentry, evbuf, cut_pos, cap);
-        return;
-    }
-    uint64_t blocks = groups;
-    if (blocks > (uint64_t)num_sms) blocks = (uint64_t)num_sms;
+    uint64_t blocks = (groups + kEmitEvWarps - 1) / kEmitEvWarps;
+    if (blocks > (uint64_t)num_sms * 4) blocks = (uint64_t)num_sms * 4;
     if (blocks < 1) blocks = 1;
-    select_emit_kernel<<<(unsigned)blocks, kEmitThreads, sizeof(EmitSmem), s>>>(
-        d, bitmap, agg, gentry, cut_pos, cap);
+    select_emit_ev_kernel<<<(unsigned)blocks, kEmitEvWarps * 32, sizeof(EmitEvSmem), s>>>(
+        d, bitmap, agg, gentry, evbuf, cut_pos, cap);
 }
 
 void launch_chunk_meta(const BatchDesc* d, const uint32_t* cut_pos, const uint32_t* n_chunks,

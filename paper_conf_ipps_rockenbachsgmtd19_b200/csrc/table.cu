@@ -38,7 +38,7 @@ __device__ __forceinline__ void load_key(const uint8_t* digest, const uint64_t* 
         const uint32_t* p = reinterpret_cast<const uint32_t*>(digest + 20 * r);
 #pragma unroll
         for (int i = 0; i < 5; ++i) key[i] = p[i];
-        myid = id != nullptr ? id[r] : 0;
+        myid = id != nullptr ? id[r] : r;  // no ids: the record index (local combine)
     }
 }
 
@@ -165,15 +165,21 @@ __device__ __forceinline__ uint32_t owner_of(const uint8_t* digest, uint64_t r, 
     return (uint32_t)(((uint64_t)be * G) >> 32);
 }
 
+// rep (optional, local combine): only records with rep[r] == r are routed.
+__device__ __forceinline__ bool routed(const uint32_t* rep, uint64_t r) {
+    return rep == nullptr || rep[r] == (uint32_t)r;
+}
+
 __global__ void route_count_kernel(const uint8_t* __restrict__ digest, const uint32_t* d_n,
-                                   uint64_t cap, uint32_t G, uint32_t* counts) {
+                                   uint64_t cap, uint32_t G, const uint32_t* __restrict__ rep,
+                                   uint32_t* counts) {
     __shared__ uint32_t h[64];
     for (int i = threadIdx.x; i < 64; i += blockDim.x) h[i] = 0;
     __syncthreads();
     const uint64_t n = min((uint64_t)*d_n, cap);
     for (uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; r < n;
          r += (uint64_t)gridDim.x * blockDim.x)
-        atomicAdd(&h[owner_of(digest, r, G)], 1u);
+        if (routed(rep, r)) atomicAdd(&h[owner_of(digest, r, G)], 1u);
     __syncthreads();
     for (uint32_t i = threadIdx.x; i < G; i += blockDim.x)
         if (h[i]) atomicAdd(&counts[i], h[i]);
@@ -194,11 +200,13 @@ __global__ void route_scan_kernel(uint32_t G, uint32_t* counts, uint32_t* send_o
 
 __global__ void route_scatter_kernel(const uint8_t* __restrict__ digest,
                                      const uint64_t* __restrict__ id, const uint32_t* d_n,
-                                     uint64_t cap, uint32_t G, uint32_t* counts, uint8_t* send,
+                                     uint64_t cap, uint32_t G, const uint32_t* __restrict__ rep,
+                                     uint32_t* counts, uint8_t* send,
                                      uint32_t* __restrict__ send_pos) {
     const uint64_t n = min((uint64_t)*d_n, cap);
     for (uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; r < n;
          r += (uint64_t)gridDim.x * blockDim.x) {
+        if (!routed(rep, r)) continue;
         const uint32_t o = owner_of(digest, r, G);
         const uint32_t pos = atomicAdd(&counts[64 + o], 1u);
         uint32_t* dst = reinterpret_cast<uint32_t*>(send + 32 * (uint64_t)pos);
@@ -213,15 +221,47 @@ __global__ void route_scatter_kernel(const uint8_t* __restrict__ digest,
 
 __global__ void scatter_kernel(const uint64_t* __restrict__ reply,
                                const uint32_t* __restrict__ send_pos,
+                               const uint32_t* __restrict__ rep,
                                const uint64_t* __restrict__ id, const uint32_t* d_n, uint64_t cap,
                                uint64_t* __restrict__ first_id, uint8_t* __restrict__ is_dup) {
     const uint64_t n = min((uint64_t)*d_n, cap);
     for (uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; r < n;
          r += (uint64_t)gridDim.x * blockDim.x) {
-        const uint64_t f = reply[send_pos[r]];
+        // with local combine a chunk takes the reply of its representative
+        const uint64_t f = reply[send_pos[rep != nullptr ? rep[r] : (uint32_t)r]];
         first_id[r] = f;
         if (is_dup != nullptr) is_dup[r] = (f != id[r]) ? 1 : 0;
     }
+}
+
+// Local combine (row A5): after the insert of records 0..n-1 with ids = the
+// record index into the ctx's local table, rep[r] = the smallest index with
+// the same digest; then the slots this batch used are cleared again (O(n),
+// no full-table memset per wave).
+__global__ void combine_rep_kernel(TableView t, const uint32_t* d_n, uint64_t cap,
+                                   const uint32_t* __restrict__ slot_idx,
+                                   uint32_t* __restrict__ rep) {
+    const uint64_t n = min((uint64_t)*d_n, cap);
+    for (uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; r < n;
+         r += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t si = slot_idx[r];
+        rep[r] = si == 0xFFFFFFFFu ? (uint32_t)r : (uint32_t)~t.slots[si].inv_min;
+    }
+}
+
+__global__ void table_clear_used_kernel(TableView t, const uint32_t* d_n, uint64_t cap,
+                                        const uint32_t* __restrict__ slot_idx) {
+    const uint64_t n = min((uint64_t)*d_n, cap);
+    for (uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; r < n;
+         r += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t si = slot_idx[r];
+        if (si != 0xFFFFFFFFu) {
+            uint4* p = reinterpret_cast<uint4*>(t.slots + si);
+            p[0] = make_uint4(0, 0, 0, 0);
+            p[1] = make_uint4(0, 0, 0, 0);
+        }
+    }
+    if (blockIdx.x == 0 && threadIdx.x < 4) t.status[threadIdx.x] = 0;
 }
 
 __global__ void pack_kernel(const BatchDesc* __restrict__ desc,
@@ -290,23 +330,36 @@ void launch_table_lookup(const TableView* t, const uint64_t* id, const void* rec
 }
 
 void launch_route(const uint8_t* digest, const uint64_t* id, const uint32_t* d_n, uint64_t cap,
-                  uint32_t num_owners, void* send, uint32_t* send_off, uint32_t* send_pos,
-                  uint32_t* scratch_counts, int num_sms, cudaStream_t s) {
+                  const uint32_t* rep, uint32_t num_owners, void* send, uint32_t* send_off,
+                  uint32_t* send_pos, uint32_t* scratch_counts, int num_sms, cudaStream_t s) {
     cudaMemsetAsync(scratch_counts, 0, sizeof(uint32_t) * 128, s);
     const unsigned g = grid_for(cap, 256, num_sms, 4);
-    if (cap) route_count_kernel<<<g, 256, 0, s>>>(digest, d_n, cap, num_owners, scratch_counts);
+    if (cap)
+        route_count_kernel<<<g, 256, 0, s>>>(digest, d_n, cap, num_owners, rep, scratch_counts);
     route_scan_kernel<<<1, 32, 0, s>>>(num_owners, scratch_counts, send_off);
     if (cap)
-        route_scatter_kernel<<<g, 256, 0, s>>>(digest, id, d_n, cap, num_owners, scratch_counts,
-                                               static_cast<uint8_t*>(send), send_pos);
+        route_scatter_kernel<<<g, 256, 0, s>>>(digest, id, d_n, cap, num_owners, rep,
+                                               scratch_counts, static_cast<uint8_t*>(send),
+                                               send_pos);
 }
 
-void launch_scatter(const uint64_t* reply, const uint32_t* send_pos, const uint64_t* id,
-                    const uint32_t* d_n, uint64_t cap, uint64_t* first_id, uint8_t* is_dup,
-                    int num_sms, cudaStream_t s) {
+void launch_scatter(const uint64_t* reply, const uint32_t* send_pos, const uint32_t* rep,
+                    const uint64_t* id, const uint32_t* d_n, uint64_t cap, uint64_t* first_id,
+                    uint8_t* is_dup, int num_sms, cudaStream_t s) {
     if (cap == 0) return;
-    scatter_kernel<<<grid_for(cap, 256, num_sms, 8), 256, 0, s>>>(reply, send_pos, id, d_n, cap,
-                                                                  first_id, is_dup);
+    scatter_kernel<<<grid_for(cap, 256, num_sms, 8), 256, 0, s>>>(reply, send_pos, rep, id, d_n,
+                                                                  cap, first_id, is_dup);
+}
+
+void launch_local_combine(TableView local, const uint8_t* digest, const uint32_t* d_n,
+                          uint64_t cap, uint32_t* slot_idx, uint32_t* rep, int num_sms,
+                          cudaStream_t s, const TableView* d_local) {
+    if (cap == 0) return;
+    const unsigned g = grid_for(cap, 256, num_sms, 4);
+    table_insert_kernel<<<g, 256, 0, s>>>(d_local, digest, nullptr, nullptr, d_n, 0, cap,
+                                          slot_idx);
+    combine_rep_kernel<<<g, 256, 0, s>>>(local, d_n, cap, slot_idx, rep);
+    table_clear_used_kernel<<<g, 256, 0, s>>>(local, d_n, cap, slot_idx);
 }
 
 void launch_pack(const BatchDesc* d, const uint32_t* n_chunks, uint64_t cap, uint32_t max_items,

@@ -1,12 +1,18 @@
 """Multi-GPU orchestration of the dedup hot path (rows A5-A8).
 
 Batches (whole items) are processed in WAVES: in wave w every rank r runs
-its own batch through the device ops of include/dedup.h, then the digests are
-routed to their owner GPU, owner(d) = floor(BE32(d[0..3]) * G / 2^32)
-(row A5, kernel ``dedup_op_route``), exchanged with an all-to-all (row A6),
+its own batch through the device ops of include/dedup.h, collapses equal
+digests of the batch to one representative (the smallest chunk index, i.e.
+the smallest id; row A5 local combine, ``dedup_op_local_combine``), then the
+representatives' digests are routed to their owner GPU,
+owner(d) = floor(BE32(d[0..3]) * G / 2^32) (row A5, kernel
+``dedup_op_route``), exchanged with an all-to-all (row A6),
 inserted + looked up in the owner's table shard (row A7, ``dedup_op_owner``),
-and the first-occurrence ids are sent back and scattered to chunk order
-(row A8, ``dedup_op_scatter``).  Owners insert every record of a wave before
+and the first-occurrence ids are sent back and scattered to chunk order,
+every chunk taking its representative's reply (row A8, ``dedup_op_scatter``).
+The combine bounds the exchange and the owner's table work by the batch's
+distinct digests: an all-duplicate stream sends one record per wave instead
+of every chunk to one hot owner (SURVEY 8(e) "skew").  Owners insert every record of a wave before
 looking any of them up, and waves are processed in order, so the result is
 the sequential stream-order answer (reading O12) whatever the GPU
 count.  The paper itself has no inter-GPU step (GPUs take batches
@@ -115,10 +121,12 @@ def loopback_all_to_all(sends, counts):
 class RankState:
     """Device buffers + ctx of one rank (owner of one table shard)."""
 
-    def __init__(self, dedup, batch_bytes: int, batch_items: int, device, num_owners: int):
+    def __init__(self, dedup, batch_bytes: int, batch_items: int, device, num_owners: int,
+                 combine: bool = True):
         import torch
         self.d = dedup
         self.G = num_owners
+        self.combine = combine  # row A5 local combine: one record per distinct digest
         self.dev = device
         cap = batch_bytes // 32 + batch_items + 2
         self.cap = cap
@@ -133,6 +141,7 @@ class RankState:
         self.send = torch.zeros((cap, REC_WORDS), **i64)
         self.send_off = torch.zeros(self.G + 1, **i32)
         self.send_pos = torch.zeros(cap, **i32)
+        self.rep = torch.zeros(cap, **i32) if combine else None
         self.first_id = torch.zeros(cap, **i64)
         self.is_dup = torch.zeros(cap, dtype=torch.uint8, device=device)
         self.item_off_dev = torch.zeros(batch_items + 1, **i64)
@@ -150,10 +159,12 @@ class RankState:
         d.op_chunk_meta(self.item_off_dev, n_items, self.cut, self.n, self.cap, first_seq,
                         self.chunk_start, self.chunk_id, self.item_first)
         d.op_sha1(data, nbytes, self.cut, self.n, self.cap, self.digest)
+        if self.combine:
+            d.op_local_combine(self.digest, self.n, self.cap, self.rep)
         d.op_route(self.digest, self.chunk_id, self.n, self.cap, self.G, self.send,
-                   self.send_off, self.send_pos)
+                   self.send_off, self.send_pos, rep=self.rep)
         off = self.send_off.cpu().numpy().astype(np.int64)   # host sync (counts)
-        self.n_host = int(off[-1])
+        self.n_host = int(off[-1])  # records sent (distinct digests with combine)
         self.send_counts = np.diff(off).tolist()
         return self.send[:self.n_host], self.send_counts
 
@@ -167,11 +178,13 @@ class RankState:
 
     # phase 3: row A8 + read-back of this rank's results
     def finish(self, reply_back) -> WaveOut:
-        n = self.n_host
+        n_sent = self.n_host
+        n = int(self.n.item())
         if n:
             self.d.op_scatter(reply_back, self.send_pos, self.chunk_id, self.n, self.cap,
-                              self.first_id, self.is_dup)
+                              self.first_id, self.is_dup, rep=self.rep)
         n_items = len(self.item_off) - 1
+        self.sent_records = n_sent
         return WaveOut(
             first_seq=self.first_seq,
             item_len=np.diff(self.item_off),

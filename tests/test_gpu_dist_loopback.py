@@ -16,8 +16,8 @@ torch = pytest.importorskip("torch")
 MiB = 1 << 20
 
 
-@pytest.mark.parametrize("G", [1, 2, 4])
-def test_loopback_routing_matches_oracle(G):
+@pytest.mark.parametrize("G,combine", [(1, True), (2, True), (4, True), (2, False), (4, False)])
+def test_loopback_routing_matches_oracle(G, combine):
     assert torch.cuda.is_available()
     from paper_conf_ipps_rockenbachsgmtd19_b200 import Dedup
     from paper_conf_ipps_rockenbachsgmtd19_b200 import dist as D
@@ -33,7 +33,7 @@ def test_loopback_routing_matches_oracle(G):
                   table_capacity=1 << 16, host_fed=False, owner_rank=r, num_owners=G)
             for r in range(G)]
     try:
-        states = [D.RankState(c, bbytes, per_batch + 1, cuda, G) for c in ctxs]
+        states = [D.RankState(c, bbytes, per_batch + 1, cuda, G, combine=combine) for c in ctxs]
         got = []
         for w in range(0, len(batches), G):
             work = []
@@ -88,3 +88,71 @@ def test_route_owner_split_is_by_digest_prefix():
         assert soff[own[r]] <= p < soff[own[r] + 1]
         assert np.array_equal(raw[p, :20], dig[r])
         assert raw[p, 24:32].view(np.uint64)[0] == ids[r]
+
+
+def test_local_combine_representatives():
+    """Row A5 local combine: rep[r] = smallest index with an equal digest, on
+    duplicate-heavy digests; the local table is left empty (second call on
+    different data gives independent answers)."""
+    from paper_conf_ipps_rockenbachsgmtd19_b200 import Dedup
+    rng = np.random.default_rng(11)
+    with Dedup(0, batch_bytes=1 << 20, batch_items=4, slots=1, table_capacity=1 << 12) as d:
+        for trial, (n, distinct) in enumerate([(5000, 37), (4000, 4000), (3000, 1)]):
+            pool = rng.integers(0, 256, (distinct, 20), dtype=np.uint8)
+            pick = rng.integers(0, distinct, n)
+            dig = pool[pick]
+            td = torch.from_numpy(dig.reshape(-1).copy()).cuda()
+            tn = torch.tensor([n], dtype=torch.int32, device="cuda")
+            rep = torch.full((n,), -1, dtype=torch.int32, device="cuda")
+            d.op_local_combine(td, tn, n, rep)
+            got = rep.cpu().numpy().astype(np.int64)
+            first = {}
+            want = np.empty(n, np.int64)
+            for r in range(n):
+                want[r] = first.setdefault(dig[r].tobytes(), r)
+            assert np.array_equal(got, want), trial
+            used, _, ovf = d.op_table_status()
+            assert ovf == 0
+
+
+def test_combined_routing_sends_one_record_per_digest():
+    """All-duplicate stream (C5b-like): with the local combine each wave sends
+    one record per distinct digest, and results still match the oracle."""
+    from paper_conf_ipps_rockenbachsgmtd19_b200 import Dedup
+    from paper_conf_ipps_rockenbachsgmtd19_b200 import dist as D
+    item = U.stream(MiB // 2, seed=77, dup_frac=0.0)
+    data = np.tile(item, 8)
+    off = synthgen.split_items(data, MiB // 2)
+    n_items = len(off) - 1
+    G = 2
+    dev = torch.from_numpy(data).cuda()
+    cuda = torch.device("cuda", 0)
+    bbytes = 2 * MiB
+    ctxs = [Dedup(0, batch_bytes=bbytes, batch_items=5, slots=1, table_capacity=1 << 14,
+                  host_fed=False, owner_rank=r, num_owners=G) for r in range(G)]
+    try:
+        states = [D.RankState(c, bbytes, 5, cuda, G) for c in ctxs]
+        got, sent, chunks = [], 0, 0
+        for w in range(0, n_items, 2 * G):
+            work = []
+            for r in range(G):
+                k = w + 2 * r
+                j = min(k + 2, n_items)
+                work.append((dev[int(off[k]):int(off[j])], off[k:j + 1] - off[k], k))
+            for st, res in zip(states, D.loopback_waves(states, work)):
+                got.extend(res.items())
+                sent += st.sent_records
+                chunks += len(res.chunk_start)
+        torch.cuda.synchronize()
+    finally:
+        for c in ctxs:
+            c.close()
+    want, _ = oracle.dedup_items([data[int(off[k]):int(off[k + 1])] for k in range(n_items)])
+    distinct_per_item = len({bytes(x) for x in want[0].digest})
+    assert sent == (n_items // 2) * distinct_per_item  # one record per digest per batch
+    assert sent < chunks
+    got.sort(key=lambda r: r[0])
+    for (seq, cs, dg, dup, fid), w in zip(got, want):
+        assert np.array_equal(cs, w.chunk_start), seq
+        assert np.array_equal(dup, w.is_dup), seq
+        assert np.array_equal(fid, w.first_id), seq
