@@ -31,6 +31,7 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "dedup_oracle.cpp")
+_SRCS = [_SRC, os.path.join(_HERE, "findmatch_oracle.cpp")]   # NEXT-1 LZSS FindMatch
 _LIB = os.path.join(_HERE, "liboracle.so")
 
 # Defaults (SURVEY 8(c) readings O1-O3, O6, O7).
@@ -42,10 +43,11 @@ VALUE = 0
 
 def build_oracle(force: bool = False) -> str:
     """Compile the oracle shared library with g++ (no CUDA)."""
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+    if force or not os.path.exists(_LIB) or any(
+            os.path.getmtime(_LIB) < os.path.getmtime(s) for s in _SRCS):
         tmp = _LIB + f".tmp{os.getpid()}"
         subprocess.check_call(
-            ["g++", "-O2", "-std=c++17", "-shared", "-fPIC", "-o", tmp, _SRC])
+            ["g++", "-O2", "-std=c++17", "-shared", "-fPIC", "-o", tmp, *_SRCS])
         os.replace(tmp, _LIB)
     return _LIB
 
@@ -83,6 +85,12 @@ def lib():
         L.oracle_ctx_counts.argtypes = [ctypes.c_void_p, u64p]
         L.oracle_max_chunks.argtypes = [ctypes.c_uint64, ctypes.c_uint32]
         L.oracle_max_chunks.restype = ctypes.c_uint64
+        L.oracle_findmatch.argtypes = [u8p, ctypes.c_uint64, u32p, ctypes.c_uint32, u8p,
+                                       ctypes.c_uint32, ctypes.c_uint32, u64p, ctypes.c_uint64,
+                                       u32p, u32p]
+        L.oracle_findmatch.restype = ctypes.c_int
+        L.oracle_findmatch_block_linear.argtypes = [u32p, ctypes.c_uint32, ctypes.c_uint64]
+        L.oracle_findmatch_block_linear.restype = ctypes.c_int64
         _lib = L
     return _lib
 
@@ -205,3 +213,40 @@ def dedup_items(items, params: Params = Params(), first_seq: int = 0):
         return [s.item(first_seq + k, it) for k, it in enumerate(items)], s.counts()
     finally:
         s.close()
+
+
+# ------------------------------------------------------------------ NEXT-1 --
+# LZSS FindMatch (Listing 3; readings L1-L6 in
+# findmatch_oracle.cpp and DESIGN.md).
+LZSS_WINDOW = 4096
+LZSS_MAX_CODED = 18
+
+
+def findmatch(data, starts, window: int = LZSS_WINDOW, max_coded: int = LZSS_MAX_CODED,
+              positions=None, skip=None):
+    """(length u32[n], offset u32[n]) for every byte of `data` (or the given
+    positions).  `starts`: strictly increasing block starts, starts[0] == 0."""
+    a, p = _u8(data)
+    st = np.ascontiguousarray(starts, dtype=np.uint32)
+    u32p = ctypes.POINTER(ctypes.c_uint32)
+    pos = None if positions is None else np.ascontiguousarray(positions, dtype=np.uint64)
+    n = len(a) if pos is None else len(pos)
+    ln = np.zeros(max(n, 1), np.uint32)
+    of = np.zeros(max(n, 1), np.uint32)
+    sk = None if skip is None else np.ascontiguousarray(skip, dtype=np.uint8)
+    rc = lib().oracle_findmatch(
+        p, len(a), st.ctypes.data_as(u32p), len(st),
+        None if sk is None else sk.ctypes.data_as(ctypes.POINTER(ctypes.c_uint8)),
+        window, max_coded,
+        None if pos is None else pos.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)), n,
+        ln.ctypes.data_as(u32p), of.ctypes.data_as(u32p))
+    if rc != 0:
+        raise ValueError("oracle_findmatch: bad arguments")
+    return ln[:n].copy(), of[:n].copy()
+
+
+def findmatch_block_linear(starts, idx: int) -> int:
+    """Listing 3 lines 4-10 as listed (linear scan): the block index of idx."""
+    st = np.ascontiguousarray(starts, dtype=np.uint32)
+    return int(lib().oracle_findmatch_block_linear(
+        st.ctypes.data_as(ctypes.POINTER(ctypes.c_uint32)), len(st), idx))

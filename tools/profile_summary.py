@@ -1,6 +1,7 @@
 """Write profiles/<tag>_ncu_summary.md + profiles/ncu_traffic.json from
 gpurun_out/bench_launches.csv and gpurun_out/prof_full.ncu-rep."""
 import csv
+import re
 import json
 import subprocess
 import sys
@@ -8,6 +9,11 @@ from collections import defaultdict
 
 tag = sys.argv[1] if len(sys.argv) > 1 else "r01"
 BATCH = 64 << 20
+
+
+def kname(full):
+    s = re.sub(r'\(anonymous namespace\)::|unnamed>::|^void ', '', full)
+    return s.split('(')[0].split('<')[0].split('::')[-1].strip()
 
 
 def launch_table(path):
@@ -21,7 +27,7 @@ def launch_table(path):
             continue
         v = float(r[vi].replace(',', ''))
         us = v / 1000.0 if r[ui] in ('nsecond', 'ns') else (v * 1000.0 if r[ui] in ('msecond', 'ms') else v)
-        agg[r[ki].split('(')[0].split('<')[0].split('::')[-1].strip()].append(us)
+        agg[kname(r[ki])].append(us)
     tot = sum(sum(v) for v in agg.values())
     out = ['| kernel | launches | mean us | share of summed time |', '|---|---|---|---|']
     for k, v in sorted(agg.items(), key=lambda kv: -sum(kv[1])):
@@ -47,7 +53,7 @@ def full_table(rep):
              '|---' * (len(M) + 2) + '|']
     traffic = {}
     for r in rows[2:]:
-        name = r[h.index('Kernel Name')].split('(')[0].split('<')[0].split('::')[-1].strip()
+        name = kname(r[h.index('Kernel Name')])
         vals = [r[h.index(m)] if m in h else '' for m in M]
         st = [(k.split('issue_stalled_')[1].split('_per')[0], float(r[i])) for i, k in enumerate(h)
               if k.startswith('smsp__average_warps_issue_stalled_') and k.endswith('per_issue_active.ratio') and r[i]]
