@@ -234,6 +234,9 @@ def reference_arm(args, data, off):
     print(json.dumps(line), flush=True)
 
 
+HBM_PEAK = 6462.1  # overwritten from MEASURED_PEAKS.json in main()
+
+
 def isolated_kernels(dd, off, int_peak, copies=4, reps=3, streams=4):
     """Live per-kernel throughput with the GPU filled by one kernel type.
 
@@ -279,6 +282,16 @@ def isolated_kernels(dd, off, int_peak, copies=4, reps=3, streams=4):
         sha_us = ev[1].elapsed_time(ev[2]) * 1e3 / (reps * streams)  # per launch's worth
         k = int(n.item())
         cp = cut[:k].cpu().numpy().astype(np.int64)
+        # row NEXT-1 (LZSS FindMatch over the same blocks; not part of the step)
+        fl = torch.empty(nb, dtype=torch.uint8, device="cuda")
+        fo = torch.empty(nb, dtype=torch.int16, device="cuda")
+        ctxs[0].op_findmatch(data, nb, cut, n, cap, fl, fo)
+        ev[0].record()
+        ctxs[0].op_findmatch(data, nb, cut, n, cap, fl, fo)
+        ev[1].record()
+        ev[1].synchronize()
+        fm_us = ev[0].elapsed_time(ev[1]) * 1e3
+        del fl, fo
     finally:
         for c in ctxs:
             c.close()
@@ -292,12 +305,19 @@ def isolated_kernels(dd, off, int_peak, copies=4, reps=3, streams=4):
                  "input_gbs": nb / (sha_us * 1e-6) / 1e9, "blocks": blocks,
                  "note": f"{streams} concurrent streams x {reps} launches; launch_us = "
                          "joint elapsed / launches"},
+        "findmatch": {"row": "NEXT-1 (LZSS FindMatch, Listing 3), W=4096, MAX_CODED=18",
+                      "bound": "hbm", "achieved": nb * 4 / (fm_us * 1e-6) / 1e9,
+                      "peak": HBM_PEAK, "unit": "GB/s",
+                      "frac": nb * 4 / (fm_us * 1e-6) / 1e9 / HBM_PEAK,
+                      "launch_us": fm_us, "input_gbs": nb / (fm_us * 1e-6) / 1e9,
+                      "note": "algorithmic HBM bytes: 1 B read + 3 B written (u8 length, "
+                              "u16 offset) per input byte; search-bound, see DESIGN.md"},
         "chunk_stage": {"bound": "alu", "achieved": scan_ops, "peak": int_peak, "unit": "Tops/s",
                         "frac": scan_ops / int_peak, "launch_us": chunk_us,
                         "input_gbs": nb / (chunk_us * 1e-6) / 1e9,
                         "note": "scan + select_scan + select_emit, one op_chunk call; "
                                 "HBM: reads 1 B/B -> "
-                                f"{nb / (chunk_us * 1e-6) / 1e9 / 6462.1:.3f} of the copy peak"},
+                                f"{nb / (chunk_us * 1e-6) / 1e9 / HBM_PEAK:.3f} of the copy peak"},
     }
 
 
@@ -375,6 +395,8 @@ def main():
 
     # ---- rooflines ----
     pk, src = peaks()
+    global HBM_PEAK
+    HBM_PEAK = float(pk.get("hbm_gbs", HBM_PEAK))
     clocks = clk.summary()
     sm_mhz = pk.get("sm_max_mhz", 1965.0)
     int_peak = 148 * INT_LANES_PER_SM_CLK * sm_mhz * 1e6 / 1e12      # Tops/s

@@ -286,6 +286,29 @@ dedup_status dedup_op_scatter(dedup_ctx* c, void* stream, const uint64_t* d_repl
                               const uint64_t* d_id, const uint32_t* d_n, uint64_t cap,
                               uint64_t* d_first_id, uint8_t* d_is_dup);
 
+/* Row NEXT-1: LZSS FindMatch over a resident batch -- stage 4
+ * of the paper's GPU Dedup ("compress every not duplicated blocks on GPU ...
+ * reuses data already on GPU"), one launch over all blocks of the
+ * batch bounded by startPos (Listing 3 at P:227-290; readings
+ * L1-L6 in DESIGN.md).  Blocks: k < n = min(*d_n_blocks, cap), block k =
+ * d_bytes[d_start[k], d_start[k+1]) (the last one ends at nbytes); d_start
+ * must be strictly increasing with d_start[0] == 0 (e.g. dedup_op_chunk's
+ * d_cut_pos) -- other lists give unspecified (but in-bounds) results.
+ * For every byte i < nbytes, inside its block [bs, be), writes the longest
+ * match length L = d_match_len[i] (u8) of block[c..c+L) == block[i..i+L) over
+ *     max(i - window, bs) <= c < i,  c + L <= i,  i + L <= be,  L <= max_coded
+ * (the earliest c among the longest; L = 0 when no earlier byte in the
+ * window equals byte i) and d_match_off[i] = (c - bs) mod window (u16; 0 when
+ * L = 0).  d_skip (optional, u8 per block): positions of blocks with a
+ * non-zero flag (duplicates) get L = 0, offset 0.
+ * d_bytes 16-byte aligned and readable to nbytes rounded up to 16;
+ * nbytes < 2^31; 1 <= window <= 32768; 1 <= max_coded <= 255; else EINVAL. */
+dedup_status dedup_op_findmatch(dedup_ctx* c, void* stream, const uint8_t* d_bytes,
+                                uint64_t nbytes, const uint32_t* d_start,
+                                const uint32_t* d_n_blocks, uint64_t cap, const uint8_t* d_skip,
+                                uint32_t window, uint32_t max_coded, uint8_t* d_match_len,
+                                uint16_t* d_match_off);
+
 /* Number of kernels this ctx has launched so far (all layers). */
 uint64_t dedup_kernel_launches(const dedup_ctx* c);
 

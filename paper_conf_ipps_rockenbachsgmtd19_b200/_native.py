@@ -33,7 +33,7 @@ EXPORTS = [
     "dedup_op_chunk", "dedup_op_chunk_meta", "dedup_op_sha1", "dedup_op_table_insert_lookup",
     "dedup_op_table_reset", "dedup_op_table_status", "dedup_op_local_combine",
     "dedup_op_route", "dedup_op_owner",
-    "dedup_op_scatter", "dedup_kernel_launches",
+    "dedup_op_scatter", "dedup_op_findmatch", "dedup_kernel_launches",
 ]
 
 
@@ -110,6 +110,7 @@ def lib():
         "dedup_op_chunk": (st, [vp, vp, vp, u64, vp, u32, vp, u64, vp]),
         "dedup_op_chunk_meta": (st, [vp, vp, vp, u32, vp, vp, u64, u64, vp, vp, vp]),
         "dedup_op_sha1": (st, [vp, vp, vp, u64, vp, vp, u64, vp]),
+        "dedup_op_findmatch": (st, [vp, vp, vp, u64, vp, vp, u64, vp, u32, u32, vp, vp]),
         "dedup_op_table_insert_lookup": (st, [vp, vp, vp, vp, vp, u64, vp, vp]),
         "dedup_op_table_reset": (st, [vp, vp]),
         "dedup_op_table_status": (st, [vp, vp, P(u64), P(u64), P(i32)]),

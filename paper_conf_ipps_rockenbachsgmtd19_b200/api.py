@@ -239,6 +239,14 @@ class Dedup:
         self._check(N.lib().dedup_op_sha1(self._ctx, _stream(stream), _ptr(data), nbytes,
                                           _ptr(cut_pos), _ptr(n_chunks), cap, _ptr(digest)))
 
+    def op_findmatch(self, data, nbytes, starts, n_blocks, cap, match_len, match_off,
+                     window=4096, max_coded=18, skip=None, stream=None):
+        """Row NEXT-1: LZSS FindMatch of every byte inside its block
+        (include/dedup.h dedup_op_findmatch; Listing 3)."""
+        self._check(N.lib().dedup_op_findmatch(
+            self._ctx, _stream(stream), _ptr(data), nbytes, _ptr(starts), _ptr(n_blocks), cap,
+            _ptr(skip), window, max_coded, _ptr(match_len), _ptr(match_off)))
+
     def op_table(self, digest, ids, n, cap, first_id, is_dup=None, stream=None):
         self._check(N.lib().dedup_op_table_insert_lookup(
             self._ctx, _stream(stream), _ptr(digest), _ptr(ids), _ptr(n), cap, _ptr(first_id),

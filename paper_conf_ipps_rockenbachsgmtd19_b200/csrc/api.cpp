@@ -887,6 +887,34 @@ dedup_status dedup_op_sha1(dedup_ctx* c, void* stream, const uint8_t* d_bytes, u
     return DEDUP_OK;
 }
 
+dedup_status dedup_op_findmatch(dedup_ctx* c, void* stream, const uint8_t* d_bytes,
+                                uint64_t nbytes, const uint32_t* d_start,
+                                const uint32_t* d_n_blocks, uint64_t cap, const uint8_t* d_skip,
+                                uint32_t window, uint32_t max_coded, uint8_t* d_match_len,
+                                uint16_t* d_match_off) {
+    if (c == nullptr) return DEDUP_EINVAL;
+    if (!usable(c)) return c->sticky;
+    if (reinterpret_cast<uintptr_t>(d_bytes) & 15)
+        return fail(c, DEDUP_EINVAL, "d_bytes must be 16-byte aligned");
+    if (reinterpret_cast<uintptr_t>(d_match_off) & 1)
+        return fail(c, DEDUP_EINVAL, "d_match_off must be 2-byte aligned");
+    if (nbytes >= (1ull << 31)) return fail(c, DEDUP_EINVAL, "nbytes >= 2^31");
+    if (window < 1 || window > 32768) return fail(c, DEDUP_EINVAL, "window not in [1, 32768]");
+    if (max_coded < 1 || max_coded > 255)
+        return fail(c, DEDUP_EINVAL, "max_coded not in [1, 255]");
+    if (nbytes > 0 && (d_start == nullptr || d_n_blocks == nullptr || cap == 0))
+        return fail(c, DEDUP_EINVAL, "no block starts");
+    CU(cudaSetDevice(c->cfg.device));
+    if (const char* k = findmatch_unlaunchable(window, max_coded))
+        return fail(c, DEDUP_EINVAL, std::string(k) + " does not fit this window");
+    launch_findmatch(d_bytes, (uint32_t)nbytes, d_start, d_n_blocks, cap, d_skip, window,
+                     max_coded, d_match_len, d_match_off, c->num_sms,
+                     static_cast<cudaStream_t>(stream));
+    c->launches += nbytes ? 1 : 0;
+    CU(cudaGetLastError());
+    return DEDUP_OK;
+}
+
 dedup_status dedup_op_table_insert_lookup(dedup_ctx* c, void* stream, const uint8_t* d_digest,
                                           const uint64_t* d_id, const uint32_t* d_n, uint64_t cap,
                                           uint64_t* d_first_id, uint8_t* d_is_dup) {

@@ -119,6 +119,14 @@ void launch_local_combine(TableView local, const uint8_t* digest, const uint32_t
                           uint64_t cap, uint32_t* slot_idx, uint32_t* rep, int num_sms,
                           cudaStream_t s, const TableView* d_local);
 
+// ---- LZSS FindMatch (lzss.cu, row NEXT-1) ----------------------------------
+uint32_t findmatch_smem(uint32_t window, uint32_t max_coded);
+const char* findmatch_unlaunchable(uint32_t window, uint32_t max_coded);
+void launch_findmatch(const uint8_t* bytes, uint32_t nbytes, const uint32_t* cut_pos,
+                      const uint32_t* n_chunks, uint64_t cap, const uint8_t* skip,
+                      uint32_t window, uint32_t max_coded, uint8_t* out_len, uint16_t* out_off,
+                      int num_sms, cudaStream_t s);
+
 // Results of one batch written straight into mapped pinned host memory.
 struct HostResultLayout {
     uint32_t* header;          // [0] n_chunks, [1] table overflow flag, [2] used slots
