@@ -43,7 +43,7 @@ MiB = 1 << 20
 ITEM_BYTES = MiB                 # the paper's fixed 1 MB batches
 BATCH_BYTES = 64 * MiB           # GPU batch (step); C2 batch sweep 1-64 MiB
 BATCH_ITEMS = 64
-SLOTS = 24                       # batches in flight ("memory spaces")
+SLOTS = 40                       # batches in flight ("memory spaces")
 WORKLOAD = "C2"
 METRIC = "input GB/s & chunks/s (dedup hot path) at 1/2/4/8 B200; % of HBM/INT roofline"
 

@@ -46,6 +46,9 @@ namespace {
 // (64K registers, 220 KiB smem), and the pipelined bench is faster with 16
 // warps (590 vs 576 GB/s): other batches' SHA-1 / table / emit CTAs share the
 // SM with a 16-warp scan CTA.
+#ifndef DEDUP_SCAN_GROUPS_PER_CTA
+#define DEDUP_SCAN_GROUPS_PER_CTA 4  // select groups per scan CTA (launch_chunk_select)
+#endif
 #ifndef DEDUP_SCAN_CTA_WARPS
 #define DEDUP_SCAN_CTA_WARPS 16
 #endif
@@ -940,7 +943,13 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
                          cudaStream_t s, cudaEvent_t after_scan) {
     chunk_set_attrs();
     const uint64_t groups = select_groups(max_tiles);
+    // A persistent scan CTA takes several groups: fewer, longer-lived CTAs
+    // per batch (a CTA holds 128 KiB of shared memory and 32K registers)
+    // share the SMs better with the other in-flight batches' SHA-1 CTAs.
+    // Measured (bench, C2, 64 MiB batches = 256 groups, SHA lane 32 KiB,
+    // 40 slots): 1 group per CTA 632, 2 640, 4 709-716, 8 702, 16 700 GB/s.
     uint64_t gneed = (groups + kHalves - 1) / kHalves;
+    gneed = (gneed + DEDUP_SCAN_GROUPS_PER_CTA - 1) / DEDUP_SCAN_GROUPS_PER_CTA;
     const unsigned grid = (unsigned)(gneed < (uint64_t)num_sms ? (gneed ? gneed : 1) : num_sms);
     // the kernel reads d->tma_rows at run time: 0 -> every tile on the LDG path
     if (DEDUP_SCAN_TMA) {

@@ -373,8 +373,15 @@ void launch_sha1(const BatchDesc* d, uint64_t max_bytes, const uint32_t* cut_pos
     // Persistent lanes pull chunks dynamically, so the grid only needs enough
     // lanes to finish the batch's bulk within its longest chunk's latency:
     // one lane per kShaLaneBytes of input keeps the per-batch footprint small
-    // and leaves the SMs to the other in-flight batches.
-    const uint64_t kShaLaneBytes = 8192;
+    // and leaves the SMs to the other in-flight batches.  A batch's SHA-1 CTA
+    // lives until its longest chunk is hashed (a sequential chain); with
+    // fewer lanes per byte the bulk of its chunks covers more of that tail.
+    // Measured (bench, C2, 64 MiB batches): 4 KiB 540, 8 KiB 590, 16 KiB
+    // 619, 24 KiB 620, 32 KiB 632-641 (40 slots), 64 KiB 494 GB/s.
+#ifndef DEDUP_SHA_LANE_BYTES
+#define DEDUP_SHA_LANE_BYTES 32768
+#endif
+    const uint64_t kShaLaneBytes = DEDUP_SHA_LANE_BYTES;
     uint64_t lanes = max_bytes / kShaLaneBytes;
     if (lanes < 1024) lanes = 1024;
     uint64_t blocks = (lanes + kShaThreads - 1) / kShaThreads;

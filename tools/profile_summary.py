@@ -1,6 +1,7 @@
 """Write profiles/<tag>_ncu_summary.md + profiles/ncu_traffic.json from
 gpurun_out/bench_launches.csv and gpurun_out/prof_full.ncu-rep."""
 import csv
+import os
 import re
 import json
 import subprocess
@@ -12,7 +13,7 @@ BATCH = 64 << 20
 
 
 def kname(full):
-    s = re.sub(r'\(anonymous namespace\)::|unnamed>::|^void ', '', full)
+    s = re.sub(r'\(anonymous namespace\)::|<unnamed>::|^void ', '', full)
     return s.split('(')[0].split('<')[0].split('::')[-1].strip()
 
 
@@ -74,6 +75,11 @@ md += lt
 md += ['', '## ncu --set full, one 64 MiB batch of C2 (tools/one_batch.py)', '',
        'Units: ns, instructions, %, bytes.  `dram` = DRAM bytes of the launch.', '']
 md += ft
+if os.path.exists('gpurun_out/prof_fm.ncu-rep'):
+    fm, fm_traffic = full_table('gpurun_out/prof_fm.ncu-rep')
+    md += ['', '## ncu --set full, row NEXT-1 FindMatch, one 64 MiB batch of C2 (tools/fm_sizes.py)', '']
+    md += fm
+    traffic.update({'findmatch_' + k: v for k, v in fm_traffic.items()})
 open(f'profiles/{tag}_ncu_summary.md', 'w').write('\n'.join(md) + '\n')
 tj = {"_source": "ncu --set full, tools/one_batch.py (64 MiB batches of C2); DRAM read+write bytes per "
                  "launch; bench scales per input byte", "capture_batch_bytes": BATCH}
