@@ -31,7 +31,8 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "dedup_oracle.cpp")
-_SRCS = [_SRC, os.path.join(_HERE, "findmatch_oracle.cpp")]   # NEXT-1 LZSS FindMatch
+_SRCS = [_SRC, os.path.join(_HERE, "findmatch_oracle.cpp"),   # NEXT-1 LZSS FindMatch
+         os.path.join(_HERE, "mandel_oracle.cpp")]      # NEXT-4 Mandelbrot
 _LIB = os.path.join(_HERE, "liboracle.so")
 
 # Defaults (SURVEY 8(c) readings O1-O3, O6, O7).
@@ -47,7 +48,8 @@ def build_oracle(force: bool = False) -> str:
             os.path.getmtime(_LIB) < os.path.getmtime(s) for s in _SRCS):
         tmp = _LIB + f".tmp{os.getpid()}"
         subprocess.check_call(
-            ["g++", "-O2", "-std=c++17", "-shared", "-fPIC", "-o", tmp, *_SRCS])
+            ["g++", "-O2", "-std=c++17", "-ffp-contract=off", "-shared", "-fPIC", "-o", tmp,
+             *_SRCS])
         os.replace(tmp, _LIB)
     return _LIB
 
@@ -91,6 +93,12 @@ def lib():
         L.oracle_findmatch.restype = ctypes.c_int
         L.oracle_findmatch_block_linear.argtypes = [u32p, ctypes.c_uint32, ctypes.c_uint64]
         L.oracle_findmatch_block_linear.restype = ctypes.c_int64
+        L.oracle_mandel_rows.argtypes = [ctypes.c_int32, ctypes.c_int32, ctypes.c_double,
+                                         ctypes.c_double, ctypes.c_double, ctypes.c_int32,
+                                         ctypes.c_int32, u8p]
+        L.oracle_mandel_rows.restype = ctypes.c_int
+        L.oracle_mandel_iters.argtypes = [ctypes.c_double, ctypes.c_double, ctypes.c_int32]
+        L.oracle_mandel_iters.restype = ctypes.c_int32
         _lib = L
     return _lib
 
@@ -250,3 +258,27 @@ def findmatch_block_linear(starts, idx: int) -> int:
     st = np.ascontiguousarray(starts, dtype=np.uint32)
     return int(lib().oracle_findmatch_block_linear(
         st.ctypes.data_as(ctypes.POINTER(ctypes.c_uint32)), len(st), idx))
+
+
+# ------------------------------------------------------------------ NEXT-4 --
+# Mandelbrot Streaming (Section IV-A, Listing 1; readings
+# M1-M4 in mandel_oracle.cpp and DESIGN.md).
+MANDEL_INIT_A, MANDEL_INIT_B, MANDEL_RANGE = -2.125, -1.5, 3.0
+
+
+def mandel_rows(dim: int, niter: int, row0: int = 0, nrows: int | None = None,
+                init_a: float = MANDEL_INIT_A, init_b: float = MANDEL_INIT_B,
+                rng: float = MANDEL_RANGE) -> np.ndarray:
+    """Rows [row0, row0 + nrows) of the dim x dim image (uint8 [nrows, dim])."""
+    nrows = dim - row0 if nrows is None else nrows
+    out = np.zeros((nrows, dim), np.uint8)
+    rc = lib().oracle_mandel_rows(dim, niter, init_a, init_b, rng, row0, nrows,
+                                  out.ctypes.data_as(ctypes.POINTER(ctypes.c_uint8)))
+    if rc != 0:
+        raise ValueError("oracle_mandel_rows: bad arguments")
+    return out
+
+
+def mandel_iters(cr: float, im: float, niter: int) -> int:
+    """Escape count k of one point (inner loop of Listing 1)."""
+    return int(lib().oracle_mandel_iters(cr, im, niter))
