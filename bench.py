@@ -321,6 +321,52 @@ def isolated_kernels(dd, off, int_peak, copies=4, reps=3, streams=4):
     }
 
 
+# Row NEXT-4 (Mandelbrot Streaming, Section IV-A): the paper's image.
+MANDEL_DIM, MANDEL_NITER = 2000, 200000
+MANDEL_BATCH_ROWS, MANDEL_SPACES = 1000, 2
+# binary64 pipe operations per iteration of Listing 1 (lines 15-19, no FMA):
+# a*a, b*b, a2+b2, 2*a, (2a)*b, +im, a2-b2, +cr and the compare with 4.0 (DSETP
+# issues to the FP64 pipe: ncu's fp64-pipe utilisation of the kernel matches
+# 9 ops x 64 lanes/clk/SM)
+MANDEL_FP64_OPS_PER_ITER = 9
+# FP64 lanes per SM per clock on B200 (derived: no FP64 figure in
+# MEASURED_PEAKS.json / B200_PROFILING.md; 64/clk/SM = the B200 FP64 rating
+# of ~37 TFLOPS FMA at 1.965 GHz; ncu's fp64-pipe utilisation checks it)
+FP64_LANES_PER_SM_CLK = 64
+
+
+def mandel_measure(sm_mhz, with_cpu=True):
+    from paper_conf_ipps_rockenbachsgmtd19_b200 import mandel as M
+    M.image(200, 1000, 32, 2)  # warm-up
+    best = None
+    for _ in range(3):
+        _, ms, iters = M.image(MANDEL_DIM, MANDEL_NITER, MANDEL_BATCH_ROWS, MANDEL_SPACES)
+        best = ms if best is None else min(best, ms)
+    peak = 148 * FP64_LANES_PER_SM_CLK * sm_mhz * 1e6 / 1e12
+    ach = iters * MANDEL_FP64_OPS_PER_ITER / (best * 1e-3) / 1e12
+    out = {"row": "NEXT-4 (Mandelbrot Streaming, Listings 1-2)",
+           "workload": f"{MANDEL_DIM}x{MANDEL_DIM}, niter {MANDEL_NITER} (P:131), frame "
+                       f"[-2.125, 0.875] x [-1.5, 1.5], batches of {MANDEL_BATCH_ROWS} rows, "
+                       f"{MANDEL_SPACES} memory spaces, D2H into pinned host memory",
+           "image_ms": best, "iterations": iters, "t_iter_per_s": iters / (best * 1e-3) / 1e12,
+           "bound": "fp64", "achieved": ach, "peak": peak, "unit": "T binary64 pipe ops/s",
+           "frac": ach / peak,
+           "peak_source": f"derived: 148 SM x {FP64_LANES_PER_SM_CLK} FP64 lanes/clk x "
+                          f"{sm_mhz:.0f} MHz",
+           "paper_context": "400 s sequential (i9-7900X), 3.02 s on 2x Titan XP (P:131, P:185)"}
+    if with_cpu:
+        import oracle
+        t0 = time.perf_counter()
+        oracle.mandel_rows(MANDEL_DIM, MANDEL_NITER, row0=1000, nrows=1)
+        dt = time.perf_counter() - t0
+        step = 3.0 / MANDEL_DIM
+        row_iters = sum(oracle.mandel_iters(-2.125 + step * j, -1.5 + step * 1000, MANDEL_NITER)
+                        for j in range(MANDEL_DIM))
+        out["cpu_baseline"] = {"value": row_iters / dt / 1e12, "unit": "T iter/s", "cores": 1,
+                               "kind": "oracle", "sample": "row 1000 (the densest) of the image"}
+    return out
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -416,6 +462,7 @@ def main():
     }
     iso = isolated_kernels(dd, off, int_peak)
     kernels.update(iso)
+    kernels["mandelbrot"] = mandel_measure(sm_mhz, with_cpu=not args.no_cpu_baseline)
     sha_blocks_per_byte = ds["sha1_blocks"] / max(ds["bytes"], 1)
     path_ops = value * 1e9 * (SCAN_OPS_PER_BYTE + sha_blocks_per_byte * SHA1_OPS_PER_BLOCK) / 1e12
     kernels["path"] = {"bound": "alu", "achieved": path_ops, "peak": int_peak, "unit": "Tops/s",

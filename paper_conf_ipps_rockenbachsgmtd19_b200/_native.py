@@ -35,6 +35,17 @@ EXPORTS = [
     "dedup_op_route", "dedup_op_owner",
     "dedup_op_scatter", "dedup_op_findmatch", "dedup_kernel_launches",
 ]
+# every symbol declared in include/mandel.h (row NEXT-4)
+MANDEL_EXPORTS = ["mandel_rows_device", "mandel_image"]
+
+
+class MandelConfig(ctypes.Structure):
+    _fields_ = [
+        ("dim", ctypes.c_int32), ("niter", ctypes.c_int32),
+        ("init_a", ctypes.c_double), ("init_b", ctypes.c_double), ("range", ctypes.c_double),
+        ("batch_rows", ctypes.c_uint32), ("spaces", ctypes.c_uint32),
+        ("num_devices", ctypes.c_uint32), ("device_ids", ctypes.POINTER(ctypes.c_int32)),
+    ]
 
 
 class Config(ctypes.Structure):
@@ -119,6 +130,9 @@ def lib():
         "dedup_op_owner": (st, [vp, vp, vp, u64, vp]),
         "dedup_op_scatter": (st, [vp, vp, vp, vp, vp, vp, vp, u64, vp, vp]),
         "dedup_kernel_launches": (u64, [vp]),
+        "mandel_rows_device": (st, [vp, i32, i32, ctypes.c_double, ctypes.c_double,
+                                    ctypes.c_double, i32, i32, vp, vp, vp]),
+        "mandel_image": (st, [P(MandelConfig), vp, P(ctypes.c_double), P(u64)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)

@@ -30,7 +30,7 @@ def sources():
 
 def deps():
     return sources() + glob.glob(os.path.join(CSRC, "*.h")) + [
-        os.path.join(ROOT, "include", "dedup.h"), __file__]
+        *glob.glob(os.path.join(ROOT, "include", "*.h")), __file__]
 
 
 def stale() -> bool:

@@ -127,6 +127,12 @@ void launch_findmatch(const uint8_t* bytes, uint32_t nbytes, const uint32_t* cut
                       uint32_t window, uint32_t max_coded, uint8_t* out_len, uint16_t* out_off,
                       int num_sms, cudaStream_t s);
 
+// ---- Mandelbrot Streaming (mandel.cu, row NEXT-4) -----------------------------
+const char* mandel_unlaunchable();
+void launch_mandel(int32_t dim, int32_t niter, double init_a, double init_b, double step,
+                   int32_t row0, int32_t nrows, uint8_t* img, uint32_t* counter,
+                   uint64_t* iters, int num_sms, cudaStream_t s);
+
 // Results of one batch written straight into mapped pinned host memory.
 struct HostResultLayout {
     uint32_t* header;          // [0] n_chunks, [1] table overflow flag, [2] used slots

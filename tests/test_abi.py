@@ -32,6 +32,26 @@ def test_header_symbols_exported(L):
         assert hasattr(L, n), n
 
 
+def test_mandel_header_symbols_exported(L):
+    src = open(os.path.join(os.path.dirname(HDR), "mandel.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    names = sorted(set(re.findall(r"\b(mandel_[a-z_0-9]+)\s*\(", src)))
+    assert set(names) == set(N.MANDEL_EXPORTS)
+    for n in names:
+        assert hasattr(L, n), n
+
+
+def test_mandel_validates_before_the_gpu(L):
+    c = N.MandelConfig(0, 100, -2.0, -1.5, 3.0, 32, 2, 1, None)
+    assert L.mandel_image(ctypes.byref(c), None, None, None) == N.DEDUP_EINVAL
+    buf = (ctypes.c_uint8 * 16)()
+    for dim, niter, spaces in ((0, 100, 2), (4, 0, 2), (4, 1 << 24, 2), (4, 100, 0)):
+        c = N.MandelConfig(dim, niter, -2.0, -1.5, 3.0, 32, spaces, 1, None)
+        assert L.mandel_image(ctypes.byref(c), buf, None, None) == N.DEDUP_EINVAL
+    assert L.mandel_rows_device(None, 10, 100, -2.0, -1.5, 3.0, 5, 6, None, None, None) == \
+        N.DEDUP_EINVAL
+
+
 def test_sm100a_only_cubin():
     B.build()
     import subprocess

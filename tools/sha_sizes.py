@@ -22,9 +22,17 @@ cap = nb // 32 + mb + 2
 for case in cases:
     cut = torch.zeros(cap, dtype=torch.int32, device="cuda")
     n = torch.zeros(1, dtype=torch.int32, device="cuda")
-    if case == "uniform":
-        c = torch.arange(0, nb, 4096, dtype=torch.int64, device="cuda").to(torch.int32)
-        cut[:len(c)] = c
+    if case in ("uniform", "jitter", "capped"):
+        rng = np.random.default_rng(1)
+        if case == "uniform":
+            lens = np.full(nb // 4096 + 1, 4096)
+        elif case == "jitter":      # lengths uniform in [2K, 6K): desynchronised switches
+            lens = rng.integers(2048, 6144, nb // 2048)
+        else:                       # geometric like C2 but no chunk above 12 KiB (no tail)
+            lens = np.minimum(32 + rng.geometric(1 / 4096, nb // 1024), 12288)
+        c = np.concatenate([[0], np.cumsum(lens)])
+        c = c[c < nb]
+        cut[:len(c)] = torch.from_numpy(c.astype(np.int32)).cuda()
         n[0] = len(c)
     else:
         off = torch.from_numpy(np.minimum(np.arange(mb + 1, dtype=np.uint64) * MiB, nb).view(np.int64)).cuda()
