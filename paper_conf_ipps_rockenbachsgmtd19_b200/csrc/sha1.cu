@@ -38,6 +38,13 @@ constexpr int kShaStateWords = 11;
 #endif
 // iterations (64-byte blocks) between compaction points
 constexpr uint32_t kCompactEvery = DEDUP_SHA_COMPACT_EVERY;
+// Idle lanes of a warp refilled together (the work pull in sha1_kernel).
+// Measured (1000 MiB of C2-like chunks / bench): 1 -> 592 GB/s / 719, 4 ->
+// 623 / 733, 8 -> - / 720, 16 -> - / 648.
+#ifndef DEDUP_SHA_REFILL_MIN
+#define DEDUP_SHA_REFILL_MIN 4
+#endif
+constexpr int kRefillMin = DEDUP_SHA_REFILL_MIN;
 constexpr uint32_t kFull = 0xFFFFFFFFu;
 
 __device__ __forceinline__ uint32_t rotl(uint32_t x, int s) { return __funnelshift_l(x, x, s); }
@@ -211,8 +218,14 @@ sha1_kernel(const BatchDesc* __restrict__ desc,
     uint32_t H[5] = {0, 0, 0, 0, 0};
     uint32_t raw[20];    // prefetched data window of the next block
     for (uint32_t iter = 1;; ++iter) {
-        // ---- pull work: long chunks first, then all others in order ----
-        while (true) {
+        // ---- pull work: long chunks first, then all others in order.  The
+        // pull is a divergent stretch of the warp (ballot, atomic, chunk
+        // bounds, first data window), so idle lanes wait until kRefillMin of
+        // them are idle (or no lane is working) and are refilled together ----
+        const uint32_t idle = __ballot_sync(kFull, !done && k < 0);
+        const bool pull = idle != 0 && (kRefillMin <= 1 || __popc(idle) >= kRefillMin ||
+                                         __ballot_sync(kFull, k >= 0) == 0);
+        while (pull) {
             const bool need = !done && k < 0;
             const uint32_t m = __ballot_sync(kFull, need);
             if (!m) break;
