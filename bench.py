@@ -377,6 +377,9 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--batch-mb", type=int, default=0, help="override the GPU batch size")
     ap.add_argument("--slots", type=int, default=0, help="override the in-flight batches")
+    ap.add_argument("--step-only", action="store_true",
+                    help="time the step only (no isolated-kernel, NEXT-row, e2e or CPU legs): "
+                         "for the ncu launch list of the step")
     args = ap.parse_args()
     global BATCH_BYTES, SLOTS, BATCH_ITEMS
     if args.batch_mb:
@@ -460,6 +463,13 @@ def main():
             "pack_d2h": ds["ms_d2h"] / nt},
         "timed_batches": ds["timed_batches"],
     }
+    if args.step_only:
+        print(json.dumps({"metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": 1,
+                          "steps": args.steps, "warmup": args.warmup,
+                          "ms_per_step": ms / args.steps, "gpu_launches": launches,
+                          "note": "--step-only"}), flush=True)
+        d.close()
+        return
     iso = isolated_kernels(dd, off, int_peak)
     kernels.update(iso)
     kernels["mandelbrot"] = mandel_measure(sm_mhz, with_cpu=not args.no_cpu_baseline)

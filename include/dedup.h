@@ -80,7 +80,10 @@ typedef struct {
     uint32_t owner_rank;     /* digest-prefix owner index of this ctx's table shard */
     uint32_t num_owners;     /* number of table shards (GPUs); 1 = single GPU */
     uint32_t host_fed;       /* 1: allocate device input slots for dedup_submit_batch */
-    uint32_t reserved[7];
+    uint32_t sha_lane_bytes; /* SHA-1 grid: one lane per this many batch bytes; 0 = 32768
+                                (tuned for many batches in flight; a ctx that runs one
+                                batch at a time wants fewer bytes per lane, e.g. 8192) */
+    uint32_t reserved[6];
 } dedup_config;
 
 /* Fills *cfg with the defaults above (struct_size set). */

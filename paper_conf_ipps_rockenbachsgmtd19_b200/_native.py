@@ -57,7 +57,8 @@ class Config(ctypes.Structure):
         ("slots", ctypes.c_uint32), ("batch_items", ctypes.c_uint32),
         ("batch_bytes", ctypes.c_uint64), ("table_capacity", ctypes.c_uint64),
         ("owner_rank", ctypes.c_uint32), ("num_owners", ctypes.c_uint32),
-        ("host_fed", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 7),
+        ("host_fed", ctypes.c_uint32), ("sha_lane_bytes", ctypes.c_uint32),
+        ("reserved", ctypes.c_uint32 * 6),
     ]
 
 

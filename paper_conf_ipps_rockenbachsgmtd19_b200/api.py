@@ -72,7 +72,8 @@ class Dedup:
                  batch_items: int = 4096, table_capacity: int = 1 << 20, host_fed: bool = True,
                  window: int = 32, poly: int = 0x45C2B6A1, anchor_mask: int = 0xFFF,
                  anchor_value: int = 0, min_chunk: int = 32, max_chunk: int = 0,
-                 owner_rank: int = 0, num_owners: int = 1, max_drain: int = 65536):
+                 owner_rank: int = 0, num_owners: int = 1, max_drain: int = 65536,
+                 sha_lane_bytes: int = 0):
         L = N.lib()
         cfg = N.Config()
         L.dedup_config_default(ctypes.byref(cfg))
@@ -81,7 +82,7 @@ class Dedup:
                          host_fed=int(host_fed), window=window, poly=poly,
                          anchor_mask=anchor_mask, anchor_value=anchor_value,
                          min_chunk=min_chunk, max_chunk=max_chunk, owner_rank=owner_rank,
-                         num_owners=num_owners).items():
+                         num_owners=num_owners, sha_lane_bytes=sha_lane_bytes).items():
             setattr(cfg, k, v)
         self.cfg = cfg
         self._ctx = _vp()

@@ -247,7 +247,7 @@ void enqueue_chunk_sha(dedup_ctx* c, Workspace& w, cudaStream_t s, const BatchDe
     if (ev_chunk) cudaEventRecordWithFlags(ev_chunk, s, cudaEventRecordExternal);
     if (digest && !(DEDUP_ATTRIB_SKIP & 1))
         launch_sha1(d, max_bytes, cut_pos, n_chunks, cap, long_bytes(c), w.counters,
-                    w.long_list, digest, c->num_sms, s);
+                    w.long_list, digest, c->num_sms, s, c->cfg.sha_lane_bytes);
 }
 
 // Records the per-batch graph of slot i (capture of the slot's stream).
@@ -416,6 +416,8 @@ dedup_status check_cfg(const dedup_config* g) {
     if (g->num_owners < 1 || g->num_owners > 64 || g->owner_rank >= g->num_owners)
         return DEDUP_EINVAL;
     if (g->table_capacity < 1 || g->table_capacity > (1ull << 31)) return DEDUP_EINVAL;
+    if (g->sha_lane_bytes != 0 && (g->sha_lane_bytes < 64 || g->sha_lane_bytes > (1u << 24)))
+        return DEDUP_EINVAL;
     if (g->window != 32 || g->min_chunk != 32 || g->max_chunk != 0) return DEDUP_EUNSUPPORTED;
     return DEDUP_OK;
 }
@@ -881,7 +883,7 @@ dedup_status dedup_op_sha1(dedup_ctx* c, void* stream, const uint8_t* d_bytes, u
     const BatchDesc* d = nullptr;
     TRY(op_desc(c, s, h, &d));
     launch_sha1(d, nbytes, d_cut_pos, d_n_chunks, cap, long_bytes(c), c->op_ws.counters,
-                c->op_ws.long_list, d_digest, c->num_sms, s);
+                c->op_ws.long_list, d_digest, c->num_sms, s, c->cfg.sha_lane_bytes);
     c->launches += 2;
     CU(cudaGetLastError());
     return DEDUP_OK;

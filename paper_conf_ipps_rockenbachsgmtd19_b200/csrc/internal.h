@@ -88,7 +88,8 @@ constexpr uint32_t kMinLongBytes = 1024;
 // max_bytes: largest nbytes this launch may see (grid sizing).
 void launch_sha1(const BatchDesc* d, uint64_t max_bytes, const uint32_t* cut_pos,
                  const uint32_t* n_chunks, uint64_t cap, uint32_t long_bytes, uint32_t* counters,
-                 uint32_t* long_list, uint8_t* digest, int num_sms, cudaStream_t s);
+                 uint32_t* long_list, uint8_t* digest, int num_sms, cudaStream_t s,
+                 uint32_t lane_bytes = 0);
 
 // ---- digest table and routing (table.cu) ----------------------------------
 // Insert records then look them up.  Records come either as (digest bytes,

@@ -381,7 +381,8 @@ const char* sha1_unlaunchable() {
 
 void launch_sha1(const BatchDesc* d, uint64_t max_bytes, const uint32_t* cut_pos,
                  const uint32_t* n_chunks, uint64_t cap, uint32_t long_bytes, uint32_t* counters,
-                 uint32_t* long_list, uint8_t* digest, int num_sms, cudaStream_t s) {
+                 uint32_t* long_list, uint8_t* digest, int num_sms, cudaStream_t s,
+                 uint32_t lane_bytes) {
     cudaMemsetAsync(counters, 0, 2 * sizeof(uint32_t), s);
     // Persistent lanes pull chunks dynamically, so the grid only needs enough
     // lanes to finish the batch's bulk within its longest chunk's latency:
@@ -394,7 +395,7 @@ void launch_sha1(const BatchDesc* d, uint64_t max_bytes, const uint32_t* cut_pos
 #ifndef DEDUP_SHA_LANE_BYTES
 #define DEDUP_SHA_LANE_BYTES 32768
 #endif
-    const uint64_t kShaLaneBytes = DEDUP_SHA_LANE_BYTES;
+    const uint64_t kShaLaneBytes = lane_bytes ? lane_bytes : DEDUP_SHA_LANE_BYTES;
     uint64_t lanes = max_bytes / kShaLaneBytes;
     if (lanes < 1024) lanes = 1024;
     uint64_t blocks = (lanes + kShaThreads - 1) / kShaThreads;

@@ -62,7 +62,7 @@ def test_sm100a_only_cubin():
 
 def test_struct_layouts_match_header(L):
     # sizes that the header fixes (the C side checks struct_size)
-    assert ctypes.sizeof(N.Config) == 96  # 10 u32, 2 u64, 3 u32, 7 reserved u32
+    assert ctypes.sizeof(N.Config) == 96  # 10 u32, 2 u64, 4 u32, 6 reserved u32
     assert ctypes.sizeof(N.Record) == 32
     c = N.Config()
     L.dedup_config_default(ctypes.byref(c))

@@ -70,7 +70,7 @@ ft, traffic = full_table('gpurun_out/prof_full.ncu-rep')
 md = [f'# {tag} profiles (B200, sm_100a)', '',
       'Commands (under gpurun, one GPU): `bash tools/gpu_profiles.sh`', '',
       '```', open('tools/gpu_profiles.sh').read().strip(), '```', '',
-      '## Launch list of the bench command (cold-cache, serialised by ncu: shares, not absolutes)', '']
+      '## Launch list of the bench step (`bench.py --step-only`: warm-up + timed steps; cold-cache, serialised by ncu: shares, not absolutes)', '']
 md += lt
 md += ['', '## ncu --set full, one 64 MiB batch of C2 (tools/one_batch.py)', '',
        'Units: ns, instructions, %, bytes.  `dram` = DRAM bytes of the launch.', '']
