@@ -399,7 +399,9 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     if world > 1 or args.gpus > 1:
         from paper_conf_ipps_rockenbachsgmtd19_b200 import dist_bench
-        return dist_bench.main(args, data, off)
+        # pass this module: under torchrun bench.py runs as __main__, and an
+        # `import bench` would see the default (un-overridden) batch settings
+        return dist_bench.main(args, data, off, sys.modules[__name__])
 
     import torch
 

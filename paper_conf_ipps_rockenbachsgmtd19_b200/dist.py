@@ -27,6 +27,8 @@ The per-rank work is split in three phases so that the same code runs
 """
 from __future__ import annotations
 
+import os
+import time
 from dataclasses import dataclass
 
 import numpy as np
@@ -97,6 +99,12 @@ class TorchDistExchange:
                                     group=self.group)
         return recv
 
+    def alltoall(self, sends, counts):
+        """Pipeline interface (one local rank per process): returns
+        ([recv], [recv_counts])."""
+        rc = self.counts(counts[0])
+        return [self.payload(sends[0], counts[0], rc)], [rc]
+
     def _device(self):
         import torch
         backend = self.dist.get_backend(self.group)
@@ -116,6 +124,13 @@ def loopback_all_to_all(sends, counts):
         recvs.append(torch.cat(parts, 0) if parts else sends[d][:0])
         rcounts.append([int(counts[s][d]) for s in range(G)])
     return recvs, rcounts
+
+
+class LoopbackExchange:
+    """Pipeline interface for G logical ranks in one process (one GPU)."""
+
+    def alltoall(self, sends, counts):
+        return loopback_all_to_all(sends, counts)
 
 
 class RankState:
@@ -250,3 +265,213 @@ def loopback_waves(states, batches):
     back_counts = [[rcounts[d][s] for s in range(len(states))] for d in range(len(states))]
     backs, _ = loopback_all_to_all(replies, back_counts)
     return [st.finish(b) for st, b in zip(states, backs)]
+
+
+# ---------------------------------------------------------------------------
+# Pipelined waves.  run_wave() finishes a wave before the next one starts, so
+# a GPU holds one batch at a time -- latency-bound (a batch's SHA-1 lasts as
+# long as its longest chunk).  WavePipeline keeps `depth` waves in flight per
+# local rank: the local rows A2-A5 of wave w + depth - 1 run on their own
+# streams while the exchange of wave w (A6-A8) runs on the owner stream; the
+# host synchronises only on wave w's route counts (to size the all-to-all)
+# and on its results.  Owner work stays in wave order on one stream per rank
+# (every record of wave w is inserted and looked up before wave w + 1's), so
+# results are the sequential stream-order answer (reading O12).
+
+
+class _Slot:
+    """One in-flight wave of one local rank: a ctx of its own (the op
+    workspace), a stream, RankState buffers, pinned staging and events."""
+
+    def __init__(self, device_index, batch_bytes, batch_items, G, sha_lane_bytes, combine):
+        import torch
+
+        from .api import Dedup
+        self.ctx = Dedup(device_index, batch_bytes=batch_bytes, batch_items=batch_items, slots=1,
+                         table_capacity=1 << 10, host_fed=False, num_owners=G,
+                         sha_lane_bytes=sha_lane_bytes)
+        dev = torch.device("cuda", device_index)
+        self.state = RankState(self.ctx, batch_bytes, batch_items, dev, G, combine=combine)
+        self.stream = torch.cuda.Stream(device=dev)
+        self.e_local = torch.cuda.Event()
+        self.e_done = torch.cuda.Event()
+        cap = self.state.cap
+        pin = dict(pin_memory=True)
+        self.h_off = torch.zeros(batch_items + 1, dtype=torch.int64, **pin)
+        self.h_send_off = torch.zeros(G + 1, dtype=torch.int32, **pin)
+        self.h_n = torch.zeros(1, dtype=torch.int32, **pin)
+        self.h_item_first = torch.zeros(batch_items + 1, dtype=torch.int32, **pin)
+        self.h_chunk_start = torch.zeros(cap, dtype=torch.int32, **pin)
+        self.h_digest = torch.zeros(cap * 20, dtype=torch.uint8, **pin)
+        self.h_first_id = torch.zeros(cap, dtype=torch.int64, **pin)
+        self.h_is_dup = torch.zeros(cap, dtype=torch.uint8, **pin)
+        self.busy = False
+
+    def local(self, data, item_off, first_seq):
+        """Rows A2-A5 on this slot's stream; no host synchronisation."""
+        import torch
+        st, S = self.state, self.stream
+        st.first_seq = first_seq
+        st.item_off = np.asarray(item_off, np.uint64)
+        n_items = len(st.item_off) - 1
+        nbytes = int(st.item_off[-1])
+        self.h_off[:n_items + 1].copy_(torch.from_numpy(st.item_off.view(np.int64)))
+        d = self.ctx
+        with torch.cuda.stream(S):
+            st.item_off_dev[:n_items + 1].copy_(self.h_off[:n_items + 1], non_blocking=True)
+            d.op_chunk(data, nbytes, st.item_off_dev, n_items, st.cut, st.cap, st.n, stream=S)
+            d.op_chunk_meta(st.item_off_dev, n_items, st.cut, st.n, st.cap, first_seq,
+                            st.chunk_start, st.chunk_id, st.item_first, stream=S)
+            d.op_sha1(data, nbytes, st.cut, st.n, st.cap, st.digest, stream=S)
+            if st.combine:
+                d.op_local_combine(st.digest, st.n, st.cap, st.rep, stream=S)
+            d.op_route(st.digest, st.chunk_id, st.n, st.cap, st.G, st.send, st.send_off,
+                       st.send_pos, rep=st.rep, stream=S)
+            self.h_send_off.copy_(st.send_off, non_blocking=True)
+            self.h_n.copy_(st.n, non_blocking=True)
+            self.e_local.record(S)
+        self.busy = True
+
+    def counts(self):
+        """Host: wait for this wave's route; per-owner record counts."""
+        self.e_local.synchronize()
+        off = self.h_send_off.numpy().astype(np.int64)
+        self.state.n_host = int(off[-1])
+        self.state.send_counts = np.diff(off).tolist()
+        return self.state.send_counts
+
+    def finish_async(self, reply_back, stream):
+        """Row A8 + D2H of the results on the owner stream."""
+        st = self.state
+        n = int(self.h_n[0])
+        if n:
+            self.ctx.op_scatter(reply_back, st.send_pos, st.chunk_id, st.n, st.cap,
+                                st.first_id, st.is_dup, rep=st.rep, stream=stream)
+        n_items = len(st.item_off) - 1
+        self.h_item_first[:n_items].copy_(st.item_first[:n_items], non_blocking=True)
+        self.h_chunk_start[:n].copy_(st.chunk_start[:n], non_blocking=True)
+        self.h_digest[:20 * n].copy_(st.digest[:20 * n], non_blocking=True)
+        self.h_first_id[:n].copy_(st.first_id[:n], non_blocking=True)
+        self.h_is_dup[:n].copy_(st.is_dup[:n], non_blocking=True)
+        self.e_done.record(stream)
+        self.n = n
+
+    def result(self) -> WaveOut:
+        self.e_done.synchronize()
+        st, n = self.state, self.n
+        n_items = len(st.item_off) - 1
+        self.busy = False
+        return WaveOut(
+            first_seq=st.first_seq, item_len=np.diff(st.item_off),
+            item_first=self.h_item_first[:n_items].numpy().view(np.uint32).copy(),
+            chunk_start=self.h_chunk_start[:n].numpy().view(np.uint32).copy(),
+            digest=self.h_digest[:20 * n].numpy().reshape(n, 20).copy(),
+            first_id=self.h_first_id[:n].numpy().view(np.uint64).copy(),
+            is_dup=self.h_is_dup[:n].numpy().copy())
+
+    def close(self):
+        self.ctx.close()
+
+
+class WavePipeline:
+    """`depth` waves in flight per local rank (rows A2-A9 at G > 1).
+
+    owners: one Dedup ctx per LOCAL rank, owning that rank's table shard
+    (owner_rank, num_owners = G); exchange: TorchDistExchange (one local rank
+    per process, NCCL) or LoopbackExchange (G local ranks on one GPU).
+    submit(batches) takes one (data_tensor, item_off, first_seq) per local
+    rank and returns the waves completed by the call (lists of WaveOut per
+    local rank, in wave order); flush() completes the rest.  Data tensors
+    must stay alive until their wave is returned."""
+
+    def __init__(self, exchange, owners, device_index: int, batch_bytes: int,
+                 batch_items: int, depth: int = 4, sha_lane_bytes: int = 8192,
+                 combine: bool = True):
+        import torch
+        self.x = exchange
+        self.owners = owners
+        self.G = owners[0].cfg.num_owners
+        self.depth = depth
+        self.slots = [[_Slot(device_index, batch_bytes, batch_items, self.G, sha_lane_bytes,
+                             combine) for _ in range(depth)] for _ in owners]
+        dev = torch.device("cuda", device_index)
+        self.owner_streams = [torch.cuda.Stream(device=dev) for _ in owners]
+        self.dev = dev
+        self.next_wave = 0
+        self.done_wave = 0
+        # host seconds: local-phase enqueue, waits for route counts / results,
+        # exchange + owner enqueue (DEDUP_PIPE_TIMES=1 prints them at close)
+        self.host_s = {"local": 0.0, "wait_counts": 0.0, "exchange": 0.0, "wait_results": 0.0}
+
+    def submit(self, batches):
+        out = []
+        w = self.next_wave
+        if w - self.done_wave >= self.depth:
+            out.append(self._complete(self.done_wave))
+        t0 = time.perf_counter()
+        for r, (data, item_off, first_seq) in enumerate(batches):
+            self.slots[r][w % self.depth].local(data, item_off, first_seq)
+        self.host_s["local"] += time.perf_counter() - t0
+        self.next_wave += 1
+        return out
+
+    def flush(self):
+        out = []
+        while self.done_wave < self.next_wave:
+            out.append(self._complete(self.done_wave))
+        return out
+
+    def end_stream(self):
+        """New dedup stream: completes every wave in flight (they belong to
+        the old stream), then clears the table shards.  Returns the waves
+        completed by the call."""
+        out = self.flush()
+        for o, S in zip(self.owners, self.owner_streams):
+            o.op_table_reset(stream=S)
+        return out
+
+    def _complete(self, w):
+        import torch
+        sl = [self.slots[r][w % self.depth] for r in range(len(self.owners))]
+        t0 = time.perf_counter()
+        counts = [s.counts() for s in sl]                       # host sync: route of wave w
+        t1 = time.perf_counter()
+        self.host_s["wait_counts"] += t1 - t0
+        for s, S in zip(sl, self.owner_streams):
+            S.wait_event(s.e_local)
+        sends = [s.state.send[:s.state.n_host] for s in sl]
+        with torch.cuda.stream(self.owner_streams[0]):
+            recvs, rcounts = self.x.alltoall(sends, counts)      # row A6
+        replies = []
+        for r, (o, S) in enumerate(zip(self.owners, self.owner_streams)):
+            S.wait_stream(self.owner_streams[0])
+            reply = torch.zeros(len(recvs[r]), dtype=torch.int64, device=self.dev)
+            if len(recvs[r]):
+                o.op_owner(recvs[r], len(recvs[r]), reply, stream=S)   # row A7
+            replies.append(reply)
+        for S in self.owner_streams[1:]:
+            self.owner_streams[0].wait_stream(S)
+        back_counts = [[rcounts[d][s] for s in range(len(sl))] for d in range(len(sl))] \
+            if len(sl) > 1 else [rcounts[0]]
+        with torch.cuda.stream(self.owner_streams[0]):
+            backs, _ = self.x.alltoall(replies, back_counts)     # row A8 (reply)
+        res = []
+        for s, b in zip(sl, backs):
+            s.finish_async(b, self.owner_streams[0])
+        t2 = time.perf_counter()
+        self.host_s["exchange"] += t2 - t1
+        for s in sl:
+            # the slot's next local phase must not overwrite buffers in use
+            s.stream.wait_event(s.e_done)
+            res.append(s.result())
+        self.host_s["wait_results"] += time.perf_counter() - t2
+        self.done_wave += 1
+        return res
+
+    def close(self):
+        if os.environ.get("DEDUP_PIPE_TIMES"):
+            print(f"WavePipeline host seconds over {self.done_wave} waves: "
+                  + ", ".join(f"{k} {v:.4f}" for k, v in self.host_s.items()), flush=True)
+        for row in self.slots:
+            for s in row:
+                s.close()

@@ -2,10 +2,13 @@
 
 Weak scaling: in every step (= wave) each rank processes one GPU batch of
 the cycled C2 stream; digests are routed to their owner GPU with NCCL
-all-to-alls (rows A5-A8, see dist.py).  A dedup stream spans
-ceil(batches / N) waves; tables are reset at every stream start.  The timed
-region is bracketed by a barrier + device synchronisation and measured with
-CUDA events; the maximum over ranks is reported.
+all-to-alls (rows A5-A8, see dist.py).  Waves are pipelined
+(dist.WavePipeline): `DEPTH` waves are in flight per rank, so a rank's GPU
+keeps chunking and hashing later batches while the exchange of the oldest
+one runs.  A dedup stream spans max(ceil(batches / N), 4 * DEPTH) waves; the
+table shards are reset at every stream start.  The timed region is bracketed by a
+barrier + device synchronisation and measured with CUDA events; the maximum
+over ranks is reported.
 """
 from __future__ import annotations
 
@@ -14,14 +17,16 @@ import os
 
 import numpy as np
 
+DEPTH = 8  # waves in flight per rank
 
-def main(args, data, off):
+
+def main(args, data, off, B):
+    """B: the running bench module (batch settings, plan_batches, metric)."""
     import torch
     import torch.distributed as dist
 
-    import bench as B
-
     from . import dist as D
+    from .api import Dedup
 
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -33,36 +38,49 @@ def main(args, data, off):
     plan = B.plan_batches(off)
     nb = len(plan)
     items_per_batch = max(j - k for k, j in plan)
-    dd = D.DistDedup(x, local, B.BATCH_BYTES, B.BATCH_ITEMS + 1,
-                     max(1 << 16, len(data) // 2048 // world))
+    # the owner receives up to `world` batches' records per wave
+    owner = Dedup(local, batch_bytes=min(1 << 30, world * B.BATCH_BYTES), batch_items=1, slots=1,
+                  table_capacity=max(1 << 16, len(data) // 2048 // world), host_fed=False,
+                  owner_rank=rank, num_owners=world)
+    pipe = D.WavePipeline(x, [owner], local, B.BATCH_BYTES, B.BATCH_ITEMS + 1, depth=DEPTH)
     ddata = torch.from_numpy(data).to(dev)
-    waves_per_stream = (nb + world - 1) // world
+    # A table reset completes every wave in flight first (end_stream), so a
+    # dedup stream spans at least 4 pipeline depths of waves (the C2 batches
+    # cycled; later passes over the data inside one stream are duplicates).
+    waves_per_stream = max((nb + world - 1) // world, 4 * DEPTH)
+    counted = {"bytes": 0, "chunks": 0}
 
-    def wave(w):
+    def take(outs, timed):
+        for wave in outs:
+            o = wave[0]
+            if timed:
+                counted["bytes"] += int(np.sum(o.item_len))
+                counted["chunks"] += len(o.chunk_start)
+
+    def wave(w, timed):
         if w % waves_per_stream == 0 and w > 0:
-            dd.end_stream()
+            take(pipe.end_stream(), timed)
         b = ((w % waves_per_stream) * world + rank) % nb
         k, j = plan[b]
         seq = (w * world + rank) * items_per_batch
-        out = dd.wave(ddata[int(off[k]):int(off[j])], off[k:j + 1] - off[k], seq)
-        return int(off[j]) - int(off[k]), len(out.chunk_start)
+        take(pipe.submit([(ddata[int(off[k]):int(off[j])], off[k:j + 1] - off[k], seq)]),
+             timed)
 
     for w in range(args.warmup):
-        wave(w)
+        wave(w, False)
+    take(pipe.flush(), False)
     torch.cuda.synchronize()
     dist.barrier()
     start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     start.record()
-    nbytes = nchunks = 0
     for w in range(args.warmup, args.warmup + args.steps):
-        a, c = wave(w)
-        nbytes += a
-        nchunks += c
+        wave(w, True)
+    take(pipe.flush(), True)
     end.record()
     torch.cuda.synchronize()
     dist.barrier()
     ms = torch.tensor([start.elapsed_time(end)], dtype=torch.float64, device=dev)
-    tot = torch.tensor([nbytes, nchunks], dtype=torch.float64, device=dev)
+    tot = torch.tensor([counted["bytes"], counted["chunks"]], dtype=torch.float64, device=dev)
     dist.all_reduce(ms, op=dist.ReduceOp.MAX)
     dist.all_reduce(tot, op=dist.ReduceOp.SUM)
     t = float(ms.item())
@@ -76,10 +94,12 @@ def main(args, data, off):
             "config": {"workload": f"{B.WORKLOAD}: 184 MiB simlarge-sized synthetic stream, "
                                    "1 MiB items, dup_frac 0.52, device-resident, one batch per "
                                    "GPU per step, digest all-to-all (NCCL) to owner GPUs",
-                       "batch_bytes": B.BATCH_BYTES, "parallelism": f"{world} GPUs, "
-                       "digest-prefix table sharding", "l2": "inputs larger than L2"},
+                       "batch_bytes": B.BATCH_BYTES, "waves_in_flight": DEPTH,
+                       "parallelism": f"{world} GPUs, digest-prefix table sharding",
+                       "l2": "inputs larger than L2"},
             "gpu_launches": None,
         }
         print(json.dumps(line), flush=True)
-    dd.close()
+    pipe.close()
+    owner.close()
     dist.destroy_process_group()

@@ -156,3 +156,60 @@ def test_combined_routing_sends_one_record_per_digest():
         assert np.array_equal(cs, w.chunk_start), seq
         assert np.array_equal(dup, w.is_dup), seq
         assert np.array_equal(fid, w.first_id), seq
+
+
+@pytest.mark.parametrize("G,depth", [(1, 3), (2, 3), (3, 2)])
+def test_wave_pipeline_matches_oracle(G, depth):
+    """dist.WavePipeline (waves in flight on their own streams, exchange on
+    the owner streams) with G logical ranks on one GPU: bit-exact vs the
+    sequential oracle, across an end_stream (fresh tables)."""
+    assert torch.cuda.is_available()
+    from paper_conf_ipps_rockenbachsgmtd19_b200 import Dedup
+    from paper_conf_ipps_rockenbachsgmtd19_b200 import dist as D
+    data = U.stream(12 * MiB, seed=61 + G, dup_frac=0.6)
+    off = synthgen.split_items(data, MiB // 2)
+    n_items = len(off) - 1
+    per_batch = 2
+    bbytes = per_batch * MiB // 2
+    batches = [(k, min(k + per_batch, n_items)) for k in range(0, n_items, per_batch)]
+    dev = torch.from_numpy(data).cuda()
+    owners = [Dedup(0, batch_bytes=G * bbytes, batch_items=1, slots=1, table_capacity=1 << 16,
+                    host_fed=False, owner_rank=r, num_owners=G) for r in range(G)]
+    pipe = D.WavePipeline(D.LoopbackExchange(), owners, 0, bbytes, per_batch + 1, depth=depth)
+    split = len(batches) // 2            # stream 1: batches [0, split), stream 2: the rest
+    got = [[], []]
+    try:
+        def take(outs, sid):
+            for wave in outs:
+                for o in wave:
+                    got[sid].extend(o.items())
+        for sid, (lo, hi) in enumerate(((0, split), (split, len(batches)))):
+            if sid:
+                take(pipe.end_stream(), 0)
+            for w in range(lo, hi, G):
+                work = []
+                for r in range(G):
+                    b = w + r
+                    if b < hi:
+                        k, j = batches[b]
+                        work.append((dev[int(off[k]):int(off[j])], off[k:j + 1] - off[k], k))
+                    else:
+                        work.append((dev[:0], np.zeros(1, np.uint64), n_items + r))
+                take(pipe.submit(work), sid)
+        take(pipe.flush(), 1)
+        torch.cuda.synchronize()
+    finally:
+        pipe.close()
+        for o in owners:
+            o.close()
+    for sid, (lo, hi) in enumerate(((0, split), (split, len(batches)))):
+        k0, k1 = batches[lo][0], batches[hi - 1][1]
+        res = sorted((g for g in got[sid] if g[0] < n_items), key=lambda r: r[0])
+        want, _ = oracle.dedup_items([data[int(off[k]):int(off[k + 1])] for k in range(k0, k1)],
+                                     first_seq=k0)
+        assert [g[0] for g in res] == [w.seq for w in want]
+        for (seq, cs, dg, dup, fid), w in zip(res, want):
+            assert np.array_equal(cs, w.chunk_start), seq
+            assert np.array_equal(dg, w.digest), seq
+            assert np.array_equal(dup, w.is_dup), seq
+            assert np.array_equal(fid, w.first_id), seq
