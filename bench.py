@@ -291,6 +291,28 @@ def isolated_kernels(dd, off, int_peak, copies=4, reps=3, streams=4):
         ev[1].record()
         ev[1].synchronize()
         fm_us = ev[0].elapsed_time(ev[1]) * 1e3
+        # row NEXT-3 (host archive writer) on the first 64 MiB of these outputs
+        from paper_conf_ipps_rockenbachsgmtd19_b200 import archive
+        an = 64 * MiB
+        kk = int(n.item())
+        cps = cut[:kk].cpu().numpy().astype(np.int64)
+        cps = cps[cps < an].astype(np.uint32)
+        a_data = dd[:an].cpu().numpy()
+        a_len = fl[:an].cpu().numpy()
+        a_off = fo[:an].cpu().numpy().view(np.uint16)
+        a_dig = digs[0][:20 * len(cps)].cpu().numpy()
+        a_dup = np.zeros(len(cps), np.uint8)
+        t0 = time.perf_counter()
+        rec = archive.encode(a_data, cps, a_dig, a_dup, a_len, a_off)
+        t1 = time.perf_counter()
+        back = archive.Decoder().decode(rec, an)
+        t2 = time.perf_counter()
+        assert np.array_equal(back, a_data)
+        arch = {"row": "NEXT-3 (host archive writer: greedy LZSS tokens from FindMatch + "
+                       "digest records; C++, 1 host thread)",
+                "encode_gbs": an / (t1 - t0) / 1e9, "decode_gbs": an / (t2 - t1) / 1e9,
+                "ratio": len(rec) / an, "sample": "first 64 MiB of the C2 stream, every chunk "
+                "encoded as unique (the step's duplicates would be 21-byte references)"}
         del fl, fo
     finally:
         for c in ctxs:
@@ -305,6 +327,7 @@ def isolated_kernels(dd, off, int_peak, copies=4, reps=3, streams=4):
                  "input_gbs": nb / (sha_us * 1e-6) / 1e9, "blocks": blocks,
                  "note": f"{streams} concurrent streams x {reps} launches; launch_us = "
                          "joint elapsed / launches"},
+        "archive": arch,
         "findmatch": {"row": "NEXT-1 (LZSS FindMatch, Listing 3), W=4096, MAX_CODED=18",
                       "bound": "hbm", "achieved": nb * 4 / (fm_us * 1e-6) / 1e9,
                       "peak": HBM_PEAK, "unit": "GB/s",

@@ -312,6 +312,43 @@ dedup_status dedup_op_findmatch(dedup_ctx* c, void* stream, const uint8_t* d_byt
                                 uint32_t window, uint32_t max_coded, uint8_t* d_match_len,
                                 uint16_t* d_match_off);
 
+/* ------------------------------------------------------------------------ */
+/* 3. Row NEXT-3: the host-side archive writer               */
+/* ------------------------------------------------------------------------ */
+/* The paper's CPU consumer of the GPU stages: "we used the result of the
+ * kernel function to run the compression on each block and generate the
+ * compressed data", then "reorders the batches and writes it in the
+ * output".  All pointers HOST; no GPU work.  Format (reading A1 in
+ * DESIGN.md): per chunk in order, 'U' digest[20] u32 raw_len u32 tok_len
+ * tokens (unique) or 'D' digest[20] (duplicate); tokens = greedy LZSS over
+ * FindMatch's output (a match of length >= 3 is a 2-byte token
+ * (offset & 0xFFF) | (length - 3) << 12, else a literal), in groups of 8
+ * behind a flag byte (bit set = literal). */
+
+/* Encodes one batch: chunk k = data[starts[k], starts[k+1]) (the last ends
+ * at nbytes; starts[0] == 0, increasing), digest[20k..] (row A4), is_dup[k]
+ * (row A7/A8), match_len / match_off per byte (dedup_op_findmatch output,
+ * copied to the host).  window must be 4096 and 3 <= max_coded <= 18 (the
+ * 12 + 4 bit token).  Returns the bytes written to out, DEDUP_ENOMEM if
+ * out_cap is too small, DEDUP_EINVAL on bad arguments. */
+int64_t dedup_archive_encode(const uint8_t* data, uint64_t nbytes, const uint32_t* starts,
+                             uint32_t n_chunks, const uint8_t* digest, const uint8_t* is_dup,
+                             const uint8_t* match_len, const uint16_t* match_off,
+                             uint32_t window, uint32_t max_coded, uint8_t* out,
+                             uint64_t out_cap);
+
+/* Decoder state across batches (the digest -> chunk map that 'D' records
+ * refer to).  new returns NULL for a window other than 4096. */
+typedef struct dedup_archive_decoder dedup_archive_decoder;
+dedup_archive_decoder* dedup_archive_decoder_new(uint32_t window);
+void dedup_archive_decoder_free(dedup_archive_decoder* d);
+
+/* Decodes the records in[0, in_len) (whole records, in stream order) into
+ * out; returns the bytes written, DEDUP_ENOMEM / DEDUP_EINVAL (malformed
+ * input or a reference to an unknown digest). */
+int64_t dedup_archive_decode(dedup_archive_decoder* d, const uint8_t* in, uint64_t in_len,
+                             uint8_t* out, uint64_t out_cap);
+
 /* Number of kernels this ctx has launched so far (all layers). */
 uint64_t dedup_kernel_launches(const dedup_ctx* c);
 

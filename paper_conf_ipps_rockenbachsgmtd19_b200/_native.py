@@ -34,6 +34,8 @@ EXPORTS = [
     "dedup_op_table_reset", "dedup_op_table_status", "dedup_op_local_combine",
     "dedup_op_route", "dedup_op_owner",
     "dedup_op_scatter", "dedup_op_findmatch", "dedup_kernel_launches",
+    "dedup_archive_encode", "dedup_archive_decoder_new", "dedup_archive_decoder_free",
+    "dedup_archive_decode",
 ]
 # every symbol declared in include/mandel.h (row NEXT-4)
 MANDEL_EXPORTS = ["mandel_rows_device", "mandel_image"]
@@ -131,6 +133,11 @@ def lib():
         "dedup_op_owner": (st, [vp, vp, vp, u64, vp]),
         "dedup_op_scatter": (st, [vp, vp, vp, vp, vp, vp, vp, u64, vp, vp]),
         "dedup_kernel_launches": (u64, [vp]),
+        "dedup_archive_encode": (ctypes.c_int64, [vp, u64, vp, u32, vp, vp, vp, vp, u32, u32,
+                                                  vp, u64]),
+        "dedup_archive_decoder_new": (vp, [u32]),
+        "dedup_archive_decoder_free": (None, [vp]),
+        "dedup_archive_decode": (ctypes.c_int64, [vp, vp, u64, vp, u64]),
         "mandel_rows_device": (st, [vp, i32, i32, ctypes.c_double, ctypes.c_double,
                                     ctypes.c_double, i32, i32, vp, vp, vp]),
         "mandel_image": (st, [P(MandelConfig), vp, P(ctypes.c_double), P(u64)]),
