@@ -46,7 +46,9 @@ struct Workspace {
     uint32_t* counters = nullptr;    // [0..1] sha1 work/long counters, [64..191] route
     uint32_t* slot_idx = nullptr;    // table slot per record
     uint32_t* long_list = nullptr;   // SHA-1 long-chunk list
+    uint32_t* item_cnt = nullptr;    // max_chunk selection: chunks per item (cap + 1)
     uint64_t max_tiles = 0;
+    uint64_t item_cap = 0;
 };
 
 struct Slot {
@@ -192,6 +194,10 @@ dedup_status ws_alloc(dedup_ctx* c, Workspace& w, uint64_t batch_bytes, uint64_t
     TRY(dalloc(c, &w.counters, 256));
     TRY(dalloc(c, &w.slot_idx, cap));
     TRY(dalloc(c, &w.long_list, batch_bytes / kMinLongBytes + 2));
+    if (c->cfg.max_chunk) {
+        TRY(dalloc(c, &w.item_cnt, cap + 1));
+        w.item_cap = cap;
+    }
     CU(cudaMemset(w.counters, 0, sizeof(uint32_t) * 256));
     return DEDUP_OK;
 }
@@ -205,6 +211,7 @@ void ws_free(Workspace& w) {
     cudaFree(w.counters);
     cudaFree(w.slot_idx);
     cudaFree(w.long_list);
+    cudaFree(w.item_cnt);
     w = Workspace{};
 }
 
@@ -240,7 +247,8 @@ void enqueue_chunk_sha(dedup_ctx* c, Workspace& w, cudaStream_t s, const BatchDe
         launch_chunk_select(d, c->d_tab, c->cfg.anchor_mask, c->cfg.anchor_value, w.bitmap,
                             w.agg, w.gagg, w.gentry, w.evbuf,
                             (max_bytes + kSelTile - 1) / kSelTile, cut_pos, cap, n_chunks,
-                            c->num_sms, s, ev_scan);
+                            c->num_sms, s, ev_scan, c->cfg.max_chunk, w.item_cnt,
+                            c->cfg.batch_items);
     if (chunk_start)
         launch_chunk_meta(d, cut_pos, n_chunks, cap, chunk_start, chunk_id, item_first,
                           max_items, c->num_sms, s);
@@ -418,7 +426,9 @@ dedup_status check_cfg(const dedup_config* g) {
     if (g->table_capacity < 1 || g->table_capacity > (1ull << 31)) return DEDUP_EINVAL;
     if (g->sha_lane_bytes != 0 && (g->sha_lane_bytes < 64 || g->sha_lane_bytes > (1u << 24)))
         return DEDUP_EINVAL;
-    if (g->window != 32 || g->min_chunk != 32 || g->max_chunk != 0) return DEDUP_EUNSUPPORTED;
+    // max_chunk (NEXT-2): forced cuts, selected by maxchunk.cu's walk
+    if (g->window != 32 || g->min_chunk != 32) return DEDUP_EUNSUPPORTED;
+    if (g->max_chunk != 0 && g->max_chunk < 64) return DEDUP_EUNSUPPORTED;
     return DEDUP_OK;
 }
 
@@ -826,6 +836,8 @@ dedup_status dedup_op_chunk(dedup_ctx* c, void* stream, const uint8_t* d_bytes, 
     if (nbytes > c->cfg.batch_bytes) return fail(c, DEDUP_EINVAL, "nbytes > batch_bytes");
     if (reinterpret_cast<uintptr_t>(d_bytes) & 15)
         return fail(c, DEDUP_EINVAL, "d_bytes must be 16-byte aligned");
+    if (c->cfg.max_chunk && n_items > c->op_ws.item_cap)
+        return fail(c, DEDUP_EINVAL, "n_items larger than the max_chunk workspace");
     CU(cudaSetDevice(c->cfg.device));
     cudaStream_t s = static_cast<cudaStream_t>(stream);
     BatchDesc h{};

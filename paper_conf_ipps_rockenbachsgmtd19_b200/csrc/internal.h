@@ -74,7 +74,13 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
                          uint32_t value, uint32_t* bitmap, uint32_t* agg, uint32_t* gagg,
                          uint32_t* gentry, uint32_t* evbuf, uint64_t max_tiles,
                          uint32_t* cut_pos, uint64_t cap, uint32_t* n_chunks, int num_sms,
-                         cudaStream_t s, cudaEvent_t after_scan);
+                         cudaStream_t s, cudaEvent_t after_scan, uint32_t max_chunk = 0,
+                         uint32_t* item_cnt = nullptr, uint32_t max_items = 0);
+// NEXT-2 max_chunk selection (maxchunk.cu): a walk per item over the scan's
+// candidate bitmap; item_cnt: max_items + 1 words of scratch.
+void launch_select_walk(const BatchDesc* d, const uint32_t* bitmap, uint32_t max_chunk,
+                        uint32_t* item_cnt, uint32_t max_items, uint32_t* cut_pos, uint64_t cap,
+                        uint32_t* n_chunks, int num_sms, cudaStream_t s);
 
 void launch_chunk_meta(const BatchDesc* d, const uint32_t* cut_pos, const uint32_t* n_chunks,
                        uint64_t cap, uint32_t* chunk_start, uint64_t* chunk_id,

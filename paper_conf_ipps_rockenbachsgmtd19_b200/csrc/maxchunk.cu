@@ -1,0 +1,139 @@
+// maxchunk.cu -- row NEXT-2, the max_chunk chunker variant:
+// cut selection with a maximum chunk length M (PARSEC-style forced cut; the
+// oracle's oracle_chunk_item with max_chunk != 0).  After a cut at c the
+// next cut is the first Rabin candidate e in [c + 32, min(c + M, r)) of the
+// item [q, r), else the forced cut c + M if c + M < r, else the item ends.
+//
+// The 32-state tile machine of rabin.cu cannot carry "distance since the
+// last cut" (up to M states), so with max_chunk the selection is a walk per
+// item over the candidate bitmap the scan kernel already wrote (bit e of the
+// e-space bitmap <=> the window ending at byte e - 1 hits): one warp per
+// item finds each next cut with one coalesced 32-word (1024-position) read
+// and a ballot, so the cost is O(chunks + candidate-free words) per item.
+// Two passes (count, then write at the item's prefix offset) keep cut_pos
+// in batch order.  Items are independent, so the grid covers items.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "internal.h"
+
+namespace dd {
+
+namespace {
+
+constexpr uint32_t kFull = 0xFFFFFFFFu;
+constexpr uint64_t kNone = ~0ull;
+constexpr int kWalkWarps = 8;
+
+// First candidate e in [lo, hi) of the e-space bitmap, or kNone (warp-wide).
+__device__ __forceinline__ uint64_t first_candidate(const uint32_t* __restrict__ bitmap,
+                                                    uint64_t lo, uint64_t hi, int lane) {
+    for (uint64_t w0 = lo >> 5; (w0 << 5) < hi; w0 += 32) {
+        const uint64_t w = w0 + lane;
+        uint32_t bits = 0;
+        if ((w << 5) < hi) {
+            bits = bitmap[w];
+            if (w == (lo >> 5)) bits &= kFull << (lo & 31);
+            if (((w + 1) << 5) > hi) {
+                const uint32_t keep = (uint32_t)(hi - (w << 5));  // 1..31
+                bits &= (1u << keep) - 1u;
+            }
+        }
+        const uint32_t m = __ballot_sync(kFull, bits != 0);
+        if (m) {
+            const int src = __ffs(m) - 1;
+            const uint32_t b = __shfl_sync(kFull, bits, src);
+            return ((w0 + (uint64_t)src) << 5) + (uint64_t)(__ffs(b) - 1);
+        }
+    }
+    return kNone;
+}
+
+// Pass 1 (write == false): item_cnt[it] = chunks of item it.
+// Pass 2 (write == true): cut_pos[item_cnt[it] + k] = k-th chunk start of it
+// (item_cnt holds the exclusive prefix by then).
+template <bool kWrite>
+__global__ void __launch_bounds__(kWalkWarps * 32)
+select_walk_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ bitmap,
+                   uint32_t max_chunk, uint32_t* __restrict__ item_cnt,
+                   uint32_t* __restrict__ cut_pos, uint64_t cap) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t n_items = desc->n_items;
+    const uint64_t* __restrict__ item_off = desc->item_off;
+    const uint64_t M = max_chunk;
+    for (uint32_t it = blockIdx.x * kWalkWarps + (threadIdx.x >> 5); it < n_items;
+         it += gridDim.x * kWalkWarps) {
+        const uint64_t q = item_off[it], r = item_off[it + 1];
+        uint64_t count = 0;
+        const uint64_t base = kWrite ? item_cnt[it] : 0;
+        uint64_t c = q;
+        while (c < r) {
+            if (kWrite && lane == 0 && base + count < cap) cut_pos[base + count] = (uint32_t)c;
+            ++count;
+            const uint64_t lim = c + M < r ? c + M : r;
+            const uint64_t e = c + 32 < lim ? first_candidate(bitmap, c + 32, lim, lane) : kNone;
+            if (e != kNone) c = e;
+            else if (c + M < r) c = c + M;
+            else break;
+        }
+        if (!kWrite && lane == 0) item_cnt[it] = (uint32_t)count;
+    }
+}
+
+// Exclusive prefix of item_cnt[0..n_items) in place; total -> *n_chunks.
+__global__ void __launch_bounds__(1024)
+item_scan_kernel(const BatchDesc* __restrict__ desc, uint32_t* __restrict__ item_cnt,
+                 uint32_t* __restrict__ n_chunks) {
+    __shared__ uint32_t s_warp[32];
+    __shared__ uint32_t s_carry;
+    const uint32_t n = desc->n_items;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    if (threadIdx.x == 0) s_carry = 0;
+    __syncthreads();
+    for (uint32_t b = 0; b < n; b += 1024) {
+        const uint32_t i = b + threadIdx.x;
+        const uint32_t v = i < n ? item_cnt[i] : 0u;
+        uint32_t x = v;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t y = __shfl_up_sync(kFull, x, d);
+            if (lane >= d) x += y;
+        }
+        if (lane == 31) s_warp[wid] = x;
+        __syncthreads();
+        if (wid == 0) {
+            uint32_t t = s_warp[lane];
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const uint32_t y = __shfl_up_sync(kFull, t, d);
+                if (lane >= d) t += y;
+            }
+            s_warp[lane] = t;  // inclusive over warps
+        }
+        __syncthreads();
+        const uint32_t carry = s_carry;
+        const uint32_t excl = carry + (wid ? s_warp[wid - 1] : 0u) + x - v;
+        if (i < n) item_cnt[i] = excl;
+        __syncthreads();
+        if (threadIdx.x == 1023) s_carry = carry + s_warp[31];
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) *n_chunks = s_carry;
+}
+
+}  // namespace
+
+void launch_select_walk(const BatchDesc* d, const uint32_t* bitmap, uint32_t max_chunk,
+                        uint32_t* item_cnt, uint32_t max_items, uint32_t* cut_pos, uint64_t cap,
+                        uint32_t* n_chunks, int num_sms, cudaStream_t s) {
+    uint64_t blocks = ((uint64_t)max_items + kWalkWarps - 1) / kWalkWarps;
+    if (blocks > (uint64_t)num_sms * 8) blocks = (uint64_t)num_sms * 8;
+    if (blocks < 1) blocks = 1;
+    select_walk_kernel<false><<<(unsigned)blocks, kWalkWarps * 32, 0, s>>>(
+        d, bitmap, max_chunk, item_cnt, cut_pos, cap);
+    item_scan_kernel<<<1, 1024, 0, s>>>(d, item_cnt, n_chunks);
+    select_walk_kernel<true><<<(unsigned)blocks, kWalkWarps * 32, 0, s>>>(
+        d, bitmap, max_chunk, item_cnt, cut_pos, cap);
+}
+
+}  // namespace dd

@@ -940,7 +940,8 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
                          uint32_t value, uint32_t* bitmap, uint32_t* agg, uint32_t* gagg,
                          uint32_t* gentry, uint32_t* evbuf, uint64_t max_tiles,
                          uint32_t* cut_pos, uint64_t cap, uint32_t* n_chunks, int num_sms,
-                         cudaStream_t s, cudaEvent_t after_scan) {
+                         cudaStream_t s, cudaEvent_t after_scan, uint32_t max_chunk,
+                         uint32_t* item_cnt, uint32_t max_items) {
     chunk_set_attrs();
     const uint64_t groups = select_groups(max_tiles);
     // A persistent scan CTA takes several groups: fewer, longer-lived CTAs
@@ -961,6 +962,11 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
         k<<<grid, kScanThreads, kScanSmem, s>>>(d, d_tab, mask, value, bitmap, agg, gagg, evbuf);
     }
     if (after_scan) cudaEventRecordWithFlags(after_scan, s, cudaEventRecordExternal);
+    if (max_chunk) {  // NEXT-2: cut selection with a maximum chunk length (maxchunk.cu)
+        launch_select_walk(d, bitmap, max_chunk, item_cnt, max_items, cut_pos, cap, n_chunks,
+                           num_sms, s);
+        return;
+    }
     select_scan_kernel<<<1, 1024, 0, s>>>(d, gagg, gentry, n_chunks);
     uint64_t blocks = (groups + kEmitEvWarps - 1) / kEmitEvWarps;
     if (blocks > (uint64_t)num_sms * 4) blocks = (uint64_t)num_sms * 4;
