@@ -46,9 +46,9 @@ struct Workspace {
     uint32_t* counters = nullptr;    // [0..1] sha1 work/long counters, [64..191] route
     uint32_t* slot_idx = nullptr;    // table slot per record
     uint32_t* long_list = nullptr;   // SHA-1 long-chunk list
-    uint32_t* item_cnt = nullptr;    // max_chunk selection: chunks per item (cap + 1)
+    uint32_t* mc_ws = nullptr;       // max_chunk selection scratch (maxchunk_ws_words)
     uint64_t max_tiles = 0;
-    uint64_t item_cap = 0;
+    uint64_t item_cap = 0;           // items the max_chunk scratch holds
 };
 
 struct Slot {
@@ -195,8 +195,8 @@ dedup_status ws_alloc(dedup_ctx* c, Workspace& w, uint64_t batch_bytes, uint64_t
     TRY(dalloc(c, &w.slot_idx, cap));
     TRY(dalloc(c, &w.long_list, batch_bytes / kMinLongBytes + 2));
     if (c->cfg.max_chunk) {
-        TRY(dalloc(c, &w.item_cnt, cap + 1));
         w.item_cap = cap;
+        TRY(dalloc(c, &w.mc_ws, maxchunk_ws_words(cap, w.item_cap)));
     }
     CU(cudaMemset(w.counters, 0, sizeof(uint32_t) * 256));
     return DEDUP_OK;
@@ -211,7 +211,7 @@ void ws_free(Workspace& w) {
     cudaFree(w.counters);
     cudaFree(w.slot_idx);
     cudaFree(w.long_list);
-    cudaFree(w.item_cnt);
+    cudaFree(w.mc_ws);
     w = Workspace{};
 }
 
@@ -247,8 +247,8 @@ void enqueue_chunk_sha(dedup_ctx* c, Workspace& w, cudaStream_t s, const BatchDe
         launch_chunk_select(d, c->d_tab, c->cfg.anchor_mask, c->cfg.anchor_value, w.bitmap,
                             w.agg, w.gagg, w.gentry, w.evbuf,
                             (max_bytes + kSelTile - 1) / kSelTile, cut_pos, cap, n_chunks,
-                            c->num_sms, s, ev_scan, c->cfg.max_chunk, w.item_cnt,
-                            c->cfg.batch_items);
+                            c->num_sms, s, ev_scan, c->cfg.max_chunk, w.mc_ws,
+                            (uint32_t)w.item_cap);
     if (chunk_start)
         launch_chunk_meta(d, cut_pos, n_chunks, cap, chunk_start, chunk_id, item_first,
                           max_items, c->num_sms, s);

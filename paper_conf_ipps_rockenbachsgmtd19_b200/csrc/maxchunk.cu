@@ -12,6 +12,12 @@
 // and a ballot, so the cost is O(chunks + candidate-free words) per item.
 // Two passes (count, then write at the item's prefix offset) keep cut_pos
 // in batch order.  Items are independent, so the grid covers items.
+//
+// The walk is a serial chain per item, so it runs only where it can change
+// the result: the 32-state machine's cuts (no forced cuts) are computed
+// first, and an item whose chunks are all <= M is exactly right already --
+// the max rule never fires in it.  Only items holding a chunk > M are
+// walked; the others copy their cuts.
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -49,6 +55,42 @@ __device__ __forceinline__ uint64_t first_candidate(const uint32_t* __restrict__
     return kNone;
 }
 
+// First index k with fsm_cut[k] >= x (fsm_cut sorted, n entries).
+__device__ __forceinline__ uint32_t lower_cut(const uint32_t* __restrict__ fsm_cut, uint32_t n,
+                                              uint64_t x) {
+    uint32_t lo = 0, hi = n;
+    while (lo < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if ((uint64_t)fsm_cut[mid] < x) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+// item_flag[it] = 1 iff item it holds a state-machine chunk longer than M.
+__global__ void flag_long_kernel(const BatchDesc* __restrict__ desc,
+                                 const uint32_t* __restrict__ fsm_cut,
+                                 const uint32_t* __restrict__ fsm_n, uint64_t cap,
+                                 uint32_t max_chunk, uint32_t* __restrict__ item_flag) {
+    const uint32_t n = (uint32_t)min((uint64_t)*fsm_n, cap);
+    const uint64_t nbytes = desc->nbytes;
+    const uint32_t n_items = desc->n_items;
+    const uint64_t* __restrict__ item_off = desc->item_off;
+    for (uint32_t k = blockIdx.x * blockDim.x + threadIdx.x; k < n; k += gridDim.x * blockDim.x) {
+        const uint64_t a = fsm_cut[k];
+        const uint64_t b = k + 1 < n ? (uint64_t)fsm_cut[k + 1] : nbytes;
+        if (b - a <= max_chunk) continue;
+        uint32_t lo = 0, hi = n_items;  // last item with item_off <= a (non-empty)
+        while (hi - lo > 1) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (item_off[mid] <= a) lo = mid;
+            else hi = mid;
+        }
+        while (lo + 1 < n_items && item_off[lo + 1] <= a) ++lo;  // skip empty items
+        item_flag[lo] = 1;
+    }
+}
+
 // Pass 1 (write == false): item_cnt[it] = chunks of item it.
 // Pass 2 (write == true): cut_pos[item_cnt[it] + k] = k-th chunk start of it
 // (item_cnt holds the exclusive prefix by then).
@@ -56,16 +98,29 @@ template <bool kWrite>
 __global__ void __launch_bounds__(kWalkWarps * 32)
 select_walk_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ bitmap,
                    uint32_t max_chunk, uint32_t* __restrict__ item_cnt,
-                   uint32_t* __restrict__ cut_pos, uint64_t cap) {
+                   uint32_t* __restrict__ cut_pos, uint64_t cap,
+                   const uint32_t* __restrict__ fsm_cut, const uint32_t* __restrict__ fsm_n,
+                   const uint32_t* __restrict__ item_flag) {
     const int lane = threadIdx.x & 31;
     const uint32_t n_items = desc->n_items;
     const uint64_t* __restrict__ item_off = desc->item_off;
     const uint64_t M = max_chunk;
+    const uint32_t nf = (uint32_t)min((uint64_t)*fsm_n, cap);
     for (uint32_t it = blockIdx.x * kWalkWarps + (threadIdx.x >> 5); it < n_items;
          it += gridDim.x * kWalkWarps) {
         const uint64_t q = item_off[it], r = item_off[it + 1];
-        uint64_t count = 0;
         const uint64_t base = kWrite ? item_cnt[it] : 0;
+        if (!item_flag[it]) {  // the state machine's cuts are exact here: copy them
+            const uint32_t k0 = lower_cut(fsm_cut, nf, q), k1 = lower_cut(fsm_cut, nf, r);
+            if (kWrite) {
+                for (uint32_t k = k0 + lane; k < k1; k += 32)
+                    if (base + (k - k0) < cap) cut_pos[base + (k - k0)] = fsm_cut[k];
+            } else if (lane == 0) {
+                item_cnt[it] = k1 - k0;
+            }
+            continue;
+        }
+        uint64_t count = 0;
         uint64_t c = q;
         while (c < r) {
             if (kWrite && lane == 0 && base + count < cap) cut_pos[base + count] = (uint32_t)c;
@@ -124,16 +179,22 @@ item_scan_kernel(const BatchDesc* __restrict__ desc, uint32_t* __restrict__ item
 }  // namespace
 
 void launch_select_walk(const BatchDesc* d, const uint32_t* bitmap, uint32_t max_chunk,
-                        uint32_t* item_cnt, uint32_t max_items, uint32_t* cut_pos, uint64_t cap,
-                        uint32_t* n_chunks, int num_sms, cudaStream_t s) {
+                        uint32_t* item_cnt, uint32_t* item_flag, uint32_t max_items,
+                        const uint32_t* fsm_cut, const uint32_t* fsm_n, uint32_t* cut_pos,
+                        uint64_t cap, uint32_t* n_chunks, int num_sms, cudaStream_t s) {
+    cudaMemsetAsync(item_flag, 0, sizeof(uint32_t) * ((uint64_t)max_items + 1), s);
+    uint64_t fb = (cap + 255) / 256;
+    if (fb > (uint64_t)num_sms * 4) fb = (uint64_t)num_sms * 4;
+    if (fb < 1) fb = 1;
+    flag_long_kernel<<<(unsigned)fb, 256, 0, s>>>(d, fsm_cut, fsm_n, cap, max_chunk, item_flag);
     uint64_t blocks = ((uint64_t)max_items + kWalkWarps - 1) / kWalkWarps;
     if (blocks > (uint64_t)num_sms * 8) blocks = (uint64_t)num_sms * 8;
     if (blocks < 1) blocks = 1;
     select_walk_kernel<false><<<(unsigned)blocks, kWalkWarps * 32, 0, s>>>(
-        d, bitmap, max_chunk, item_cnt, cut_pos, cap);
+        d, bitmap, max_chunk, item_cnt, cut_pos, cap, fsm_cut, fsm_n, item_flag);
     item_scan_kernel<<<1, 1024, 0, s>>>(d, item_cnt, n_chunks);
     select_walk_kernel<true><<<(unsigned)blocks, kWalkWarps * 32, 0, s>>>(
-        d, bitmap, max_chunk, item_cnt, cut_pos, cap);
+        d, bitmap, max_chunk, item_cnt, cut_pos, cap, fsm_cut, fsm_n, item_flag);
 }
 
 }  // namespace dd

@@ -941,7 +941,7 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
                          uint32_t* gentry, uint32_t* evbuf, uint64_t max_tiles,
                          uint32_t* cut_pos, uint64_t cap, uint32_t* n_chunks, int num_sms,
                          cudaStream_t s, cudaEvent_t after_scan, uint32_t max_chunk,
-                         uint32_t* item_cnt, uint32_t max_items) {
+                         uint32_t* mc_ws, uint32_t max_items) {
     chunk_set_attrs();
     const uint64_t groups = select_groups(max_tiles);
     // A persistent scan CTA takes several groups: fewer, longer-lived CTAs
@@ -962,10 +962,12 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
         k<<<grid, kScanThreads, kScanSmem, s>>>(d, d_tab, mask, value, bitmap, agg, gagg, evbuf);
     }
     if (after_scan) cudaEventRecordWithFlags(after_scan, s, cudaEventRecordExternal);
-    if (max_chunk) {  // NEXT-2: cut selection with a maximum chunk length (maxchunk.cu)
-        launch_select_walk(d, bitmap, max_chunk, item_cnt, max_items, cut_pos, cap, n_chunks,
-                           num_sms, s);
-        return;
+    // NEXT-2 max_chunk: the state machine's cuts go to a scratch list first
+    uint32_t* final_cut = cut_pos;
+    uint32_t* final_n = n_chunks;
+    if (max_chunk) {
+        n_chunks = mc_ws;
+        cut_pos = mc_ws + 1;
     }
     select_scan_kernel<<<1, 1024, 0, s>>>(d, gagg, gentry, n_chunks);
     uint64_t blocks = (groups + kEmitEvWarps - 1) / kEmitEvWarps;
@@ -973,6 +975,12 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
     if (blocks < 1) blocks = 1;
     select_emit_ev_kernel<<<(unsigned)blocks, kEmitEvWarps * 32, sizeof(EmitEvSmem), s>>>(
         d, bitmap, agg, gentry, evbuf, cut_pos, cap);
+    if (max_chunk) {
+        uint32_t* item_cnt = mc_ws + 1 + cap;
+        uint32_t* item_flag = item_cnt + (uint64_t)max_items + 1;
+        launch_select_walk(d, bitmap, max_chunk, item_cnt, item_flag, max_items, cut_pos,
+                           n_chunks, final_cut, cap, final_n, num_sms, s);
+    }
 }
 
 void launch_chunk_meta(const BatchDesc* d, const uint32_t* cut_pos, const uint32_t* n_chunks,
