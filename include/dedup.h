@@ -70,7 +70,7 @@ typedef struct {
     uint32_t poly;           /* P(t) = t^32 + poly over GF(2) */
     uint32_t anchor_mask;    /* cut iff (fp & anchor_mask) == anchor_value */
     uint32_t anchor_value;
-    uint32_t min_chunk;      /* GPU v1 requires == window */
+    uint32_t min_chunk;      /* >= window; != 32 selects cuts by a walk per item (NEXT-2) */
     uint32_t max_chunk;      /* 0 = none; else >= 64: forced cut at c + max_chunk (NEXT-2) */
     int32_t device;          /* CUDA device ordinal of this ctx */
     uint32_t slots;          /* in-flight batches ("memory spaces"), 1..64 */
@@ -92,8 +92,8 @@ void dedup_config_default(dedup_config* cfg);
 /* Creates a ctx on cfg->device: copies the config, builds the Rabin tables,
  * allocates `slots` batch slots (device + pinned host result buffers) and two
  * digest tables of >= 2 * table_capacity slots (power of two).
- * Errors: EINVAL (bad config), EUNSUPPORTED (window/min_chunk other than
- * 32, or 0 < max_chunk < 64), ENOMEM, ECUDA.  *out is NULL on error. */
+ * Errors: EINVAL (bad config), EUNSUPPORTED (window other than 32, or
+ * 0 < max_chunk < 64), ENOMEM, ECUDA.  *out is NULL on error. */
 dedup_status dedup_init(const dedup_config* cfg, dedup_ctx** out);
 
 /* Releases everything; waits for in-flight work.  Accepts NULL. */

@@ -194,7 +194,7 @@ dedup_status ws_alloc(dedup_ctx* c, Workspace& w, uint64_t batch_bytes, uint64_t
     TRY(dalloc(c, &w.counters, 256));
     TRY(dalloc(c, &w.slot_idx, cap));
     TRY(dalloc(c, &w.long_list, batch_bytes / kMinLongBytes + 2));
-    if (c->cfg.max_chunk) {
+    if (c->cfg.max_chunk || c->cfg.min_chunk != 32) {
         w.item_cap = cap;
         TRY(dalloc(c, &w.mc_ws, maxchunk_ws_words(cap, w.item_cap)));
     }
@@ -248,7 +248,7 @@ void enqueue_chunk_sha(dedup_ctx* c, Workspace& w, cudaStream_t s, const BatchDe
                             w.agg, w.gagg, w.gentry, w.evbuf,
                             (max_bytes + kSelTile - 1) / kSelTile, cut_pos, cap, n_chunks,
                             c->num_sms, s, ev_scan, c->cfg.max_chunk, w.mc_ws,
-                            (uint32_t)w.item_cap);
+                            (uint32_t)w.item_cap, c->cfg.min_chunk);
     if (chunk_start)
         launch_chunk_meta(d, cut_pos, n_chunks, cap, chunk_start, chunk_id, item_first,
                           max_items, c->num_sms, s);
@@ -426,8 +426,8 @@ dedup_status check_cfg(const dedup_config* g) {
     if (g->table_capacity < 1 || g->table_capacity > (1ull << 31)) return DEDUP_EINVAL;
     if (g->sha_lane_bytes != 0 && (g->sha_lane_bytes < 64 || g->sha_lane_bytes > (1u << 24)))
         return DEDUP_EINVAL;
-    // max_chunk (NEXT-2): forced cuts, selected by maxchunk.cu's walk
-    if (g->window != 32 || g->min_chunk != 32) return DEDUP_EUNSUPPORTED;
+    // max_chunk and min_chunk > window (NEXT-2): selected by maxchunk.cu's walk
+    if (g->window != 32) return DEDUP_EUNSUPPORTED;
     if (g->max_chunk != 0 && g->max_chunk < 64) return DEDUP_EUNSUPPORTED;
     return DEDUP_OK;
 }
@@ -836,7 +836,7 @@ dedup_status dedup_op_chunk(dedup_ctx* c, void* stream, const uint8_t* d_bytes, 
     if (nbytes > c->cfg.batch_bytes) return fail(c, DEDUP_EINVAL, "nbytes > batch_bytes");
     if (reinterpret_cast<uintptr_t>(d_bytes) & 15)
         return fail(c, DEDUP_EINVAL, "d_bytes must be 16-byte aligned");
-    if (c->cfg.max_chunk && n_items > c->op_ws.item_cap)
+    if ((c->cfg.max_chunk || c->cfg.min_chunk != 32) && n_items > c->op_ws.item_cap)
         return fail(c, DEDUP_EINVAL, "n_items larger than the max_chunk workspace");
     CU(cudaSetDevice(c->cfg.device));
     cudaStream_t s = static_cast<cudaStream_t>(stream);

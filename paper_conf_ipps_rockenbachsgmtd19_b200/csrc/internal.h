@@ -75,7 +75,8 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
                          uint32_t* gentry, uint32_t* evbuf, uint64_t max_tiles,
                          uint32_t* cut_pos, uint64_t cap, uint32_t* n_chunks, int num_sms,
                          cudaStream_t s, cudaEvent_t after_scan, uint32_t max_chunk = 0,
-                         uint32_t* mc_ws = nullptr, uint32_t max_items = 0);
+                         uint32_t* mc_ws = nullptr, uint32_t max_items = 0,
+                         uint32_t min_chunk = 32);
 // max_chunk workspace words: fsm count (1) + fsm cuts (cap) + item counts and
 // flags (2 x (max_items + 1)).
 inline uint64_t maxchunk_ws_words(uint64_t cap, uint64_t max_items) {
@@ -85,9 +86,10 @@ inline uint64_t maxchunk_ws_words(uint64_t cap, uint64_t max_items) {
 // (fsm_cut, *fsm_n) are kept for items without a chunk > max_chunk; the
 // other items are walked over the scan's candidate bitmap.
 void launch_select_walk(const BatchDesc* d, const uint32_t* bitmap, uint32_t max_chunk,
-                        uint32_t* item_cnt, uint32_t* item_flag, uint32_t max_items,
-                        const uint32_t* fsm_cut, const uint32_t* fsm_n, uint32_t* cut_pos,
-                        uint64_t cap, uint32_t* n_chunks, int num_sms, cudaStream_t s);
+                        uint32_t min_chunk, uint32_t* item_cnt, uint32_t* item_flag,
+                        uint32_t max_items, const uint32_t* fsm_cut, const uint32_t* fsm_n,
+                        uint32_t* cut_pos, uint64_t cap, uint32_t* n_chunks, int num_sms,
+                        cudaStream_t s);
 
 void launch_chunk_meta(const BatchDesc* d, const uint32_t* cut_pos, const uint32_t* n_chunks,
                        uint64_t cap, uint32_t* chunk_start, uint64_t* chunk_id,

@@ -1,4 +1,5 @@
-// maxchunk.cu -- row NEXT-2, the max_chunk chunker variant:
+// maxchunk.cu -- row NEXT-2, the max_chunk and min_chunk >
+// window chunker variants.  max_chunk:
 // cut selection with a maximum chunk length M (PARSEC-style forced cut; the
 // oracle's oracle_chunk_item with max_chunk != 0).  After a cut at c the
 // next cut is the first Rabin candidate e in [c + 32, min(c + M, r)) of the
@@ -18,6 +19,10 @@
 // first, and an item whose chunks are all <= M is exactly right already --
 // the max rule never fires in it.  Only items holding a chunk > M are
 // walked; the others copy their cuts.
+//
+// min_chunk > 32 (the hash restarts at a cut; the next cut is the first
+// candidate >= c + min_chunk): the 32-state machine does not apply at all,
+// every item is walked with that lower bound.
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -97,14 +102,15 @@ __global__ void flag_long_kernel(const BatchDesc* __restrict__ desc,
 template <bool kWrite>
 __global__ void __launch_bounds__(kWalkWarps * 32)
 select_walk_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ bitmap,
-                   uint32_t max_chunk, uint32_t* __restrict__ item_cnt,
+                   uint32_t max_chunk, uint32_t min_chunk, uint32_t* __restrict__ item_cnt,
                    uint32_t* __restrict__ cut_pos, uint64_t cap,
                    const uint32_t* __restrict__ fsm_cut, const uint32_t* __restrict__ fsm_n,
                    const uint32_t* __restrict__ item_flag) {
     const int lane = threadIdx.x & 31;
     const uint32_t n_items = desc->n_items;
     const uint64_t* __restrict__ item_off = desc->item_off;
-    const uint64_t M = max_chunk;
+    const uint64_t M = max_chunk ? max_chunk : ~0ull >> 1;  // 0: no forced cut
+    const uint64_t m = min_chunk;
     const uint32_t nf = (uint32_t)min((uint64_t)*fsm_n, cap);
     for (uint32_t it = blockIdx.x * kWalkWarps + (threadIdx.x >> 5); it < n_items;
          it += gridDim.x * kWalkWarps) {
@@ -126,7 +132,7 @@ select_walk_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restric
             if (kWrite && lane == 0 && base + count < cap) cut_pos[base + count] = (uint32_t)c;
             ++count;
             const uint64_t lim = c + M < r ? c + M : r;
-            const uint64_t e = c + 32 < lim ? first_candidate(bitmap, c + 32, lim, lane) : kNone;
+            const uint64_t e = c + m < lim ? first_candidate(bitmap, c + m, lim, lane) : kNone;
             if (e != kNone) c = e;
             else if (c + M < r) c = c + M;
             else break;
@@ -179,22 +185,29 @@ item_scan_kernel(const BatchDesc* __restrict__ desc, uint32_t* __restrict__ item
 }  // namespace
 
 void launch_select_walk(const BatchDesc* d, const uint32_t* bitmap, uint32_t max_chunk,
-                        uint32_t* item_cnt, uint32_t* item_flag, uint32_t max_items,
-                        const uint32_t* fsm_cut, const uint32_t* fsm_n, uint32_t* cut_pos,
-                        uint64_t cap, uint32_t* n_chunks, int num_sms, cudaStream_t s) {
-    cudaMemsetAsync(item_flag, 0, sizeof(uint32_t) * ((uint64_t)max_items + 1), s);
-    uint64_t fb = (cap + 255) / 256;
-    if (fb > (uint64_t)num_sms * 4) fb = (uint64_t)num_sms * 4;
-    if (fb < 1) fb = 1;
-    flag_long_kernel<<<(unsigned)fb, 256, 0, s>>>(d, fsm_cut, fsm_n, cap, max_chunk, item_flag);
+                        uint32_t min_chunk, uint32_t* item_cnt, uint32_t* item_flag,
+                        uint32_t max_items, const uint32_t* fsm_cut, const uint32_t* fsm_n,
+                        uint32_t* cut_pos, uint64_t cap, uint32_t* n_chunks, int num_sms,
+                        cudaStream_t s) {
+    if (min_chunk != 32) {
+        // the state machine assumes min chunk = window = 32: walk every item
+        cudaMemsetAsync(item_flag, 1, sizeof(uint32_t) * ((uint64_t)max_items + 1), s);
+    } else {
+        cudaMemsetAsync(item_flag, 0, sizeof(uint32_t) * ((uint64_t)max_items + 1), s);
+        uint64_t fb = (cap + 255) / 256;
+        if (fb > (uint64_t)num_sms * 4) fb = (uint64_t)num_sms * 4;
+        if (fb < 1) fb = 1;
+        flag_long_kernel<<<(unsigned)fb, 256, 0, s>>>(d, fsm_cut, fsm_n, cap, max_chunk,
+                                                      item_flag);
+    }
     uint64_t blocks = ((uint64_t)max_items + kWalkWarps - 1) / kWalkWarps;
     if (blocks > (uint64_t)num_sms * 8) blocks = (uint64_t)num_sms * 8;
     if (blocks < 1) blocks = 1;
     select_walk_kernel<false><<<(unsigned)blocks, kWalkWarps * 32, 0, s>>>(
-        d, bitmap, max_chunk, item_cnt, cut_pos, cap, fsm_cut, fsm_n, item_flag);
+        d, bitmap, max_chunk, min_chunk, item_cnt, cut_pos, cap, fsm_cut, fsm_n, item_flag);
     item_scan_kernel<<<1, 1024, 0, s>>>(d, item_cnt, n_chunks);
     select_walk_kernel<true><<<(unsigned)blocks, kWalkWarps * 32, 0, s>>>(
-        d, bitmap, max_chunk, item_cnt, cut_pos, cap, fsm_cut, fsm_n, item_flag);
+        d, bitmap, max_chunk, min_chunk, item_cnt, cut_pos, cap, fsm_cut, fsm_n, item_flag);
 }
 
 }  // namespace dd

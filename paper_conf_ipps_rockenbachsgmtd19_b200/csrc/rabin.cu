@@ -941,7 +941,7 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
                          uint32_t* gentry, uint32_t* evbuf, uint64_t max_tiles,
                          uint32_t* cut_pos, uint64_t cap, uint32_t* n_chunks, int num_sms,
                          cudaStream_t s, cudaEvent_t after_scan, uint32_t max_chunk,
-                         uint32_t* mc_ws, uint32_t max_items) {
+                         uint32_t* mc_ws, uint32_t max_items, uint32_t min_chunk) {
     chunk_set_attrs();
     const uint64_t groups = select_groups(max_tiles);
     // A persistent scan CTA takes several groups: fewer, longer-lived CTAs
@@ -965,7 +965,8 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
     // NEXT-2 max_chunk: the state machine's cuts go to a scratch list first
     uint32_t* final_cut = cut_pos;
     uint32_t* final_n = n_chunks;
-    if (max_chunk) {
+    const bool walk = max_chunk != 0 || min_chunk != 32;
+    if (walk) {
         n_chunks = mc_ws;
         cut_pos = mc_ws + 1;
     }
@@ -975,11 +976,11 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
     if (blocks < 1) blocks = 1;
     select_emit_ev_kernel<<<(unsigned)blocks, kEmitEvWarps * 32, sizeof(EmitEvSmem), s>>>(
         d, bitmap, agg, gentry, evbuf, cut_pos, cap);
-    if (max_chunk) {
+    if (walk) {
         uint32_t* item_cnt = mc_ws + 1 + cap;
         uint32_t* item_flag = item_cnt + (uint64_t)max_items + 1;
-        launch_select_walk(d, bitmap, max_chunk, item_cnt, item_flag, max_items, cut_pos,
-                           n_chunks, final_cut, cap, final_n, num_sms, s);
+        launch_select_walk(d, bitmap, max_chunk, min_chunk, item_cnt, item_flag, max_items,
+                           cut_pos, n_chunks, final_cut, cap, final_n, num_sms, s);
     }
 }
 

@@ -73,7 +73,6 @@ def test_struct_layouts_match_header(L):
 
 @pytest.mark.parametrize("fields,status", [
     (dict(window=48, min_chunk=48), N.DEDUP_EUNSUPPORTED),
-    (dict(min_chunk=64), N.DEDUP_EUNSUPPORTED),
     (dict(max_chunk=48), N.DEDUP_EUNSUPPORTED),
     (dict(max_chunk=16), N.DEDUP_EINVAL),         # max_chunk < min_chunk
     (dict(window=48), N.DEDUP_EINVAL),          # min_chunk < window
