@@ -60,6 +60,22 @@ SCAN_OPS_PER_BYTE = 8
 INT_LANES_PER_SM_CLK = 128
 
 
+def h2d_bandwidth(pin, dev, nbytes=64 * MiB, reps=10):
+    """Plain pinned host -> device copy bandwidth (the e2e roofline, PCIe)."""
+    import torch
+    src = torch.from_numpy(pin[:nbytes])
+    dst = dev[:nbytes]
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
+    dst.copy_(src, non_blocking=True)
+    torch.cuda.synchronize()
+    ev[0].record()
+    for _ in range(reps):
+        dst.copy_(src, non_blocking=True)
+    ev[1].record()
+    ev[1].synchronize()
+    return nbytes * reps / (ev[0].elapsed_time(ev[1]) * 1e-3) / 1e9
+
+
 def engine_kwargs(stream_bytes: int) -> dict:
     return dict(batch_bytes=BATCH_BYTES, batch_items=BATCH_ITEMS, slots=SLOTS,
                 table_capacity=max(1 << 16, stream_bytes // 2048), host_fed=True)
@@ -546,7 +562,8 @@ def main():
            "d2h_bytes_per_step": (33 * de["chunks"] + 4 * de["items"] + 8 * de["batches"])
            / e2e_steps,
            "steps": e2e_steps, "items_per_step": items_per_step,
-           "api": "dedup_submit_batch (pinned host buffers) + dedup_drain"}
+           "api": "dedup_submit_batch (pinned host buffers) + dedup_drain",
+           "pcie_h2d_gbs": h2d_bandwidth(pin, dd)}
     d.close()
 
     line = {

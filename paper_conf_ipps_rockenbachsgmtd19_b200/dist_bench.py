@@ -1,12 +1,15 @@
 """bench.py --gpus N (N > 1) under torchrun: one process per GPU, NCCL.
 
-Weak scaling: in every step (= wave) each rank processes one GPU batch of
-the cycled C2 stream; digests are routed to their owner GPU with NCCL
-all-to-alls (rows A5-A8, see dist.py).  Waves are pipelined
-(dist.WavePipeline): `DEPTH` waves are in flight per rank, so a rank's GPU
-keeps chunking and hashing later batches while the exchange of the oldest
-one runs.  A dedup stream spans max(ceil(batches / N), 4 * DEPTH) waves; the
-table shards are reset at every stream start.  The timed region is bracketed by a
+Weak scaling: in every step (= wave) each rank processes one pass over the
+whole C2 stream (184 MiB, 184 items of 1 MiB) as one GPU batch; digests are
+routed to their owner GPU with NCCL all-to-alls (rows A5-A8, see dist.py).
+Waves are pipelined (dist.WavePipeline): `DEPTH` waves are in flight per
+rank, so a rank's GPU keeps chunking and hashing later waves while the
+exchange of the oldest one runs.  The wave is the whole stream because the
+pipeline's host orchestration costs ~1 ms per wave.
+A dedup stream spans 4 * DEPTH waves; the table shards are reset at every
+stream start (every rank passes over the same bytes, so within a stream
+the other ranks' and later passes' chunks are duplicates).  The timed region is bracketed by a
 barrier + device synchronisation and measured with CUDA events; the maximum
 over ranks is reported.
 """
@@ -17,7 +20,7 @@ import os
 
 import numpy as np
 
-DEPTH = 8  # waves in flight per rank
+DEPTH = 4  # waves in flight per rank
 
 
 def main(args, data, off, B):
@@ -35,19 +38,21 @@ def main(args, data, off, B):
     dev = torch.device("cuda", local)
     dist.init_process_group("nccl", device_id=dev)
     x = D.TorchDistExchange()
-    plan = B.plan_batches(off)
-    nb = len(plan)
-    items_per_batch = max(j - k for k, j in plan)
+    n_items = len(off) - 1
+    plan = [(0, n_items)]                # one wave batch = the whole stream
+    nb = 1
+    items_per_batch = n_items
+    wave_bytes = int(off[-1])
     # the owner receives up to `world` batches' records per wave
-    owner = Dedup(local, batch_bytes=min(1 << 30, world * B.BATCH_BYTES), batch_items=1, slots=1,
+    owner = Dedup(local, batch_bytes=min(1 << 30, world * wave_bytes), batch_items=1, slots=1,
                   table_capacity=max(1 << 16, len(data) // 2048 // world), host_fed=False,
                   owner_rank=rank, num_owners=world)
-    pipe = D.WavePipeline(x, [owner], local, B.BATCH_BYTES, B.BATCH_ITEMS + 1, depth=DEPTH)
+    pipe = D.WavePipeline(x, [owner], local, wave_bytes, n_items + 1, depth=DEPTH)
     ddata = torch.from_numpy(data).to(dev)
     # A table reset completes every wave in flight first (end_stream), so a
     # dedup stream spans at least 4 pipeline depths of waves (the C2 batches
     # cycled; later passes over the data inside one stream are duplicates).
-    waves_per_stream = max((nb + world - 1) // world, 4 * DEPTH)
+    waves_per_stream = 4 * DEPTH
     counted = {"bytes": 0, "chunks": 0}
 
     def take(outs, timed):
@@ -92,9 +97,10 @@ def main(args, data, off, B):
             "vs_baseline": None, "dtype": "u32", "data": "synthetic",
             "chunks_per_s": float(tot[1]) / (t / 1e3),
             "config": {"workload": f"{B.WORKLOAD}: 184 MiB simlarge-sized synthetic stream, "
-                                   "1 MiB items, dup_frac 0.52, device-resident, one batch per "
-                                   "GPU per step, digest all-to-all (NCCL) to owner GPUs",
-                       "batch_bytes": B.BATCH_BYTES, "waves_in_flight": DEPTH,
+                                   "1 MiB items, dup_frac 0.52, device-resident, one pass over "
+                                   "the stream per GPU per step, digest all-to-all (NCCL) to "
+                                   "owner GPUs",
+                       "batch_bytes": wave_bytes, "waves_in_flight": DEPTH,
                        "parallelism": f"{world} GPUs, digest-prefix table sharding",
                        "l2": "inputs larger than L2"},
             "gpu_launches": None,
