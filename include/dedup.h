@@ -305,7 +305,7 @@ dedup_status dedup_op_scatter(dedup_ctx* c, void* stream, const uint64_t* d_repl
  * L = 0).  d_skip (optional, u8 per block): positions of blocks with a
  * non-zero flag (duplicates) get L = 0, offset 0.
  * d_bytes 16-byte aligned and readable to nbytes rounded up to 16;
- * nbytes < 2^31; 1 <= window <= 32768; 1 <= max_coded <= 255; else EINVAL. */
+ * nbytes < 2^31; 1 <= window <= 16384; 1 <= max_coded <= 255; else EINVAL. */
 dedup_status dedup_op_findmatch(dedup_ctx* c, void* stream, const uint8_t* d_bytes,
                                 uint64_t nbytes, const uint32_t* d_start,
                                 const uint32_t* d_n_blocks, uint64_t cap, const uint8_t* d_skip,

@@ -913,7 +913,7 @@ dedup_status dedup_op_findmatch(dedup_ctx* c, void* stream, const uint8_t* d_byt
     if (reinterpret_cast<uintptr_t>(d_match_off) & 1)
         return fail(c, DEDUP_EINVAL, "d_match_off must be 2-byte aligned");
     if (nbytes >= (1ull << 31)) return fail(c, DEDUP_EINVAL, "nbytes >= 2^31");
-    if (window < 1 || window > 32768) return fail(c, DEDUP_EINVAL, "window not in [1, 32768]");
+    if (window < 1 || window > 16384) return fail(c, DEDUP_EINVAL, "window not in [1, 16384]");
     if (max_coded < 1 || max_coded > 255)
         return fail(c, DEDUP_EINVAL, "max_coded not in [1, 255]");
     if (nbytes > 0 && (d_start == nullptr || d_n_blocks == nullptr || cap == 0))

@@ -75,7 +75,7 @@ def test_findmatch_random_starts(cuda, entropy):
 
 
 @pytest.mark.parametrize("W,MC", [(1, 1), (7, 3), (64, 18), (300, 40), (2048, 255),
-                                  (32768, 18)])
+                                  (16384, 18)])
 def test_findmatch_window_and_length_limits(cuda, W, MC):
     rng = np.random.default_rng(W + MC)
     n = 70_001
