@@ -51,6 +51,7 @@ METRIC = "input GB/s & chunks/s (dedup hot path) at 1/2/4/8 B200; % of HBM/INT r
 # counting a 3-input logic/add as one op and a rotate as one op):
 #   80 rounds x (f 1 + rotl5 1 + adds 2 + rotl30 1) + 64 x schedule 3 + 5.
 SHA1_OPS_PER_BLOCK = 80 * 5 + 64 * 3 + 5
+SHA1_ALU_OPS_PER_BLOCK = 80 * 3 + 64 * 3       # of which on the ALU pipe
 # Rabin rolling step per input byte: 2 table lookups, shift-in,
 # 2 address formations, 1 3-way XOR, test + bit = 8 ops.
 SCAN_OPS_PER_BYTE = 8
@@ -530,8 +531,17 @@ def main():
         tj = json.load(open(tp))  # scaled from its batch size to this launch's bytes
         if "sha1" in tj:
             traffic = tj["sha1"] / tj["capture_batch_bytes"] * kd["launch_bytes"]
+    # the same launch against the ALU pipe alone (16 lanes/clk/SMSP): the
+    # round function and message schedule need 432 ALU-pipe ops per block
+    # (f LOP3 80, rotl30 SHF 80, rotl5+add LEA 80, schedule 2 LOP3 + SHF
+    # per word x 64), the adds go to the FMA pipe
+    alu_peak = int_peak / 2
+    alu_ach = kd["achieved"] * SHA1_ALU_OPS_PER_BLOCK / SHA1_OPS_PER_BLOCK
     roofline = {"kernel": "sha1_kernel", "bound": "alu", "achieved": kd["achieved"],
                 "peak": int_peak, "unit": "Tops/s", "frac": kd["achieved"] / int_peak,
+                "alu_pipe_view": {"achieved": alu_ach, "peak": alu_peak,
+                                  "frac": alu_ach / alu_peak, "ops_per_block":
+                                  SHA1_ALU_OPS_PER_BLOCK},
                 "traffic": traffic, "peak_source": peak_source,
                 "launch": f"{kd['launch_bytes'] / MiB:.0f} MiB of C2 chunks per launch, "
                           f"{kd['launch_us']:.0f} us per launch (CUDA events, "
