@@ -407,6 +407,44 @@ def mandel_measure(sm_mhz, with_cpu=True):
     return out
 
 
+def batch_sweep(dd, off, sizes=(1, 2, 4, 8, 16, 32), target_bytes=3 << 30):
+    """BASELINE.json configs[1]: the C2 stream at GPU batch sizes 1..32 MiB
+    (the 64 MiB point is the headline `value`), device-resident, 40 batches
+    in flight, CUDA events around the submissions; GB/s per batch size."""
+    import torch
+
+    from paper_conf_ipps_rockenbachsgmtd19_b200 import Dedup
+    out = {}
+    for mb in sizes:
+        bb = mb * MiB
+        plan, k, n = [], 0, len(off) - 1
+        while k < n:
+            j = k + 1
+            while j < n and int(off[j + 1]) - int(off[k]) <= bb:
+                j += 1
+            plan.append((k, j))
+            k = j
+        subs = [(dd[int(off[a]):int(off[b])], (off[a:b + 1] - off[a]).copy()) for a, b in plan]
+        d = Dedup(0, batch_bytes=bb, batch_items=max(mb, 1) + 1, slots=SLOTS,
+                  table_capacity=max(1 << 16, len(dd) // 2048), host_fed=False)
+        producer = torch.cuda.current_stream().cuda_stream
+        sub = lambda b: d.submit_device(subs[b][0], subs[b][1], producer)  # noqa: E731
+        steps = max(60, target_bytes // bb)
+        run_steps(d, sub, len(plan), 8, 0)
+        torch.cuda.synchronize()
+        s0 = d.stats()
+        ev = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
+        ev[0].record()
+        run_steps(d, sub, len(plan), steps, 8)
+        d.join()
+        ev[1].record()
+        ev[1].synchronize()
+        nbytes = d.stats()["bytes"] - s0["bytes"]
+        out[f"{mb}MiB"] = nbytes / (ev[0].elapsed_time(ev[1]) * 1e-3) / 1e9
+        d.close()
+    return out
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -515,6 +553,8 @@ def main():
     iso = isolated_kernels(dd, off, int_peak)
     kernels.update(iso)
     kernels["mandelbrot"] = mandel_measure(sm_mhz, with_cpu=not args.no_cpu_baseline)
+    sweep = batch_sweep(dd, off)
+    sweep[f"{BATCH_BYTES // MiB}MiB"] = value
     sha_blocks_per_byte = ds["sha1_blocks"] / max(ds["bytes"], 1)
     path_ops = value * 1e9 * (SCAN_OPS_PER_BYTE + sha_blocks_per_byte * SHA1_OPS_PER_BLOCK) / 1e12
     kernels["path"] = {"bound": "alu", "achieved": path_ops, "peak": int_peak, "unit": "Tops/s",
@@ -586,6 +626,7 @@ def main():
                                "1 MiB items, dup_frac 0.52, device-resident",
                    "batch_bytes": BATCH_BYTES, "batch_items": BATCH_ITEMS, "slots": SLOTS,
                    "batches_per_stream": nb, "parallelism": "1 GPU",
+                   "batch_sweep_gbs": sweep,
                    "l2": "inputs larger than L2 (184 MiB stream cycled, 126 MB L2)"},
         "clocks": clocks, "gpu_launches": launches, "roofline": roofline, "kernels": kernels,
         "e2e": e2e,
