@@ -429,7 +429,7 @@ def batch_sweep(dd, off, sizes=(1, 2, 4, 8, 16, 32), target_bytes=3 << 30):
                   table_capacity=max(1 << 16, len(dd) // 2048), host_fed=False)
         producer = torch.cuda.current_stream().cuda_stream
         sub = lambda b: d.submit_device(subs[b][0], subs[b][1], producer)  # noqa: E731
-        steps = max(60, target_bytes // bb)
+        steps = max(400, target_bytes // bb)
         run_steps(d, sub, len(plan), 8, 0)
         torch.cuda.synchronize()
         s0 = d.stats()
