@@ -18,7 +18,8 @@
 // the result: the 32-state machine's cuts (no forced cuts) are computed
 // first, and an item whose chunks are all <= M is exactly right already --
 // the max rule never fires in it.  Only items holding a chunk > M are
-// walked; the others copy their cuts.
+// walked, and only from the start of their first such chunk (the chain
+// before it is the machine's); the others copy their cuts.
 //
 // min_chunk > 32 (the hash restarts at a cut; the next cut is the first
 // candidate >= c + min_chunk): the 32-state machine does not apply at all,
@@ -128,6 +129,31 @@ select_walk_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restric
         }
         uint64_t count = 0;
         uint64_t c = q;
+        if (m == 32) {
+            // the chain is the state machine's up to the first chunk longer
+            // than M: copy those cuts and walk from that chunk's start on
+            const uint32_t k0 = lower_cut(fsm_cut, nf, q), k1 = lower_cut(fsm_cut, nf, r);
+            const uint64_t nbytes = desc->nbytes;
+            uint32_t kf = k1;
+            for (uint32_t kb = k0; kb < k1; kb += 32) {
+                const uint32_t k = kb + lane;
+                bool lng = false;
+                if (k < k1) {
+                    const uint64_t e = k + 1 < nf ? (uint64_t)fsm_cut[k + 1] : nbytes;
+                    lng = e - fsm_cut[k] > M;
+                }
+                const uint32_t bl = __ballot_sync(kFull, lng);
+                if (bl) {
+                    kf = kb + (uint32_t)(__ffs(bl) - 1);
+                    break;
+                }
+            }
+            if (kWrite)
+                for (uint32_t k = k0 + lane; k < kf; k += 32)
+                    if (base + (k - k0) < cap) cut_pos[base + (k - k0)] = fsm_cut[k];
+            count = kf - k0;
+            c = kf < k1 ? (uint64_t)fsm_cut[kf] : r;
+        }
         while (c < r) {
             if (kWrite && lane == 0 && base + count < cap) cut_pos[base + count] = (uint32_t)c;
             ++count;
