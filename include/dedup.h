@@ -349,6 +349,65 @@ void dedup_archive_decoder_free(dedup_archive_decoder* d);
 int64_t dedup_archive_decode(dedup_archive_decoder* d, const uint8_t* in, uint64_t in_len,
                              uint8_t* out, uint64_t out_cap);
 
+/* ------------------------------------------------------------------------ */
+/* 4. Multi-GPU wave pipeline (rows A5-A8 at G > 1), NCCL      */
+/* ------------------------------------------------------------------------ */
+/* One process (and one dedup_dist) per GPU.  In wave w every rank submits
+ * one batch; its local rows (chunk, SHA-1, local combine, route by digest
+ * owner) run on one of `depth` slots; when `depth` waves are in flight the
+ * oldest completes: per-owner counts and 32-byte records are exchanged with
+ * grouped ncclSend/ncclRecv, the owner inserts + looks up its shard (row
+ * A7), the first ids come back (row A8) and the results are copied to
+ * pinned host memory.  Every rank must make the same sequence of submit /
+ * flush / end_stream calls (NCCL matches them in order). */
+typedef struct dedup_dist dedup_dist;
+
+/* A 128-byte NCCL unique id (rank 0 creates it, the others receive it). */
+dedup_status dedup_nccl_unique_id(uint8_t out[128]);
+
+/* cfg: the owner config of this rank (device, owner_rank = rank,
+ * num_owners = nranks, table_capacity = this shard's expected distinct
+ * digests; the chunker fields apply to every batch).  batch_bytes /
+ * batch_items: the largest batch a wave may submit on this rank. */
+dedup_status dedup_dist_create(const dedup_config* cfg, const uint8_t nccl_id[128], int nranks,
+                               int rank, uint32_t depth, uint64_t batch_bytes,
+                               uint32_t batch_items, dedup_dist** out);
+void dedup_dist_destroy(dedup_dist* d);
+const char* dedup_dist_last_error(const dedup_dist* d);
+
+/* Submits this rank's batch of the next wave: d_bytes (device, 16-byte
+ * aligned, after `producer`'s current work), item_off (host, n_items + 1
+ * offsets), items get seq = first_seq + k.  If `depth` waves were in
+ * flight, the oldest completes first and *completed = 1: read it with
+ * dedup_dist_result before the next call. */
+dedup_status dedup_dist_submit(dedup_dist* d, const uint8_t* d_bytes, uint64_t nbytes,
+                               const uint64_t* item_off, uint32_t n_items, uint64_t first_seq,
+                               void* producer, uint32_t* completed);
+/* Completes the oldest wave in flight if any (*completed = 1). */
+dedup_status dedup_dist_flush(dedup_dist* d, uint32_t* completed);
+/* New dedup stream (clears this rank's table shard); no wave may be in
+ * flight (flush first), else DEDUP_EAGAIN. */
+dedup_status dedup_dist_end_stream(dedup_dist* d);
+
+typedef struct {
+    uint64_t first_seq;
+    uint32_t n_items, n_chunks;
+    const uint64_t* item_off;          /* [n_items + 1] batch-relative */
+    const uint32_t* item_first_chunk;  /* [n_items], 0xFFFFFFFF for empty items */
+    const uint32_t* chunk_start;       /* [n_chunks] item-relative */
+    const uint8_t* digest;             /* [n_chunks * 20] */
+    const uint64_t* first_id;          /* [n_chunks] */
+    const uint8_t* is_dup;             /* [n_chunks] */
+} dedup_wave_result;
+/* The last completed wave's results: waits until they are in host memory;
+ * the views stay valid until that slot completes again (`depth`
+ * completions later). */
+dedup_status dedup_dist_result(const dedup_dist* d, dedup_wave_result* out);
+/* The last completed wave's item count, chunk count and bytes, without
+ * waiting for its results to reach host memory. */
+dedup_status dedup_dist_last_counts(const dedup_dist* d, uint32_t* n_items, uint32_t* n_chunks,
+                                    uint64_t* nbytes);
+
 /* Number of kernels this ctx has launched so far (all layers). */
 uint64_t dedup_kernel_launches(const dedup_ctx* c);
 

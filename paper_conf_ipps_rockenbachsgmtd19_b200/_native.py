@@ -36,9 +36,25 @@ EXPORTS = [
     "dedup_op_scatter", "dedup_op_findmatch", "dedup_kernel_launches",
     "dedup_archive_encode", "dedup_archive_decoder_new", "dedup_archive_decoder_free",
     "dedup_archive_decode",
+    "dedup_nccl_unique_id", "dedup_dist_create", "dedup_dist_destroy", "dedup_dist_last_error",
+    "dedup_dist_submit", "dedup_dist_flush", "dedup_dist_end_stream", "dedup_dist_result",
+    "dedup_dist_last_counts",
 ]
 # every symbol declared in include/mandel.h (row NEXT-4)
 MANDEL_EXPORTS = ["mandel_rows_device", "mandel_image"]
+
+
+class WaveResult(ctypes.Structure):
+    _fields_ = [
+        ("first_seq", ctypes.c_uint64), ("n_items", ctypes.c_uint32),
+        ("n_chunks", ctypes.c_uint32),
+        ("item_off", ctypes.POINTER(ctypes.c_uint64)),
+        ("item_first_chunk", ctypes.POINTER(ctypes.c_uint32)),
+        ("chunk_start", ctypes.POINTER(ctypes.c_uint32)),
+        ("digest", ctypes.POINTER(ctypes.c_uint8)),
+        ("first_id", ctypes.POINTER(ctypes.c_uint64)),
+        ("is_dup", ctypes.POINTER(ctypes.c_uint8)),
+    ]
 
 
 class MandelConfig(ctypes.Structure):
@@ -138,6 +154,15 @@ def lib():
         "dedup_archive_decoder_new": (vp, [u32]),
         "dedup_archive_decoder_free": (None, [vp]),
         "dedup_archive_decode": (ctypes.c_int64, [vp, vp, u64, vp, u64]),
+        "dedup_nccl_unique_id": (st, [vp]),
+        "dedup_dist_create": (st, [P(Config), vp, i32, i32, u32, u64, u32, P(vp)]),
+        "dedup_dist_destroy": (None, [vp]),
+        "dedup_dist_last_error": (ctypes.c_char_p, [vp]),
+        "dedup_dist_submit": (st, [vp, vp, u64, vp, u32, u64, vp, P(u32)]),
+        "dedup_dist_flush": (st, [vp, P(u32)]),
+        "dedup_dist_end_stream": (st, [vp]),
+        "dedup_dist_result": (st, [vp, P(WaveResult)]),
+        "dedup_dist_last_counts": (st, [vp, P(u32), P(u32), P(u64)]),
         "mandel_rows_device": (st, [vp, i32, i32, ctypes.c_double, ctypes.c_double,
                                     ctypes.c_double, i32, i32, vp, vp, vp]),
         "mandel_image": (st, [P(MandelConfig), vp, P(ctypes.c_double), P(u64)]),

@@ -16,12 +16,27 @@ CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libdedup_b200.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
+def _nccl():
+    """The NCCL that torch loads (the wheel's)."""
+    try:
+        import nvidia.nccl
+        base = list(nvidia.nccl.__path__)[0]
+        return os.path.join(base, "include"), os.path.join(base, "lib")
+    except Exception:
+        return None, None
+
+
+NCCL_INC, NCCL_LIB = _nccl()
+
 FLAGS = [
     "-O3", "-std=c++17", "-lineinfo",
     "-gencode", "arch=compute_100a,code=sm_100a",
     "-Xcompiler", "-fPIC", "-shared",
     "-I", os.path.join(ROOT, "include"),
 ]
+if NCCL_INC:
+    FLAGS += ["-I", NCCL_INC, "-L", NCCL_LIB, "-l:libnccl.so.2",
+              "-Xlinker", f"-rpath={NCCL_LIB}"]
 
 
 def sources():

@@ -213,3 +213,49 @@ def test_wave_pipeline_matches_oracle(G, depth):
             assert np.array_equal(dg, w.digest), seq
             assert np.array_equal(dup, w.is_dup), seq
             assert np.array_equal(fid, w.first_id), seq
+
+
+@pytest.mark.parametrize("depth", [1, 3])
+def test_native_wave_pipeline_world1(depth):
+    """The C++ wave pipeline (csrc/dist.cpp) through NCCL with one rank: the
+    exchange sends every record to itself; bit-exact vs the oracle across an
+    end_stream."""
+    assert torch.cuda.is_available()
+    from paper_conf_ipps_rockenbachsgmtd19_b200 import dist as D
+    data = U.stream(10 * MiB, seed=71 + depth, dup_frac=0.6)
+    off = synthgen.split_items(data, MiB // 2)
+    n_items = len(off) - 1
+    per_batch = 3
+    bbytes = per_batch * MiB // 2
+    batches = [(k, min(k + per_batch, n_items)) for k in range(0, n_items, per_batch)]
+    dev = torch.from_numpy(data).cuda()
+    pipe = D.NativeWavePipeline(D.nccl_unique_id(), 1, 0, 0, bbytes, per_batch + 1, 1 << 16,
+                                depth=depth)
+    split = len(batches) // 2
+    got = [[], []]
+    try:
+        def take(outs, sid):
+            for wave in outs:
+                for o in wave:
+                    got[sid].extend(o.items())
+        for sid, (lo, hi) in enumerate(((0, split), (split, len(batches)))):
+            if sid:
+                take(pipe.end_stream(), 0)
+            for b in range(lo, hi):
+                k, j = batches[b]
+                take(pipe.submit([(dev[int(off[k]):int(off[j])], off[k:j + 1] - off[k], k)]), sid)
+        take(pipe.flush(), 1)
+        torch.cuda.synchronize()
+    finally:
+        pipe.close()
+    for sid, (lo, hi) in enumerate(((0, split), (split, len(batches)))):
+        k0, k1 = batches[lo][0], batches[hi - 1][1]
+        res = sorted(got[sid], key=lambda r: r[0])
+        want, _ = oracle.dedup_items([data[int(off[k]):int(off[k + 1])] for k in range(k0, k1)],
+                                     first_seq=k0)
+        assert [g[0] for g in res] == [w.seq for w in want]
+        for (seq, cs, dg, dup, fid), w in zip(res, want):
+            assert np.array_equal(cs, w.chunk_start), seq
+            assert np.array_equal(dg, w.digest), seq
+            assert np.array_equal(dup, w.is_dup), seq
+            assert np.array_equal(fid, w.first_id), seq
