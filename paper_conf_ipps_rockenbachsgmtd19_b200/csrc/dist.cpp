@@ -21,6 +21,7 @@
 #include <nccl.h>
 
 #include <cstdint>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -30,7 +31,11 @@
 namespace {
 
 struct DSlot {
+    // ctx: its op-descriptor ring is used only by the first (warm-up) wave and
+    // the graph captures, so the descriptors the graphs copy from are never
+    // reused; ctx2 runs every uncaptured op after that (chunk_meta each wave).
     dedup_ctx* ctx = nullptr;
+    dedup_ctx* ctx2 = nullptr;
     cudaStream_t s = nullptr;
     cudaEvent_t e_local = nullptr, e_done = nullptr;
     uint64_t cap = 0;
@@ -56,7 +61,20 @@ struct DSlot {
     uint32_t n_items = 0;
     uint32_t n_chunks = 0;
     bool busy = false;
+    bool warm = false;  // one uncaptured wave done (lazy allocations inside the ops)
+    // The local rows as two CUDA graphs per batch geometry (bytes, nbytes,
+    // n_items): chunk (A2-A3), then chunk_meta uncaptured (its first_seq
+    // changes every wave), then SHA-1 + local combine + route (A4-A5).
+    struct G {
+        const uint8_t* bytes;
+        uint64_t nbytes;
+        uint32_t n_items;
+        cudaGraphExec_t g1, g2;
+    };
+    std::vector<G> graphs;
 };
+
+constexpr size_t kMaxGraphs = 8;  // per slot
 
 }  // namespace
 
@@ -69,6 +87,7 @@ struct dedup_dist {
     uint32_t depth = 1;
     uint64_t next_wave = 0, done_wave = 0;
     int last_done = -1;  // slot of the last completed wave (results readable)
+    bool use_graphs = true;  // DEDUP_DIST_GRAPHS=0: plain op calls
     // metadata of the last completed wave (its slot is reused right away)
     uint64_t res_first_seq = 0;
     uint32_t res_n_items = 0, res_n_chunks = 0;
@@ -120,6 +139,7 @@ dedup_status slot_alloc(dedup_dist* d, DSlot& sl, const dedup_config& base, uint
     c.table_capacity = 1024;  // the slot's own table is not used
     if (c.sha_lane_bytes == 0) c.sha_lane_bytes = 8192;
     dedup_status st = dedup_init(&c, &sl.ctx);
+    if (st == DEDUP_OK) st = dedup_init(&c, &sl.ctx2);
     if (st != DEDUP_OK) return dfail(d, st, "dedup_init of a wave slot failed");
     const uint32_t G = (uint32_t)d->nranks;
     sl.cap = batch_bytes / 32 + batch_items + 2;
@@ -158,7 +178,12 @@ void slot_free(DSlot& sl) {
     if (sl.e_local) cudaEventDestroy(sl.e_local);
     if (sl.e_done) cudaEventDestroy(sl.e_done);
     if (sl.s) cudaStreamDestroy(sl.s);
+    for (auto& g : sl.graphs) {
+        if (g.g1) cudaGraphExecDestroy(g.g1);
+        if (g.g2) cudaGraphExecDestroy(g.g2);
+    }
     if (sl.ctx) dedup_destroy(sl.ctx);
+    if (sl.ctx2) dedup_destroy(sl.ctx2);
     sl = DSlot{};
 }
 
@@ -271,6 +296,7 @@ dedup_status dedup_dist_create(const dedup_config* cfg, const uint8_t nccl_id[12
     d->rank = rank;
     d->depth = depth;
     d->device = cfg->device;
+    if (const char* e = std::getenv("DEDUP_DIST_GRAPHS")) d->use_graphs = std::atoi(e) != 0;
     auto bail = [&](dedup_status st) {
         dedup_dist_destroy(d);
         return st;
@@ -339,14 +365,53 @@ dedup_status dedup_dist_submit(dedup_dist* d, const uint8_t* d_bytes, uint64_t n
     DCU(cudaMemcpyAsync(sl.item_off, sl.h_off, sizeof(uint64_t) * (n_items + 1),
                         cudaMemcpyHostToDevice, sl.s));
     // rows A2-A5 on the slot's stream
-    DTRY(dedup_op_chunk(sl.ctx, sl.s, d_bytes, nbytes, sl.item_off, n_items, sl.cut, sl.cap,
-                        sl.n));
-    DTRY(dedup_op_chunk_meta(sl.ctx, sl.s, sl.item_off, n_items, sl.cut, sl.n, sl.cap,
-                             first_seq, sl.chunk_start, sl.chunk_id, sl.item_first));
-    DTRY(dedup_op_sha1(sl.ctx, sl.s, d_bytes, nbytes, sl.cut, sl.n, sl.cap, sl.digest));
-    DTRY(dedup_op_local_combine(sl.ctx, sl.s, sl.digest, sl.n, sl.cap, sl.rep));
-    DTRY(dedup_op_route(sl.ctx, sl.s, sl.digest, sl.chunk_id, sl.n, sl.cap, sl.rep, G, sl.send,
-                        sl.send_off, sl.send_pos));
+    auto part1 = [&](dedup_ctx* c) -> dedup_status {
+        return dedup_op_chunk(c, sl.s, d_bytes, nbytes, sl.item_off, n_items, sl.cut, sl.cap,
+                              sl.n);
+    };
+    auto part2 = [&](dedup_ctx* c) -> dedup_status {
+        dedup_status st = dedup_op_sha1(c, sl.s, d_bytes, nbytes, sl.cut, sl.n, sl.cap,
+                                        sl.digest);
+        if (st == DEDUP_OK) st = dedup_op_local_combine(c, sl.s, sl.digest, sl.n, sl.cap, sl.rep);
+        if (st == DEDUP_OK)
+            st = dedup_op_route(c, sl.s, sl.digest, sl.chunk_id, sl.n, sl.cap, sl.rep, G,
+                                sl.send, sl.send_off, sl.send_pos);
+        return st;
+    };
+    auto meta = [&](dedup_ctx* c) -> dedup_status {
+        return dedup_op_chunk_meta(c, sl.s, sl.item_off, n_items, sl.cut, sl.n, sl.cap,
+                                   first_seq, sl.chunk_start, sl.chunk_id, sl.item_first);
+    };
+    DSlot::G* g = nullptr;
+    for (auto& x : sl.graphs)
+        if (x.bytes == d_bytes && x.nbytes == nbytes && x.n_items == n_items) g = &x;
+    if (g == nullptr && sl.warm && d->use_graphs && sl.graphs.size() < kMaxGraphs) {
+        // capture both parts once for this geometry (on ctx)
+        DSlot::G ng{d_bytes, nbytes, n_items, nullptr, nullptr};
+        for (int part = 0; part < 2; ++part) {
+            cudaGraph_t graph = nullptr;
+            DCU(cudaStreamBeginCapture(sl.s, cudaStreamCaptureModeRelaxed));
+            const dedup_status st = part == 0 ? part1(sl.ctx) : part2(sl.ctx);
+            const cudaError_t ce = cudaStreamEndCapture(sl.s, &graph);
+            if (st != DEDUP_OK) return dfail(d, st, dedup_last_error(sl.ctx));
+            if (ce != cudaSuccess) return dfail(d, DEDUP_ECUDA, cudaGetErrorString(ce));
+            DCU(cudaGraphInstantiate(part == 0 ? &ng.g1 : &ng.g2, graph, 0));
+            cudaGraphDestroy(graph);
+        }
+        sl.graphs.push_back(ng);
+        g = &sl.graphs.back();
+    }
+    if (g != nullptr) {
+        DCU(cudaGraphLaunch(g->g1, sl.s));
+        DTRY(meta(sl.ctx2));
+        DCU(cudaGraphLaunch(g->g2, sl.s));
+    } else {
+        dedup_ctx* c = sl.warm ? sl.ctx2 : sl.ctx;  // ctx's ring: warm-up and captures only
+        DTRY(part1(c));
+        DTRY(meta(c));
+        DTRY(part2(c));
+        sl.warm = true;
+    }
     // the per-owner offsets and n to pinned host memory (read at completion)
     DCU(cudaMemcpyAsync(sl.h_send_off, sl.send_off, sizeof(uint32_t) * (G + 1),
                         cudaMemcpyDeviceToHost, sl.s));

@@ -17,7 +17,12 @@ import json
 import os
 
 
-DEPTH = 16  # waves in flight per rank
+# waves in flight per rank and SHA-1 bytes per lane of a wave.  Measured
+# (world 1, 64 MiB waves): depth 16 / 8 KiB 320-365 GB/s; 16 / 32 KiB 277;
+# 40 / 32 KiB 217; 40 / 8 KiB 157; 56 / 32 KiB 54 (more slot streams than
+# hardware queues)
+DEPTH = int(os.environ.get("DEDUP_DIST_DEPTH", "16"))
+SHA_LANE_BYTES = int(os.environ.get("DEDUP_DIST_SHA_LANE", "8192"))
 
 
 def main(args, data, off, B):
@@ -43,7 +48,8 @@ def main(args, data, off, B):
     dist.broadcast(idt, 0)
     pipe = D.NativeWavePipeline(bytes(idt.cpu().numpy()), world, rank, local, wave_bytes,
                                 items_per_batch + 1,
-                                max(1 << 16, len(data) // 2048 // world), depth=DEPTH)
+                                max(1 << 16, len(data) // 2048 // world), depth=DEPTH,
+                                sha_lane_bytes=SHA_LANE_BYTES)
     ddata = torch.from_numpy(data).to(dev)
     # A table reset completes every wave in flight first (end_stream), so a
     # dedup stream spans at least 4 pipeline depths of waves (the C2 batches

@@ -218,8 +218,10 @@ def test_wave_pipeline_matches_oracle(G, depth):
 @pytest.mark.parametrize("depth", [1, 3])
 def test_native_wave_pipeline_world1(depth):
     """The C++ wave pipeline (csrc/dist.cpp) through NCCL with one rank: the
-    exchange sends every record to itself; bit-exact vs the oracle across an
-    end_stream."""
+    exchange sends every record to itself.  Three dedup streams: the first
+    half of the batches, the second half, then the first half again from the
+    same device buffers (the local phase replays its captured CUDA graphs);
+    bit-exact vs the oracle each time."""
     assert torch.cuda.is_available()
     from paper_conf_ipps_rockenbachsgmtd19_b200 import dist as D
     data = U.stream(10 * MiB, seed=71 + depth, dup_frac=0.6)
@@ -229,30 +231,32 @@ def test_native_wave_pipeline_world1(depth):
     bbytes = per_batch * MiB // 2
     batches = [(k, min(k + per_batch, n_items)) for k in range(0, n_items, per_batch)]
     dev = torch.from_numpy(data).cuda()
+    views = [dev[int(off[k]):int(off[j])] for k, j in batches]
     pipe = D.NativeWavePipeline(D.nccl_unique_id(), 1, 0, 0, bbytes, per_batch + 1, 1 << 16,
                                 depth=depth)
     split = len(batches) // 2
-    got = [[], []]
+    plan = [(0, split, 0), (split, len(batches), 0), (0, split, n_items)]  # (lo, hi, seq base)
+    got = [[] for _ in plan]
     try:
         def take(outs, sid):
             for wave in outs:
                 for o in wave:
                     got[sid].extend(o.items())
-        for sid, (lo, hi) in enumerate(((0, split), (split, len(batches)))):
+        for sid, (lo, hi, base) in enumerate(plan):
             if sid:
-                take(pipe.end_stream(), 0)
+                take(pipe.end_stream(), sid - 1)
             for b in range(lo, hi):
                 k, j = batches[b]
-                take(pipe.submit([(dev[int(off[k]):int(off[j])], off[k:j + 1] - off[k], k)]), sid)
-        take(pipe.flush(), 1)
+                take(pipe.submit([(views[b], off[k:j + 1] - off[k], base + k)]), sid)
+        take(pipe.flush(), len(plan) - 1)
         torch.cuda.synchronize()
     finally:
         pipe.close()
-    for sid, (lo, hi) in enumerate(((0, split), (split, len(batches)))):
+    for sid, (lo, hi, base) in enumerate(plan):
         k0, k1 = batches[lo][0], batches[hi - 1][1]
         res = sorted(got[sid], key=lambda r: r[0])
         want, _ = oracle.dedup_items([data[int(off[k]):int(off[k + 1])] for k in range(k0, k1)],
-                                     first_seq=k0)
+                                     first_seq=base + k0)
         assert [g[0] for g in res] == [w.seq for w in want]
         for (seq, cs, dg, dup, fid), w in zip(res, want):
             assert np.array_equal(cs, w.chunk_start), seq
