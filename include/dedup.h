@@ -385,8 +385,11 @@ dedup_status dedup_dist_submit(dedup_dist* d, const uint8_t* d_bytes, uint64_t n
                                void* producer, uint32_t* completed);
 /* Completes the oldest wave in flight if any (*completed = 1). */
 dedup_status dedup_dist_flush(dedup_dist* d, uint32_t* completed);
-/* New dedup stream (clears this rank's table shard); no wave may be in
- * flight (flush first), else DEDUP_EAGAIN. */
+/* New dedup stream (clears this rank's table shard).  With waves in flight
+ * the reset is deferred: it is issued on the owner stream right before the
+ * owner work of the next wave submitted, so the waves in flight still see
+ * the old stream's table and the pipeline is not drained (every rank must
+ * call it at the same wave). */
 dedup_status dedup_dist_end_stream(dedup_dist* d);
 
 typedef struct {

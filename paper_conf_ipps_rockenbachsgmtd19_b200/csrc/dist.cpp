@@ -4,10 +4,12 @@
 // Waves: in wave w every rank submits one batch.  Its local rows run on one
 // of `depth` slots (each a ctx of its own for the op workspace, a stream and
 // device buffers): A2-A4 chunk + SHA-1, A5 local combine + route by digest
-// owner.  When `depth` waves are in flight, the oldest completes on the
-// owner stream: per-owner record counts (NCCL grouped send/recv of one u32
-// per peer), the host reads them (the only synchronisation: it sizes the
-// payload), the 32-byte records go to their owners (A6), the owner inserts
+// owner.  Right behind its local rows each wave exchanges its per-owner
+// record counts on the owner stream (NCCL grouped send/recv of two u32 per
+// peer) into pinned memory.  When `depth` waves are in flight, the oldest
+// completes on the owner stream: the host reads its counts (the only
+// synchronisation: it sizes the payload; the event was recorded `depth`
+// waves ago, so it does not wait for newer owner work), the 32-byte records go to their owners (A6), the owner inserts
 // then looks up all of them in its table shard (A7, dedup_op_owner), the
 // first-occurrence ids go back (A8), are scattered to chunk order, and the
 // results are copied to pinned host memory.  Owner work stays in wave order
@@ -23,6 +25,7 @@
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
+#include <deque>
 #include <string>
 #include <vector>
 
@@ -38,6 +41,7 @@ struct DSlot {
     dedup_ctx* ctx2 = nullptr;
     cudaStream_t s = nullptr;
     cudaEvent_t e_local = nullptr, e_done = nullptr;
+    cudaEvent_t e_cnt = nullptr;  // the wave's counts exchange landed in h_cnt
     uint64_t cap = 0;
     uint32_t max_items = 0;
     // device
@@ -80,14 +84,21 @@ constexpr size_t kMaxGraphs = 8;  // per slot
 
 struct dedup_dist {
     ncclComm_t comm = nullptr;
+    ncclComm_t ccomm = nullptr;  // counts exchange (split of comm), on stream cs
+    cudaStream_t cs = nullptr;
     int nranks = 1, rank = 0, device = 0;
     dedup_ctx* owner = nullptr;
     cudaStream_t os = nullptr;  // owner stream
     std::vector<DSlot> slots;
+    // table resets deferred by dedup_dist_end_stream with waves in flight:
+    // each is issued on the owner stream right before the owner work of
+    // the wave it names (the first wave of the next stream)
+    std::deque<uint64_t> resets;
     uint32_t depth = 1;
     uint64_t next_wave = 0, done_wave = 0;
     int last_done = -1;  // slot of the last completed wave (results readable)
     bool use_graphs = true;  // DEDUP_DIST_GRAPHS=0: plain op calls
+    bool early_counts = true;  // DEDUP_DIST_EARLY_COUNTS=0: counts exchanged at completion
     // metadata of the last completed wave (its slot is reused right away)
     uint64_t res_first_seq = 0;
     uint32_t res_n_items = 0, res_n_chunks = 0;
@@ -147,6 +158,7 @@ dedup_status slot_alloc(dedup_dist* d, DSlot& sl, const dedup_config& base, uint
     DCU(cudaStreamCreateWithFlags(&sl.s, cudaStreamNonBlocking));
     DCU(cudaEventCreateWithFlags(&sl.e_local, cudaEventDisableTiming));
     DCU(cudaEventCreateWithFlags(&sl.e_done, cudaEventDisableTiming));
+    DCU(cudaEventCreateWithFlags(&sl.e_cnt, cudaEventDisableTiming));
     const uint64_t cap = sl.cap;
     if (dmalloc(d, &sl.cut, cap) || dmalloc(d, &sl.n, 1) || dmalloc(d, &sl.chunk_start, cap) ||
         dmalloc(d, &sl.item_first, batch_items + 1) || dmalloc(d, &sl.send_off, G + 1) ||
@@ -177,6 +189,7 @@ void slot_free(DSlot& sl) {
         if (p) cudaFreeHost(p);
     if (sl.e_local) cudaEventDestroy(sl.e_local);
     if (sl.e_done) cudaEventDestroy(sl.e_done);
+    if (sl.e_cnt) cudaEventDestroy(sl.e_cnt);
     if (sl.s) cudaStreamDestroy(sl.s);
     for (auto& g : sl.graphs) {
         if (g.g1) cudaGraphExecDestroy(g.g1);
@@ -187,24 +200,50 @@ void slot_free(DSlot& sl) {
     sl = DSlot{};
 }
 
+// Row A6's first half, issued at submit time on the owner stream right after
+// the wave's local rows: per-owner record counts -> every peer (peer p gets
+// this rank's (send_off[p], send_off[p + 1]) and returns its own pair), then
+// to pinned host memory.  complete_oldest waits only for this event, so the
+// host never blocks on the owner stream's newest work (the previous wave's
+// exchange, insert and D2H).  Every rank issues the same NCCL sequence.
+dedup_status exchange_counts(dedup_dist* d, DSlot& sl) {
+    const uint32_t G = (uint32_t)d->nranks;
+    // early: own communicator and stream, so the owner stream (and through
+    // e_done the next wave's slot) never waits for the newest local rows
+    cudaStream_t st = d->early_counts ? d->cs : d->os;
+    ncclComm_t cm = d->early_counts ? d->ccomm : d->comm;
+    DCU(cudaStreamWaitEvent(st, sl.e_local, 0));
+    DNC(ncclGroupStart());
+    for (uint32_t p = 0; p < G; ++p) {
+        DNC(ncclSend(sl.send_off + p, 2, ncclUint32, (int)p, cm, st));
+        DNC(ncclRecv(sl.cnt_recv + 2 * p, 2, ncclUint32, (int)p, cm, st));
+    }
+    DNC(ncclGroupEnd());
+    DCU(cudaMemcpyAsync(sl.h_cnt, sl.cnt_recv, sizeof(uint32_t) * 2 * G,
+                        cudaMemcpyDeviceToHost, st));
+    DCU(cudaEventRecord(sl.e_cnt, st));
+    return DEDUP_OK;
+}
+
 // Completes the oldest wave in flight (rows A6-A8 + D2H on the owner stream).
 dedup_status complete_oldest(dedup_dist* d) {
     const int i = (int)(d->done_wave % d->depth);
     DSlot& sl = d->slots[i];
     const uint32_t G = (uint32_t)d->nranks;
     cudaStream_t os = d->os;
-    DCU(cudaStreamWaitEvent(os, sl.e_local, 0));
-    // per-owner record counts -> every peer: peer p gets this rank's
-    // (send_off[p], send_off[p + 1]) and returns its own pair for us
-    DNC(ncclGroupStart());
-    for (uint32_t p = 0; p < G; ++p) {
-        DNC(ncclSend(sl.send_off + p, 2, ncclUint32, (int)p, d->comm, os));
-        DNC(ncclRecv(sl.cnt_recv + 2 * p, 2, ncclUint32, (int)p, d->comm, os));
+    // the counts were exchanged when the wave was submitted (exchange_counts);
+    // waiting for them does not wait for the owner stream's newer work
+    while (!d->resets.empty() && d->resets.front() <= d->done_wave) {
+        const dedup_status st = dedup_op_table_reset(d->owner, os);
+        if (st != DEDUP_OK) return dfail(d, st, dedup_last_error(d->owner));
+        d->resets.pop_front();
     }
-    DNC(ncclGroupEnd());
-    DCU(cudaMemcpyAsync(sl.h_cnt, sl.cnt_recv, sizeof(uint32_t) * 2 * G,
-                        cudaMemcpyDeviceToHost, os));
-    DCU(cudaStreamSynchronize(os));  // sizes of the payload (host); local rows done too
+    if (!d->early_counts) {
+        const dedup_status st = exchange_counts(d, sl);
+        if (st != DEDUP_OK) return st;
+    }
+    DCU(cudaEventSynchronize(sl.e_cnt));  // sizes of the payload (host); local rows done too
+    DCU(cudaStreamWaitEvent(os, sl.e_cnt, 0));  // the records (send) come from the local rows
     const uint32_t* soff = sl.h_send_off;
     sl.n_chunks = sl.h_send_off[G + 1];
     uint64_t roff = 0;
@@ -297,6 +336,7 @@ dedup_status dedup_dist_create(const dedup_config* cfg, const uint8_t nccl_id[12
     d->depth = depth;
     d->device = cfg->device;
     if (const char* e = std::getenv("DEDUP_DIST_GRAPHS")) d->use_graphs = std::atoi(e) != 0;
+    if (const char* e = std::getenv("DEDUP_DIST_EARLY_COUNTS")) d->early_counts = std::atoi(e) != 0;
     auto bail = [&](dedup_status st) {
         dedup_dist_destroy(d);
         return st;
@@ -315,6 +355,12 @@ dedup_status dedup_dist_create(const dedup_config* cfg, const uint8_t nccl_id[12
     ncclUniqueId id;
     std::memcpy(&id, nccl_id, 128);
     if (ncclCommInitRank(&d->comm, nranks, id, rank) != ncclSuccess) return bail(DEDUP_ECUDA);
+    if (d->early_counts) {
+        if (cudaStreamCreateWithFlags(&d->cs, cudaStreamNonBlocking) != cudaSuccess)
+            return bail(DEDUP_ECUDA);
+        if (ncclCommSplit(d->comm, 0, rank, &d->ccomm, nullptr) != ncclSuccess)
+            return bail(DEDUP_ECUDA);
+    }
     d->slots.resize(depth);
     for (auto& sl : d->slots)
         if (slot_alloc(d, sl, *cfg, batch_bytes, batch_items) != DEDUP_OK)
@@ -327,7 +373,9 @@ void dedup_dist_destroy(dedup_dist* d) {
     if (d == nullptr) return;
     cudaSetDevice(d->device);
     for (auto& sl : d->slots) slot_free(sl);
+    if (d->ccomm) ncclCommDestroy(d->ccomm);
     if (d->comm) ncclCommDestroy(d->comm);
+    if (d->cs) cudaStreamDestroy(d->cs);
     if (d->os) cudaStreamDestroy(d->os);
     if (d->owner) dedup_destroy(d->owner);
     delete d;
@@ -418,6 +466,10 @@ dedup_status dedup_dist_submit(dedup_dist* d, const uint8_t* d_bytes, uint64_t n
     DCU(cudaMemcpyAsync(sl.h_send_off + G + 1, sl.n, sizeof(uint32_t), cudaMemcpyDeviceToHost,
                         sl.s));
     DCU(cudaEventRecord(sl.e_local, sl.s));
+    if (d->early_counts) {
+        const dedup_status st = exchange_counts(d, sl);
+        if (st != DEDUP_OK) return st;
+    }
     sl.busy = true;
     ++d->next_wave;
     return DEDUP_OK;
@@ -435,9 +487,15 @@ dedup_status dedup_dist_flush(dedup_dist* d, uint32_t* completed) {
 
 dedup_status dedup_dist_end_stream(dedup_dist* d) {
     if (d == nullptr) return DEDUP_EINVAL;
-    if (d->done_wave != d->next_wave)
-        return dfail(d, DEDUP_EAGAIN, "complete every wave in flight first (dedup_dist_flush)");
+    if (d->done_wave != d->next_wave) {
+        // waves of this stream still in flight: their owner work is issued in
+        // wave order on the owner stream, so the reset goes in right before
+        // the next stream's first wave (no drain of the pipeline)
+        d->resets.push_back(d->next_wave);
+        return DEDUP_OK;
+    }
     if (cudaSetDevice(d->device) != cudaSuccess) return DEDUP_ECUDA;
+    d->resets.clear();  // every deferred reset is subsumed by this one
     const dedup_status st = dedup_op_table_reset(d->owner, d->os);
     return st == DEDUP_OK ? st : dfail(d, st, dedup_last_error(d->owner));
 }

@@ -567,8 +567,11 @@ class NativeWavePipeline:
                 return out
             out.append(self._result() if collect else self._counts())
 
-    def end_stream(self, collect: bool = True):
-        out = self.flush(collect)
+    def end_stream(self, collect: bool = True, drain: bool = True):
+        """New dedup stream.  drain=False keeps the waves in flight (their
+        results come out of later submit/flush calls); the table reset is
+        then issued in wave order before the next stream's first wave."""
+        out = self.flush(collect) if drain else []
         self._check(self.N.lib().dedup_dist_end_stream(self._d))
         return out
 

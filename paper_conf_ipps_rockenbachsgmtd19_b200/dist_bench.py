@@ -18,11 +18,14 @@ import os
 
 
 # waves in flight per rank and SHA-1 bytes per lane of a wave.  Measured
-# (world 1, 64 MiB waves): depth 16 / 8 KiB 320-365 GB/s; 16 / 32 KiB 277;
+# (world 1, 64 MiB waves): depth 16 / 8 KiB 320-365 GB/s (405-433 with early counts); 16 / 32 KiB 277;
 # 40 / 32 KiB 217; 40 / 8 KiB 157; 56 / 32 KiB 54 (more slot streams than
 # hardware queues)
 DEPTH = int(os.environ.get("DEDUP_DIST_DEPTH", "16"))
 SHA_LANE_BYTES = int(os.environ.get("DEDUP_DIST_SHA_LANE", "8192"))
+# end_stream without draining the waves in flight (the table reset goes in
+# before the next stream's first wave on the owner stream)
+DRAIN = os.environ.get("DEDUP_DIST_DRAIN", "0") != "0"
 
 
 def main(args, data, off, B):
@@ -65,7 +68,7 @@ def main(args, data, off, B):
 
     def wave(w, timed):
         if w % waves_per_stream == 0 and w > 0:
-            take(pipe.end_stream(collect=False), timed)
+            take(pipe.end_stream(collect=False, drain=DRAIN), timed)
         b = ((w % waves_per_stream) * world + rank) % nb
         k, j = plan[b]
         seq = (w * world + rank) * items_per_batch

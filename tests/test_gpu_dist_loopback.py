@@ -215,14 +215,20 @@ def test_wave_pipeline_matches_oracle(G, depth):
             assert np.array_equal(fid, w.first_id), seq
 
 
+@pytest.mark.parametrize("early", ["0", "1"])
+@pytest.mark.parametrize("drain", [True, False])
 @pytest.mark.parametrize("depth", [1, 3])
-def test_native_wave_pipeline_world1(depth):
+def test_native_wave_pipeline_world1(depth, drain, early, monkeypatch):
     """The C++ wave pipeline (csrc/dist.cpp) through NCCL with one rank: the
     exchange sends every record to itself.  Three dedup streams: the first
     half of the batches, the second half, then the first half again from the
     same device buffers (the local phase replays its captured CUDA graphs);
-    bit-exact vs the oracle each time."""
+    bit-exact vs the oracle each time.  drain=False: end_stream with waves in
+    flight (the table reset deferred to the next stream's first wave);
+    early: counts exchanged right behind the local rows on their own
+    communicator (DEDUP_DIST_EARLY_COUNTS)."""
     assert torch.cuda.is_available()
+    monkeypatch.setenv("DEDUP_DIST_EARLY_COUNTS", early)
     from paper_conf_ipps_rockenbachsgmtd19_b200 import dist as D
     data = U.stream(10 * MiB, seed=71 + depth, dup_frac=0.6)
     off = synthgen.split_items(data, MiB // 2)
@@ -238,13 +244,17 @@ def test_native_wave_pipeline_world1(depth):
     plan = [(0, split, 0), (split, len(batches), 0), (0, split, n_items)]  # (lo, hi, seq base)
     got = [[] for _ in plan]
     try:
-        def take(outs, sid):
+        def sid_of(seq):  # the three streams' seq ranges are disjoint
+            return 2 if seq >= n_items else (0 if seq < batches[split][0] else 1)
+
+        def take(outs, _sid):
             for wave in outs:
                 for o in wave:
-                    got[sid].extend(o.items())
+                    for r in o.items():
+                        got[sid_of(r[0])].append(r)
         for sid, (lo, hi, base) in enumerate(plan):
             if sid:
-                take(pipe.end_stream(), sid - 1)
+                take(pipe.end_stream(drain=drain), sid - 1)
             for b in range(lo, hi):
                 k, j = batches[b]
                 take(pipe.submit([(views[b], off[k:j + 1] - off[k], base + k)]), sid)
