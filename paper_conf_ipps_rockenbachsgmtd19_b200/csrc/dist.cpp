@@ -22,7 +22,9 @@
 #include <cuda_runtime.h>
 #include <nccl.h>
 
+#include <chrono>
 #include <cstdint>
+#include <cstdio>
 #include <cstdlib>
 #include <cstring>
 #include <deque>
@@ -104,6 +106,11 @@ struct dedup_dist {
     uint32_t res_n_items = 0, res_n_chunks = 0;
     std::vector<uint64_t> res_item_off;
     std::string err = "no error";
+    // DEDUP_DIST_HOST_TIMING=1: host seconds spent in submit (issue) and in
+    // the completion's wait for the counts, printed to stderr at destroy
+    bool host_timing = false;
+    double t_submit = 0, t_wait = 0;
+    uint64_t n_submit = 0;
 };
 
 namespace {
@@ -242,7 +249,10 @@ dedup_status complete_oldest(dedup_dist* d) {
         const dedup_status st = exchange_counts(d, sl);
         if (st != DEDUP_OK) return st;
     }
+    const auto tw0 = std::chrono::steady_clock::now();
     DCU(cudaEventSynchronize(sl.e_cnt));  // sizes of the payload (host); local rows done too
+    if (d->host_timing)
+        d->t_wait += std::chrono::duration<double>(std::chrono::steady_clock::now() - tw0).count();
     DCU(cudaStreamWaitEvent(os, sl.e_cnt, 0));  // the records (send) come from the local rows
     const uint32_t* soff = sl.h_send_off;
     sl.n_chunks = sl.h_send_off[G + 1];
@@ -337,6 +347,7 @@ dedup_status dedup_dist_create(const dedup_config* cfg, const uint8_t nccl_id[12
     d->device = cfg->device;
     if (const char* e = std::getenv("DEDUP_DIST_GRAPHS")) d->use_graphs = std::atoi(e) != 0;
     if (const char* e = std::getenv("DEDUP_DIST_EARLY_COUNTS")) d->early_counts = std::atoi(e) != 0;
+    if (const char* e = std::getenv("DEDUP_DIST_HOST_TIMING")) d->host_timing = std::atoi(e) != 0;
     auto bail = [&](dedup_status st) {
         dedup_dist_destroy(d);
         return st;
@@ -371,6 +382,12 @@ dedup_status dedup_dist_create(const dedup_config* cfg, const uint8_t nccl_id[12
 
 void dedup_dist_destroy(dedup_dist* d) {
     if (d == nullptr) return;
+    if (d->host_timing && d->n_submit)
+        std::fprintf(stderr,
+                     "dedup_dist host timing: %llu submits, %.1f us/submit total, of which "
+                     "%.1f us waiting for the oldest wave's counts\n",
+                     (unsigned long long)d->n_submit, 1e6 * d->t_submit / d->n_submit,
+                     1e6 * d->t_wait / d->n_submit);
     cudaSetDevice(d->device);
     for (auto& sl : d->slots) slot_free(sl);
     if (d->ccomm) ncclCommDestroy(d->ccomm);
@@ -390,6 +407,16 @@ dedup_status dedup_dist_submit(dedup_dist* d, const uint8_t* d_bytes, uint64_t n
                                void* producer, uint32_t* completed) {
     if (d == nullptr || item_off == nullptr || completed == nullptr) return DEDUP_EINVAL;
     *completed = 0;
+    struct Timer {
+        dedup_dist* d;
+        std::chrono::steady_clock::time_point t0 = std::chrono::steady_clock::now();
+        ~Timer() {
+            if (!d->host_timing) return;
+            d->t_submit +=
+                std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+            ++d->n_submit;
+        }
+    } timer{d};
     if (cudaSetDevice(d->device) != cudaSuccess) return DEDUP_ECUDA;
     if (d->next_wave - d->done_wave >= d->depth) {
         const dedup_status st = complete_oldest(d);
