@@ -109,7 +109,7 @@ struct dedup_dist {
     // DEDUP_DIST_HOST_TIMING=1: host seconds spent in submit (issue) and in
     // the completion's wait for the counts, printed to stderr at destroy
     bool host_timing = false;
-    double t_submit = 0, t_wait = 0;
+    double t_submit = 0, t_wait = 0, t_complete = 0, t_local = 0;
     uint64_t n_submit = 0;
 };
 
@@ -385,9 +385,11 @@ void dedup_dist_destroy(dedup_dist* d) {
     if (d->host_timing && d->n_submit)
         std::fprintf(stderr,
                      "dedup_dist host timing: %llu submits, %.1f us/submit total, of which "
-                     "%.1f us waiting for the oldest wave's counts\n",
+                     "%.1f us completing the oldest wave (%.1f us waiting for its counts), "
+                     "%.1f us issuing the local rows\n",
                      (unsigned long long)d->n_submit, 1e6 * d->t_submit / d->n_submit,
-                     1e6 * d->t_wait / d->n_submit);
+                     1e6 * d->t_complete / d->n_submit, 1e6 * d->t_wait / d->n_submit,
+                     1e6 * d->t_local / d->n_submit);
     cudaSetDevice(d->device);
     for (auto& sl : d->slots) slot_free(sl);
     if (d->ccomm) ncclCommDestroy(d->ccomm);
@@ -419,7 +421,11 @@ dedup_status dedup_dist_submit(dedup_dist* d, const uint8_t* d_bytes, uint64_t n
     } timer{d};
     if (cudaSetDevice(d->device) != cudaSuccess) return DEDUP_ECUDA;
     if (d->next_wave - d->done_wave >= d->depth) {
+        const auto tc0 = std::chrono::steady_clock::now();
         const dedup_status st = complete_oldest(d);
+        if (d->host_timing)
+            d->t_complete +=
+                std::chrono::duration<double>(std::chrono::steady_clock::now() - tc0).count();
         if (st != DEDUP_OK) return st;
         *completed = 1;
     }
@@ -457,6 +463,7 @@ dedup_status dedup_dist_submit(dedup_dist* d, const uint8_t* d_bytes, uint64_t n
         return dedup_op_chunk_meta(c, sl.s, sl.item_off, n_items, sl.cut, sl.n, sl.cap,
                                    first_seq, sl.chunk_start, sl.chunk_id, sl.item_first);
     };
+    const auto tl0 = std::chrono::steady_clock::now();
     DSlot::G* g = nullptr;
     for (auto& x : sl.graphs)
         if (x.bytes == d_bytes && x.nbytes == nbytes && x.n_items == n_items) g = &x;
@@ -487,6 +494,8 @@ dedup_status dedup_dist_submit(dedup_dist* d, const uint8_t* d_bytes, uint64_t n
         DTRY(part2(c));
         sl.warm = true;
     }
+    if (d->host_timing)
+        d->t_local += std::chrono::duration<double>(std::chrono::steady_clock::now() - tl0).count();
     // the per-owner offsets and n to pinned host memory (read at completion)
     DCU(cudaMemcpyAsync(sl.h_send_off, sl.send_off, sizeof(uint32_t) * (G + 1),
                         cudaMemcpyDeviceToHost, sl.s));
