@@ -355,8 +355,12 @@ int64_t dedup_archive_decode(dedup_archive_decoder* d, const uint8_t* in, uint64
 /* One process (and one dedup_dist) per GPU.  In wave w every rank submits
  * one batch; its local rows (chunk, SHA-1, local combine, route by digest
  * owner) run on one of `depth` slots; when `depth` waves are in flight the
- * oldest completes: per-owner counts and 32-byte records are exchanged with
- * grouped ncclSend/ncclRecv, the owner inserts + looks up its shard (row
+ * oldest completes: the 32-byte records are exchanged with grouped
+ * ncclSend/ncclRecv (their per-owner counts were exchanged right behind the
+ * wave's local rows, on a communicator split from the first, so the host
+ * waits only for those; DEDUP_DIST_EARLY_COUNTS=0 exchanges them at
+ * completion on the first one and must then be set alike on every rank,
+ * as the split is collective), the owner inserts + looks up its shard (row
  * A7), the first ids come back (row A8) and the results are copied to
  * pinned host memory.  Every rank must make the same sequence of submit /
  * flush / end_stream calls (NCCL matches them in order). */
