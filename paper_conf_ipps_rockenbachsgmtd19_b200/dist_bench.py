@@ -18,11 +18,12 @@ import os
 
 
 # waves in flight per rank and SHA-1 bytes per lane of a wave.  Measured
-# (world 1, 64 MiB waves): depth 16 / 8 KiB 320-365 GB/s (570 with early counts, graphs primed); 16 / 32 KiB 277;
-# 40 / 32 KiB 217; 40 / 8 KiB 157; 56 / 32 KiB 54 (more slot streams than
-# hardware queues)
-DEPTH = int(os.environ.get("DEDUP_DIST_DEPTH", "16"))
-SHA_LANE_BYTES = int(os.environ.get("DEDUP_DIST_SHA_LANE", "8192"))
+# (world 1, 64 MiB waves, early counts, graphs primed;
+# profiles/r01_dist_depth_lane_sweep.txt): depth 24 / 16 KiB 632-643 GB/s;
+# 24 / 32 KiB 606-632; 32 / 8 KiB 578; 24 / 8 KiB 578; 16 / 16 KiB 593-595;
+# 16 / 8 KiB 570; 16 / 32 KiB 501-503; 12 / 8 KiB 524; 8 / 8 KiB 400
+DEPTH = int(os.environ.get("DEDUP_DIST_DEPTH", "24"))
+SHA_LANE_BYTES = int(os.environ.get("DEDUP_DIST_SHA_LANE", "16384"))
 # end_stream without draining the waves in flight (the table reset goes in
 # before the next stream's first wave on the owner stream)
 DRAIN = os.environ.get("DEDUP_DIST_DRAIN", "0") != "0"
@@ -79,7 +80,7 @@ def main(args, data, off, B):
     # waves_per_stream waves visits every (slot, batch geometry) pair the
     # timed waves use (slot = w % DEPTH, batch = (w * N + rank) % nb; all of
     # them whenever lcm(DEPTH, nb) <= waves_per_stream, e.g. C2's 3 batches
-    # at depth 16: 48 <= 64), so each slot's
+    # at depth 24: 24 <= 96), so each slot's
     # local-row CUDA graphs are captured here, not inside the timed region;
     # then a fresh table.
     for w in range(waves_per_stream):
