@@ -273,3 +273,50 @@ def test_native_wave_pipeline_world1(depth, drain, early, monkeypatch):
             assert np.array_equal(dg, w.digest), seq
             assert np.array_equal(dup, w.is_dup), seq
             assert np.array_equal(fid, w.first_id), seq
+
+
+@pytest.mark.parametrize("depth", [2, 4])
+def test_native_wave_pipeline_deferred_resets(depth):
+    """end_stream twice in a row with waves in flight (an empty dedup stream
+    between two), then a stream that repeats the first one's data: every
+    deferred reset lands before the right wave, so the repeat is all-new
+    again (bit-exact vs the oracle per stream)."""
+    assert torch.cuda.is_available()
+    from paper_conf_ipps_rockenbachsgmtd19_b200 import dist as D
+    data = U.stream(6 * MiB, seed=97 + depth, dup_frac=0.5)
+    off = synthgen.split_items(data, MiB // 2)
+    n_items = len(off) - 1
+    per_batch = 2
+    bbytes = per_batch * MiB // 2
+    batches = [(k, min(k + per_batch, n_items)) for k in range(0, n_items, per_batch)]
+    dev = torch.from_numpy(data).cuda()
+    views = [dev[int(off[k]):int(off[j])] for k, j in batches]
+    pipe = D.NativeWavePipeline(D.nccl_unique_id(), 1, 0, 0, bbytes, per_batch + 1, 1 << 16,
+                                depth=depth)
+    got = {0: [], 1: []}
+    try:
+        def take(outs):
+            for wave in outs:
+                for o in wave:
+                    for r in o.items():
+                        got[0 if r[0] < n_items else 1].append(r)
+        for b, (k, j) in enumerate(batches):
+            take(pipe.submit([(views[b], off[k:j + 1] - off[k], k)]))
+        take(pipe.end_stream(drain=False))
+        take(pipe.end_stream(drain=False))  # an empty stream
+        for b, (k, j) in enumerate(batches):
+            take(pipe.submit([(views[b], off[k:j + 1] - off[k], n_items + k)]))
+        take(pipe.flush())
+        torch.cuda.synchronize()
+    finally:
+        pipe.close()
+    for sid, base in ((0, 0), (1, n_items)):
+        res = sorted(got[sid], key=lambda r: r[0])
+        want, _ = oracle.dedup_items([data[int(off[k]):int(off[k + 1])] for k in range(n_items)],
+                                     first_seq=base)
+        assert [g[0] for g in res] == [w.seq for w in want]
+        for (seq, cs, dg, dup, fid), w in zip(res, want):
+            assert np.array_equal(cs, w.chunk_start), seq
+            assert np.array_equal(dg, w.digest), seq
+            assert np.array_equal(dup, w.is_dup), seq
+            assert np.array_equal(fid, w.first_id), seq
