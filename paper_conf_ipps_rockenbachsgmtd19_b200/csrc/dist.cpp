@@ -44,6 +44,7 @@ struct DSlot {
     cudaStream_t s = nullptr;
     cudaEvent_t e_local = nullptr, e_done = nullptr;
     cudaEvent_t e_cnt = nullptr;  // the wave's counts exchange landed in h_cnt
+    cudaEvent_t e_prod = nullptr;  // the producer stream's bytes are ready
     uint64_t cap = 0;
     uint32_t max_items = 0;
     // device
@@ -166,6 +167,7 @@ dedup_status slot_alloc(dedup_dist* d, DSlot& sl, const dedup_config& base, uint
     DCU(cudaEventCreateWithFlags(&sl.e_local, cudaEventDisableTiming));
     DCU(cudaEventCreateWithFlags(&sl.e_done, cudaEventDisableTiming));
     DCU(cudaEventCreateWithFlags(&sl.e_cnt, cudaEventDisableTiming));
+    DCU(cudaEventCreateWithFlags(&sl.e_prod, cudaEventDisableTiming));
     const uint64_t cap = sl.cap;
     if (dmalloc(d, &sl.cut, cap) || dmalloc(d, &sl.n, 1) || dmalloc(d, &sl.chunk_start, cap) ||
         dmalloc(d, &sl.item_first, batch_items + 1) || dmalloc(d, &sl.send_off, G + 1) ||
@@ -197,6 +199,7 @@ void slot_free(DSlot& sl) {
     if (sl.e_local) cudaEventDestroy(sl.e_local);
     if (sl.e_done) cudaEventDestroy(sl.e_done);
     if (sl.e_cnt) cudaEventDestroy(sl.e_cnt);
+    if (sl.e_prod) cudaEventDestroy(sl.e_prod);
     if (sl.s) cudaStreamDestroy(sl.s);
     for (auto& g : sl.graphs) {
         if (g.g1) cudaGraphExecDestroy(g.g1);
@@ -438,11 +441,9 @@ dedup_status dedup_dist_submit(dedup_dist* d, const uint8_t* d_bytes, uint64_t n
     sl.first_seq = first_seq;
     sl.n_items = n_items;
     std::memcpy(sl.h_off, item_off, sizeof(uint64_t) * (n_items + 1));
-    cudaEvent_t ev = nullptr;
-    DCU(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
-    DCU(cudaEventRecord(ev, static_cast<cudaStream_t>(producer)));
-    DCU(cudaStreamWaitEvent(sl.s, ev, 0));
-    cudaEventDestroy(ev);
+    // (the wait takes the event's state now, so the slot's event is reusable)
+    DCU(cudaEventRecord(sl.e_prod, static_cast<cudaStream_t>(producer)));
+    DCU(cudaStreamWaitEvent(sl.s, sl.e_prod, 0));
     DCU(cudaMemcpyAsync(sl.item_off, sl.h_off, sizeof(uint64_t) * (n_items + 1),
                         cudaMemcpyHostToDevice, sl.s));
     // rows A2-A5 on the slot's stream
