@@ -48,7 +48,8 @@ def build_oracle(force: bool = False) -> str:
             os.path.getmtime(_LIB) < os.path.getmtime(s) for s in _SRCS):
         tmp = _LIB + f".tmp{os.getpid()}"
         subprocess.check_call(
-            ["g++", "-O2", "-std=c++17", "-ffp-contract=off", "-shared", "-fPIC", "-o", tmp,
+            ["g++", "-O2", "-std=c++17", "-ffp-contract=off", "-shared", "-fPIC", "-pthread",
+             "-o", tmp,
              *_SRCS])
         os.replace(tmp, _LIB)
     return _LIB
@@ -85,6 +86,14 @@ def lib():
                                       u32p, u8p, u8p, u64p, ctypes.c_uint64]
         L.oracle_ctx_item.restype = ctypes.c_uint64
         L.oracle_ctx_counts.argtypes = [ctypes.c_void_p, u64p]
+        L.oracle_ctx_items_parallel.argtypes = [ctypes.c_void_p, ctypes.c_uint64, u8p, u64p,
+                                                ctypes.c_uint64, ctypes.c_uint32]
+        L.oracle_ctx_items_parallel.restype = ctypes.c_void_p
+        L.oracle_batch_chunks.argtypes = [ctypes.c_void_p]
+        L.oracle_batch_chunks.restype = ctypes.c_uint64
+        L.oracle_batch_times.argtypes = [ctypes.c_void_p, ctypes.POINTER(ctypes.c_double)]
+        L.oracle_batch_fetch.argtypes = [ctypes.c_void_p, u64p, u32p, u8p, u8p, u64p]
+        L.oracle_batch_free.argtypes = [ctypes.c_void_p]
         L.oracle_max_chunks.argtypes = [ctypes.c_uint64, ctypes.c_uint32]
         L.oracle_max_chunks.restype = ctypes.c_uint64
         L.oracle_findmatch.argtypes = [u8p, ctypes.c_uint64, u32p, ctypes.c_uint32, u8p,
@@ -172,6 +181,24 @@ class ItemResult:
     first_id: np.ndarray     # u64 [n]
 
 
+@dataclass
+class BatchResult:
+    """Results of Stream.items_parallel: item k's chunks are
+    [item_first[k], item_first[k + 1]) of the per-chunk arrays."""
+    item_first: np.ndarray   # u64 [n_items + 1]
+    chunk_start: np.ndarray  # u32 [m] item-relative
+    digest: np.ndarray       # u8 [m, 20]
+    is_dup: np.ndarray       # u8 [m]
+    first_id: np.ndarray     # u64 [m]
+    s_chunk_sha: float       # wall seconds, threaded chunking + SHA-1
+    s_dedup: float           # wall seconds, sequential dedup
+    threads: int
+
+    def item(self, k: int) -> tuple:
+        a, b = int(self.item_first[k]), int(self.item_first[k + 1])
+        return (self.chunk_start[a:b], self.digest[a:b], self.is_dup[a:b], self.first_id[a:b])
+
+
 class Stream:
     """Stateful oracle over one dedup stream (global table across items)."""
 
@@ -206,6 +233,34 @@ class Stream:
         assert k <= cap
         return ItemResult(seq, len(a), cs[:k].copy(), dg[:k].copy(), dup[:k].copy(),
                           fid[:k].copy())
+
+    def items_parallel(self, seq0: int, buf, item_off, threads: int | None = None):
+        """Items buf[item_off[k]:item_off[k+1]] (seq = seq0 + k) with chunking
+        and SHA-1 on `threads` host threads (default: all cores) and the dedup
+        step sequential.  Returns a BatchResult."""
+        a, p = _u8(buf)
+        off = np.ascontiguousarray(item_off, dtype=np.uint64)
+        n = len(off) - 1
+        T = threads or os.cpu_count() or 1
+        h = lib().oracle_ctx_items_parallel(
+            self._ctx, seq0, p, off.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)), n, T)
+        try:
+            m = int(lib().oracle_batch_chunks(h))
+            r = BatchResult(np.zeros(n + 1, np.uint64), np.zeros(m, np.uint32),
+                            np.zeros((m, 20), np.uint8), np.zeros(m, np.uint8),
+                            np.zeros(m, np.uint64), 0.0, 0.0, T)
+            tt = (ctypes.c_double * 2)()
+            lib().oracle_batch_times(h, tt)
+            r.s_chunk_sha, r.s_dedup = tt[0], tt[1]
+            lib().oracle_batch_fetch(
+                h, r.item_first.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)),
+                r.chunk_start.ctypes.data_as(ctypes.POINTER(ctypes.c_uint32)),
+                r.digest.ctypes.data_as(ctypes.POINTER(ctypes.c_uint8)),
+                r.is_dup.ctypes.data_as(ctypes.POINTER(ctypes.c_uint8)),
+                r.first_id.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)))
+        finally:
+            lib().oracle_batch_free(h)
+        return r
 
     def counts(self) -> dict:
         out = np.zeros(5, np.uint64)

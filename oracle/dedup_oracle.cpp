@@ -26,9 +26,12 @@
 //      std::unordered_map digest -> first id, id = (seq << 32) | chunk index.
 //   5. Output per item in seq order.
 // ============================================================================
+#include <atomic>
+#include <chrono>
 #include <cstdint>
 #include <cstring>
 #include <string>
+#include <thread>
 #include <unordered_map>
 #include <vector>
 
@@ -249,5 +252,112 @@ uint64_t oracle_max_chunks(uint64_t n, uint32_t min_chunk) {
     uint32_t m = min_chunk ? min_chunk : 1;
     return n / m + 1;
 }
+
+// ----------------------------------------------------------------------------
+// Threaded variant: steps 2-3 (chunking + SHA-1) of the
+// items of one buffer spread over T host threads -- items are independent --
+// then step 4 (the dedup table) sequentially in stream order, with exactly
+// the functions above.  Used for the CPU baseline on all host cores and to
+// run the oracle over the full-size configurations in the tests.
+// ----------------------------------------------------------------------------
+struct oracle_batch {
+    std::vector<uint64_t> item_first;  // [n_items + 1] chunk offsets
+    std::vector<uint32_t> chunk_start;
+    std::vector<uint8_t> digest;
+    std::vector<uint8_t> is_dup;
+    std::vector<uint64_t> first_id;
+    double s_chunk_sha = 0, s_dedup = 0;  // wall seconds of the two phases
+};
+
+// buf[item_off[k] .. item_off[k+1]) is item k (seq = seq0 + k).  Returns a
+// result handle (free with oracle_batch_free); the dedup state continues the
+// stream of ctx.
+oracle_batch* oracle_ctx_items_parallel(oracle_ctx* c, uint64_t seq0, const uint8_t* buf,
+                                        const uint64_t* item_off, uint64_t n_items,
+                                        uint32_t threads) {
+    auto* r = new oracle_batch();
+    const auto t0 = std::chrono::steady_clock::now();
+    std::vector<std::vector<uint32_t>> starts(n_items);
+    std::vector<std::vector<uint8_t>> digs(n_items);
+    std::atomic<uint64_t> next{0};
+    auto work = [&]() {
+        for (uint64_t k; (k = next.fetch_add(1)) < n_items;) {
+            const uint8_t* p = buf + item_off[k];
+            const uint64_t n = item_off[k + 1] - item_off[k];
+            std::vector<uint32_t>& s = starts[k];
+            s.resize(oracle_max_chunks(n, c->prm.min_chunk));
+            s.resize(oracle_chunk_item(p, n, &c->prm, s.data(), s.size()));
+            digs[k].resize(20 * s.size());
+            for (uint64_t j = 0; j < s.size(); ++j) {
+                const uint64_t e = j + 1 < s.size() ? s[j + 1] : n;
+                oracle_sha1(p + s[j], e - s[j], digs[k].data() + 20 * j);
+            }
+        }
+    };
+    if (threads < 1) threads = 1;
+    std::vector<std::thread> pool;
+    for (uint32_t t = 1; t < threads; ++t) pool.emplace_back(work);
+    work();
+    for (auto& t : pool) t.join();
+    const auto t1 = std::chrono::steady_clock::now();
+    r->item_first.resize(n_items + 1, 0);
+    for (uint64_t k = 0; k < n_items; ++k)
+        r->item_first[k + 1] = r->item_first[k] + starts[k].size();
+    const uint64_t total = r->item_first[n_items];
+    r->chunk_start.resize(total);
+    r->digest.resize(20 * total);
+    r->is_dup.resize(total);
+    r->first_id.resize(total);
+    for (uint64_t k = 0; k < n_items; ++k) {  // step 4, sequential, stream order
+        const uint64_t f = r->item_first[k], n = item_off[k + 1] - item_off[k];
+        const std::vector<uint32_t>& s = starts[k];
+        for (uint64_t j = 0; j < s.size(); ++j) {
+            const uint64_t e = j + 1 < s.size() ? s[j + 1] : n;
+            const uint8_t* d = digs[k].data() + 20 * j;
+            r->chunk_start[f + j] = s[j];
+            std::memcpy(r->digest.data() + 20 * (f + j), d, 20);
+            std::string key((const char*)d, 20);
+            const uint64_t id = ((seq0 + k) << 32) | j;
+            auto it = c->table.find(key);
+            if (it != c->table.end()) {
+                r->is_dup[f + j] = 1;
+                r->first_id[f + j] = it->second;
+                c->dup_chunks++;
+                c->dup_bytes += e - s[j];
+            } else {
+                c->table.emplace(key, id);
+                r->is_dup[f + j] = 0;
+                r->first_id[f + j] = id;
+            }
+        }
+        c->chunks += s.size();
+        c->bytes += n;
+        c->items += 1;
+    }
+    const auto t2 = std::chrono::steady_clock::now();
+    r->s_chunk_sha = std::chrono::duration<double>(t1 - t0).count();
+    r->s_dedup = std::chrono::duration<double>(t2 - t1).count();
+    return r;
+}
+
+uint64_t oracle_batch_chunks(const oracle_batch* r) { return r->chunk_start.size(); }
+
+void oracle_batch_times(const oracle_batch* r, double out[2]) {
+    out[0] = r->s_chunk_sha;
+    out[1] = r->s_dedup;
+}
+
+// Copies the results out: item_first[n_items + 1], then per chunk.
+void oracle_batch_fetch(const oracle_batch* r, uint64_t* item_first, uint32_t* chunk_start,
+                        uint8_t* digest, uint8_t* is_dup, uint64_t* first_id) {
+    std::memcpy(item_first, r->item_first.data(), 8 * r->item_first.size());
+    const uint64_t n = r->chunk_start.size();
+    std::memcpy(chunk_start, r->chunk_start.data(), 4 * n);
+    std::memcpy(digest, r->digest.data(), 20 * n);
+    std::memcpy(is_dup, r->is_dup.data(), n);
+    std::memcpy(first_id, r->first_id.data(), 8 * n);
+}
+
+void oracle_batch_free(oracle_batch* r) { delete r; }
 
 }  // extern "C"

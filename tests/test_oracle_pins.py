@@ -241,3 +241,34 @@ def test_tiny_and_empty_items():
     assert [len(r.chunk_start) for r in res] == [0, 1, 0, 1]
     assert res[1].is_dup[0] == 0 and res[3].is_dup[0] == 1
     assert int(res[3].first_id[0]) == (1 << 32)
+
+
+# ------------------------------------------------ threaded variant (8c.6) --
+@pytest.mark.parametrize("threads", [1, 3, 8])
+def test_items_parallel_equals_sequential_and_hashlib(threads):
+    """The threaded driver (steps 2-3 on T threads, step 4 sequential) gives
+    the sequential stream's results item by item, across two calls on one
+    stream; every digest is re-checked with hashlib and every dup flag with a
+    dict over (digest) in stream order."""
+    data = synthgen.make_stream(3 << 20, seed=11, dup_frac=0.5, segment=64 * 1024)
+    off = list(synthgen.split_items(data, 200 * 1024))
+    off = np.array(off[:5] + [off[4], off[4] + 7] + off[5:], np.uint64)  # empty + tiny item
+    items = [data[int(off[k]):int(off[k + 1])] for k in range(len(off) - 1)]
+    want, _ = oracle.dedup_items(items)
+    s = oracle.Stream()
+    h = len(items) // 2
+    r1 = s.items_parallel(0, data, off[:h + 1], threads)
+    r2 = s.items_parallel(h, data[int(off[h]):], off[h:] - off[h], threads)
+    s.close()
+    got = [r1.item(k) for k in range(h)] + [r2.item(k) for k in range(len(items) - h)]
+    seen = {}
+    for k, (w, g) in enumerate(zip(want, got)):
+        cs, dg, dup, fid = g
+        assert np.array_equal(cs, w.chunk_start) and np.array_equal(dg, w.digest)
+        assert np.array_equal(dup, w.is_dup) and np.array_equal(fid, w.first_id)
+        ends = list(cs[1:]) + [len(items[k])]
+        for j, (a, b) in enumerate(zip(cs, ends)):
+            d = hashlib.sha1(items[k][a:b].tobytes()).digest()
+            assert bytes(dg[j]) == d
+            assert dup[j] == (d in seen)
+            assert fid[j] == seen.setdefault(d, (k << 32) | j)
