@@ -5,14 +5,17 @@ Contract (README / DESIGN.md "Measurement"):
   python bench.py --gpus N --steps K --warmup W [--impl b200|reference]
 prints ONE JSON line on rank 0.
 
-A step is one pass of the whole hot path (rows A1-A9 of SURVEY 8(a)) over
-one GPU batch of the BASELINE.json configs[1] workload: the 184 MiB
-simlarge-sized synthetic stream (1 MiB items, ~50 % duplicate chunks),
-cycled; at every wrap of the stream a new dedup stream (fresh digest table)
-starts.  `value` is input GB/s (1e9 B/s) with the stream resident in HBM
-(device-timed with CUDA events around submit..drain); `e2e` is the same
-metric through dedup_submit_batch with pinned HOST buffers (H2D and the
-result read-back inside the timed region).
+Workload: BASELINE.json configs[2], the 672 MiB native-sized synthetic stream
+C3 (1 MiB items, dup_frac 0.52), resident in HBM.  A step is one pass of the
+whole hot path (rows A1-A9 of SURVEY 8(a)) over the WHOLE C3 stream as a new
+dedup stream (fresh digest table): 11 GPU batches (64 MiB of whole items
+each).  The engine keeps up to SLOTS batches in flight and consecutive steps
+run back to back (a step's batches enter the pipeline while the previous
+step's are still in flight), so the timed region -- W warm-up steps drained,
+then K steps bracketed by CUDA events -- measures the pipeline in steady
+state plus one fill and one drain.  `value` is input GB/s (1e9 B/s); `e2e`
+is the same metric through dedup_submit_batch with pinned HOST buffers (H2D
+and the result read-back inside the timed region).
 """
 from __future__ import annotations
 
@@ -30,7 +33,7 @@ import numpy as np
 # concurrently (must be set before CUDA is initialised).
 os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
 # per-stage CUDA-event times are read for every 8th batch (event queries cost
-# host time); the roofline uses those samples
+# host time)
 os.environ.setdefault("DEDUP_TIME_EVERY", "8")
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
@@ -41,52 +44,33 @@ import synthgen  # noqa: E402
 
 MiB = 1 << 20
 ITEM_BYTES = MiB                 # the paper's fixed 1 MB batches
-BATCH_BYTES = 64 * MiB           # GPU batch (step); C2 batch sweep 1-64 MiB
+BATCH_BYTES = 64 * MiB           # GPU batch; configs[1] sweeps 1-64 MiB
 BATCH_ITEMS = 64
 SLOTS = 40                       # batches in flight ("memory spaces")
-WORKLOAD = "C2"
+WORKLOAD = "C3"
+WORKLOAD_DESC = ("C3: 672 MiB native-sized synthetic stream (seed 3), 1 MiB items, "
+                 "dup_frac 0.52, device-resident; one step = one pass over the whole stream "
+                 "as a new dedup stream (11 GPU batches of <= 64 MiB)")
 METRIC = "input GB/s & chunks/s (dedup hot path) at 1/2/4/8 B200; % of HBM/INT roofline"
 
 # SHA-1 algorithmic 32-bit integer ops per 64-byte block (FIPS 180-4 6.1.2,
 # counting a 3-input logic/add as one op and a rotate as one op):
 #   80 rounds x (f 1 + rotl5 1 + adds 2 + rotl30 1) + 64 x schedule 3 + 5.
 SHA1_OPS_PER_BLOCK = 80 * 5 + 64 * 3 + 5
-SHA1_ALU_OPS_PER_BLOCK = 80 * 3 + 64 * 3       # of which on the ALU pipe
+# of which, as the minimal sm_100a mapping issues them:
+# on the ALU pipe f LOP3 80, rotl30 SHF 80, rotl5 + add LEA.HI 80, schedule
+# 2 LOP3 + 1 SHF per word x 64 = 432; on the FMA pipe the other adds 165
+SHA1_ALU_OPS_PER_BLOCK = 80 * 3 + 64 * 3
+SHA1_FMA_OPS_PER_BLOCK = SHA1_OPS_PER_BLOCK - SHA1_ALU_OPS_PER_BLOCK
 # Rabin rolling step per input byte: 2 table lookups, shift-in,
 # 2 address formations, 1 3-way XOR, test + bit = 8 ops.
 SCAN_OPS_PER_BYTE = 8
-# Integer-op peak = instruction issue: 148 SM x 4 SMSP x 1 warp-instr/clk x 32
-# lanes (B300_MICROARCH.md: 4 SMSPs, ALU and FMA pipes 16 lanes/clk each per
-# SMSP, so a mix of ALU-pipe and IMAD ops can fill every issue slot).
-INT_LANES_PER_SM_CLK = 128
-
-
-def h2d_bandwidth(pin, dev, nbytes=64 * MiB, reps=10):
-    """Plain pinned host -> device copy bandwidth (the e2e roofline, PCIe)."""
-    import torch
-    src = torch.from_numpy(pin[:nbytes])
-    dst = dev[:nbytes]
-    ev = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
-    dst.copy_(src, non_blocking=True)
-    torch.cuda.synchronize()
-    ev[0].record()
-    for _ in range(reps):
-        dst.copy_(src, non_blocking=True)
-    ev[1].record()
-    ev[1].synchronize()
-    return nbytes * reps / (ev[0].elapsed_time(ev[1]) * 1e-3) / 1e9
-
-
-def engine_kwargs(stream_bytes: int) -> dict:
-    return dict(batch_bytes=BATCH_BYTES, batch_items=BATCH_ITEMS, slots=SLOTS,
-                table_capacity=max(1 << 16, stream_bytes // 2048), host_fed=True)
 
 
 def peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
-        d = json.load(open(p))
-        return d, "measured"
+        return json.load(open(p)), "measured"
     return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}, "fallback"
 
 
@@ -121,7 +105,7 @@ class ClockSampler:
                         self.reasons.add(name)
             except Exception:
                 pass
-            time.sleep(0.005)
+            time.sleep(0.002)
 
     def __enter__(self):
         if self.nv is not None:
@@ -142,23 +126,33 @@ class ClockSampler:
                 "reasons": sorted(self.reasons), "samples": len(self.samples)}
 
 
-def plan_batches(off):
+def plan_batches(off, batch_bytes=None, batch_items=None):
+    """Greedy grouping of whole items into GPU batches (item index ranges)."""
+    bb = batch_bytes or BATCH_BYTES
+    bi = batch_items or BATCH_ITEMS
     out, k, n = [], 0, len(off) - 1
     while k < n:
         j = k + 1
-        while j < n and j - k < BATCH_ITEMS and int(off[j + 1]) - int(off[k]) <= BATCH_BYTES:
+        while j < n and j - k < bi and int(off[j + 1]) - int(off[k]) <= bb:
             j += 1
         out.append((k, j))
         k = j
     return out
 
 
-def run_steps(d, submit, n_batches, steps, first_step):
-    """Submit `steps` consecutive steps (batches, cycling the stream)."""
-    for s in range(first_step, first_step + steps):
-        b = s % n_batches
-        if b == 0 and s > 0:
-            d.end_stream()
+def engine_kwargs(stream_bytes: int) -> dict:
+    return dict(batch_bytes=BATCH_BYTES, batch_items=BATCH_ITEMS, slots=SLOTS,
+                table_capacity=max(1 << 16, stream_bytes // 2048), host_fed=True)
+
+
+def submit_pass(d, submit, n_batches, new_stream=True):
+    """One step: every batch of the stream, as a new dedup stream.  A full
+    slot ring is relieved by a non-blocking drain (results of the batches
+    handed out by the previous drain are released), blocking only if nothing
+    has completed."""
+    if new_stream:
+        d.end_stream()
+    for b in range(n_batches):
         while True:
             try:
                 submit(b)
@@ -166,10 +160,11 @@ def run_steps(d, submit, n_batches, steps, first_step):
             except Exception as e:
                 if "EAGAIN" not in str(e):
                     raise
-                # a non-blocking drain first releases the slots handed out by
-                # the previous drain; block only if nothing has completed
                 if d.drain_raw(wait_ms=0) == 0:
                     d.drain_raw(wait_ms=-1)
+
+
+def drain_all(d):
     while d.pending():
         d.drain_raw(wait_ms=-1)
 
@@ -178,100 +173,146 @@ def stat_delta(a, b):
     return {k: b[k] - a[k] for k in a if isinstance(a[k], (int, float))}
 
 
-def cpu_baseline(data, off, seconds_budget=12.0):
-    """The oracle as it stands, 1 host thread, on a bounded prefix sample."""
-    import oracle
-    t_total, nbytes, items = 0.0, 0, 0
-    st = oracle.Stream()
-    k = 0
-    n = len(off) - 1
-    while k < n and t_total < seconds_budget:
-        it = data[int(off[k]):int(off[k + 1])]
-        t0 = time.perf_counter()
-        st.item(k, it)
-        t_total += time.perf_counter() - t0
-        nbytes += len(it)
-        items += 1
-        k += 1
-    c = st.counts()
-    st.close()
-    return {"value": nbytes / t_total / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle",
-            "sample": f"first {items} items ({nbytes / MiB:.0f} MiB) of the {WORKLOAD} stream, "
-                      f"sequential C++ oracle (chunk+SHA-1+dedup), {c['chunks']} chunks",
-            "chunks_per_s": c["chunks"] / t_total}
+def timed_passes(d, submit, n_batches, steps, warmup, sampler=None):
+    """W warm-up passes (drained), then K passes between CUDA events on
+    torch's stream; dedup_join makes the end event wait for every batch."""
+    import torch
+    for _ in range(warmup):
+        submit_pass(d, submit, n_batches)
+    drain_all(d)
+    torch.cuda.synchronize()
+    s0, l0 = d.stats(), d.kernel_launches()
+    start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ctx = sampler if sampler is not None else _Null()
+    with ctx:
+        start.record()
+        for _ in range(steps):
+            submit_pass(d, submit, n_batches)
+        d.join()
+        end.record()
+        end.synchronize()
+    drain_all(d)
+    ms = start.elapsed_time(end)
+    return ms, stat_delta(s0, d.stats()), d.kernel_launches() - l0
 
 
-def reference_arm(args, data, off):
-    """--impl reference: the oracle on the host cores, same metric/config."""
-    import oracle
-    rank = int(os.environ.get("RANK", "0"))
-    if rank != 0:
-        return
-    n = len(off) - 1
-    total_steps = args.steps + args.warmup
-    budget_bytes = 60.0 * 60e6       # ~60 s of oracle work (~60 MB/s) over the whole run
-    per_step_items = max(1, min(BATCH_ITEMS, int(budget_bytes / max(total_steps, 1) / ITEM_BYTES)))
-    st = oracle.Stream()
-    k, seq = 0, 0
-    t_timed, bytes_timed, chunks_timed = 0.0, 0, 0
-    for s in range(total_steps):
-        t0 = time.perf_counter()
-        nb = nc = 0
-        for _ in range(per_step_items):
-            if k == n:
-                st.close()
-                st = oracle.Stream()
-                k = 0
-            it = data[int(off[k]):int(off[k + 1])]
-            r = st.item(seq, it)
-            nb += len(it)
-            nc += len(r.chunk_start)
-            k += 1
-            seq += 1
-        dt = time.perf_counter() - t0
-        if s >= args.warmup:
-            t_timed += dt
-            bytes_timed += nb
-            chunks_timed += nc
-    st.close()
-    v = bytes_timed / t_timed / 1e9
-    line = {
-        "impl": "reference", "metric": METRIC, "value": v, "unit": "GB/s",
-        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
-        "ms_per_step": 1e3 * t_timed / max(args.steps, 1), "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-        "chunks_per_s": chunks_timed / t_timed,
-        "config": {"workload": f"{WORKLOAD}: 184 MiB simlarge-sized stream, 1 MiB items, "
-                               "dup_frac 0.52", "step_sample_items": per_step_items},
-        "cpu_baseline": {"value": v, "unit": "GB/s", "cores": 1, "kind": "oracle",
-                         "sample": f"{per_step_items} x 1 MiB items per step, cycling the "
-                                   f"{WORKLOAD} stream"},
-        "e2e": {"value": v, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
-    }
-    print(json.dumps(line), flush=True)
+class _Null:
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        return False
 
 
-HBM_PEAK = 6462.1  # overwritten from MEASURED_PEAKS.json in main()
+def device_subs(dd, off, plan):
+    return [(dd[int(off[k]):int(off[j])], (off[k:j + 1] - off[k]).copy()) for k, j in plan]
 
 
-def isolated_kernels(dd, off, int_peak, copies=4, reps=3, streams=4):
-    """Live per-kernel throughput with the GPU filled by one kernel type.
-
-    chunk stage: one op_chunk call (scan + select) over the C2 stream tiled
-    `copies` times (a full-GPU grid).  SHA-1: one launch's duration is floored
-    by the longest chunk's serial chain of 64-byte compressions (latency, not
-    throughput), so `streams` contexts launch the same SHA-1 work concurrently
-    on their own streams and the throughput is all their blocks over the
-    joint elapsed time.  CUDA events on torch's current stream bracket both."""
+def stream_throughput(name, data, steps=3, warmup=1):
+    """GB/s and chunks/s of the engine on one named config (device-resident,
+    the bench's engine configuration, each pass a new dedup stream)."""
     import torch
 
     from paper_conf_ipps_rockenbachsgmtd19_b200 import Dedup
-    nb1 = int(off[-1])
-    data = dd.repeat(copies)
-    nb = nb1 * copies
-    n_items = (len(off) - 1) * copies
-    offs = np.concatenate([off[:-1] + k * nb1 for k in range(copies)] + [np.array([nb], off.dtype)])
-    item_off = torch.from_numpy(offs.astype(np.int64)).cuda()
+    off = synthgen.split_items(data, ITEM_BYTES)
+    plan = plan_batches(off)
+    dd = torch.from_numpy(data).cuda()
+    subs = device_subs(dd, off, plan)
+    with Dedup(0, **dict(engine_kwargs(len(data)), host_fed=False)) as d:
+        prod = torch.cuda.current_stream().cuda_stream
+        ms, ds, _ = timed_passes(d, lambda b: d.submit_device(subs[b][0], subs[b][1], prod),
+                                 len(plan), steps, warmup)
+    del dd, subs
+    torch.cuda.empty_cache()
+    return {"gbs": ds["bytes"] / (ms * 1e-3) / 1e9, "chunks_per_s": ds["chunks"] / (ms * 1e-3),
+            "chunks_per_pass": ds["chunks"] // steps,
+            "dup_ratio": ds["dup_chunks"] / max(ds["chunks"], 1),
+            "bytes_per_pass": ds["bytes"] // steps, "passes": steps}
+
+
+def config_lines(steps):
+    """Throughput of the other BASELINE.json configs (single GPU)."""
+    out = {}
+    specs = [
+        ("C1", "10 MiB simsmall-sized, dup_frac 0.52 (seed 1)", lambda: synthgen.config_stream("C1")),
+        ("C4_share", "the 2 GiB per-GPU share (1/8) of the 16 GiB dup_frac-0 stream (seed 4)",
+         lambda: synthgen.config_stream("C4", nbytes=2 << 30)),
+        ("C5a", "672 MiB all-unique (seed 51)", lambda: synthgen.config_stream("C5a")),
+        ("C5b", "672 MiB all-duplicate: every item = item 0 (seed 52)",
+         lambda: synthgen.config_stream("C5b")),
+        ("C5c_zero", "672 MiB all-zero: 22 M identical 32-byte chunks",
+         lambda: synthgen.config_stream("C5c_zero")),
+        ("C5c_hit", "672 MiB constructed-hit: 22 M distinct 32-byte chunks",
+         lambda: synthgen.config_stream("C5c_hit")),
+        ("C5d", "672 MiB constructed no-hit: one 1 MiB chunk per item",
+         lambda: synthgen.config_stream("C5d")),
+    ]
+    for key, desc, gen in specs:
+        data = gen()
+        # about 0.3-3 GB of work per config: C1 is tiny, repeat it more
+        n = max(1, min(steps, int(3e9 // len(data))))
+        r = stream_throughput(key, data, steps=n)
+        r["workload"] = desc
+        out[key] = r
+        del data
+    return out
+
+
+def batch_sweep(data, sizes=(1, 2, 4, 8, 16, 32, 64), target_bytes=2 << 30):
+    """BASELINE.json configs[1]: the C2 stream at GPU batch sizes 1..64 MiB,
+    device-resident, SLOTS batches in flight; GB/s per batch size."""
+    import torch
+
+    from paper_conf_ipps_rockenbachsgmtd19_b200 import Dedup
+    out = {}
+    off = synthgen.split_items(data, ITEM_BYTES)
+    dd = torch.from_numpy(data).cuda()
+    for mb in sizes:
+        bb = mb * MiB
+        plan = plan_batches(off, bb, max(mb, 1) + 1)
+        subs = device_subs(dd, off, plan)
+        with Dedup(0, batch_bytes=bb, batch_items=max(mb, 1) + 1, slots=SLOTS,
+                   table_capacity=max(1 << 16, len(data) // 2048), host_fed=False) as d:
+            prod = torch.cuda.current_stream().cuda_stream
+            passes = max(2, int(target_bytes // len(data)))
+            ms, ds, _ = timed_passes(
+                d, lambda b: d.submit_device(subs[b][0], subs[b][1], prod), len(plan),
+                passes, 1)
+        out[f"{mb}MiB"] = ds["bytes"] / (ms * 1e-3) / 1e9
+    del dd
+    torch.cuda.empty_cache()
+    return out
+
+
+def int_rates():
+    """Measured integer-pipe rates (include/dedup.h dedup_probe_int_rates)."""
+    from paper_conf_ipps_rockenbachsgmtd19_b200 import probe_int_rates
+    return probe_int_rates(0)
+
+
+def sha1_peak(r):
+    """Attainable int ops/s for SHA-1's op mix from the measured pipe rates:
+    a block needs 432 ALU-pipe ops, 165 FMA-pipe ops and 597 issue slots, so
+    its time is max(432 / R_alu, 165 / R_fma, 597 / R_issue)."""
+    t = max(SHA1_ALU_OPS_PER_BLOCK / r["lop3"], SHA1_FMA_OPS_PER_BLOCK / r["imad"],
+            SHA1_OPS_PER_BLOCK / r["mix_lop3_imad"])
+    return SHA1_OPS_PER_BLOCK / t
+
+
+def isolated_kernels(dd, off, int_peak, alu_peak, reps=3, streams=4):
+    """Live per-kernel throughput with the GPU filled by one kernel type, on
+    the C3 stream.  chunk stage: one op_chunk call (scan + cut selection)
+    over the whole stream.  SHA-1: one launch's duration is floored by its
+    longest chunk's serial chain of 64-byte compressions (latency, not
+    throughput), so `streams` contexts launch the same SHA-1 work
+    concurrently on their own streams and the throughput is all their blocks
+    over the joint elapsed time.  CUDA events on torch's stream bracket both."""
+    import torch
+
+    from paper_conf_ipps_rockenbachsgmtd19_b200 import Dedup
+    nb = int(off[-1])
+    n_items = len(off) - 1
+    item_off = torch.from_numpy(off.astype(np.int64)).cuda()
     cap = nb // 32 + n_items + 2
     ctxs = [Dedup(0, batch_bytes=nb, batch_items=n_items + 1, slots=1, table_capacity=1 << 12,
                   host_fed=False) for _ in range(streams)]
@@ -281,17 +322,17 @@ def isolated_kernels(dd, off, int_peak, copies=4, reps=3, streams=4):
         digs = [torch.zeros(cap * 20, dtype=torch.uint8, device="cuda") for _ in range(streams)]
         sts = [torch.cuda.Stream() for _ in range(streams)]
         ev = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
-        ctxs[0].op_chunk(data, nb, item_off, n_items, cut, cap, n)   # warm-up
-        ctxs[0].op_sha1(data, nb, cut, n, cap, digs[0])
+        ctxs[0].op_chunk(dd, nb, item_off, n_items, cut, cap, n)   # warm-up
+        ctxs[0].op_sha1(dd, nb, cut, n, cap, digs[0])
         torch.cuda.synchronize()
         ev[0].record()
         for _ in range(reps):
-            ctxs[0].op_chunk(data, nb, item_off, n_items, cut, cap, n)
+            ctxs[0].op_chunk(dd, nb, item_off, n_items, cut, cap, n)
         ev[1].record()
         for k in range(streams):
             sts[k].wait_event(ev[1])
             for _ in range(reps):
-                ctxs[k].op_sha1(data, nb, cut, n, cap, digs[k], stream=sts[k].cuda_stream)
+                ctxs[k].op_sha1(dd, nb, cut, n, cap, digs[k], stream=sts[k].cuda_stream)
             torch.cuda.current_stream().wait_stream(sts[k])
         ev[2].record()
         ev[2].synchronize()
@@ -302,18 +343,16 @@ def isolated_kernels(dd, off, int_peak, copies=4, reps=3, streams=4):
         # row NEXT-1 (LZSS FindMatch over the same blocks; not part of the step)
         fl = torch.empty(nb, dtype=torch.uint8, device="cuda")
         fo = torch.empty(nb, dtype=torch.int16, device="cuda")
-        ctxs[0].op_findmatch(data, nb, cut, n, cap, fl, fo)
+        ctxs[0].op_findmatch(dd, nb, cut, n, cap, fl, fo)
         ev[0].record()
-        ctxs[0].op_findmatch(data, nb, cut, n, cap, fl, fo)
+        ctxs[0].op_findmatch(dd, nb, cut, n, cap, fl, fo)
         ev[1].record()
         ev[1].synchronize()
         fm_us = ev[0].elapsed_time(ev[1]) * 1e3
         # row NEXT-3 (host archive writer) on the first 64 MiB of these outputs
         from paper_conf_ipps_rockenbachsgmtd19_b200 import archive
         an = 64 * MiB
-        kk = int(n.item())
-        cps = cut[:kk].cpu().numpy().astype(np.int64)
-        cps = cps[cps < an].astype(np.uint32)
+        cps = cp[cp < an].astype(np.uint32)
         a_data = dd[:an].cpu().numpy()
         a_len = fl[:an].cpu().numpy()
         a_off = fo[:an].cpu().numpy().view(np.uint16)
@@ -328,7 +367,7 @@ def isolated_kernels(dd, off, int_peak, copies=4, reps=3, streams=4):
         arch = {"row": "NEXT-3 (host archive writer: greedy LZSS tokens from FindMatch + "
                        "digest records; C++, 1 host thread)",
                 "encode_gbs": an / (t1 - t0) / 1e9, "decode_gbs": an / (t2 - t1) / 1e9,
-                "ratio": len(rec) / an, "sample": "first 64 MiB of the C2 stream, every chunk "
+                "ratio": len(rec) / an, "sample": "first 64 MiB of the C3 stream, every chunk "
                 "encoded as unique (the step's duplicates would be 21-byte references)"}
         del fl, fo
     finally:
@@ -338,26 +377,29 @@ def isolated_kernels(dd, off, int_peak, copies=4, reps=3, streams=4):
     blocks = int(((lens + 9 + 63) // 64).sum())
     sha_ops = blocks * SHA1_OPS_PER_BLOCK / (sha_us * 1e-6) / 1e12
     scan_ops = nb * SCAN_OPS_PER_BYTE / (chunk_us * 1e-6) / 1e12
+    pk, _ = peaks()
+    hbm = float(pk.get("hbm_gbs", 6550.1))
     return {
         "sha1": {"bound": "alu", "achieved": sha_ops, "peak": int_peak, "unit": "Tops/s",
                  "frac": sha_ops / int_peak, "launch_us": sha_us, "launch_bytes": nb,
                  "input_gbs": nb / (sha_us * 1e-6) / 1e9, "blocks": blocks,
-                 "note": f"{streams} concurrent streams x {reps} launches; launch_us = "
-                         "joint elapsed / launches"},
+                 "note": f"{streams} concurrent streams x {reps} launches over the C3 chunks; "
+                         "launch_us = joint elapsed / launches"},
         "archive": arch,
         "findmatch": {"row": "NEXT-1 (LZSS FindMatch, Listing 3), W=4096, MAX_CODED=18",
                       "bound": "hbm", "achieved": nb * 4 / (fm_us * 1e-6) / 1e9,
-                      "peak": HBM_PEAK, "unit": "GB/s",
-                      "frac": nb * 4 / (fm_us * 1e-6) / 1e9 / HBM_PEAK,
+                      "peak": hbm, "unit": "GB/s",
+                      "frac": nb * 4 / (fm_us * 1e-6) / 1e9 / hbm,
                       "launch_us": fm_us, "input_gbs": nb / (fm_us * 1e-6) / 1e9,
                       "note": "algorithmic HBM bytes: 1 B read + 3 B written (u8 length, "
                               "u16 offset) per input byte; search-bound, see DESIGN.md"},
-        "chunk_stage": {"bound": "alu", "achieved": scan_ops, "peak": int_peak, "unit": "Tops/s",
-                        "frac": scan_ops / int_peak, "launch_us": chunk_us,
+        "chunk_stage": {"bound": "alu", "achieved": scan_ops, "peak": alu_peak, "unit": "Tops/s",
+                        "frac": scan_ops / alu_peak, "launch_us": chunk_us,
                         "input_gbs": nb / (chunk_us * 1e-6) / 1e9,
-                        "note": "scan + select_scan + select_emit, one op_chunk call; "
-                                "HBM: reads 1 B/B -> "
-                                f"{nb / (chunk_us * 1e-6) / 1e9 / HBM_PEAK:.3f} of the copy peak"},
+                        "hbm_frac": nb / (chunk_us * 1e-6) / 1e9 / hbm,
+                        "note": "scan + select_scan + select_emit, one op_chunk call over C3; "
+                                "peak = measured LOP3 (ALU-pipe) rate; hbm_frac = read "
+                                "bytes / the HBM copy peak"},
     }
 
 
@@ -365,13 +407,10 @@ def isolated_kernels(dd, off, int_peak, copies=4, reps=3, streams=4):
 MANDEL_DIM, MANDEL_NITER = 2000, 200000
 MANDEL_BATCH_ROWS, MANDEL_SPACES = 1000, 2
 # binary64 pipe operations per iteration of Listing 1 (lines 15-19, no FMA):
-# a*a, b*b, a2+b2, 2*a, (2a)*b, +im, a2-b2, +cr and the compare with 4.0 (DSETP
-# issues to the FP64 pipe: ncu's fp64-pipe utilisation of the kernel matches
-# 9 ops x 64 lanes/clk/SM)
+# a*a, b*b, a2+b2, 2*a, (2a)*b, +im, a2-b2, +cr and the compare with 4.0
 MANDEL_FP64_OPS_PER_ITER = 9
 # FP64 lanes per SM per clock on B200 (derived: no FP64 figure in
-# MEASURED_PEAKS.json / B200_PROFILING.md; 64/clk/SM = the B200 FP64 rating
-# of ~37 TFLOPS FMA at 1.965 GHz; ncu's fp64-pipe utilisation checks it)
+# MEASURED_PEAKS.json / B200_PROFILING.md; ncu's fp64-pipe utilisation checks it)
 FP64_LANES_PER_SM_CLK = 64
 
 
@@ -407,62 +446,138 @@ def mandel_measure(sm_mhz, with_cpu=True):
     return out
 
 
-def batch_sweep(dd, off, sizes=(1, 2, 4, 8, 16, 32), target_bytes=3 << 30):
-    """BASELINE.json configs[1]: the C2 stream at GPU batch sizes 1..32 MiB
-    (the 64 MiB point is the headline `value`), device-resident, 40 batches
-    in flight, CUDA events around the submissions; GB/s per batch size."""
-    import torch
+def host_info():
+    info = {"nproc": os.cpu_count()}
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                info["cpu"] = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return info
 
-    from paper_conf_ipps_rockenbachsgmtd19_b200 import Dedup
-    out = {}
-    for mb in sizes:
-        bb = mb * MiB
-        plan, k, n = [], 0, len(off) - 1
-        while k < n:
-            j = k + 1
-            while j < n and int(off[j + 1]) - int(off[k]) <= bb:
-                j += 1
-            plan.append((k, j))
-            k = j
-        subs = [(dd[int(off[a]):int(off[b])], (off[a:b + 1] - off[a]).copy()) for a, b in plan]
-        d = Dedup(0, batch_bytes=bb, batch_items=max(mb, 1) + 1, slots=SLOTS,
-                  table_capacity=max(1 << 16, len(dd) // 2048), host_fed=False)
-        producer = torch.cuda.current_stream().cuda_stream
-        sub = lambda b: d.submit_device(subs[b][0], subs[b][1], producer)  # noqa: E731
-        steps = max(400, target_bytes // bb)
-        run_steps(d, sub, len(plan), 8, 0)
-        torch.cuda.synchronize()
-        s0 = d.stats()
-        ev = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
-        ev[0].record()
-        run_steps(d, sub, len(plan), steps, 8)
-        d.join()
-        ev[1].record()
-        ev[1].synchronize()
-        nbytes = d.stats()["bytes"] - s0["bytes"]
-        out[f"{mb}MiB"] = nbytes / (ev[0].elapsed_time(ev[1]) * 1e-3) / 1e9
-        d.close()
+
+def cpu_baseline(data, off, seconds_budget=12.0):
+    """The oracle as it stands on the host cores, on a bounded prefix of the
+    stream: (1) the threaded driver (chunking + SHA-1 of the items on all
+    cores, the dedup table sequential) and (2) the
+    sequential oracle on one core."""
+    import oracle
+    T = os.cpu_count() or 1
+    n = len(off) - 1
+    # calibrate the threaded driver on a few items, then size the sample
+    k0 = min(n, max(4, T))
+    st = oracle.Stream()
+    t0 = time.perf_counter()
+    st.items_parallel(0, data[:int(off[k0])], off[:k0 + 1], T)
+    rate = int(off[k0]) / (time.perf_counter() - t0)
+    st.close()
+    k = int(min(n, max(k0, rate * seconds_budget * 0.6 // ITEM_BYTES)))
+    st = oracle.Stream()
+    t0 = time.perf_counter()
+    r = st.items_parallel(0, data[:int(off[k])], off[:k + 1], T)
+    dt = time.perf_counter() - t0
+    st.close()
+    nbytes = int(off[k])
+    out = {"value": nbytes / dt / 1e9, "unit": "GB/s", "cores": T, "kind": "oracle",
+           "sample": f"first {k} items ({nbytes / MiB:.0f} MiB) of the {WORKLOAD} stream, "
+                     f"threaded oracle driver: chunking + SHA-1 on {T} threads "
+                     f"({r.s_chunk_sha:.2f} s), dedup table sequential ({r.s_dedup:.3f} s)",
+           "chunks_per_s": len(r.chunk_start) / dt, "host": host_info()}
+    # one core, the sequential oracle (about a third of the budget)
+    st = oracle.Stream()
+    t1, nb1, j = 0.0, 0, 0
+    while j < n and t1 < seconds_budget * 0.3:
+        it = data[int(off[j]):int(off[j + 1])]
+        t0 = time.perf_counter()
+        st.item(j, it)
+        t1 += time.perf_counter() - t0
+        nb1 += len(it)
+        j += 1
+    st.close()
+    out["one_core"] = {"value": nb1 / t1 / 1e9, "unit": "GB/s", "cores": 1,
+                       "sample": f"first {j} items, sequential oracle"}
     return out
+
+
+def reference_arm(args, data, off):
+    """--impl reference: the oracle on the host cores, same metric/config.
+    Each step is a bounded sample of the C3 stream (its first items, one new
+    dedup stream per step) through the threaded oracle driver on all cores,
+    sized from a calibration so the whole run takes about a minute."""
+    import oracle
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    T = os.cpu_count() or 1
+    n = len(off) - 1
+    total_steps = args.steps + args.warmup
+    k0 = min(n, max(4, T))
+    st = oracle.Stream()
+    t0 = time.perf_counter()
+    st.items_parallel(0, data[:int(off[k0])], off[:k0 + 1], T)
+    rate = int(off[k0]) / (time.perf_counter() - t0)
+    st.close()
+    per_step = int(min(n, max(k0, rate * 60.0 / max(total_steps, 1) // ITEM_BYTES)))
+    t_timed, bytes_timed, chunks_timed = 0.0, 0, 0
+    for s in range(total_steps):
+        st = oracle.Stream()
+        t0 = time.perf_counter()
+        r = st.items_parallel(0, data[:int(off[per_step])], off[:per_step + 1], T)
+        dt = time.perf_counter() - t0
+        st.close()
+        if s >= args.warmup:
+            t_timed += dt
+            bytes_timed += int(off[per_step])
+            chunks_timed += len(r.chunk_start)
+    v = bytes_timed / t_timed / 1e9
+    line = {
+        "impl": "reference", "metric": METRIC, "value": v, "unit": "GB/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": 1e3 * t_timed / max(args.steps, 1), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "chunks_per_s": chunks_timed / t_timed,
+        "config": {"workload": WORKLOAD_DESC, "step_sample_items": per_step},
+        "cpu_baseline": {"value": v, "unit": "GB/s", "cores": T, "kind": "oracle",
+                         "sample": f"first {per_step} x 1 MiB items of the {WORKLOAD} stream "
+                                   "per step (a new dedup stream each step), threaded oracle "
+                                   f"driver on {T} threads", "host": host_info()},
+        "e2e": {"value": v, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def h2d_bandwidth(pin, dev, nbytes=64 * MiB, reps=10):
+    """Plain pinned host -> device copy bandwidth (the e2e roofline, PCIe)."""
+    import torch
+    src = torch.from_numpy(pin[:nbytes])
+    dst = dev[:nbytes]
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
+    dst.copy_(src, non_blocking=True)
+    torch.cuda.synchronize()
+    ev[0].record()
+    for _ in range(reps):
+        dst.copy_(src, non_blocking=True)
+    ev[1].record()
+    ev[1].synchronize()
+    return nbytes * reps / (ev[0].elapsed_time(ev[1]) * 1e-3) / 1e9
 
 
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=600)
-    ap.add_argument("--warmup", type=int, default=12)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="b200", choices=["b200", "reference"])
-    ap.add_argument("--e2e-steps", type=int, default=0, help="0 = min(steps, 120)")
+    ap.add_argument("--e2e-steps", type=int, default=0, help="0 = steps")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--batch-mb", type=int, default=0, help="override the GPU batch size")
     ap.add_argument("--slots", type=int, default=0, help="override the in-flight batches")
     ap.add_argument("--step-only", action="store_true",
-                    help="time the step only (no isolated-kernel, NEXT-row, e2e or CPU legs): "
-                         "for the ncu launch list of the step")
+                    help="time the step only (no isolated-kernel, config, NEXT-row, e2e or CPU "
+                         "legs): for the ncu launch list of the step")
     args = ap.parse_args()
-    global BATCH_BYTES, SLOTS, BATCH_ITEMS
-    if args.batch_mb:
-        BATCH_BYTES = args.batch_mb * MiB
-        BATCH_ITEMS = max(BATCH_ITEMS, BATCH_BYTES // ITEM_BYTES)
+    global SLOTS
     if args.slots:
         SLOTS = args.slots
     if args.warmup < 3:
@@ -477,8 +592,7 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     if world > 1 or args.gpus > 1:
         from paper_conf_ipps_rockenbachsgmtd19_b200 import dist_bench
-        # pass this module: under torchrun bench.py runs as __main__, and an
-        # `import bench` would see the default (un-overridden) batch settings
+        # pass this module: under torchrun bench.py runs as __main__
         return dist_bench.main(args, data, off, sys.modules[__name__])
 
     import torch
@@ -490,51 +604,36 @@ def main():
     plan = plan_batches(off)
     nb = len(plan)
     dd = torch.from_numpy(data).to(dev)
-    subs = []
-    for k, j in plan:
-        subs.append((dd[int(off[k]):int(off[j])], (off[k:j + 1] - off[k]).copy()))
-    batch_bytes = [int(off[j]) - int(off[k]) for k, j in plan]
-
+    subs = device_subs(dd, off, plan)
     d = Dedup(0, **engine_kwargs(len(data)))
     producer = torch.cuda.current_stream().cuda_stream
     submit_dev = lambda b: d.submit_device(subs[b][0], subs[b][1], producer)  # noqa: E731
     torch.cuda.synchronize()
 
     # ---- device-resident (value) ----
-    run_steps(d, submit_dev, nb, args.warmup, 0)
-    torch.cuda.synchronize()
-    s0 = d.stats()
-    l0 = d.kernel_launches()
-    start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with ClockSampler(0) as clk:
-        start.record()
-        run_steps(d, submit_dev, nb, args.steps, args.warmup)
-        d.join()
-        end.record()
-        end.synchronize()
-    ms = start.elapsed_time(end)
-    s1 = d.stats()
-    launches = d.kernel_launches() - l0
-    ds = stat_delta(s0, s1)
-    step_ids = [(args.warmup + s) % nb for s in range(args.steps)]
-    bytes_timed = sum(batch_bytes[b] for b in step_ids)
+    clk = ClockSampler(0)
+    ms, ds, launches = timed_passes(d, submit_dev, nb, args.steps, args.warmup, clk)
+    bytes_timed = args.steps * int(off[-1])
     assert ds["bytes"] == bytes_timed, (ds["bytes"], bytes_timed)
     value = bytes_timed / (ms / 1e3) / 1e9
     chunks_per_s = ds["chunks"] / (ms / 1e3)
-
-    # ---- rooflines ----
-    pk, src = peaks()
-    global HBM_PEAK
-    HBM_PEAK = float(pk.get("hbm_gbs", HBM_PEAK))
     clocks = clk.summary()
+    if args.step_only:
+        print(json.dumps({"metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": 1,
+                          "steps": args.steps, "warmup": args.warmup,
+                          "ms_per_step": ms / args.steps, "gpu_launches": launches,
+                          "chunks_per_s": chunks_per_s, "clocks": clocks,
+                          "note": "--step-only"}), flush=True)
+        d.close()
+        return
+
+    # ---- measured roofline denominators ----
+    pk, src = peaks()
+    hbm_peak = float(pk.get("hbm_gbs", 6550.1))
     sm_mhz = pk.get("sm_max_mhz", 1965.0)
-    int_peak = 148 * INT_LANES_PER_SM_CLK * sm_mhz * 1e6 / 1e12      # Tops/s
-    peak_source = (f"derived: 148 SM x 4 SMSP x 32 lanes (1 warp-instr/clk/SMSP) x "
-                   f"{sm_mhz:.0f} MHz ({src} max SM clock); B200_PROFILING.md has no "
-                   "integer peak")
-    # pipeline stage latencies: CUDA events of every DEDUP_TIME_EVERY-th batch on
-    # the slot's own stream (the stages of ~SLOTS batches overlap, so these are
-    # latencies, not costs)
+    rates = int_rates()
+    int_peak = sha1_peak(rates)
+    alu_peak = rates["lop3"]
     nt = max(ds["timed_batches"], 1)
     kernels = {
         "stage_latency_ms_per_batch": {
@@ -542,28 +641,18 @@ def main():
             "sha1": ds["ms_sha1"] / nt, "table": ds["ms_table"] / nt,
             "pack_d2h": ds["ms_d2h"] / nt},
         "timed_batches": ds["timed_batches"],
+        "int_rates_tops": rates,
     }
-    if args.step_only:
-        print(json.dumps({"metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": 1,
-                          "steps": args.steps, "warmup": args.warmup,
-                          "ms_per_step": ms / args.steps, "gpu_launches": launches,
-                          "note": "--step-only"}), flush=True)
-        d.close()
-        return
-    iso = isolated_kernels(dd, off, int_peak)
-    kernels.update(iso)
+    kernels.update(isolated_kernels(dd, off, int_peak, alu_peak))
     kernels["mandelbrot"] = mandel_measure(sm_mhz, with_cpu=not args.no_cpu_baseline)
-    sweep = batch_sweep(dd, off)
-    sweep[f"{BATCH_BYTES // MiB}MiB"] = value
     sha_blocks_per_byte = ds["sha1_blocks"] / max(ds["bytes"], 1)
     path_ops = value * 1e9 * (SCAN_OPS_PER_BYTE + sha_blocks_per_byte * SHA1_OPS_PER_BLOCK) / 1e12
     kernels["path"] = {"bound": "alu", "achieved": path_ops, "peak": int_peak, "unit": "Tops/s",
                        "frac": path_ops / int_peak,
                        "ops_per_byte": SCAN_OPS_PER_BYTE + sha_blocks_per_byte * SHA1_OPS_PER_BLOCK,
                        "note": "whole step: algorithmic scan + SHA-1 int ops at `value`"}
-    # dominant kernel: SHA-1 (largest marginal cost per batch in the pipeline,
-    # DESIGN.md section 8); achieved = its algorithmic ops per launch / launch
-    # duration of an isolated full-GPU launch on the C2 data
+    # dominant kernel: SHA-1 (largest share of the step, profiles/); achieved =
+    # its algorithmic ops per launch / launch duration of full-GPU launches
     kd = kernels["sha1"]
     traffic = None
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -571,47 +660,38 @@ def main():
         tj = json.load(open(tp))  # scaled from its batch size to this launch's bytes
         if "sha1" in tj:
             traffic = tj["sha1"] / tj["capture_batch_bytes"] * kd["launch_bytes"]
-    # the same launch against the ALU pipe alone (16 lanes/clk/SMSP): the
-    # round function and message schedule need 432 ALU-pipe ops per block
-    # (f LOP3 80, rotl30 SHF 80, rotl5+add LEA 80, schedule 2 LOP3 + SHF
-    # per word x 64), the adds go to the FMA pipe
-    alu_peak = int_peak / 2
     alu_ach = kd["achieved"] * SHA1_ALU_OPS_PER_BLOCK / SHA1_OPS_PER_BLOCK
     roofline = {"kernel": "sha1_kernel", "bound": "alu", "achieved": kd["achieved"],
                 "peak": int_peak, "unit": "Tops/s", "frac": kd["achieved"] / int_peak,
                 "alu_pipe_view": {"achieved": alu_ach, "peak": alu_peak,
-                                  "frac": alu_ach / alu_peak, "ops_per_block":
-                                  SHA1_ALU_OPS_PER_BLOCK},
-                "traffic": traffic, "peak_source": peak_source,
-                "launch": f"{kd['launch_bytes'] / MiB:.0f} MiB of C2 chunks per launch, "
+                                  "frac": alu_ach / alu_peak,
+                                  "ops_per_block": SHA1_ALU_OPS_PER_BLOCK},
+                "traffic": traffic,
+                "peak_source": "measured (dedup_probe_int_rates, this run): SHA-1's op mix "
+                               f"(432 ALU + 165 FMA ops per block) at the measured LOP3 "
+                               f"{rates['lop3']:.1f}, IMAD {rates['imad']:.1f} and mixed-issue "
+                               f"{rates['mix_lop3_imad']:.1f} T ops/s",
+                "launch": f"{kd['launch_bytes'] / MiB:.0f} MiB of C3 chunks per launch, "
                           f"{kd['launch_us']:.0f} us per launch (CUDA events, "
                           "4 concurrent streams)"}
 
+    # ---- the other BASELINE.json configs ----
+    cfgs = config_lines(args.steps)
+    cfgs["C2_batch_sweep_gbs"] = batch_sweep(synthgen.config_stream("C2"))
+
     # ---- end-to-end through the host-fed C ABI ----
-    e2e_steps = args.e2e_steps or min(args.steps, 120)
+    e2e_steps = args.e2e_steps or args.steps
     pin = d.host_empty(len(data))
     pin[:] = data
     submit_host = lambda b: d.submit_buffer(  # noqa: E731
         pin[int(off[plan[b][0]]):int(off[plan[b][1]])], subs[b][1])
-    d.end_stream()
-    run_steps(d, submit_host, nb, args.warmup, 0)
-    torch.cuda.synchronize()
-    e0 = d.stats()
-    start.record()
-    run_steps(d, submit_host, nb, e2e_steps, args.warmup)
-    d.join()
-    end.record()
-    end.synchronize()
-    ems = start.elapsed_time(end)
-    e1 = d.stats()
-    de = stat_delta(e0, e1)
+    ems, de, _ = timed_passes(d, submit_host, nb, e2e_steps, args.warmup)
     e2e_value = de["bytes"] / (ems / 1e3) / 1e9
-    items_per_step = de["items"] / e2e_steps
     e2e = {"value": e2e_value, "unit": "GB/s",
            "h2d_bytes_per_step": (de["bytes"] + 8 * (de["items"] + de["batches"])) / e2e_steps,
            "d2h_bytes_per_step": (33 * de["chunks"] + 4 * de["items"] + 8 * de["batches"])
            / e2e_steps,
-           "steps": e2e_steps, "items_per_step": items_per_step,
+           "steps": e2e_steps, "chunks_per_s": de["chunks"] / (ems / 1e3),
            "api": "dedup_submit_batch (pinned host buffers) + dedup_drain",
            "pcie_h2d_gbs": h2d_bandwidth(pin, dd)}
     d.close()
@@ -622,14 +702,12 @@ def main():
         "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
         "chunks_per_s": chunks_per_s,
         "dup_ratio": ds["dup_chunks"] / max(ds["chunks"], 1),
-        "config": {"workload": f"{WORKLOAD}: 184 MiB simlarge-sized synthetic stream (seed 2), "
-                               "1 MiB items, dup_frac 0.52, device-resident",
-                   "batch_bytes": BATCH_BYTES, "batch_items": BATCH_ITEMS, "slots": SLOTS,
-                   "batches_per_stream": nb, "parallelism": "1 GPU",
-                   "batch_sweep_gbs": sweep,
-                   "l2": "inputs larger than L2 (184 MiB stream cycled, 126 MB L2)"},
-        "clocks": clocks, "gpu_launches": launches, "roofline": roofline, "kernels": kernels,
-        "e2e": e2e,
+        "config": {"workload": WORKLOAD_DESC, "batch_bytes": BATCH_BYTES,
+                   "batch_items": BATCH_ITEMS, "slots": SLOTS, "batches_per_step": nb,
+                   "parallelism": "1 GPU",
+                   "l2": "inputs larger than L2 (672 MiB stream, 126 MB L2)"},
+        "clocks": clocks, "gpu_launches": launches, "roofline": roofline,
+        "configs": cfgs, "kernels": kernels, "e2e": e2e,
     }
     if not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(data, off)

@@ -418,6 +418,24 @@ dedup_status dedup_dist_last_counts(const dedup_dist* d, uint32_t* n_items, uint
 /* Number of kernels this ctx has launched so far (all layers). */
 uint64_t dedup_kernel_launches(const dedup_ctx* c);
 
+/* ------------------------------------------------------------------------ */
+/* 5. Measured roofline denominators ("Integer-op peak. Not in */
+/*    MEASURED_PEAKS: microbenchmark LOP3/SHF/IADD3 throughput on B200")     */
+/* ------------------------------------------------------------------------ */
+typedef struct {
+    /* thread-level integer ops per second (1e12) of one instruction kind on
+     * the whole GPU: 8 independent chains per thread, 2 x 1024 threads per
+     * SM.  lop3 / shf / iadd3 / prmt / lea_hi issue to the ALU pipe, imad /
+     * imad_hi to the FMA pipe; mix_lop3_imad alternates LOP3 and IMAD (both
+     * pipes, the issue-slot limit). */
+    double lop3, shf, iadd3, imad, imad_hi, prmt, lea_hi, mix_lop3_imad;
+    int32_t num_sms, clock_mhz_attr;
+} dedup_int_rates;
+
+/* Runs the probe kernels on `device` (about 1 s; device-wide, do not run
+ * beside other work).  Errors: EINVAL (out NULL), ENOMEM, ECUDA. */
+dedup_status dedup_probe_int_rates(int32_t device, dedup_int_rates* out);
+
 #ifdef __cplusplus
 }
 #endif

@@ -11,6 +11,6 @@ import os as _os
 _os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
 
 from ._native import DedupError, lib  # noqa: F401
-from .api import Dedup, ItemResult, result_from_c  # noqa: F401
+from .api import Dedup, ItemResult, probe_int_rates, result_from_c  # noqa: F401
 
-__all__ = ["Dedup", "DedupError", "ItemResult", "lib", "result_from_c"]
+__all__ = ["Dedup", "DedupError", "ItemResult", "lib", "probe_int_rates", "result_from_c"]

@@ -38,7 +38,7 @@ EXPORTS = [
     "dedup_archive_decode",
     "dedup_nccl_unique_id", "dedup_dist_create", "dedup_dist_destroy", "dedup_dist_last_error",
     "dedup_dist_submit", "dedup_dist_flush", "dedup_dist_end_stream", "dedup_dist_result",
-    "dedup_dist_last_counts",
+    "dedup_dist_last_counts", "dedup_probe_int_rates",
 ]
 # every symbol declared in include/mandel.h (row NEXT-4)
 MANDEL_EXPORTS = ["mandel_rows_device", "mandel_image"]
@@ -102,6 +102,12 @@ class Stats(ctypes.Structure):
         ("timed_bytes", ctypes.c_uint64), ("timed_sha1_blocks", ctypes.c_uint64)]
 
 
+class IntRates(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_double) for n in (
+        "lop3", "shf", "iadd3", "imad", "imad_hi", "prmt", "lea_hi", "mix_lop3_imad")] + [
+        ("num_sms", ctypes.c_int32), ("clock_mhz_attr", ctypes.c_int32)]
+
+
 class Record(ctypes.Structure):
     _fields_ = [("digest", ctypes.c_uint8 * 20), ("pad", ctypes.c_uint32),
                 ("id", ctypes.c_uint64)]
@@ -163,6 +169,7 @@ def lib():
         "dedup_dist_end_stream": (st, [vp]),
         "dedup_dist_result": (st, [vp, P(WaveResult)]),
         "dedup_dist_last_counts": (st, [vp, P(u32), P(u32), P(u64)]),
+        "dedup_probe_int_rates": (st, [i32, P(IntRates)]),
         "mandel_rows_device": (st, [vp, i32, i32, ctypes.c_double, ctypes.c_double,
                                     ctypes.c_double, i32, i32, vp, vp, vp]),
         "mandel_image": (st, [P(MandelConfig), vp, P(ctypes.c_double), P(u64)]),

@@ -65,6 +65,14 @@ def result_from_c(r: N.ItemResult, copy: bool = True) -> ItemResult:
     return ItemResult(int(r.seq), int(r.item_len), cs, dg, dup, fid)
 
 
+def probe_int_rates(device: int = 0) -> dict:
+    """Measured integer-pipe throughput (T thread-ops/s) of `device`
+    (include/dedup.h dedup_probe_int_rates)."""
+    r = N.IntRates()
+    N.check(N.lib().dedup_probe_int_rates(device, ctypes.byref(r)))
+    return {k: getattr(r, k) for k, _ in N.IntRates._fields_}
+
+
 class Dedup:
     """One dedup context on one GPU (streaming API of include/dedup.h)."""
 

@@ -117,6 +117,58 @@ def all_duplicate(nbytes: int, seed: int, item_bytes: int = MiB) -> np.ndarray:
     return np.tile(base, reps)[:nbytes].copy()
 
 
+_PATTERNS = None
+
+
+def _patterns():
+    """Stored inputs of C5c(ii)/C5d (synthgen/data/c5_patterns.npz, written by
+    tools/make_c5_patterns.py with the oracle fingerprint; here they are only
+    XORed and tiled)."""
+    global _PATTERNS
+    if _PATTERNS is None:
+        import os
+        z = np.load(os.path.join(os.path.dirname(os.path.abspath(__file__)), "data",
+                                 "c5_patterns.npz"))
+        _PATTERNS = {k: z[k] for k in z.files}
+    return _PATTERNS
+
+
+def constructed_hit(nbytes: int, seed: int = 53) -> np.ndarray:
+    """consecutive 32-byte blocks, each the XOR of a seeded
+    random subset of the 32 stored hit blocks (bits of one splitmix64 word per
+    block); every block's window hits, so every chunk is one 32-byte block and
+    almost all of them are distinct.  Trailing bytes (< 32) are zero."""
+    basis = _patterns()["hit_basis"]                  # u8 [32, 32]
+    nb = nbytes // 32
+    # XOR tables over each byte of the selector word: T[i][b] = XOR of the
+    # basis blocks 8i + j for the set bits j of b
+    T = np.zeros((4, 256, 32), np.uint8)
+    for i in range(4):
+        for b in range(1, 256):
+            low = b & -b
+            j = low.bit_length() - 1
+            T[i, b] = T[i, b ^ low] ^ basis[8 * i + j]
+    T = T.view(np.uint64)                             # [4, 256, 4] (same bytes)
+    sel = splitmix64_words(seed, 0, nb).astype(np.uint32)
+    out = np.zeros(nbytes, np.uint8)
+    blocks = out[:nb * 32].view(np.uint64).reshape(nb, 4)
+    for i in range(4):
+        blocks ^= T[i][(sel >> np.uint32(8 * i)) & np.uint32(0xFF)]
+    return out
+
+
+def constructed_no_hit(nbytes: int, item_bytes: int = MiB) -> np.ndarray:
+    """item k is the k-th stored 64-byte no-hit pattern tiled
+    (no window of the item hits: every item is ONE chunk)."""
+    pats = _patterns()["nohit_period"]                # u8 [672, 64]
+    out = np.empty(nbytes, np.uint8)
+    for k, lo in enumerate(range(0, nbytes, item_bytes)):
+        hi = min(lo + item_bytes, nbytes)
+        p = pats[k % len(pats)]
+        out[lo:hi] = np.tile(p, (hi - lo + 63) // 64)[:hi - lo]
+    return out
+
+
 # Named workloads (SURVEY 8(d) table; BASELINE.json configs).
 CONFIGS = {
     "C1": dict(nbytes=10 * MiB, seed=1, dup_frac=0.52, entropy=8),
@@ -127,7 +179,18 @@ CONFIGS = {
 }
 
 
+# adversarial streams of BASELINE.json configs[4]
+ADVERSARIAL = {
+    "C5b": lambda n: all_duplicate(n, seed=52),
+    "C5c_zero": all_zero,
+    "C5c_hit": lambda n: constructed_hit(n, seed=53),
+    "C5d": constructed_no_hit,
+}
+
+
 def config_stream(name: str, nbytes: int | None = None) -> np.ndarray:
+    if name in ADVERSARIAL:
+        return ADVERSARIAL[name](nbytes if nbytes is not None else 672 * MiB)
     cfg = dict(CONFIGS[name])
     if nbytes is not None:
         cfg["nbytes"] = nbytes
