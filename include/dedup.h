@@ -59,8 +59,9 @@ typedef int32_t dedup_status;
 #define DEDUP_EUNSUPPORTED (-5) /* config valid for the method, not for GPU v1 */
 #define DEDUP_ECUDA (-6)        /* CUDA error (sticky) */
 #define DEDUP_ETIMEDOUT (-7)    /* dedup_drain: nothing completed within wait_ms */
+#define DEDUP_ENCCL (-8)        /* NCCL error or a failed peer of the exchange (sticky) */
 
-#define DEDUP_ABI_VERSION 1
+#define DEDUP_ABI_VERSION 2
 
 typedef struct dedup_ctx dedup_ctx; /* opaque; owns its device buffers and tables */
 
@@ -83,7 +84,23 @@ typedef struct {
     uint32_t sha_lane_bytes; /* SHA-1 grid: one lane per this many batch bytes; 0 = 32768
                                 (tuned for many batches in flight; a ctx that runs one
                                 batch at a time wants fewer bytes per lane, e.g. 8192) */
-    uint32_t reserved[6];
+    /* Multi-GPU (the paper's GPUs take batches round-robin,
+     * P:185, one host thread per device).  num_devices >= 2 (or
+     * transport != 0) selects the multi-GPU engine: G = num_devices logical
+     * ranks, rank r on device_ids[r]; batches go to the ranks round-robin
+     * (batch b -> rank b % G, wave b / G), rank r owns the digest-table shard
+     * of the digests whose BE32 prefix p has floor(p G / 2^32) = r, and
+     * dedup_drain returns every rank's items merged in sequence order
+     * (P:217).  `slots` is then the waves in flight per rank and
+     * table_capacity the expected distinct digests of the whole stream.
+     * owner_rank / num_owners must be 0 / 1 (they describe the op layer). */
+    uint32_t num_devices;       /* 0 or 1: single-GPU engine on `device`; 2..64: ranks */
+    uint32_t transport;         /* exchange of rows A6/A8: 0 auto (NCCL if the devices are
+                                   distinct, else copy), 1 NCCL (ncclCommInitAll; distinct
+                                   devices), 2 in-process copy (peer loads over NVLink, or
+                                   the loopback when device ids repeat) */
+    const int32_t* device_ids;  /* [num_devices] CUDA ordinals, may repeat; NULL = 0..G-1 */
+    uint32_t reserved[2];
 } dedup_config;
 
 /* Fills *cfg with the defaults above (struct_size set). */
@@ -162,6 +179,11 @@ dedup_status dedup_drain(dedup_ctx* c, uint32_t max_items, int32_t wait_ms,
 /* Number of submitted items not yet returned by dedup_drain. */
 uint64_t dedup_pending(const dedup_ctx* c);
 
+/* CUDA device of the rank that receives the next batch (multi-GPU ctx:
+ * dedup_submit_device's d_bytes should live there; on another device it is
+ * read over peer access).  The single-GPU engine returns cfg.device. */
+int32_t dedup_next_device(const dedup_ctx* c);
+
 typedef struct {
     uint64_t items, bytes, chunks, dup_chunks, dup_bytes, unique_chunks;
     uint64_t batches, table_used, table_slots, kernel_launches;
@@ -176,6 +198,12 @@ typedef struct {
      * DEDUP_TIME_EVERY-th drained batch, default 1; none if
      * DEDUP_STAGE_EVENTS=0): their count, bytes and SHA-1 blocks */
     uint64_t timed_batches, timed_bytes, timed_sha1_blocks;
+    /* multi-GPU engine: waves completed, bytes of 32-byte records and 8-byte
+     * replies that left their rank (rows A6 + A8), and the summed device time
+     * of the exchange + owner phase (records .. scatter) of the sampled waves */
+    uint64_t waves, a2a_bytes;
+    double ms_a2a;
+    uint32_t num_devices, reserved_;
 } dedup_stats_t;
 
 /* Counters over all drained batches of the ctx (all streams). */
@@ -381,14 +409,23 @@ const char* dedup_dist_last_error(const dedup_dist* d);
 
 /* Submits this rank's batch of the next wave: d_bytes (device, 16-byte
  * aligned, after `producer`'s current work), item_off (host, n_items + 1
- * offsets), items get seq = first_seq + k.  If `depth` waves were in
- * flight, the oldest completes first and *completed = 1: read it with
- * dedup_dist_result before the next call. */
+ * offsets, item_off[0] = 0, non-decreasing, item_off[n_items] = nbytes),
+ * items get seq = first_seq + k.  Arguments are checked before anything is
+ * enqueued (EINVAL).  If `depth` waves were in flight, the oldest completes
+ * first and *completed = 1: read it with dedup_dist_result before the next
+ * call.  A digest-table overflow of any owner shard (replies of ~0) makes
+ * the completing call return the sticky DEDUP_ETABLEFULL; an NCCL error
+ * (polled with ncclCommGetAsyncError while the host waits) aborts the
+ * communicators and returns the sticky DEDUP_ENCCL. */
 dedup_status dedup_dist_submit(dedup_dist* d, const uint8_t* d_bytes, uint64_t nbytes,
                                const uint64_t* item_off, uint32_t n_items, uint64_t first_seq,
                                void* producer, uint32_t* completed);
 /* Completes the oldest wave in flight if any (*completed = 1). */
 dedup_status dedup_dist_flush(dedup_dist* d, uint32_t* completed);
+/* Makes `stream` (cudaStream_t as void*) wait for the results of every
+ * completed wave (no host synchronisation); call after the flushes, e.g. to
+ * bracket the pipeline with CUDA events. */
+dedup_status dedup_dist_join(dedup_dist* d, void* stream);
 /* New dedup stream (clears this rank's table shard).  With waves in flight
  * the reset is deferred: it is issued on the owner stream right before the
  * owner work of the next wave submitted, so the waves in flight still see
@@ -414,6 +451,9 @@ dedup_status dedup_dist_result(const dedup_dist* d, dedup_wave_result* out);
  * waiting for its results to reach host memory. */
 dedup_status dedup_dist_last_counts(const dedup_dist* d, uint32_t* n_items, uint32_t* n_chunks,
                                     uint64_t* nbytes);
+
+/* Kernels this rank's pipeline has launched so far. */
+uint64_t dedup_dist_kernel_launches(const dedup_dist* d);
 
 /* Number of kernels this ctx has launched so far (all layers). */
 uint64_t dedup_kernel_launches(const dedup_ctx* c);

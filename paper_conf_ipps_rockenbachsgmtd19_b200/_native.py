@@ -21,15 +21,16 @@ DEDUP_ETABLEFULL = -4
 DEDUP_EUNSUPPORTED = -5
 DEDUP_ECUDA = -6
 DEDUP_ETIMEDOUT = -7
+DEDUP_ENCCL = -8
 
 STATUS_NAMES = {0: "OK", -1: "EINVAL", -2: "EAGAIN", -3: "ENOMEM", -4: "ETABLEFULL",
-                -5: "EUNSUPPORTED", -6: "ECUDA", -7: "ETIMEDOUT"}
+                -5: "EUNSUPPORTED", -6: "ECUDA", -7: "ETIMEDOUT", -8: "ENCCL"}
 
 # every symbol declared in include/dedup.h (checked by tests/test_abi.py)
 EXPORTS = [
     "dedup_config_default", "dedup_init", "dedup_destroy", "dedup_last_error",
     "dedup_submit_batch", "dedup_submit_device", "dedup_join", "dedup_end_stream", "dedup_drain",
-    "dedup_pending", "dedup_stats", "dedup_host_alloc", "dedup_host_free",
+    "dedup_pending", "dedup_next_device", "dedup_stats", "dedup_host_alloc", "dedup_host_free",
     "dedup_op_chunk", "dedup_op_chunk_meta", "dedup_op_sha1", "dedup_op_table_insert_lookup",
     "dedup_op_table_reset", "dedup_op_table_status", "dedup_op_local_combine",
     "dedup_op_route", "dedup_op_owner",
@@ -37,7 +38,8 @@ EXPORTS = [
     "dedup_archive_encode", "dedup_archive_decoder_new", "dedup_archive_decoder_free",
     "dedup_archive_decode",
     "dedup_nccl_unique_id", "dedup_dist_create", "dedup_dist_destroy", "dedup_dist_last_error",
-    "dedup_dist_submit", "dedup_dist_flush", "dedup_dist_end_stream", "dedup_dist_result",
+    "dedup_dist_submit", "dedup_dist_flush", "dedup_dist_join", "dedup_dist_end_stream",
+    "dedup_dist_result", "dedup_dist_kernel_launches",
     "dedup_dist_last_counts", "dedup_probe_int_rates",
 ]
 # every symbol declared in include/mandel.h (row NEXT-4)
@@ -76,7 +78,8 @@ class Config(ctypes.Structure):
         ("batch_bytes", ctypes.c_uint64), ("table_capacity", ctypes.c_uint64),
         ("owner_rank", ctypes.c_uint32), ("num_owners", ctypes.c_uint32),
         ("host_fed", ctypes.c_uint32), ("sha_lane_bytes", ctypes.c_uint32),
-        ("reserved", ctypes.c_uint32 * 6),
+        ("num_devices", ctypes.c_uint32), ("transport", ctypes.c_uint32),
+        ("device_ids", ctypes.POINTER(ctypes.c_int32)), ("reserved", ctypes.c_uint32 * 2),
     ]
 
 
@@ -99,7 +102,9 @@ class Stats(ctypes.Structure):
         (n, ctypes.c_double) for n in ("ms_h2d", "ms_scan", "ms_select", "ms_sha1", "ms_table",
                                        "ms_d2h", "ms_host_launch", "ms_host_parse")] + [
         ("sha1_blocks", ctypes.c_uint64), ("timed_batches", ctypes.c_uint64),
-        ("timed_bytes", ctypes.c_uint64), ("timed_sha1_blocks", ctypes.c_uint64)]
+        ("timed_bytes", ctypes.c_uint64), ("timed_sha1_blocks", ctypes.c_uint64),
+        ("waves", ctypes.c_uint64), ("a2a_bytes", ctypes.c_uint64), ("ms_a2a", ctypes.c_double),
+        ("num_devices", ctypes.c_uint32), ("reserved_", ctypes.c_uint32)]
 
 
 class IntRates(ctypes.Structure):
@@ -140,6 +145,7 @@ def lib():
         "dedup_end_stream": (st, [vp]),
         "dedup_drain": (st, [vp, u32, i32, P(ItemResult), P(u32)]),
         "dedup_pending": (u64, [vp]),
+        "dedup_next_device": (i32, [vp]),
         "dedup_stats": (st, [vp, P(Stats)]),
         "dedup_host_alloc": (vp, [vp, ctypes.c_size_t]),
         "dedup_host_free": (None, [vp, vp]),
@@ -166,6 +172,8 @@ def lib():
         "dedup_dist_last_error": (ctypes.c_char_p, [vp]),
         "dedup_dist_submit": (st, [vp, vp, u64, vp, u32, u64, vp, P(u32)]),
         "dedup_dist_flush": (st, [vp, P(u32)]),
+        "dedup_dist_join": (st, [vp, vp]),
+        "dedup_dist_kernel_launches": (u64, [vp]),
         "dedup_dist_end_stream": (st, [vp]),
         "dedup_dist_result": (st, [vp, P(WaveResult)]),
         "dedup_dist_last_counts": (st, [vp, P(u32), P(u32), P(u64)]),

@@ -81,7 +81,13 @@ class Dedup:
                  window: int = 32, poly: int = 0x45C2B6A1, anchor_mask: int = 0xFFF,
                  anchor_value: int = 0, min_chunk: int = 32, max_chunk: int = 0,
                  owner_rank: int = 0, num_owners: int = 1, max_drain: int = 65536,
-                 sha_lane_bytes: int = 0):
+                 sha_lane_bytes: int = 0, num_devices: int = 0, device_ids=None,
+                 transport: int = 0):
+        """num_devices >= 2 (or transport != 0) selects the multi-GPU engine
+        (include/dedup.h): G ranks on device_ids (default 0..G-1; ids may
+        repeat: then the ranks share a GPU and exchange through the in-process
+        copy transport), transport 0 auto / 1 NCCL / 2 copy; `slots` is then
+        the waves in flight per rank."""
         L = N.lib()
         cfg = N.Config()
         L.dedup_config_default(ctypes.byref(cfg))
@@ -90,8 +96,13 @@ class Dedup:
                          host_fed=int(host_fed), window=window, poly=poly,
                          anchor_mask=anchor_mask, anchor_value=anchor_value,
                          min_chunk=min_chunk, max_chunk=max_chunk, owner_rank=owner_rank,
-                         num_owners=num_owners, sha_lane_bytes=sha_lane_bytes).items():
+                         num_owners=num_owners, sha_lane_bytes=sha_lane_bytes,
+                         num_devices=num_devices, transport=transport).items():
             setattr(cfg, k, v)
+        self._dev_ids = None
+        if device_ids is not None:
+            self._dev_ids = (ctypes.c_int32 * len(device_ids))(*device_ids)
+            cfg.device_ids = self._dev_ids
         self.cfg = cfg
         self._ctx = _vp()
         st = L.dedup_init(ctypes.byref(cfg), ctypes.byref(self._ctx))
@@ -214,6 +225,10 @@ class Dedup:
 
     def pending(self) -> int:
         return int(N.lib().dedup_pending(self._ctx))
+
+    def next_device(self) -> int:
+        """CUDA device of the rank that receives the next batch."""
+        return int(N.lib().dedup_next_device(self._ctx))
 
     def stats(self) -> dict:
         s = N.Stats()

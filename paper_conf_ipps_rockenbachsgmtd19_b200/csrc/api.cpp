@@ -30,6 +30,7 @@
 
 #include "dedup.h"
 #include "internal.h"
+#include "mg.h"
 
 using namespace dd;
 
@@ -96,6 +97,7 @@ struct TableBuf {
 
 struct dedup_ctx {
     dedup_config cfg{};
+    dd::mg::CtxEngine* mg = nullptr;  // num_devices >= 2: the multi-GPU engine (mg.cpp)
     int num_sms = 0;
     uint32_t* d_tab = nullptr;  // R[256] then W256[256]
     std::vector<Slot> slots;
@@ -152,13 +154,6 @@ dedup_status fail(dedup_ctx* c, dedup_status s, const std::string& msg) {
         dedup_status s_ = (x);         \
         if (s_ != DEDUP_OK) return s_; \
     } while (0)
-
-// ---- product-side Rabin tables (independent of the oracle) ----------------
-// Multiply a degree<32 polynomial by t^k modulo P(t) = t^32 + poly.
-uint32_t mul_tk(uint32_t x, unsigned k, uint32_t poly) {
-    while (k--) x = (x & 0x80000000u) ? ((x << 1) ^ poly) : (x << 1);
-    return x;
-}
 
 uint64_t next_pow2(uint64_t v) {
     uint64_t p = 1;
@@ -217,6 +212,12 @@ void ws_free(Workspace& w) {
 
 bool usable(const dedup_ctx* c) { return c != nullptr && c->sticky == DEDUP_OK; }
 
+// dedup_op_* apply to a single-GPU ctx
+#define NO_MG(c)                                                                        \
+    do {                                                                                \
+        if ((c)->mg) return fail(c, DEDUP_EUNSUPPORTED, "dedup_op_* need a single-GPU ctx"); \
+    } while (0)
+
 // Attribution builds (tools/attrib.sh) only: 1 = omit the SHA-1 kernels,
 // 2 = omit the table kernels, 4 = omit chunk selection.  Results are invalid;
 // the product build has 0.
@@ -224,13 +225,7 @@ bool usable(const dedup_ctx* c) { return c != nullptr && c->sticky == DEDUP_OK; 
 #define DEDUP_ATTRIB_SKIP 0
 #endif
 
-// Chunks at least 4x the mean anchor distance are hashed first.
-uint32_t long_bytes(const dedup_ctx* c) {
-    uint64_t v = 4ull * ((uint64_t)c->cfg.anchor_mask + 1);
-    if (v < kMinLongBytes) v = kMinLongBytes;
-    if (v > (1u << 20)) v = 1u << 20;
-    return (uint32_t)v;
-}
+uint32_t long_bytes(const dedup_ctx* c) { return long_chunk_bytes(c->cfg.anchor_mask); }
 
 TableView table_view(const dedup_ctx* c) {
     const TableBuf& t = c->tables[c->cur_table];
@@ -424,6 +419,8 @@ dedup_status check_cfg(const dedup_config* g) {
     if (g->num_owners < 1 || g->num_owners > 64 || g->owner_rank >= g->num_owners)
         return DEDUP_EINVAL;
     if (g->table_capacity < 1 || g->table_capacity > (1ull << 31)) return DEDUP_EINVAL;
+    if (g->num_devices > 64 || g->transport > 2) return DEDUP_EINVAL;
+    if (mg::wanted(g) && (g->owner_rank != 0 || g->num_owners != 1)) return DEDUP_EINVAL;
     if (g->sha_lane_bytes != 0 && (g->sha_lane_bytes < 64 || g->sha_lane_bytes > (1u << 24)))
         return DEDUP_EINVAL;
     // max_chunk and min_chunk > window (NEXT-2): selected by maxchunk.cu's walk
@@ -543,6 +540,18 @@ dedup_status dedup_init(const dedup_config* cfg, dedup_ctx** out) {
     if (s != DEDUP_OK) return s;
     dedup_ctx* c = new dedup_ctx();
     c->cfg = *cfg;
+    if (mg::wanted(cfg)) {  // G ranks, one worker thread per rank (mg.cpp)
+        const char* why = nullptr;
+        s = mg::create(cfg, &c->mg, &why);
+        if (s != DEDUP_OK) {
+            std::fprintf(stderr, "dedup_init (multi-GPU): %s\n", why ? why : "failed");
+            delete c;
+            return s;
+        }
+        c->cfg.device_ids = nullptr;  // not retained
+        *out = c;
+        return DEDUP_OK;
+    }
     auto bail = [&](dedup_status r) {
         dedup_destroy(c);
         return r;
@@ -560,10 +569,7 @@ dedup_status dedup_init(const dedup_config* cfg, dedup_ctx** out) {
     }
     c->chunk_cap = cfg->batch_bytes / 32 + cfg->batch_items + 2;
     uint32_t tab[512];
-    for (uint32_t b = 0; b < 256; ++b) {
-        tab[b] = mul_tk(b, 32, cfg->poly);         // R[b]    = b t^32  mod P
-        tab[256 + b] = mul_tk(b, 256, cfg->poly);  // W256[b] = b t^256 mod P
-    }
+    rabin_tables(cfg->poly, tab);
     if ((s = dalloc(c, &c->d_tab, 512)) != DEDUP_OK) return bail(s);
     if (cudaMemcpy(c->d_tab, tab, sizeof(tab), cudaMemcpyHostToDevice) != cudaSuccess)
         return bail(DEDUP_ECUDA);
@@ -602,6 +608,11 @@ dedup_status dedup_init(const dedup_config* cfg, dedup_ctx** out) {
 
 void dedup_destroy(dedup_ctx* c) {
     if (c == nullptr) return;
+    if (c->mg) {
+        mg::destroy(c->mg);
+        delete c;
+        return;
+    }
     cudaSetDevice(c->cfg.device);
     for (Slot& sl : c->slots) slot_free(sl);
     ws_free(c->op_ws);
@@ -623,12 +634,14 @@ void dedup_destroy(dedup_ctx* c) {
 }
 
 const char* dedup_last_error(const dedup_ctx* c) {
+    if (c != nullptr && c->mg && c->err == "no error") return mg::last_error(c->mg);
     return c == nullptr ? "null ctx" : c->err.c_str();
 }
 
 dedup_status dedup_submit_batch(dedup_ctx* c, uint32_t n_items, const uint8_t* const* item_ptr,
                                 const uint64_t* item_len, uint64_t* first_seq_out) {
     if (c == nullptr) return DEDUP_EINVAL;
+    if (c->mg) return mg::submit_host(c->mg, n_items, item_ptr, item_len, first_seq_out);
     if (!usable(c)) return c->sticky;
     if (!c->cfg.host_fed) return fail(c, DEDUP_EINVAL, "ctx was created with host_fed = 0");
     if (c->cfg.num_owners != 1)
@@ -691,6 +704,9 @@ dedup_status dedup_submit_device(dedup_ctx* c, const uint8_t* d_bytes, uint64_t 
                                  const uint64_t* item_off, uint32_t n_items, void* producer,
                                  uint64_t* first_seq_out) {
     if (c == nullptr) return DEDUP_EINVAL;
+    if (c->mg)
+        return mg::submit_device(c->mg, d_bytes, nbytes, item_off, n_items, producer,
+                                 first_seq_out);
     if (!usable(c)) return c->sticky;
     if (c->cfg.num_owners != 1)
         return fail(c, DEDUP_EUNSUPPORTED, "num_owners > 1: use the dedup_op_* orchestration");
@@ -725,6 +741,7 @@ dedup_status dedup_submit_device(dedup_ctx* c, const uint8_t* d_bytes, uint64_t 
 
 dedup_status dedup_join(dedup_ctx* c, void* stream) {
     if (c == nullptr) return DEDUP_EINVAL;
+    if (c->mg) return mg::join(c->mg, stream);
     if (!usable(c)) return c->sticky;
     CU(cudaSetDevice(c->cfg.device));
     for (int i : c->inflight)
@@ -734,6 +751,7 @@ dedup_status dedup_join(dedup_ctx* c, void* stream) {
 
 dedup_status dedup_end_stream(dedup_ctx* c) {
     if (c == nullptr) return DEDUP_EINVAL;
+    if (c->mg) return mg::end_stream(c->mg);
     if (!usable(c)) return c->sticky;
     c->cur_table ^= 1;
     c->stream_fresh = true;
@@ -744,6 +762,7 @@ dedup_status dedup_drain(dedup_ctx* c, uint32_t max_items, int32_t wait_ms,
                          dedup_item_result* out, uint32_t* n_out) {
     if (c == nullptr || n_out == nullptr || (max_items > 0 && out == nullptr)) return DEDUP_EINVAL;
     *n_out = 0;
+    if (c->mg) return mg::drain(c->mg, max_items, wait_ms, out, n_out);
     if (!usable(c)) return c->sticky;
     CU(cudaSetDevice(c->cfg.device));
     for (int i : c->to_release) c->slots[i].busy = false;
@@ -801,18 +820,28 @@ dedup_status dedup_drain(dedup_ctx* c, uint32_t max_items, int32_t wait_ms,
     return DEDUP_OK;
 }
 
-uint64_t dedup_pending(const dedup_ctx* c) { return c ? c->pending_items : 0; }
+uint64_t dedup_pending(const dedup_ctx* c) {
+    if (c && c->mg) return mg::pending(c->mg);
+    return c ? c->pending_items : 0;
+}
+
+int32_t dedup_next_device(const dedup_ctx* c) {
+    if (c == nullptr) return -1;
+    return c->mg ? mg::next_device(c->mg) : c->cfg.device;
+}
 
 dedup_status dedup_stats(const dedup_ctx* c, dedup_stats_t* out) {
     if (c == nullptr || out == nullptr) return DEDUP_EINVAL;
+    if (c->mg) return mg::stats(c->mg, out);
     *out = c->st;
     out->kernel_launches = c->launches;
+    out->num_devices = 1;
     return DEDUP_OK;
 }
 
 void* dedup_host_alloc(dedup_ctx* c, size_t bytes) {
     if (c == nullptr) return nullptr;
-    cudaSetDevice(c->cfg.device);
+    if (!c->mg) cudaSetDevice(c->cfg.device);
     void* p = nullptr;
     if (cudaHostAlloc(&p, bytes, cudaHostAllocPortable) != cudaSuccess) return nullptr;
     return p;
@@ -823,7 +852,10 @@ void dedup_host_free(dedup_ctx* c, void* p) {
     if (p) cudaFreeHost(p);
 }
 
-uint64_t dedup_kernel_launches(const dedup_ctx* c) { return c ? c->launches : 0; }
+uint64_t dedup_kernel_launches(const dedup_ctx* c) {
+    if (c && c->mg) return mg::kernel_launches(c->mg);
+    return c ? c->launches : 0;
+}
 
 // ---------------------------------------------------------------------------
 // Stream-ordered device operations
@@ -832,6 +864,7 @@ dedup_status dedup_op_chunk(dedup_ctx* c, void* stream, const uint8_t* d_bytes, 
                             const uint64_t* d_item_off, uint32_t n_items, uint32_t* d_cut_pos,
                             uint64_t cap, uint32_t* d_n_chunks) {
     if (c == nullptr) return DEDUP_EINVAL;
+    NO_MG(c);
     if (!usable(c)) return c->sticky;
     if (nbytes > c->cfg.batch_bytes) return fail(c, DEDUP_EINVAL, "nbytes > batch_bytes");
     if (reinterpret_cast<uintptr_t>(d_bytes) & 15)
@@ -861,6 +894,7 @@ dedup_status dedup_op_chunk_meta(dedup_ctx* c, void* stream, const uint64_t* d_i
                                  uint32_t* d_chunk_start, uint64_t* d_chunk_id,
                                  uint32_t* d_item_first_chunk) {
     if (c == nullptr) return DEDUP_EINVAL;
+    NO_MG(c);
     if (!usable(c)) return c->sticky;
     CU(cudaSetDevice(c->cfg.device));
     cudaStream_t s = static_cast<cudaStream_t>(stream);
@@ -907,6 +941,7 @@ dedup_status dedup_op_findmatch(dedup_ctx* c, void* stream, const uint8_t* d_byt
                                 uint32_t window, uint32_t max_coded, uint8_t* d_match_len,
                                 uint16_t* d_match_off) {
     if (c == nullptr) return DEDUP_EINVAL;
+    NO_MG(c);
     if (!usable(c)) return c->sticky;
     if (reinterpret_cast<uintptr_t>(d_bytes) & 15)
         return fail(c, DEDUP_EINVAL, "d_bytes must be 16-byte aligned");
@@ -933,6 +968,7 @@ dedup_status dedup_op_table_insert_lookup(dedup_ctx* c, void* stream, const uint
                                           const uint64_t* d_id, const uint32_t* d_n, uint64_t cap,
                                           uint64_t* d_first_id, uint8_t* d_is_dup) {
     if (c == nullptr) return DEDUP_EINVAL;
+    NO_MG(c);
     if (!usable(c)) return c->sticky;
     if (cap > c->chunk_cap) return fail(c, DEDUP_EINVAL, "cap larger than the ctx workspace");
     CU(cudaSetDevice(c->cfg.device));
@@ -952,6 +988,7 @@ dedup_status dedup_op_table_insert_lookup(dedup_ctx* c, void* stream, const uint
 
 dedup_status dedup_op_table_reset(dedup_ctx* c, void* stream) {
     if (c == nullptr) return DEDUP_EINVAL;
+    NO_MG(c);
     if (!usable(c)) return c->sticky;
     CU(cudaSetDevice(c->cfg.device));
     TableBuf& t = c->tables[c->cur_table];
@@ -964,6 +1001,7 @@ dedup_status dedup_op_table_reset(dedup_ctx* c, void* stream) {
 dedup_status dedup_op_table_status(dedup_ctx* c, void* stream, uint64_t* used, uint64_t* slots,
                                    int32_t* overflow) {
     if (c == nullptr) return DEDUP_EINVAL;
+    NO_MG(c);
     CU(cudaSetDevice(c->cfg.device));
     TableBuf& t = c->tables[c->cur_table];
     uint32_t st[4];
@@ -979,6 +1017,7 @@ dedup_status dedup_op_table_status(dedup_ctx* c, void* stream, uint64_t* used, u
 dedup_status dedup_op_local_combine(dedup_ctx* c, void* stream, const uint8_t* d_digest,
                                     const uint32_t* d_n, uint64_t cap, uint32_t* d_rep) {
     if (c == nullptr) return DEDUP_EINVAL;
+    NO_MG(c);
     if (!usable(c)) return c->sticky;
     if (cap > c->chunk_cap) return fail(c, DEDUP_EINVAL, "cap larger than the ctx workspace");
     if (d_rep == nullptr || (cap > 0 && (d_digest == nullptr || d_n == nullptr)))
@@ -1008,6 +1047,7 @@ dedup_status dedup_op_route(dedup_ctx* c, void* stream, const uint8_t* d_digest,
                             const uint32_t* d_rep, uint32_t num_owners, dedup_record* d_send,
                             uint32_t* d_send_off, uint32_t* d_send_pos) {
     if (c == nullptr) return DEDUP_EINVAL;
+    NO_MG(c);
     if (!usable(c)) return c->sticky;
     if (num_owners < 1 || num_owners > 64) return fail(c, DEDUP_EINVAL, "num_owners in 1..64");
     CU(cudaSetDevice(c->cfg.device));
@@ -1021,6 +1061,7 @@ dedup_status dedup_op_route(dedup_ctx* c, void* stream, const uint8_t* d_digest,
 dedup_status dedup_op_owner(dedup_ctx* c, void* stream, const dedup_record* d_recv,
                             uint64_t n_recv, uint64_t* d_reply) {
     if (c == nullptr) return DEDUP_EINVAL;
+    NO_MG(c);
     if (!usable(c)) return c->sticky;
     if (n_recv > c->chunk_cap) return fail(c, DEDUP_EINVAL, "n_recv larger than the workspace");
     CU(cudaSetDevice(c->cfg.device));
@@ -1046,6 +1087,7 @@ dedup_status dedup_op_scatter(dedup_ctx* c, void* stream, const uint64_t* d_repl
                               const uint64_t* d_id, const uint32_t* d_n, uint64_t cap,
                               uint64_t* d_first_id, uint8_t* d_is_dup) {
     if (c == nullptr) return DEDUP_EINVAL;
+    NO_MG(c);
     if (!usable(c)) return c->sticky;
     CU(cudaSetDevice(c->cfg.device));
     launch_scatter(d_reply_back, d_send_pos, d_rep, d_id, d_n, cap, d_first_id, d_is_dup,

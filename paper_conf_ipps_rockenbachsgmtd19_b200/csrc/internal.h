@@ -42,6 +42,31 @@ struct alignas(64) BatchDesc {
 // tma_rows = 0 if the driver cannot encode it, the scan then uses LDG).
 bool encode_scan_tmap(BatchDesc& d);
 
+// ---- product-side Rabin tables (independent of the oracle) ---------------
+// P(t) = t^32 + poly over GF(2); tab[b] = R[b] = b t^32 mod P (reduction of
+// the byte shifted out of the top), tab[256 + b] = W256[b] = b t^256 mod P
+// (the byte leaving the 32-byte window, applied after the shift).
+inline uint32_t gf2_mul_tk(uint32_t x, unsigned k, uint32_t poly) {
+    while (k--) x = (x & 0x80000000u) ? ((x << 1) ^ poly) : (x << 1);
+    return x;
+}
+inline void rabin_tables(uint32_t poly, uint32_t tab[512]) {
+    for (uint32_t b = 0; b < 256; ++b) {
+        tab[b] = gf2_mul_tk(b, 32, poly);
+        tab[256 + b] = gf2_mul_tk(b, 256, poly);
+    }
+}
+
+// Chunks at least this long are hashed first (longest-processing-time-first):
+// 4x the mean anchor distance, clamped to [kMinLongBytes, 1 MiB].
+constexpr uint32_t kMinLongBytes = 1024;
+inline uint32_t long_chunk_bytes(uint32_t anchor_mask) {
+    uint64_t v = 4ull * ((uint64_t)anchor_mask + 1);
+    if (v < kMinLongBytes) v = kMinLongBytes;
+    if (v > (1u << 20)) v = 1u << 20;
+    return (uint32_t)v;
+}
+
 // ---- chunking (rabin.cu) --------------------------------------------------
 // Positions per cut-selection tile (e-space), words of the candidate bitmap.
 constexpr uint32_t kSelTile = 8192;
@@ -99,7 +124,6 @@ void launch_chunk_meta(const BatchDesc* d, const uint32_t* cut_pos, const uint32
 // ---- SHA-1 (sha1.cu) -------------------------------------------------------
 // counters: 2 words of scratch (work counter, long-chunk count); long_list:
 // capacity nbytes / kMinLongBytes + 2.
-constexpr uint32_t kMinLongBytes = 1024;
 // max_bytes: largest nbytes this launch may see (grid sizing).
 void launch_sha1(const BatchDesc* d, uint64_t max_bytes, const uint32_t* cut_pos,
                  const uint32_t* n_chunks, uint64_t cap, uint32_t long_bytes, uint32_t* counters,
@@ -125,9 +149,21 @@ void launch_table_lookup(const TableView* tv, const uint64_t* id, const void* re
 void launch_route(const uint8_t* digest, const uint64_t* id, const uint32_t* d_n, uint64_t cap,
                   const uint32_t* rep, uint32_t num_owners, void* send, uint32_t* send_off,
                   uint32_t* send_pos, uint32_t* scratch_counts, int num_sms, cudaStream_t s);
+// overflow (optional): set to 1 if a reply is ~0 (the owner's shard overflowed)
 void launch_scatter(const uint64_t* reply, const uint32_t* send_pos, const uint32_t* rep,
                     const uint64_t* id, const uint32_t* d_n, uint64_t cap, uint64_t* first_id,
-                    uint8_t* is_dup, int num_sms, cudaStream_t s);
+                    uint8_t* is_dup, int num_sms, cudaStream_t s, uint32_t* overflow = nullptr);
+// Copy exchange of the multi-GPU engine (mg.cpp): rank `me` pulls rows
+// [src_off[s][me], src_off[s][me+1]) of src[s] for every rank s (pointer
+// arrays in device memory) to dst_off[s] or, without dst_off, to the prefix
+// of the counts, which is written to out_off[0..G].
+void launch_gather_rows(const uint8_t* const* src, const uint32_t* const* src_off, uint32_t me,
+                        uint32_t G, uint32_t row_bytes, uint8_t* dst, const uint32_t* dst_off,
+                        uint32_t* out_off, uint64_t max_rows_per_src, int num_sms,
+                        cudaStream_t s);
+// cnt[2s], cnt[2s+1] = src_off[s][me], src_off[s][me+1]
+void launch_gather_counts(const uint32_t* const* src_off, uint32_t me, uint32_t G, uint32_t* cnt,
+                          cudaStream_t s);
 // Row A5 local combine: rep[r] = smallest record index with digest r's digest,
 // through the (empty) local table `local` (*d_local: the same view in device
 // memory); the used slots are cleared again afterwards.

@@ -30,6 +30,8 @@
 // if its 32-byte window lies inside one item.
 #include <cuda.h>
 #include <cuda_runtime.h>
+
+#include <mutex>
 #include <stdint.h>
 
 #include "internal.h"
@@ -895,9 +897,17 @@ uint64_t select_groups(uint64_t max_tiles) { return (max_tiles + kGroup - 1) / k
 uint64_t event_words(uint64_t max_tiles) { return max_tiles * kEvWords; }
 
 namespace {
+// Function attributes are per device: set once for every device this process
+// launches the chunker on (the multi-GPU engine drives several from worker
+// threads).
 void chunk_set_attrs() {
-    static bool attr_set = false;
-    if (attr_set) return;
+    static std::mutex mu;
+    static uint64_t done_mask = 0;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    const uint64_t bit = 1ull << (dev & 63);
+    std::lock_guard<std::mutex> lock(mu);
+    if (done_mask & bit) return;
     for (const void* f : {(const void*)rabin_scan_agg2_kernel<true, false>,
                           (const void*)rabin_scan_agg2_kernel<false, false>})
         cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
@@ -907,7 +917,7 @@ void chunk_set_attrs() {
             cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmemTma);
     cudaFuncSetAttribute(select_emit_ev_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)sizeof(EmitEvSmem));
-    attr_set = true;
+    done_mask |= bit;
 }
 }  // namespace
 

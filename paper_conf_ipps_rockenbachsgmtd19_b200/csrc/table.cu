@@ -223,14 +223,60 @@ __global__ void scatter_kernel(const uint64_t* __restrict__ reply,
                                const uint32_t* __restrict__ send_pos,
                                const uint32_t* __restrict__ rep,
                                const uint64_t* __restrict__ id, const uint32_t* d_n, uint64_t cap,
-                               uint64_t* __restrict__ first_id, uint8_t* __restrict__ is_dup) {
+                               uint64_t* __restrict__ first_id, uint8_t* __restrict__ is_dup,
+                               uint32_t* overflow) {
     const uint64_t n = min((uint64_t)*d_n, cap);
+    bool bad = false;
     for (uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; r < n;
          r += (uint64_t)gridDim.x * blockDim.x) {
         // with local combine a chunk takes the reply of its representative
         const uint64_t f = reply[send_pos[rep != nullptr ? rep[r] : (uint32_t)r]];
         first_id[r] = f;
         if (is_dup != nullptr) is_dup[r] = (f != id[r]) ? 1 : 0;
+        bad |= f == ~0ull;  // the owner's shard overflowed (table_lookup_kernel)
+    }
+    if (overflow != nullptr && bad) atomicExch(overflow, 1u);
+}
+
+// Copy exchange (the in-process transport of the multi-GPU engine, mg.cpp):
+// rank `me` pulls its rows from every rank s.  Source s's rows for `me` are
+// rows [src_off[s][me], src_off[s][me + 1]) of src[s] (row_bytes each, a
+// multiple of 8); they land at dst_off[s] (if given) or at the prefix of
+// the counts over s, which is then written to out_off[0..G] (out_off[G] =
+// total rows).  One CTA group per source; peer pointers are device memory
+// of this GPU or of a peer GPU with peer access enabled (NVLink).
+__global__ void gather_rows_kernel(const uint8_t* const* __restrict__ src,
+                                   const uint32_t* const* __restrict__ src_off, uint32_t me,
+                                   uint32_t G, uint32_t row_bytes, uint8_t* __restrict__ dst,
+                                   const uint32_t* __restrict__ dst_off,
+                                   uint32_t* __restrict__ out_off) {
+    const uint32_t s = blockIdx.y;
+    uint64_t base = 0;
+    if (dst_off != nullptr) {
+        base = dst_off[s];
+    } else {
+        for (uint32_t q = 0; q < s; ++q) base += src_off[q][me + 1] - src_off[q][me];
+        if (blockIdx.x == 0 && threadIdx.x == 0) {
+            out_off[s] = (uint32_t)base;
+            if (s == G - 1) out_off[G] = (uint32_t)(base + src_off[s][me + 1] - src_off[s][me]);
+        }
+    }
+    const uint32_t b = src_off[s][me], e = src_off[s][me + 1];
+    const uint64_t words = (uint64_t)(e - b) * (row_bytes / 8);
+    const uint64_t* __restrict__ sp =
+        reinterpret_cast<const uint64_t*>(src[s] + (uint64_t)b * row_bytes);
+    uint64_t* __restrict__ dp = reinterpret_cast<uint64_t*>(dst + base * row_bytes);
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < words;
+         i += (uint64_t)gridDim.x * blockDim.x)
+        dp[i] = sp[i];
+}
+
+// counts: cnt[2 s], cnt[2 s + 1] = rank s's send_off[me], send_off[me + 1]
+__global__ void gather_counts_kernel(const uint32_t* const* __restrict__ src_off, uint32_t me,
+                                     uint32_t G, uint32_t* __restrict__ cnt) {
+    for (uint32_t s = threadIdx.x; s < G; s += blockDim.x) {
+        cnt[2 * s] = src_off[s][me];
+        cnt[2 * s + 1] = src_off[s][me + 1];
     }
 }
 
@@ -345,10 +391,28 @@ void launch_route(const uint8_t* digest, const uint64_t* id, const uint32_t* d_n
 
 void launch_scatter(const uint64_t* reply, const uint32_t* send_pos, const uint32_t* rep,
                     const uint64_t* id, const uint32_t* d_n, uint64_t cap, uint64_t* first_id,
-                    uint8_t* is_dup, int num_sms, cudaStream_t s) {
+                    uint8_t* is_dup, int num_sms, cudaStream_t s, uint32_t* overflow) {
     if (cap == 0) return;
     scatter_kernel<<<grid_for(cap, 256, num_sms, 8), 256, 0, s>>>(reply, send_pos, rep, id, d_n,
-                                                                  cap, first_id, is_dup);
+                                                                  cap, first_id, is_dup, overflow);
+}
+
+void launch_gather_rows(const uint8_t* const* src, const uint32_t* const* src_off, uint32_t me,
+                        uint32_t G, uint32_t row_bytes, uint8_t* dst, const uint32_t* dst_off,
+                        uint32_t* out_off, uint64_t max_rows_per_src, int num_sms,
+                        cudaStream_t s) {
+    const uint64_t words = max_rows_per_src * (row_bytes / 8);
+    uint64_t bx = (words + 255) / 256;
+    const uint64_t mx = (uint64_t)num_sms * 4 / G + 1;
+    if (bx > mx) bx = mx;
+    if (bx < 1) bx = 1;
+    gather_rows_kernel<<<dim3((unsigned)bx, G), 256, 0, s>>>(src, src_off, me, G, row_bytes, dst,
+                                                             dst_off, out_off);
+}
+
+void launch_gather_counts(const uint32_t* const* src_off, uint32_t me, uint32_t G, uint32_t* cnt,
+                          cudaStream_t s) {
+    gather_counts_kernel<<<1, 64, 0, s>>>(src_off, me, G, cnt);
 }
 
 void launch_local_combine(TableView local, const uint8_t* digest, const uint32_t* d_n,

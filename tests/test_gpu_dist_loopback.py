@@ -1,8 +1,7 @@
-"""GPU parity of the multi-GPU routing (rows A5-A8) on ONE GPU: G logical
-ranks, each a ctx owning one digest-table shard (owner_rank r of G), run the
-real route / owner / scatter kernels; the all-to-all is replaced by
-in-process tensor copies (dist.loopback_all_to_all).  Results must equal the
-sequential oracle bit for bit, for any G (grouping invariance)."""
+"""GPU tests of the routing ops (row A5: owner split by digest prefix, local
+combine) and of the one-process-per-GPU front end of the multi-GPU engine
+(dedup_dist_*, NCCL at world size 1).  The engine at G > 1 is tested in
+tests/test_gpu_mg.py (G logical ranks on one GPU, the copy transport)."""
 import numpy as np
 import pytest
 
@@ -14,50 +13,6 @@ pytestmark = pytest.mark.gpu
 torch = pytest.importorskip("torch")
 
 MiB = 1 << 20
-
-
-@pytest.mark.parametrize("G,combine", [(1, True), (2, True), (4, True), (2, False), (4, False)])
-def test_loopback_routing_matches_oracle(G, combine):
-    assert torch.cuda.is_available()
-    from paper_conf_ipps_rockenbachsgmtd19_b200 import Dedup
-    from paper_conf_ipps_rockenbachsgmtd19_b200 import dist as D
-    data = U.stream(10 * MiB, seed=41 + G, dup_frac=0.6)
-    off = synthgen.split_items(data, MiB // 2)
-    n_items = len(off) - 1
-    per_batch = 3
-    batches = [(k, min(k + per_batch, n_items)) for k in range(0, n_items, per_batch)]
-    dev = torch.from_numpy(data).cuda()
-    cuda = torch.device("cuda", 0)
-    bbytes = per_batch * MiB // 2
-    ctxs = [Dedup(0, batch_bytes=bbytes, batch_items=per_batch + 1, slots=1,
-                  table_capacity=1 << 16, host_fed=False, owner_rank=r, num_owners=G)
-            for r in range(G)]
-    try:
-        states = [D.RankState(c, bbytes, per_batch + 1, cuda, G, combine=combine) for c in ctxs]
-        got = []
-        for w in range(0, len(batches), G):
-            work = []
-            for r in range(G):
-                b = w + r
-                if b < len(batches):
-                    k, j = batches[b]
-                    work.append((dev[int(off[k]):int(off[j])], off[k:j + 1] - off[k], k))
-                else:
-                    work.append((dev[:0], np.zeros(1, np.uint64), n_items))
-            for res in D.loopback_waves(states, work):
-                got.extend(res.items())
-        torch.cuda.synchronize()
-    finally:
-        for c in ctxs:
-            c.close()
-    got.sort(key=lambda r: r[0])
-    want, _ = oracle.dedup_items([data[int(off[k]):int(off[k + 1])] for k in range(n_items)])
-    assert [g[0] for g in got] == [w.seq for w in want]
-    for (seq, cs, dg, dup, fid), w in zip(got, want):
-        assert np.array_equal(cs, w.chunk_start), seq
-        assert np.array_equal(dg, w.digest), seq
-        assert np.array_equal(dup, w.is_dup), seq
-        assert np.array_equal(fid, w.first_id), seq
 
 
 def test_route_owner_split_is_by_digest_prefix():
@@ -115,120 +70,16 @@ def test_local_combine_representatives():
             assert ovf == 0
 
 
-def test_combined_routing_sends_one_record_per_digest():
-    """All-duplicate stream (C5b-like): with the local combine each wave sends
-    one record per distinct digest, and results still match the oracle."""
-    from paper_conf_ipps_rockenbachsgmtd19_b200 import Dedup
-    from paper_conf_ipps_rockenbachsgmtd19_b200 import dist as D
-    item = U.stream(MiB // 2, seed=77, dup_frac=0.0)
-    data = np.tile(item, 8)
-    off = synthgen.split_items(data, MiB // 2)
-    n_items = len(off) - 1
-    G = 2
-    dev = torch.from_numpy(data).cuda()
-    cuda = torch.device("cuda", 0)
-    bbytes = 2 * MiB
-    ctxs = [Dedup(0, batch_bytes=bbytes, batch_items=5, slots=1, table_capacity=1 << 14,
-                  host_fed=False, owner_rank=r, num_owners=G) for r in range(G)]
-    try:
-        states = [D.RankState(c, bbytes, 5, cuda, G) for c in ctxs]
-        got, sent, chunks = [], 0, 0
-        for w in range(0, n_items, 2 * G):
-            work = []
-            for r in range(G):
-                k = w + 2 * r
-                j = min(k + 2, n_items)
-                work.append((dev[int(off[k]):int(off[j])], off[k:j + 1] - off[k], k))
-            for st, res in zip(states, D.loopback_waves(states, work)):
-                got.extend(res.items())
-                sent += st.sent_records
-                chunks += len(res.chunk_start)
-        torch.cuda.synchronize()
-    finally:
-        for c in ctxs:
-            c.close()
-    want, _ = oracle.dedup_items([data[int(off[k]):int(off[k + 1])] for k in range(n_items)])
-    distinct_per_item = len({bytes(x) for x in want[0].digest})
-    assert sent == (n_items // 2) * distinct_per_item  # one record per digest per batch
-    assert sent < chunks
-    got.sort(key=lambda r: r[0])
-    for (seq, cs, dg, dup, fid), w in zip(got, want):
-        assert np.array_equal(cs, w.chunk_start), seq
-        assert np.array_equal(dup, w.is_dup), seq
-        assert np.array_equal(fid, w.first_id), seq
-
-
-@pytest.mark.parametrize("G,depth", [(1, 3), (2, 3), (3, 2)])
-def test_wave_pipeline_matches_oracle(G, depth):
-    """dist.WavePipeline (waves in flight on their own streams, exchange on
-    the owner streams) with G logical ranks on one GPU: bit-exact vs the
-    sequential oracle, across an end_stream (fresh tables)."""
-    assert torch.cuda.is_available()
-    from paper_conf_ipps_rockenbachsgmtd19_b200 import Dedup
-    from paper_conf_ipps_rockenbachsgmtd19_b200 import dist as D
-    data = U.stream(12 * MiB, seed=61 + G, dup_frac=0.6)
-    off = synthgen.split_items(data, MiB // 2)
-    n_items = len(off) - 1
-    per_batch = 2
-    bbytes = per_batch * MiB // 2
-    batches = [(k, min(k + per_batch, n_items)) for k in range(0, n_items, per_batch)]
-    dev = torch.from_numpy(data).cuda()
-    owners = [Dedup(0, batch_bytes=G * bbytes, batch_items=1, slots=1, table_capacity=1 << 16,
-                    host_fed=False, owner_rank=r, num_owners=G) for r in range(G)]
-    pipe = D.WavePipeline(D.LoopbackExchange(), owners, 0, bbytes, per_batch + 1, depth=depth)
-    split = len(batches) // 2            # stream 1: batches [0, split), stream 2: the rest
-    got = [[], []]
-    try:
-        def take(outs, sid):
-            for wave in outs:
-                for o in wave:
-                    got[sid].extend(o.items())
-        for sid, (lo, hi) in enumerate(((0, split), (split, len(batches)))):
-            if sid:
-                take(pipe.end_stream(), 0)
-            for w in range(lo, hi, G):
-                work = []
-                for r in range(G):
-                    b = w + r
-                    if b < hi:
-                        k, j = batches[b]
-                        work.append((dev[int(off[k]):int(off[j])], off[k:j + 1] - off[k], k))
-                    else:
-                        work.append((dev[:0], np.zeros(1, np.uint64), n_items + r))
-                take(pipe.submit(work), sid)
-        take(pipe.flush(), 1)
-        torch.cuda.synchronize()
-    finally:
-        pipe.close()
-        for o in owners:
-            o.close()
-    for sid, (lo, hi) in enumerate(((0, split), (split, len(batches)))):
-        k0, k1 = batches[lo][0], batches[hi - 1][1]
-        res = sorted((g for g in got[sid] if g[0] < n_items), key=lambda r: r[0])
-        want, _ = oracle.dedup_items([data[int(off[k]):int(off[k + 1])] for k in range(k0, k1)],
-                                     first_seq=k0)
-        assert [g[0] for g in res] == [w.seq for w in want]
-        for (seq, cs, dg, dup, fid), w in zip(res, want):
-            assert np.array_equal(cs, w.chunk_start), seq
-            assert np.array_equal(dg, w.digest), seq
-            assert np.array_equal(dup, w.is_dup), seq
-            assert np.array_equal(fid, w.first_id), seq
-
-
-@pytest.mark.parametrize("early", ["0", "1"])
 @pytest.mark.parametrize("drain", [True, False])
 @pytest.mark.parametrize("depth", [1, 3])
-def test_native_wave_pipeline_world1(depth, drain, early, monkeypatch):
-    """The C++ wave pipeline (csrc/dist.cpp) through NCCL with one rank: the
-    exchange sends every record to itself.  Three dedup streams: the first
-    half of the batches, the second half, then the first half again from the
-    same device buffers (the local phase replays its captured CUDA graphs);
-    bit-exact vs the oracle each time.  drain=False: end_stream with waves in
-    flight (the table reset deferred to the next stream's first wave);
-    early: counts exchanged right behind the local rows on their own
-    communicator (DEDUP_DIST_EARLY_COUNTS)."""
+def test_native_wave_pipeline_world1(depth, drain):
+    """The one-process-per-GPU front end of the multi-GPU engine (csrc/mg.cpp,
+    dedup_dist_*) through NCCL with one rank: the exchange sends every record
+    to itself.  Three dedup streams: the first half of the batches, the second
+    half, then the first half again from the same device buffers; bit-exact vs
+    the oracle each time.  drain=False: end_stream with waves in flight (the
+    table reset deferred to the next stream's first wave)."""
     assert torch.cuda.is_available()
-    monkeypatch.setenv("DEDUP_DIST_EARLY_COUNTS", early)
     from paper_conf_ipps_rockenbachsgmtd19_b200 import dist as D
     data = U.stream(10 * MiB, seed=71 + depth, dup_frac=0.6)
     off = synthgen.split_items(data, MiB // 2)
@@ -320,3 +171,52 @@ def test_native_wave_pipeline_deferred_resets(depth):
             assert np.array_equal(dg, w.digest), seq
             assert np.array_equal(dup, w.is_dup), seq
             assert np.array_equal(fid, w.first_id), seq
+
+
+def test_native_wave_pipeline_rejects_bad_offsets_before_enqueue():
+    """Argument checks run before anything is enqueued: a bad
+    offset array is EINVAL and the pipeline still works afterwards."""
+    from paper_conf_ipps_rockenbachsgmtd19_b200 import dist as D
+    from paper_conf_ipps_rockenbachsgmtd19_b200._native import DedupError
+    data = U.stream(2 * MiB, seed=5, dup_frac=0.3)
+    off = synthgen.split_items(data, MiB // 2)
+    dev = torch.from_numpy(data).cuda()
+    pipe = D.NativeWavePipeline(D.nccl_unique_id(), 1, 0, 0, 2 * MiB, 8, 1 << 14, depth=2)
+    try:
+        bad = off.copy()
+        bad[1], bad[2] = bad[2], bad[1]          # decreasing
+        with pytest.raises(DedupError, match="EINVAL"):
+            pipe.submit([(dev, bad, 0)])
+        with pytest.raises(DedupError, match="EINVAL"):
+            pipe.submit([(dev, off + np.uint64(1), 0)])   # item_off[0] != 0
+        got = []
+        for outs in (pipe.submit([(dev, off, 0)]), pipe.flush()):
+            for wave in outs:
+                for o in wave:
+                    got.extend(o.items())
+    finally:
+        pipe.close()
+    want, _ = oracle.dedup_items([data[int(off[k]):int(off[k + 1])] for k in range(len(off) - 1)])
+    assert [g[0] for g in got] == [w.seq for w in want]
+    for (seq, cs, dg, dup, fid), w in zip(got, want):
+        assert np.array_equal(cs, w.chunk_start) and np.array_equal(fid, w.first_id), seq
+
+
+def test_native_wave_pipeline_table_overflow_is_sticky():
+    """A full owner shard is reported, not silently turned into wrong dup
+    flags: DEDUP_ETABLEFULL, and it stays."""
+    from paper_conf_ipps_rockenbachsgmtd19_b200 import dist as D
+    from paper_conf_ipps_rockenbachsgmtd19_b200._native import DedupError
+    data = U.stream(4 * MiB, seed=9, dup_frac=0.0)
+    off = synthgen.split_items(data, MiB)
+    dev = torch.from_numpy(data).cuda()
+    pipe = D.NativeWavePipeline(D.nccl_unique_id(), 1, 0, 0, 4 * MiB, 8, 16, depth=1)
+    try:
+        with pytest.raises(DedupError, match="ETABLEFULL"):
+            pipe.submit([(dev, off, 0)])
+            for _ in range(2):
+                pipe.flush()
+        with pytest.raises(DedupError, match="ETABLEFULL"):
+            pipe.submit([(dev, off, 100)])
+    finally:
+        pipe.close()
