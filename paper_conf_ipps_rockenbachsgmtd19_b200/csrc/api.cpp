@@ -46,7 +46,7 @@ struct Workspace {
     uint32_t* evbuf = nullptr;       // per-tile event lists (scan -> cut emission)
     uint32_t* counters = nullptr;    // [0..1] sha1 work/long counters, [64..191] route
     uint32_t* slot_idx = nullptr;    // table slot per record
-    uint32_t* long_list = nullptr;   // SHA-1 long-chunk list
+    uint32_t* sha_ws = nullptr;      // SHA-1 sort of the chunks by length + task counter
     uint32_t* mc_ws = nullptr;       // max_chunk selection scratch (maxchunk_ws_words)
     uint64_t max_tiles = 0;
     uint64_t item_cap = 0;           // items the max_chunk scratch holds
@@ -188,7 +188,7 @@ dedup_status ws_alloc(dedup_ctx* c, Workspace& w, uint64_t batch_bytes, uint64_t
     TRY(dalloc(c, &w.evbuf, event_words(w.max_tiles)));
     TRY(dalloc(c, &w.counters, 256));
     TRY(dalloc(c, &w.slot_idx, cap));
-    TRY(dalloc(c, &w.long_list, batch_bytes / kMinLongBytes + 2));
+    TRY(dalloc(c, &w.sha_ws, sha1_ws_words(cap)));
     if (c->cfg.max_chunk || c->cfg.min_chunk != 32) {
         w.item_cap = cap;
         TRY(dalloc(c, &w.mc_ws, maxchunk_ws_words(cap, w.item_cap)));
@@ -205,7 +205,7 @@ void ws_free(Workspace& w) {
     cudaFree(w.evbuf);
     cudaFree(w.counters);
     cudaFree(w.slot_idx);
-    cudaFree(w.long_list);
+    cudaFree(w.sha_ws);
     cudaFree(w.mc_ws);
     w = Workspace{};
 }
@@ -224,8 +224,6 @@ bool usable(const dedup_ctx* c) { return c != nullptr && c->sticky == DEDUP_OK; 
 #ifndef DEDUP_ATTRIB_SKIP
 #define DEDUP_ATTRIB_SKIP 0
 #endif
-
-uint32_t long_bytes(const dedup_ctx* c) { return long_chunk_bytes(c->cfg.anchor_mask); }
 
 TableView table_view(const dedup_ctx* c) {
     const TableBuf& t = c->tables[c->cur_table];
@@ -249,8 +247,8 @@ void enqueue_chunk_sha(dedup_ctx* c, Workspace& w, cudaStream_t s, const BatchDe
                           max_items, c->num_sms, s);
     if (ev_chunk) cudaEventRecordWithFlags(ev_chunk, s, cudaEventRecordExternal);
     if (digest && !(DEDUP_ATTRIB_SKIP & 1))
-        launch_sha1(d, max_bytes, cut_pos, n_chunks, cap, long_bytes(c), w.counters,
-                    w.long_list, digest, c->num_sms, s, c->cfg.sha_lane_bytes);
+        launch_sha1(d, max_bytes, cut_pos, n_chunks, cap, w.sha_ws, digest, c->num_sms, s,
+                    c->cfg.sha_lane_bytes);
 }
 
 // Records the per-batch graph of slot i (capture of the slot's stream).
@@ -928,8 +926,9 @@ dedup_status dedup_op_sha1(dedup_ctx* c, void* stream, const uint8_t* d_bytes, u
     h.nbytes = nbytes;
     const BatchDesc* d = nullptr;
     TRY(op_desc(c, s, h, &d));
-    launch_sha1(d, nbytes, d_cut_pos, d_n_chunks, cap, long_bytes(c), c->op_ws.counters,
-                c->op_ws.long_list, d_digest, c->num_sms, s, c->cfg.sha_lane_bytes);
+    if (cap > c->chunk_cap) return fail(c, DEDUP_EINVAL, "cap larger than the ctx workspace");
+    launch_sha1(d, nbytes, d_cut_pos, d_n_chunks, cap, c->op_ws.sha_ws, d_digest, c->num_sms, s,
+                c->cfg.sha_lane_bytes);
     c->launches += 2;
     CU(cudaGetLastError());
     return DEDUP_OK;

@@ -57,16 +57,6 @@ inline void rabin_tables(uint32_t poly, uint32_t tab[512]) {
     }
 }
 
-// Chunks at least this long are hashed first (longest-processing-time-first):
-// 4x the mean anchor distance, clamped to [kMinLongBytes, 1 MiB].
-constexpr uint32_t kMinLongBytes = 1024;
-inline uint32_t long_chunk_bytes(uint32_t anchor_mask) {
-    uint64_t v = 4ull * ((uint64_t)anchor_mask + 1);
-    if (v < kMinLongBytes) v = kMinLongBytes;
-    if (v > (1u << 20)) v = 1u << 20;
-    return (uint32_t)v;
-}
-
 // ---- chunking (rabin.cu) --------------------------------------------------
 // Positions per cut-selection tile (e-space), words of the candidate bitmap.
 constexpr uint32_t kSelTile = 8192;
@@ -122,13 +112,13 @@ void launch_chunk_meta(const BatchDesc* d, const uint32_t* cut_pos, const uint32
                        cudaStream_t s);
 
 // ---- SHA-1 (sha1.cu) -------------------------------------------------------
-// counters: 2 words of scratch (work counter, long-chunk count); long_list:
-// capacity nbytes / kMinLongBytes + 2.
-// max_bytes: largest nbytes this launch may see (grid sizing).
+// ws: sha1_ws_words(cap) words of scratch (the sort of the chunks by length
+// and the warps' task counter).  max_bytes: largest nbytes this launch may see
+// (grid sizing); lane_bytes: batch bytes per SHA-1 lane (0 = 32 KiB).
+uint64_t sha1_ws_words(uint64_t cap);
 void launch_sha1(const BatchDesc* d, uint64_t max_bytes, const uint32_t* cut_pos,
-                 const uint32_t* n_chunks, uint64_t cap, uint32_t long_bytes, uint32_t* counters,
-                 uint32_t* long_list, uint8_t* digest, int num_sms, cudaStream_t s,
-                 uint32_t lane_bytes = 0);
+                 const uint32_t* n_chunks, uint64_t cap, uint32_t* ws, uint8_t* digest,
+                 int num_sms, cudaStream_t s, uint32_t lane_bytes = 0);
 
 // ---- digest table and routing (table.cu) ----------------------------------
 // Insert records then look them up.  Records come either as (digest bytes,

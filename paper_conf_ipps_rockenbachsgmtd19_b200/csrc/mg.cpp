@@ -106,7 +106,7 @@ struct Slot {
     uint8_t* d_in = nullptr;  // host-fed input
     // chunking / SHA-1 workspace (as the single-GPU engine's)
     uint32_t *bitmap = nullptr, *agg = nullptr, *gagg = nullptr, *gentry = nullptr,
-             *evbuf = nullptr, *counters = nullptr, *slot_idx = nullptr, *long_list = nullptr,
+             *evbuf = nullptr, *counters = nullptr, *slot_idx = nullptr, *sha_ws = nullptr,
              *mc_ws = nullptr;
     uint64_t max_tiles = 0, item_cap = 0;
     // per-chunk arrays
@@ -258,7 +258,7 @@ void slot_free(Slot& sl) {
         if (e) cudaEventDestroy(e);
     for (void* p : {(void*)sl.d_desc, (void*)sl.d_item_off, (void*)sl.d_in, (void*)sl.bitmap,
                     (void*)sl.agg, (void*)sl.gagg, (void*)sl.gentry, (void*)sl.evbuf,
-                    (void*)sl.counters, (void*)sl.slot_idx, (void*)sl.long_list, (void*)sl.mc_ws,
+                    (void*)sl.counters, (void*)sl.slot_idx, (void*)sl.sha_ws, (void*)sl.mc_ws,
                     (void*)sl.cut, (void*)sl.small, (void*)sl.chunk_start, (void*)sl.item_first,
                     (void*)sl.send_off, (void*)sl.send_pos, (void*)sl.rep, (void*)sl.cnt_recv,
                     (void*)sl.route_scratch, (void*)sl.chunk_id, (void*)sl.first_id,
@@ -309,8 +309,7 @@ dedup_status capture_local(Engine* E, Rank& r, Slot& sl) {
                         c.min_chunk);
     launch_chunk_meta(sl.d_desc, sl.cut, sl.small, E->cap, sl.chunk_start, sl.chunk_id,
                       sl.item_first, E->batch_items, r.num_sms, s);
-    launch_sha1(sl.d_desc, E->batch_bytes, sl.cut, sl.small, E->cap,
-                long_chunk_bytes(c.anchor_mask), sl.counters, sl.long_list, sl.digest,
+    launch_sha1(sl.d_desc, E->batch_bytes, sl.cut, sl.small, E->cap, sl.sha_ws, sl.digest,
                 r.num_sms, s, E->lane_bytes);
     const TableView lv{sl.lt, sl.lt_cap - 1, sl.lt_status};
     launch_local_combine(lv, sl.digest, sl.small, E->cap, sl.slot_idx, sl.rep, r.num_sms, s,
@@ -368,7 +367,7 @@ dedup_status slot_alloc(Engine* E, Rank& r, Slot& sl) {
     MTRY(dmalloc(E, &sl.counters, 256));
     MCU(cudaMemset(sl.counters, 0, sizeof(uint32_t) * 256));
     MTRY(dmalloc(E, &sl.slot_idx, cap));
-    MTRY(dmalloc(E, &sl.long_list, bb / kMinLongBytes + 2));
+    MTRY(dmalloc(E, &sl.sha_ws, sha1_ws_words(cap)));
     if (E->cfg.max_chunk || E->cfg.min_chunk != 32) {
         sl.item_cap = cap;
         MTRY(dmalloc(E, &sl.mc_ws, maxchunk_ws_words(cap, sl.item_cap)));

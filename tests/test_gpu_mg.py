@@ -176,10 +176,10 @@ def test_mg_join_brackets_all_work():
 def test_mg_table_overflow_is_sticky():
     """A full shard is DEDUP_ETABLEFULL (sticky), never wrong dup flags."""
     from paper_conf_ipps_rockenbachsgmtd19_b200._native import DedupError
-    data = U.stream(4 * MiB, seed=505, dup_frac=0.0)
+    data = U.stream(48 * MiB, seed=505, dup_frac=0.0)      # ~12 k distinct chunks
     off = synthgen.split_items(data, MiB // 2)
     dev = torch.from_numpy(data).cuda()
-    with mg(2, 2, table_capacity=16) as d:
+    with mg(2, 2, table_capacity=16) as d:                  # 2 shards of 4096 slots
         with pytest.raises(DedupError, match="ETABLEFULL"):
             got = []
             submit_device_batches(d, dev, off, 0, len(off) - 1, MiB, 8, got)
