@@ -393,7 +393,6 @@ dedup_status launch_batch(dedup_ctx* c, int i, const uint8_t* d_bytes) {
     d.table = table_view(c);
     c->stream_fresh = false;
     const auto t0 = std::chrono::steady_clock::now();
-    encode_scan_tmap(d);  // TMA view for the scan (tma_rows = 0: LDG path)
     CU(cudaGraphLaunch(sl.graph, sl.stream));
     c->st.ms_host_launch +=
         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
@@ -876,7 +875,6 @@ dedup_status dedup_op_chunk(dedup_ctx* c, void* stream, const uint8_t* d_bytes, 
     h.nbytes = nbytes;
     h.item_off = d_item_off;
     h.n_items = n_items;
-    encode_scan_tmap(h);
     const BatchDesc* d = nullptr;
     TRY(op_desc(c, s, h, &d));
     enqueue_chunk_sha(c, c->op_ws, s, d, nbytes, d_cut_pos, cap, d_n_chunks, nullptr, nullptr,

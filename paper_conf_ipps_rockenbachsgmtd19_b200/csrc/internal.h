@@ -30,17 +30,7 @@ struct alignas(64) BatchDesc {
     uint32_t n_items;
     uint32_t fresh;            // 1: clear the table before inserting
     TableView table;
-    // TMA view of the batch for the scan (encode_scan_tmap): bytes as a 2-D
-    // tensor of tma_rows rows x 256 B (the lane segments), 32 x 32 B boxes.
-    // tma_rows = 0: no tensor map, the scan loads with LDG.
-    uint32_t tma_rows;
-    uint32_t pad_[7];
-    alignas(64) unsigned char tmap[128];
 };
-
-// Fills d.tmap / d.tma_rows from d.bytes, d.nbytes (host; false and
-// tma_rows = 0 if the driver cannot encode it, the scan then uses LDG).
-bool encode_scan_tmap(BatchDesc& d);
 
 // ---- product-side Rabin tables (independent of the oracle) ---------------
 // P(t) = t^32 + poly over GF(2); tab[b] = R[b] = b t^32 mod P (reduction of

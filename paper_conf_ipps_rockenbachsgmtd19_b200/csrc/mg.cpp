@@ -748,7 +748,6 @@ void stage_batch(Engine* E, Slot& sl, uint64_t w, uint64_t first_seq, const uint
     d.n_items = n_items;
     d.fresh = 0;
     d.table = TableView{nullptr, 0, nullptr};
-    encode_scan_tmap(d);
     sl.busy = true;
     sl.parsed = false;
     sl.next_item = 0;

@@ -5,9 +5,9 @@
 //
 // The paper ran this on the CPU; here it is three sm_100a kernels:
 //
-//  rabin_scan_agg2_kernel  persistent, one CTA of 16 warps per SM.  A CTA
-//      takes groups of 32 tiles of 8 KiB; warp w rolls tiles w and w + 16 of
-//      the group together (two independent chains per lane, ILP 2); each lane
+//  rabin_scan_kernel  persistent, one CTA of 16 warps per SM.  A CTA takes
+//      groups of 32 tiles of 8 KiB; a warp rolls 4 tiles of a group together
+//      (four independent chains per lane, ILP 4); each lane
 //      rolls the 32-byte window hash over its 256 bytes (after a 32-byte
 //      warm-up) with the post-shift recurrence
 //          h' = ((h << 8) | in) ^ R[h >> 24] ^ W256[out]
@@ -28,7 +28,6 @@
 //      writing the cut positions (the paper's startPos).
 // Item starts are forced cuts and reset the state; a candidate is valid only
 // if its 32-byte window lies inside one item.
-#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <mutex>
@@ -40,31 +39,30 @@ namespace dd {
 
 namespace {
 
-// Scan CTA: DEDUP_SCAN_CTA_WARPS warps (64 registers each).  A select group
-// is 32 tiles rolled by 16 warps (2 tiles per warp, ILP 2); a 32-warp CTA
-// runs two groups at once (its two halves share the 64 KiB table).  Measured:
-// the 32-warp CTA scans faster alone (736 MiB chunk stage 1647 vs 1527 GB/s:
-// 16 warps x 2 chains leave the roll latency-bound) but it takes a whole SM
-// (64K registers, 220 KiB smem), and the pipelined bench is faster with 16
-// warps (590 vs 576 GB/s): other batches' SHA-1 / table / emit CTAs share the
-// SM with a 16-warp scan CTA.
+// Scan CTA: 16 warps.  A select group is 32 tiles of 8 KiB; a warp rolls
+// kChains tiles of a group together (kChains independent rolling chains per
+// lane: the PRMT -> LDS -> LOP3 dependency of one chain overlaps with the
+// others'), so kGroupWarps = 32 / kChains warps make a group and the CTA runs
+// kHalves = 16 / kGroupWarps groups at once (its halves share the 64 KiB
+// table).  One scan CTA per SM (the table is 64 KiB-aligned, see below).
 #ifndef DEDUP_SCAN_GROUPS_PER_CTA
 #define DEDUP_SCAN_GROUPS_PER_CTA 4  // select groups per scan CTA (launch_chunk_select)
 #endif
-#ifndef DEDUP_SCAN_CTA_WARPS
-#define DEDUP_SCAN_CTA_WARPS 16
+#ifndef DEDUP_SCAN_CHAINS
+#define DEDUP_SCAN_CHAINS 4
 #endif
-constexpr int kScanWarps = DEDUP_SCAN_CTA_WARPS;
+constexpr int kChains = DEDUP_SCAN_CHAINS;
+static_assert(kChains == 2 || kChains == 4, "2 or 4 chains per lane");
+constexpr int kScanWarps = 16;
 constexpr int kScanThreads = kScanWarps * 32;
-constexpr int kGroupWarps = 16;                    // warps per select group
+constexpr int kGroup = 32;                         // tiles per select group
+constexpr int kGroupWarps = kGroup / kChains;      // warps per select group
 constexpr int kHalves = kScanWarps / kGroupWarps;  // groups in flight per CTA
-static_assert(kHalves == 1 || kHalves == 2, "16 or 32 warps per scan CTA");
 constexpr int kTabBytes = 256 * 256;  // [x][R|W][lane] u32 = 64 KiB
 constexpr uint32_t kLaneBytes = kSelTile / 32;  // 256 bytes per lane per tile
 constexpr uint32_t kFull = 0xFFFFFFFFu;
 constexpr uint32_t kInf = 0xFFFFFFFFu;
 constexpr uint32_t kM27 = (1u << 27) - 1;
-constexpr int kGroup = kGroupWarps * 2;  // tiles per select group (2 per warp)
 constexpr int kItemCache = 1024;  // item offsets cached in shared memory
 
 constexpr uint32_t kListCap = 128;  // events per tile kept as a sorted list
@@ -85,7 +83,7 @@ struct SelWarpSmem {
 // assumes at least kStaticMin bytes of static smem; the kernel traps if the
 // runtime layout disagrees.
 constexpr int kScanAux = kScanWarps * (int)sizeof(SelWarpSmem) + kItemCache * 8;
-constexpr int kStaticMin = kHalves == 1 ? 8192 : 16384;
+constexpr int kStaticMin = 2048 + kHalves * 8192;  // src table + fun buffers
 constexpr bool kAuxInPad = kScanAux <= 65536 - 1024 - 10752;
 constexpr int kScanSmem = kAuxInPad ? 65536 + kTabBytes : 2 * 65536 - kStaticMin + kScanAux;
 
@@ -98,33 +96,13 @@ __device__ __forceinline__ uint32_t lds(uint32_t addr) {
     return v;
 }
 
-#ifndef DEDUP_SCAN_EXPERIMENT
-#define DEDUP_SCAN_EXPERIMENT 0  // timing experiments only (results invalid): 4 = no
-                                 // global loads in the scan, 8 = no per-tile epilogue
-#endif
-
-#ifndef DEDUP_SCAN_LDHINT
-#define DEDUP_SCAN_LDHINT 1  // 1: L1::no_allocate (measured +10 %), 2: L2::256B (no gain)
-#endif
-#if DEDUP_SCAN_LDHINT == 1
-#define DEDUP_LDV8 "ld.global.nc.L1::no_allocate.v8.u32"
-#elif DEDUP_SCAN_LDHINT == 2
-#define DEDUP_LDV8 "ld.global.nc.L2::256B.v8.u32"
-#else
-#define DEDUP_LDV8 "ld.global.nc.v8.u32"
-#endif
-
 // One 256-bit load (LDG.E.256, sm_100) of 32 bytes at a 32-byte aligned p.
 // One request per lane-sector instead of two halves the L1 tag work of the
 // lane-strided scan loads; L1::no_allocate keeps the streamed bytes out of
 // the L1 that the table lookups share.
+// (measured: the no-allocate hint +10 %.)
 __device__ __forceinline__ void ldg_v8(const uint8_t* p, uint32_t v[8]) {
-    if (DEDUP_SCAN_EXPERIMENT & 4) {
-#pragma unroll
-        for (int i = 0; i < 8; ++i) v[i] = (uint32_t)(uintptr_t)p * 2654435761u + i;
-        return;
-    }
-    asm(DEDUP_LDV8 " {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+    asm("ld.global.nc.L1::no_allocate.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
         : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]),
           "=r"(v[7])
         : "l"(p));
@@ -324,149 +302,60 @@ __device__ __forceinline__ uint32_t walk_any(const SelWarpSmem& sm, uint32_t n_e
     return walk_tile(sm, s, exit_state, out, out_base, cap, T0);
 }
 
-// Two independent rolling chains per lane (ILP 2): the LDS -> LOP3 -> PRMT
-// dependency of one chain overlaps with the other's.
-// Words [W0, W1) of the 32-byte step; bits accumulate into bitsA / bitsB.
-template <bool kZeroValue, int W0 = 0, int W1 = 8>
-__device__ __forceinline__ void roll32x2(uint32_t& hA, const uint32_t curA[8],
-                                         const uint32_t oldA[8], uint32_t& bitsA, uint32_t& hB,
-                                         const uint32_t curB[8], const uint32_t oldB[8],
-                                         uint32_t& bitsB, uint32_t laneR, uint32_t laneW,
-                                         uint32_t mask, uint32_t value) {
-    if (W0 == 0) bitsA = bitsB = 0;
+// One rolling step of kChains independent chains over words [W0, W1) of a
+// 32-byte step (post-shift recurrence h' = ((h << 8) | in) ^ R[h >> 24] ^
+// W256[out]); candidate bits accumulate in bits[c].  kMul: the anchor test
+// (h & mask) == 0 with mask = 2^k - 1 as (h * 2^(32-k)) == 0 -- the IMAD and
+// the bit insert (a predicated add) issue to the FMA pipe, leaving three
+// PRMT, one LOP3 and one ISETP per byte on the ALU pipe; otherwise
+// ((h & mask) ^ value) == 0 (one LOP3) and a predicated OR.
+template <bool kMul, int W0, int W1>
+__device__ __forceinline__ void roll_step(uint32_t (&h)[kChains], const uint32_t (&cur)[kChains][8],
+                                          const uint32_t (&old)[kChains][8],
+                                          uint32_t (&bits)[kChains], uint32_t laneR,
+                                          uint32_t laneW, uint32_t mask, uint32_t value,
+                                          uint32_t mul) {
+    if (W0 == 0) {
+#pragma unroll
+        for (int c = 0; c < kChains; ++c) bits[c] = 0;
+    }
 #pragma unroll
     for (int w = W0; w < W1; ++w) {
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
-            const uint32_t aRA = __byte_perm(hA, laneR, 0x7634);
-            const uint32_t aRB = __byte_perm(hB, laneR, 0x7634);
-            const uint32_t aWA = __byte_perm(oldA[w], laneW, 0x7604 | (k << 4));
-            const uint32_t aWB = __byte_perm(oldB[w], laneW, 0x7604 | (k << 4));
-            const uint32_t hsA = __byte_perm(curA[w], hA, 0x6540 | k);
-            const uint32_t hsB = __byte_perm(curB[w], hB, 0x6540 | k);
-            hA = hsA ^ lds(aRA) ^ lds(aWA);
-            hB = hsB ^ lds(aRB) ^ lds(aWB);
-            const uint32_t tA = kZeroValue ? (hA & mask) : ((hA & mask) ^ value);
-            const uint32_t tB = kZeroValue ? (hB & mask) : ((hB & mask) ^ value);
-            asm("{\n\t.reg .pred p;\n\tsetp.eq.u32 p, %1, 0;\n\t@p or.b32 %0, %0, %2;\n\t}"
-                : "+r"(bitsA)
-                : "r"(tA), "r"(1u << (4 * w + k)));
-            asm("{\n\t.reg .pred p;\n\tsetp.eq.u32 p, %1, 0;\n\t@p or.b32 %0, %0, %2;\n\t}"
-                : "+r"(bitsB)
-                : "r"(tB), "r"(1u << (4 * w + k)));
+#pragma unroll
+            for (int c = 0; c < kChains; ++c) {
+                const uint32_t aR = __byte_perm(h[c], laneR, 0x7634);
+                const uint32_t aW = __byte_perm(old[c][w], laneW, 0x7604 | (k << 4));
+                const uint32_t hs = __byte_perm(cur[c][w], h[c], 0x6540 | k);
+                h[c] = hs ^ lds(aR) ^ lds(aW);
+                if (kMul) {
+                    asm("{\n\t.reg .pred p;\n\t.reg .u32 t;\n\tmul.lo.u32 t, %1, %2;\n\t"
+                        "setp.eq.u32 p, t, 0;\n\t@p add.u32 %0, %0, %3;\n\t}"
+                        : "+r"(bits[c])
+                        : "r"(h[c]), "r"(mul), "r"(1u << (4 * w + k)));
+                } else {
+                    const uint32_t t = (h[c] & mask) ^ value;
+                    asm("{\n\t.reg .pred p;\n\tsetp.eq.u32 p, %1, 0;\n\t@p or.b32 %0, %0, %2;\n\t}"
+                        : "+r"(bits[c])
+                        : "r"(t), "r"(1u << (4 * w + k)));
+                }
+            }
         }
     }
 }
 
-// L2 prefetch of tile t's bytes (and the 32 warm-up bytes before it) by the
-// TMA unit: one bulk request per tile, no registers, issued a whole group
-// ahead so that the per-step loads of the roll hit L2 instead of HBM.
-__device__ __forceinline__ void prefetch_tile_l2(const uint8_t* bytes, uint64_t t,
-                                                 uint64_t lim16) {
-    uint64_t a = t * kSelTile;
-    if (a >= lim16) return;
-    a = a >= 32 ? a - 32 : 0;
-    uint64_t n = kSelTile + 32;
-    if (a + n > lim16) n = lim16 - a;
-    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(bytes + a), "r"((uint32_t)n)
-                 : "memory");
-}
-
-// L1 prefetch of the next group's first bytes per lane (the group-start
-// loads stall the whole CTA: ~7 % of the scan's stall samples).  Measured:
-// isolated chunk stage 1357 -> 1270 GB/s, bench 742 -> 725: off.
-#ifndef DEDUP_SCAN_L1PF
-#define DEDUP_SCAN_L1PF 0
+// Persistent scan: a CTA of kScanWarps warps takes groups of 32 tiles; warp
+// hw of a group rolls its tiles hw + kGroupWarps * c (c < kChains) together.
+#ifndef DEDUP_SCAN_MAXREG
+#define DEDUP_SCAN_MAXREG 96
 #endif
-__device__ __forceinline__ void prefetch_l1(const uint8_t* p) {
-    asm volatile("prefetch.global.L1 [%0];" ::"l"(p));
-}
-
-// Measured (isolated chunk stage, 256 MiB of C2-like data): next-step loads
-// issued one step ahead into the recycled registers 949 GB/s (none: 938);
-// one LDG.E.256 per step instead of two LDG.128: 996; an L2 bulk prefetch of
-// the next group's tiles: slightly slower (899 / 938), off.
-#ifndef DEDUP_SCAN_L2PF
-#define DEDUP_SCAN_L2PF 0
-#endif
-
-// ---- TMA staging of the scan's input (kTma) ----------------------------------
-// The lane-strided LDGs of the scan (32 lanes x 32 B at a 256 B stride per
-// step) cost 32 L1 tag lookups per warp instruction and contend with the
-// table LDS in the L1/shared pipeline (ncu: short-scoreboard stalls 0.4 -> 2.9
-// per issue when the loads are present; the scan without loads is 39 %
-// faster).  With kTma one lane per warp asks the TMA unit for the next steps'
-// 32 rows x 32 B boxes (2-D tensor map: rows = lane segments of 256 B) into a
-// per-warp ring of kScanStages shared-memory stages, and the lanes read their
-// rows with two conflict-free LDS.128 (SWIZZLE_32B: the 16-byte halves of row
-// r are swapped when bit 2 of r is set, so 8 consecutive lanes cover all 32
-// banks).  Tiles whose rows are not all inside the tensor (the batch's ragged
-// end) keep the LDG path.
-#ifndef DEDUP_SCAN_TMA
-#define DEDUP_SCAN_TMA 0
-#endif
-#if DEDUP_SCAN_TMA && DEDUP_SCAN_CTA_WARPS != 16
-#error "the TMA ring fits the shared memory of a 16-warp scan CTA only"
-#endif
-#ifndef DEDUP_SCAN_STAGES
-#define DEDUP_SCAN_STAGES 3
-#endif
-constexpr int kScanStages = DEDUP_SCAN_STAGES;
-constexpr int kBoxBytes = 32 * 32;                 // one step of 32 lane rows
-constexpr int kUnitsPerTile = 1 + kLaneBytes / 32;  // warm-up box + 8 steps
-constexpr int kRingBytes = kScanWarps * kScanStages * 2 * kBoxBytes;
-// dynamic smem: [pad to the 64 KiB boundary (aux)][table 64 KiB][ring].  The
-// pad is 64 KiB minus the static smem (~10.4 KiB), so 10 KiB less than the
-// worst case is requested (the kernel traps if the runtime layout disagrees).
-constexpr int kScanSmemTma = 2 * 65536 - 10240 + kRingBytes;
-
-__device__ __forceinline__ void mbar_init(uint32_t mbar, uint32_t count) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(mbar), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive_tx(uint32_t mbar, uint32_t bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mbar), "r"(bytes)
-                 : "memory");
-}
-// Bounded wait: a lost transfer traps (the context fails) instead of hanging.
-__device__ __forceinline__ void mbar_wait(uint32_t mbar, uint32_t parity) {
-    uint32_t done = 0;
-    for (uint32_t spin = 0;; ++spin) {
-        asm volatile(
-            "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
-            "selp.u32 %0, 1, 0, p;\n\t}"
-            : "=r"(done)
-            : "r"(mbar), "r"(parity)
-            : "memory");
-        if (done) return;
-        if (spin > (1u << 24)) __trap();
-    }
-}
-__device__ __forceinline__ void tma_box(uint32_t dst, const void* tmap, int x, int y,
-                                        uint32_t mbar) {
-    asm volatile(
-        "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
-        " [%0], [%1, {%2, %3}], [%4];" ::"r"(dst),
-        "l"(tmap), "r"(x), "r"(y), "r"(mbar)
-        : "memory");
-}
-// Row `lane` of a 32 x 32 B box (SWIZZLE_32B) -> v[0..7].
-__device__ __forceinline__ void lds_row(uint32_t box, int lane, uint32_t v[8]) {
-    const uint32_t sw = ((uint32_t)lane >> 2) & 1u;
-    const uint32_t a0 = box + lane * 32 + 16 * sw, a1 = box + lane * 32 + 16 * (sw ^ 1u);
-    asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];"
-                 : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]) : "r"(a0));
-    asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];"
-                 : "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]) : "r"(a1));
-}
-
-// ILP-2 scan: a CTA of kScanWarps warps takes groups of 2 x kScanWarps tiles;
-// warp w rolls tiles w and w + kScanWarps of the group together.
-template <bool kZeroValue, bool kTma>
-__global__ void __launch_bounds__(kScanThreads, 1024 / kScanThreads)  // <= 64 registers
-rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ gtab,
-                       uint32_t mask, uint32_t value, uint32_t* __restrict__ bitmap,
-                       uint32_t* __restrict__ agg, uint32_t* __restrict__ gagg,
-                       uint32_t* __restrict__ evbuf) {
+template <bool kMul>
+__global__ void __maxnreg__(DEDUP_SCAN_MAXREG)
+rabin_scan_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ gtab,
+                  uint32_t mask, uint32_t value, uint32_t mul, uint32_t* __restrict__ bitmap,
+                  uint32_t* __restrict__ agg, uint32_t* __restrict__ gagg,
+                  uint32_t* __restrict__ evbuf) {
     extern __shared__ __align__(16) uint8_t smem[];
     __shared__ uint32_t src[512];
     __shared__ uint32_t fun[kFunBufs][kHalves][kGroup][32];
@@ -489,10 +378,6 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
     const uint32_t lim16 = (nbytes + 15) & ~15u;
     // CTA b, half h takes groups b * kHalves + h + k * gridDim.x * kHalves
     const uint32_t g0 = blockIdx.x * kHalves + half, gstride = gridDim.x * kHalves;
-    if (DEDUP_SCAN_L2PF && lane == 0 && g0 < n_groups) {  // first group, during the table build
-        prefetch_tile_l2(bytes, (uint64_t)g0 * kGroup + hw, lim16);
-        prefetch_tile_l2(bytes, (uint64_t)g0 * kGroup + hw + kGroupWarps, lim16);
-    }
     if (threadIdx.x < 512) src[threadIdx.x] = gtab[threadIdx.x];
     const uint64_t* items = cache_items(icache, desc);
     const uint32_t n_items = desc->n_items;
@@ -502,181 +387,108 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
         for (int idx = threadIdx.x; idx < kTabBytes / 4; idx += blockDim.x)
             t32[idx] = src[((idx >> 5) & 1) * 256 + (idx >> 6)];
     }
-    // TMA ring: per warp kScanStages stages x 2 chains x 1 KiB after the table
-    __shared__ __align__(8) uint64_t mbar_s[kScanWarps][kScanStages];
-    const uint32_t ring = base + kTabBytes + (uint32_t)wid * (kScanStages * 2 * kBoxBytes);
-    if (kTma && base + kTabBytes + kRingBytes > win + (uint32_t)kScanSmemTma) __trap();
-    const uint32_t mbar0 = (uint32_t)__cvta_generic_to_shared(&mbar_s[wid][0]);
-    const uint32_t tma_rows = kTma ? desc->tma_rows : 0u;
-    const void* tmap = desc->tmap;
-    if (kTma && lane == 0) {
-        for (int i = 0; i < kScanStages; ++i) mbar_init(mbar0 + 8 * i, 1);
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        asm volatile("fence.proxy.tensormap::generic.acquire.gpu [%0], 128;" ::"l"(tmap)
-                     : "memory");
-    }
     __syncthreads();
     if (nbytes == 0) return;
     const uint32_t laneR = base | (lane * 4);
     const uint32_t laneW = laneR + 128;
     const bool a32 = (reinterpret_cast<uintptr_t>(bytes) & 31) == 0;
-    // Unit v of this warp = box s = v % 9 (0: warm-up, 1..8: steps) of the
-    // k = v / 9-th group of the CTA.  Unit v lives in stage v % kScanStages,
-    // phase (v / kScanStages) & 1.  Lane 0 issues unit v + kScanStages - 1
-    // when the lanes start reading unit v (its stage was read and released by
-    // the __syncwarp that ended unit v - 1).
-    auto tile_tma = [&](uint32_t t) { return (t + 1) * 32u <= tma_rows; };
-    auto issue = [&](uint32_t v) {
-        const uint32_t k = v / kUnitsPerTile, sidx = v % kUnitsPerTile;
-        const uint32_t g = g0 + k * gstride;
-        if (g >= n_groups) return;
-        const uint32_t st = v % kScanStages, mb = mbar0 + 8 * st;
-        const uint32_t t0 = g * kGroup + hw, t1 = t0 + kGroupWarps;
-        const bool c0 = tile_tma(t0), c1 = tile_tma(t1);
-        mbar_arrive_tx(mb, (c0 ? kBoxBytes : 0) + (c1 ? kBoxBytes : 0));
-        const int x = sidx == 0 ? (int)(kLaneBytes - 32) : 32 * (int)(sidx - 1);
-        const int dy = sidx == 0 ? -1 : 0;
-        const uint32_t dst = ring + st * 2 * kBoxBytes;
-        if (c0) tma_box(dst, tmap, x, (int)(t0 * 32) + dy, mb);
-        if (c1) tma_box(dst + kBoxBytes, tmap, x, (int)(t1 * 32) + dy, mb);
-    };
-    if (kTma && lane == 0)
-        for (uint32_t v = 0; v + 1 < (uint32_t)kScanStages; ++v) issue(v);
-    uint32_t unit = 0;  // next unit to read (kTma)
-    // The bytes of unit `unit` for both chains (TMA ring or LDG fallback).
-    auto fetch = [&](uint32_t offA, uint32_t offB, bool okA, bool okB, bool tA_tma,
-                     bool tB_tma, uint32_t (&vA)[8], uint32_t (&vB)[8]) {
-        if (kTma) {
-            if (lane == 0) issue(unit + kScanStages - 1);
-            const uint32_t st = unit % kScanStages;
-            if (tA_tma || tB_tma) mbar_wait(mbar0 + 8 * st, (unit / kScanStages) & 1u);
-            const uint32_t box = ring + st * 2 * kBoxBytes;
-            if (tA_tma) lds_row(box, lane, vA);
-            else if (okA) load32_v8(bytes, offA, lim16, a32, vA);
-            if (tB_tma) lds_row(box + kBoxBytes, lane, vB);
-            else if (okB) load32_v8(bytes, offB, lim16, a32, vB);
-            __syncwarp();
-            ++unit;
-        } else {
-            if (okA) load32_v8(bytes, offA, lim16, a32, vA);
-            if (okB) load32_v8(bytes, offB, lim16, a32, vB);
-        }
-    };
     int par = 0;
     for (uint32_t g = g0; g < n_groups; g += gstride, par ^= 1) {
-        const uint32_t tA = g * kGroup + hw, tB = tA + kGroupWarps;
-        if (DEDUP_SCAN_L2PF && lane == 0 && g + gstride < n_groups) {  // next group
-            prefetch_tile_l2(bytes, tA + gstride * kGroup, lim16);
-            prefetch_tile_l2(bytes, tB + gstride * kGroup, lim16);
-        }
-        if (DEDUP_SCAN_L1PF && g + gstride < n_groups) {
-            // the next group's first bytes of this lane's segments (warm-up
-            // window + first step) into L1: every warp of the CTA starts a
-            // group at the same time, so these loads would otherwise stall
-            // the whole CTA once per group
-            const uint64_t nA = (uint64_t)(tA + gstride * kGroup) * kSelTile + lane * kLaneBytes;
-            const uint64_t nB = nA + (uint64_t)kGroupWarps * kSelTile;
-            if (nA < lim16) {
-                if (nA >= 32) prefetch_l1(bytes + nA - 32);
-                prefetch_l1(bytes + nA);
-            }
-            if (nB < lim16) {
-                prefetch_l1(bytes + nB - 32);
-                prefetch_l1(bytes + nB);
-            }
-        }
-        const uint32_t qA = tA * kSelTile + lane * kLaneBytes;
-        const uint32_t qB = tB * kSelTile + lane * kLaneBytes;
-        uint32_t prevA[8], curA[8], prevB[8], curB[8];
+        uint32_t t[kChains], q[kChains];
 #pragma unroll
-        for (int i = 0; i < 8; ++i) prevA[i] = curA[i] = prevB[i] = curB[i] = 0;
-        const bool tmaA = kTma && tile_tma(tA), tmaB = kTma && tile_tma(tB);
-        // both tiles inside the batch and 32-byte aligned loads: no guards
-        const bool full = !kTma && a32 && (tB + 1) * kSelTile <= nbytes;
-        fetch(qA - 32, qB - 32, qA >= 32 && qA < nbytes, qB >= 32 && qB < nbytes, tmaA, tmaB,
-              prevA, prevB);
-        fetch(qA, qB, qA < nbytes, qB < nbytes, tmaA, tmaB, curA, curB);
-        uint32_t hA = 0, hB = 0, pbA = 0, pbB = 0;
-        {   // warm-up of both chains: the windows ending at q-1
-            const uint32_t zero[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-            uint32_t bA, bB;
-            roll32x2<kZeroValue>(hA, prevA, zero, bA, hB, prevB, zero, bB, laneR, laneW, mask,
-                                 value);
-            pbA = qA >= 32 ? bA : 0;
-            pbB = qB >= 32 ? bB : 0;
-            if (qA < 32) hA = 0;
-            if (qB < 32) hB = 0;
+        for (int c = 0; c < kChains; ++c) {
+            t[c] = g * kGroup + hw + c * kGroupWarps;
+            q[c] = t[c] * kSelTile + lane * kLaneBytes;
         }
-        // One 32-byte step of both chains: roll `in` against `old`, then the
-        // bits in e-space.  Once `old` has been rolled out, its registers
-        // receive the NEXT step's bytes (TMA ring or LDG), so `in` and `old`
-        // swap roles every step (the loop body holds two steps) and no extra
-        // registers are needed.
-        auto step = [&](int j, uint32_t (&inA)[8], uint32_t (&oldA)[8], uint32_t (&inB)[8],
-                        uint32_t (&oldB)[8]) {
-            const uint32_t bA0 = qA + 32 * j, bB0 = qB + 32 * j;
-            uint32_t bitsA, bitsB;
-            roll32x2<kZeroValue, 0, 4>(hA, inA, oldA, bitsA, hB, inB, oldB, bitsB, laneR, laneW,
-                                       mask, value);
-            roll32x2<kZeroValue, 4, 8>(hA, inA, oldA, bitsA, hB, inB, oldB, bitsB, laneR, laneW,
-                                       mask, value);
+        uint32_t prev[kChains][8], cur[kChains][8];
+#pragma unroll
+        for (int c = 0; c < kChains; ++c)
+#pragma unroll
+            for (int i = 0; i < 8; ++i) prev[c][i] = cur[c][i] = 0;
+        // every tile inside the batch and 32-byte aligned loads: no guards
+        const bool full = a32 && (t[kChains - 1] + 1) * kSelTile <= nbytes;
+#pragma unroll
+        for (int c = 0; c < kChains; ++c) {
+            if (q[c] >= 32 && q[c] < nbytes) load32_v8(bytes, q[c] - 32, lim16, a32, prev[c]);
+            if (q[c] < nbytes) load32_v8(bytes, q[c], lim16, a32, cur[c]);
+        }
+        uint32_t h[kChains], pb[kChains];
+        {   // warm-up of the chains: the windows ending at q - 1
+            uint32_t zero[kChains][8], b0[kChains];
+#pragma unroll
+            for (int c = 0; c < kChains; ++c) {
+                h[c] = 0;
+#pragma unroll
+                for (int i = 0; i < 8; ++i) zero[c][i] = 0;
+            }
+            roll_step<kMul, 0, 8>(h, prev, zero, b0, laneR, laneW, mask, value, mul);
+#pragma unroll
+            for (int c = 0; c < kChains; ++c) {
+                pb[c] = q[c] >= 32 ? b0[c] : 0;
+                if (q[c] < 32) h[c] = 0;
+            }
+        }
+        // One 32-byte step of the chains, then the bits in e-space.  Once
+        // `old` has been rolled out, its registers receive the NEXT step's
+        // bytes, so `in` and `old` swap roles every step (the loop body holds
+        // two steps) and no extra registers are needed.
+        auto step = [&](int j, uint32_t (&in)[kChains][8], uint32_t (&old)[kChains][8]) {
+            uint32_t bits[kChains];
+            roll_step<kMul, 0, 4>(h, in, old, bits, laneR, laneW, mask, value, mul);
+            roll_step<kMul, 4, 8>(h, in, old, bits, laneR, laneW, mask, value, mul);
             if (j < 7) {  // the next step's bytes into the registers `old` just freed
-                if (full) {
-                    ldg_v8(bytes + bA0 + 32, oldA);
-                    ldg_v8(bytes + bB0 + 32, oldB);
-                } else {
 #pragma unroll
-                    for (int i = 0; i < 8; ++i) oldA[i] = oldB[i] = 0;
-                    fetch(bA0 + 32, bB0 + 32, bA0 + 32 < nbytes, bB0 + 32 < nbytes, tmaA, tmaB,
-                          oldA, oldB);
+                for (int c = 0; c < kChains; ++c) {
+                    const uint32_t nq = q[c] + 32 * (j + 1);
+                    if (full) {
+                        ldg_v8(bytes + nq, old[c]);
+                    } else {
+#pragma unroll
+                        for (int i = 0; i < 8; ++i) old[c][i] = 0;
+                        if (nq < nbytes) load32_v8(bytes, nq, lim16, a32, old[c]);
+                    }
                 }
             }
-            uint32_t ewA = __funnelshift_l(pbA, bitsA, 1), ewB = __funnelshift_l(pbB, bitsB, 1);
-            if (!full) {  // the batch's ragged end
-                if (bA0 >= nbytes) ewA = 0;
-                else if (bA0 + 32 > nbytes) ewA &= (1u << (uint32_t)(nbytes - bA0)) - 1u;
-                if (bB0 >= nbytes) ewB = 0;
-                else if (bB0 + 32 > nbytes) ewB &= (1u << (uint32_t)(nbytes - bB0)) - 1u;
-                if (bA0 + 32 > nbytes)
-                    bitsA &= bA0 < nbytes ? (1u << (uint32_t)(nbytes - bA0)) - 1u : 0u;
-                if (bB0 + 32 > nbytes)
-                    bitsB &= bB0 < nbytes ? (1u << (uint32_t)(nbytes - bB0)) - 1u : 0u;
+#pragma unroll
+            for (int c = 0; c < kChains; ++c) {
+                const uint32_t b0 = q[c] + 32 * j;
+                uint32_t ew = __funnelshift_l(pb[c], bits[c], 1);
+                if (!full) {  // the batch's ragged end
+                    if (b0 >= nbytes) ew = 0;
+                    else if (b0 + 32 > nbytes) ew &= (1u << (uint32_t)(nbytes - b0)) - 1u;
+                    if (b0 + 32 > nbytes)
+                        bits[c] &= b0 < nbytes ? (1u << (uint32_t)(nbytes - b0)) - 1u : 0u;
+                }
+                if (full || t[c] < n_tiles) bitmap[t[c] * kSelTileWords + lane * 8 + j] = ew;
+                pb[c] = bits[c];
             }
-            sm.cand[lane * 8 + j] = ewA;
-            if (full || tA < n_tiles) bitmap[tA * kSelTileWords + lane * 8 + j] = ewA;
-            if (full || tB < n_tiles) bitmap[tB * kSelTileWords + lane * 8 + j] = ewB;
-            pbA = bitsA;
-            pbB = bitsB;
         };
 #pragma unroll 1
         for (int j = 0; j < 8; j += 2) {
-            step(j, curA, prevA, curB, prevB);      // prev now holds step j+1's bytes
-            step(j + 1, prevA, curA, prevB, curB);  // cur now holds step j+2's bytes
-        }
-        // transfer functions of tile A (candidate words already in smem), then B
-        uint32_t fA = (uint32_t)lane << 27, fB = fA;
-        if (tA < n_tiles && !(DEDUP_SCAN_EXPERIMENT & 8)) {
-            const uint32_t n_ev = apply_items(sm, tA * kSelTile, nbytes, items, n_items, lane);
-            store_events(sm, n_ev, evbuf + (size_t)tA * kEvWords, lane);
-            uint32_t ex;
-            const uint32_t cnt = walk_any(sm, n_ev, lane, ex, nullptr, 0, 0, 0);
-            fA = (ex << 27) | cnt;
-            agg[32 * tA + lane] = fA;
+            step(j, cur, prev);      // prev now holds step j+1's bytes
+            step(j + 1, prev, cur);  // cur now holds step j+2's bytes
         }
         __syncwarp();
-        if (tB < n_tiles && !(DEDUP_SCAN_EXPERIMENT & 8)) {
+        // transfer functions of the warp's tiles (entry state = lane)
+#pragma unroll 1
+        for (int c = 0; c < kChains; ++c) {
+            const uint32_t tc = g * kGroup + hw + c * kGroupWarps;
+            uint32_t f = (uint32_t)lane << 27;
+            if (tc < n_tiles) {
 #pragma unroll
-            for (int k = 0; k < 8; ++k)
-                sm.cand[lane * 8 + k] = bitmap[tB * kSelTileWords + lane * 8 + k];
-            const uint32_t n_ev = apply_items(sm, tB * kSelTile, nbytes, items, n_items, lane);
-            store_events(sm, n_ev, evbuf + (size_t)tB * kEvWords, lane);
-            uint32_t ex;
-            const uint32_t cnt = walk_any(sm, n_ev, lane, ex, nullptr, 0, 0, 0);
-            fB = (ex << 27) | cnt;
-            agg[32 * tB + lane] = fB;
+                for (int k = 0; k < 8; ++k)
+                    sm.cand[lane * 8 + k] = bitmap[tc * kSelTileWords + lane * 8 + k];
+                const uint32_t n_ev = apply_items(sm, (uint64_t)tc * kSelTile, nbytes, items,
+                                                  n_items, lane);
+                store_events(sm, n_ev, evbuf + (size_t)tc * kEvWords, lane);
+                uint32_t ex;
+                const uint32_t cnt = walk_any(sm, n_ev, lane, ex, nullptr, 0, 0, 0);
+                f = (ex << 27) | cnt;
+                agg[32 * tc + lane] = f;
+            }
+            fun[par][half][hw + c * kGroupWarps][lane] = f;
+            __syncwarp();
         }
-        fun[par][half][hw][lane] = fA;
-        fun[par][half][hw + kGroupWarps][lane] = fB;
         if (kHalves == 1) __syncthreads();
         else asm volatile("bar.sync %0, %1;" ::"r"(1 + half), "r"(kGroupWarps * 32) : "memory");
         if (hw == 0) {
@@ -908,13 +720,8 @@ void chunk_set_attrs() {
     const uint64_t bit = 1ull << (dev & 63);
     std::lock_guard<std::mutex> lock(mu);
     if (done_mask & bit) return;
-    for (const void* f : {(const void*)rabin_scan_agg2_kernel<true, false>,
-                          (const void*)rabin_scan_agg2_kernel<false, false>})
+    for (const void* f : {(const void*)rabin_scan_kernel<true>, (const void*)rabin_scan_kernel<false>})
         cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
-    if (DEDUP_SCAN_TMA)
-        for (const void* f : {(const void*)rabin_scan_agg2_kernel<true, true>,
-                              (const void*)rabin_scan_agg2_kernel<false, true>})
-            cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmemTma);
     cudaFuncSetAttribute(select_emit_ev_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)sizeof(EmitEvSmem));
     done_mask |= bit;
@@ -923,53 +730,13 @@ void chunk_set_attrs() {
 
 const char* chunk_unlaunchable() {
     chunk_set_attrs();
-    for (const void* f : {(const void*)rabin_scan_agg2_kernel<true, false>,
-                          (const void*)rabin_scan_agg2_kernel<false, false>})
-        if (!fits(f, kScanThreads, kScanSmem)) return "rabin_scan_agg2_kernel";
-    if (DEDUP_SCAN_TMA)
-        for (const void* f : {(const void*)rabin_scan_agg2_kernel<true, true>,
-                              (const void*)rabin_scan_agg2_kernel<false, true>})
-            if (!fits(f, kScanThreads, kScanSmemTma)) return "rabin_scan_agg2_kernel (TMA)";
+    for (const void* f : {(const void*)rabin_scan_kernel<true>, (const void*)rabin_scan_kernel<false>})
+        if (!fits(f, kScanThreads, kScanSmem)) return "rabin_scan_kernel";
     if (!fits((const void*)select_scan_kernel, 1024, 0)) return "select_scan_kernel";
     if (!fits((const void*)select_emit_ev_kernel, kEmitEvWarps * 32, sizeof(EmitEvSmem)))
         return "select_emit_ev_kernel";
     if (!fits((const void*)chunk_meta_kernel, 256, 0)) return "chunk_meta_kernel";
     return nullptr;
-}
-
-// Host side of the TMA view (internal.h).  The driver's tensor-map encoder is
-// resolved once through the runtime's entry-point query (no libcuda link).
-bool encode_scan_tmap(BatchDesc& d) {
-    d.tma_rows = 0;
-    if (!DEDUP_SCAN_TMA) return false;
-    using EncodeFn = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
-                                  const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
-                                  const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
-                                  CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
-    static EncodeFn enc = [] {
-        void* fn = nullptr;
-        cudaDriverEntryPointQueryResult q;
-        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) !=
-                cudaSuccess ||
-            q != cudaDriverEntryPointSuccess)
-            fn = nullptr;
-        cudaGetLastError();
-        return reinterpret_cast<EncodeFn>(fn);
-    }();
-    const uint64_t rows = d.nbytes / kLaneBytes;
-    if (enc == nullptr || rows < 32 || (reinterpret_cast<uintptr_t>(d.bytes) & 15)) return false;
-    const cuuint64_t dims[2] = {kLaneBytes, rows};
-    const cuuint64_t strides[1] = {kLaneBytes};
-    const cuuint32_t box[2] = {32, 32};
-    const cuuint32_t estr[2] = {1, 1};
-    CUtensorMap* m = reinterpret_cast<CUtensorMap*>(d.tmap);
-    const CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<uint8_t*>(d.bytes),
-                           dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                           CU_TENSOR_MAP_SWIZZLE_32B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-    if (r != CUDA_SUCCESS) return false;
-    d.tma_rows = (uint32_t)rows;
-    return true;
 }
 
 void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mask,
@@ -988,15 +755,12 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
     uint64_t gneed = (groups + kHalves - 1) / kHalves;
     gneed = (gneed + DEDUP_SCAN_GROUPS_PER_CTA - 1) / DEDUP_SCAN_GROUPS_PER_CTA;
     const unsigned grid = (unsigned)(gneed < (uint64_t)num_sms ? (gneed ? gneed : 1) : num_sms);
-    // the kernel reads d->tma_rows at run time: 0 -> every tile on the LDG path
-    if (DEDUP_SCAN_TMA) {
-        auto k = value == 0 ? rabin_scan_agg2_kernel<true, true> : rabin_scan_agg2_kernel<false, true>;
-        k<<<grid, kScanThreads, kScanSmemTma, s>>>(d, d_tab, mask, value, bitmap, agg, gagg, evbuf);
-    } else {
-        auto k = value == 0 ? rabin_scan_agg2_kernel<true, false>
-                            : rabin_scan_agg2_kernel<false, false>;
-        k<<<grid, kScanThreads, kScanSmem, s>>>(d, d_tab, mask, value, bitmap, agg, gagg, evbuf);
-    }
+    // (h & mask) == value for a low-bit mask and value 0 as an IMAD test
+    const bool low = value == 0 && (mask & (mask + 1u)) == 0;
+    const int kbits = __builtin_popcount(mask);  // low: mask = 2^kbits - 1
+    const uint32_t mul = kbits == 0 ? 0u : (kbits == 32 ? 1u : (1u << (32 - kbits)));
+    auto k = low ? rabin_scan_kernel<true> : rabin_scan_kernel<false>;
+    k<<<grid, kScanThreads, kScanSmem, s>>>(d, d_tab, mask, value, mul, bitmap, agg, gagg, evbuf);
     if (after_scan) cudaEventRecordWithFlags(after_scan, s, cudaEventRecordExternal);
     // NEXT-2 max_chunk: the state machine's cuts go to a scratch list first
     uint32_t* final_cut = cut_pos;

@@ -72,18 +72,23 @@ md = [f'# {tag} profiles (B200, sm_100a)', '',
       '```', open('tools/gpu_profiles.sh').read().strip(), '```', '',
       '## Launch list of the bench step (`bench.py --step-only`: warm-up + timed steps; cold-cache, serialised by ncu: shares, not absolutes)', '']
 md += lt
-md += ['', '## ncu --set full, one 64 MiB batch of C2 (tools/one_batch.py)', '',
+md += ['', '## ncu --set full, 64 MiB batches of C3 (tools/one_batch.py)', '',
        'Units: ns, instructions, %, bytes.  `dram` = DRAM bytes of the launch.', '']
 md += ft
+if os.path.exists('gpurun_out/prof_sha.ncu-rep'):
+    sh, _ = full_table('gpurun_out/prof_sha.ncu-rep')
+    md += ['', '## ncu --set full, the SHA-1 kernel alone on all 672 MiB of C3 chunks '
+               '(tools/sha_sizes.py, one launch)', '']
+    md += sh
 if os.path.exists('gpurun_out/prof_fm.ncu-rep'):
     fm, fm_traffic = full_table('gpurun_out/prof_fm.ncu-rep')
     md += ['', '## ncu --set full, row NEXT-1 FindMatch, one 64 MiB batch of C2 (tools/fm_sizes.py)', '']
     md += fm
     traffic.update({'findmatch_' + k: v for k, v in fm_traffic.items()})
 open(f'profiles/{tag}_ncu_summary.md', 'w').write('\n'.join(md) + '\n')
-tj = {"_source": "ncu --set full, tools/one_batch.py (64 MiB batches of C2); DRAM read+write bytes per "
+tj = {"_source": "ncu --set full, tools/one_batch.py (64 MiB batches of C3); DRAM read+write bytes per "
                  "launch; bench scales per input byte", "capture_batch_bytes": BATCH}
-name_map = {'sha1_kernel': 'sha1', 'rabin_scan_agg2_kernel': 'rabin_scan', 'select_emit_ev_kernel': 'select_emit',
+name_map = {'sha1_kernel': 'sha1', 'rabin_scan_kernel': 'rabin_scan', 'select_emit_ev_kernel': 'select_emit',
             'table_insert_kernel': 'table_insert'}
 for k, v in traffic.items():
     tj[name_map.get(k, k)] = v
