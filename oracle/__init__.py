@@ -58,7 +58,8 @@ def build_oracle(force: bool = False) -> str:
 class _Params(ctypes.Structure):
     _fields_ = [("window", ctypes.c_uint32), ("poly", ctypes.c_uint32),
                 ("anchor_mask", ctypes.c_uint32), ("anchor_value", ctypes.c_uint32),
-                ("min_chunk", ctypes.c_uint32), ("max_chunk", ctypes.c_uint32)]
+                ("min_chunk", ctypes.c_uint32), ("max_chunk", ctypes.c_uint32),
+                ("literal_window", ctypes.c_uint32)]
 
 
 _lib = None
@@ -125,10 +126,11 @@ class Params:
     anchor_value: int = VALUE
     min_chunk: int = WINDOW
     max_chunk: int = 0
+    literal_window: bool = False  # PARSEC rabinwintab with rf_win = 0 (reading O5-L)
 
     def c(self) -> _Params:
         return _Params(self.window, self.poly, self.anchor_mask, self.anchor_value,
-                       self.min_chunk, self.max_chunk)
+                       self.min_chunk, self.max_chunk, int(self.literal_window))
 
 
 def fp_window(window_bytes, poly: int = POLY) -> int:

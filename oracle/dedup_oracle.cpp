@@ -84,6 +84,7 @@ typedef struct {
     uint32_t anchor_value;  // 0
     uint32_t min_chunk;     // >= window; 32 (reading O6)
     uint32_t max_chunk;     // 0 = none (reading O7)
+    uint32_t literal_window;  // 1: PARSEC's rabininit(rf_win = 0) table (reading O5-L)
 } oracle_params;
 
 // Fingerprint of the window ending at every byte i (inclusive) of p, with the
@@ -109,10 +110,17 @@ void oracle_rolling_fp(const uint8_t* p, uint64_t n, uint32_t poly, uint32_t win
 //   e in [c+min_chunk, n) with (fp(p[e-window..e-1]) & mask) == value, or the
 //   forced cut e = c+max_chunk (max_chunk != 0, e < n); else e = n.
 // Returns the number of chunks; starts[] receives item-relative chunk starts.
+//
+// literal_window (row NEXT-2, reading O5-L): PARSEC's chunker as
+// called with a window-table length of 0, rabinwintab[x] = x * t^0 = x: the
+// byte leaving the window is XORed in at degree 0 instead of removed, so the
+// hash at a position depends on every byte since the last cut (restart).
 uint64_t oracle_chunk_item(const uint8_t* p, uint64_t n, const oracle_params* prm,
                            uint32_t* starts, uint64_t cap) {
     uint32_t R[256], Wt[256];
     oracle_rabin_tables(prm->poly, prm->window, R, Wt);
+    if (prm->literal_window)
+        for (uint32_t b = 0; b < 256; ++b) Wt[b] = b;
     const uint32_t W = prm->window;
     uint64_t count = 0;
     uint64_t c = 0;

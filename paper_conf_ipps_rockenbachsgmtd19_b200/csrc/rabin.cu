@@ -83,8 +83,11 @@ struct SelWarpSmem {
 // assumes at least kStaticMin bytes of static smem; the kernel traps if the
 // runtime layout disagrees.
 constexpr int kScanAux = kScanWarps * (int)sizeof(SelWarpSmem) + kItemCache * 8;
-constexpr int kStaticMin = 2048 + kHalves * 8192;  // src table + fun buffers
-constexpr bool kAuxInPad = kScanAux <= 65536 - 1024 - 10752;
+// static smem of the scan kernel (src table + group function buffers) and a
+// bound on what precedes the dynamic window (static + system reserved)
+constexpr int kStaticMin = 2048 + kHalves * 8192;
+constexpr int kStaticMax = kStaticMin + 2048;
+constexpr bool kAuxInPad = kScanAux <= 65536 - kStaticMax;
 constexpr int kScanSmem = kAuxInPad ? 65536 + kTabBytes : 2 * 65536 - kStaticMin + kScanAux;
 
 // Group buffers in the scan (double buffering across the group barrier).

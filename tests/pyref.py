@@ -43,3 +43,36 @@ def chunk_bruteforce(data: bytes, mask=0xFFF, value=0, window=WINDOW, min_chunk=
                 break
         c = e
     return starts
+
+
+def literal_fp(seg: bytes, poly: int = POLY, window: int = WINDOW) -> int:
+    """PARSEC's hash with the window table of length 0 (reading O5-L) after
+    reading seg = data[c:n] from a restart at c, as a closed form: every byte
+    p[k] enters at degree 8 (n - 1 - k), and every byte with k <= n - 1 -
+    window is XORed in once more when it leaves the window, then shifted
+    n - window - k times:  h = sum_k p[k] t^{8(n-1-k)} + sum_{k <= n-1-window}
+    p[k] t^{8(n-window-k)}  (mod P), by big-integer long division."""
+    n = len(seg)
+    x = 0
+    for k, b in enumerate(seg):
+        x ^= b << (8 * (n - 1 - k))
+        if k <= n - 1 - window:
+            x ^= b << (8 * (n - window - k))
+    return gf2_mod(x, poly)
+
+
+def chunk_bruteforce_literal(data: bytes, mask=0xFFF, value=0, window=WINDOW, poly=POLY):
+    """Greedy definition for the literal mode: from a cut c, the next cut is
+    the smallest e >= c + window (e < n) with (literal_fp(data[c:e]) & mask)
+    == value; the item end closes the last chunk."""
+    n = len(data)
+    starts, c = [], 0
+    while c < n:
+        starts.append(c)
+        e = n
+        for x in range(c + window, n):
+            if (literal_fp(data[c:x], poly, window) & mask) == value:
+                e = x
+                break
+        c = e
+    return starts

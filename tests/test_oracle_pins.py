@@ -272,3 +272,29 @@ def test_items_parallel_equals_sequential_and_hashlib(threads):
             assert bytes(dg[j]) == d
             assert dup[j] == (d in seen)
             assert fid[j] == seen.setdefault(d, (k << 32) | j)
+
+
+# ------------------------------------- NEXT-2: PARSEC literal window (O5-L) --
+@pytest.mark.parametrize("seed", range(6))
+def test_literal_window_bruteforce(seed):
+    """oracle chunk_item(literal_window) == the greedy definition over the
+    closed-form literal hash (big-integer long division, tests/pyref.py) on
+    small random inputs, dense masks so that cuts happen often."""
+    rng = np.random.default_rng(1000 + seed)
+    data = rng.integers(0, 256, 300 + 97 * seed, dtype=np.uint8)
+    for mask in (0x3, 0xF, 0x3F):
+        got = oracle.chunk_item(data, oracle.Params(anchor_mask=mask, literal_window=True))
+        want = pyref.chunk_bruteforce_literal(data.tobytes(), mask=mask)
+        assert list(got) == want, mask
+
+
+def test_literal_window_differs_from_true_window_and_zero_closed_form():
+    """The literal hash is history-dependent: on random data it cuts
+    elsewhere than the true 32-byte window (reading O5); on all-zero data both
+    are the same closed form (cuts every 32 bytes)."""
+    data = synthgen.splitmix64_bytes(42, 1 << 17)
+    lit = oracle.chunk_item(data, oracle.Params(literal_window=True))
+    assert list(lit) != list(oracle.chunk_item(data))
+    assert lit[0] == 0 and np.all(np.diff(lit.astype(np.int64)) >= 32)
+    z = np.zeros(100, np.uint8)
+    assert list(oracle.chunk_item(z, oracle.Params(literal_window=True))) == [0, 32, 64, 96]
