@@ -140,9 +140,13 @@ def plan_batches(off, batch_bytes=None, batch_items=None):
     return out
 
 
+SHA_LANE = 0                     # batch bytes per SHA-1 lane (0: the engine's 32 KiB)
+
+
 def engine_kwargs(stream_bytes: int) -> dict:
     return dict(batch_bytes=BATCH_BYTES, batch_items=BATCH_ITEMS, slots=SLOTS,
-                table_capacity=max(1 << 16, stream_bytes // 2048), host_fed=True)
+                table_capacity=max(1 << 16, stream_bytes // 2048), host_fed=True,
+                sha_lane_bytes=SHA_LANE)
 
 
 def submit_pass(d, submit, n_batches, new_stream=True):
@@ -581,13 +585,17 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=0, help="0 = steps")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--slots", type=int, default=0, help="override the in-flight batches")
+    ap.add_argument("--sha-lane", type=int, default=0,
+                    help="override the batch bytes per SHA-1 lane (0 = the engine default)")
     ap.add_argument("--step-only", action="store_true",
                     help="time the step only (no isolated-kernel, config, NEXT-row, e2e or CPU "
                          "legs): for the ncu launch list of the step")
     args = ap.parse_args()
-    global SLOTS
+    global SLOTS, SHA_LANE
     if args.slots:
         SLOTS = args.slots
+    if args.sha_lane:
+        SHA_LANE = args.sha_lane
     if args.warmup < 3:
         args.warmup = 3
 

@@ -5,9 +5,9 @@
 //
 // The paper ran this on the CPU; here it is three sm_100a kernels:
 //
-//  rabin_scan_kernel  persistent, one CTA of 16 warps per SM.  A CTA takes
-//      groups of 32 tiles of 8 KiB; a warp rolls 4 tiles of a group together
-//      (four independent chains per lane, ILP 4); each lane
+//  rabin_scan_agg2_kernel  persistent, one CTA of 16 warps per SM.  A CTA
+//      takes groups of 32 tiles of 8 KiB; warp w rolls tiles w and w + 16 of
+//      the group together (two independent chains per lane, ILP 2); each lane
 //      rolls the 32-byte window hash over its 256 bytes (after a 32-byte
 //      warm-up) with the post-shift recurrence
 //          h' = ((h << 8) | in) ^ R[h >> 24] ^ W256[out]
@@ -39,30 +39,29 @@ namespace dd {
 
 namespace {
 
-// Scan CTA: 16 warps.  A select group is 32 tiles of 8 KiB; a warp rolls
-// kChains tiles of a group together (kChains independent rolling chains per
-// lane: the PRMT -> LDS -> LOP3 dependency of one chain overlaps with the
-// others'), so kGroupWarps = 32 / kChains warps make a group and the CTA runs
-// kHalves = 16 / kGroupWarps groups at once (its halves share the 64 KiB
-// table).  One scan CTA per SM (the table is 64 KiB-aligned, see below).
+// Scan CTA: 16 warps (64 registers each).  A select group is 32 tiles rolled
+// by 16 warps (2 tiles per warp, ILP 2).  Measured (round 1): a 32-warp CTA
+// running two groups at once scans faster alone (736 MiB chunk stage 1647 vs
+// 1527 GB/s) but takes a whole SM, and the pipelined bench is faster with 16
+// warps (590 vs 576 GB/s): other batches' SHA-1 / table / emit CTAs share the
+// SM.  Measured (round 2, C3, 672 MiB chunk stage): 4 chains per lane (8
+// warps per group, two groups per CTA) 1220 GB/s at 128 registers and 1171
+// at 96; the anchor test as IMAD + predicated add (FMA pipe) 1341; this
+// kernel 1480 -- neither kept.
 #ifndef DEDUP_SCAN_GROUPS_PER_CTA
 #define DEDUP_SCAN_GROUPS_PER_CTA 4  // select groups per scan CTA (launch_chunk_select)
 #endif
-#ifndef DEDUP_SCAN_CHAINS
-#define DEDUP_SCAN_CHAINS 4
-#endif
-constexpr int kChains = DEDUP_SCAN_CHAINS;
-static_assert(kChains == 2 || kChains == 4, "2 or 4 chains per lane");
 constexpr int kScanWarps = 16;
 constexpr int kScanThreads = kScanWarps * 32;
-constexpr int kGroup = 32;                         // tiles per select group
-constexpr int kGroupWarps = kGroup / kChains;      // warps per select group
+constexpr int kGroupWarps = 16;                    // warps per select group
 constexpr int kHalves = kScanWarps / kGroupWarps;  // groups in flight per CTA
+static_assert(kHalves == 1, "one group per scan CTA");
 constexpr int kTabBytes = 256 * 256;  // [x][R|W][lane] u32 = 64 KiB
 constexpr uint32_t kLaneBytes = kSelTile / 32;  // 256 bytes per lane per tile
 constexpr uint32_t kFull = 0xFFFFFFFFu;
 constexpr uint32_t kInf = 0xFFFFFFFFu;
 constexpr uint32_t kM27 = (1u << 27) - 1;
+constexpr int kGroup = kGroupWarps * 2;  // tiles per select group (2 per warp)
 constexpr int kItemCache = 1024;  // item offsets cached in shared memory
 
 constexpr uint32_t kListCap = 128;  // events per tile kept as a sorted list
@@ -83,11 +82,8 @@ struct SelWarpSmem {
 // assumes at least kStaticMin bytes of static smem; the kernel traps if the
 // runtime layout disagrees.
 constexpr int kScanAux = kScanWarps * (int)sizeof(SelWarpSmem) + kItemCache * 8;
-// static smem of the scan kernel (src table + group function buffers) and a
-// bound on what precedes the dynamic window (static + system reserved)
-constexpr int kStaticMin = 2048 + kHalves * 8192;
-constexpr int kStaticMax = kStaticMin + 2048;
-constexpr bool kAuxInPad = kScanAux <= 65536 - kStaticMax;
+constexpr int kStaticMin = kHalves == 1 ? 8192 : 16384;
+constexpr bool kAuxInPad = kScanAux <= 65536 - 1024 - 10752;
 constexpr int kScanSmem = kAuxInPad ? 65536 + kTabBytes : 2 * 65536 - kStaticMin + kScanAux;
 
 // Group buffers in the scan (double buffering across the group barrier).
@@ -305,60 +301,48 @@ __device__ __forceinline__ uint32_t walk_any(const SelWarpSmem& sm, uint32_t n_e
     return walk_tile(sm, s, exit_state, out, out_base, cap, T0);
 }
 
-// One rolling step of kChains independent chains over words [W0, W1) of a
-// 32-byte step (post-shift recurrence h' = ((h << 8) | in) ^ R[h >> 24] ^
-// W256[out]); candidate bits accumulate in bits[c].  kMul: the anchor test
-// (h & mask) == 0 with mask = 2^k - 1 as (h * 2^(32-k)) == 0 -- the IMAD and
-// the bit insert (a predicated add) issue to the FMA pipe, leaving three
-// PRMT, one LOP3 and one ISETP per byte on the ALU pipe; otherwise
-// ((h & mask) ^ value) == 0 (one LOP3) and a predicated OR.
-template <bool kMul, int W0, int W1>
-__device__ __forceinline__ void roll_step(uint32_t (&h)[kChains], const uint32_t (&cur)[kChains][8],
-                                          const uint32_t (&old)[kChains][8],
-                                          uint32_t (&bits)[kChains], uint32_t laneR,
-                                          uint32_t laneW, uint32_t mask, uint32_t value,
-                                          uint32_t mul) {
-    if (W0 == 0) {
-#pragma unroll
-        for (int c = 0; c < kChains; ++c) bits[c] = 0;
-    }
+// Two independent rolling chains per lane (ILP 2): the LDS -> LOP3 -> PRMT
+// dependency of one chain overlaps with the other's.
+// Words [W0, W1) of the 32-byte step; bits accumulate into bitsA / bitsB.
+template <bool kZeroValue, int W0 = 0, int W1 = 8>
+__device__ __forceinline__ void roll32x2(uint32_t& hA, const uint32_t curA[8],
+                                         const uint32_t oldA[8], uint32_t& bitsA, uint32_t& hB,
+                                         const uint32_t curB[8], const uint32_t oldB[8],
+                                         uint32_t& bitsB, uint32_t laneR, uint32_t laneW,
+                                         uint32_t mask, uint32_t value) {
+    if (W0 == 0) bitsA = bitsB = 0;
 #pragma unroll
     for (int w = W0; w < W1; ++w) {
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
-#pragma unroll
-            for (int c = 0; c < kChains; ++c) {
-                const uint32_t aR = __byte_perm(h[c], laneR, 0x7634);
-                const uint32_t aW = __byte_perm(old[c][w], laneW, 0x7604 | (k << 4));
-                const uint32_t hs = __byte_perm(cur[c][w], h[c], 0x6540 | k);
-                h[c] = hs ^ lds(aR) ^ lds(aW);
-                if (kMul) {
-                    asm("{\n\t.reg .pred p;\n\t.reg .u32 t;\n\tmul.lo.u32 t, %1, %2;\n\t"
-                        "setp.eq.u32 p, t, 0;\n\t@p add.u32 %0, %0, %3;\n\t}"
-                        : "+r"(bits[c])
-                        : "r"(h[c]), "r"(mul), "r"(1u << (4 * w + k)));
-                } else {
-                    const uint32_t t = (h[c] & mask) ^ value;
-                    asm("{\n\t.reg .pred p;\n\tsetp.eq.u32 p, %1, 0;\n\t@p or.b32 %0, %0, %2;\n\t}"
-                        : "+r"(bits[c])
-                        : "r"(t), "r"(1u << (4 * w + k)));
-                }
-            }
+            const uint32_t aRA = __byte_perm(hA, laneR, 0x7634);
+            const uint32_t aRB = __byte_perm(hB, laneR, 0x7634);
+            const uint32_t aWA = __byte_perm(oldA[w], laneW, 0x7604 | (k << 4));
+            const uint32_t aWB = __byte_perm(oldB[w], laneW, 0x7604 | (k << 4));
+            const uint32_t hsA = __byte_perm(curA[w], hA, 0x6540 | k);
+            const uint32_t hsB = __byte_perm(curB[w], hB, 0x6540 | k);
+            hA = hsA ^ lds(aRA) ^ lds(aWA);
+            hB = hsB ^ lds(aRB) ^ lds(aWB);
+            const uint32_t tA = kZeroValue ? (hA & mask) : ((hA & mask) ^ value);
+            const uint32_t tB = kZeroValue ? (hB & mask) : ((hB & mask) ^ value);
+            asm("{\n\t.reg .pred p;\n\tsetp.eq.u32 p, %1, 0;\n\t@p or.b32 %0, %0, %2;\n\t}"
+                : "+r"(bitsA)
+                : "r"(tA), "r"(1u << (4 * w + k)));
+            asm("{\n\t.reg .pred p;\n\tsetp.eq.u32 p, %1, 0;\n\t@p or.b32 %0, %0, %2;\n\t}"
+                : "+r"(bitsB)
+                : "r"(tB), "r"(1u << (4 * w + k)));
         }
     }
 }
 
-// Persistent scan: a CTA of kScanWarps warps takes groups of 32 tiles; warp
-// hw of a group rolls its tiles hw + kGroupWarps * c (c < kChains) together.
-#ifndef DEDUP_SCAN_MAXREG
-#define DEDUP_SCAN_MAXREG 96
-#endif
-template <bool kMul>
-__global__ void __maxnreg__(DEDUP_SCAN_MAXREG)
-rabin_scan_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ gtab,
-                  uint32_t mask, uint32_t value, uint32_t mul, uint32_t* __restrict__ bitmap,
-                  uint32_t* __restrict__ agg, uint32_t* __restrict__ gagg,
-                  uint32_t* __restrict__ evbuf) {
+// ILP-2 scan: a CTA of kScanWarps warps takes groups of 2 x kScanWarps tiles;
+// warp w rolls tiles w and w + kScanWarps of the group together.
+template <bool kZeroValue>
+__global__ void __launch_bounds__(kScanThreads, 1024 / kScanThreads)  // <= 64 registers
+rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ gtab,
+                       uint32_t mask, uint32_t value, uint32_t* __restrict__ bitmap,
+                       uint32_t* __restrict__ agg, uint32_t* __restrict__ gagg,
+                       uint32_t* __restrict__ evbuf) {
     extern __shared__ __align__(16) uint8_t smem[];
     __shared__ uint32_t src[512];
     __shared__ uint32_t fun[kFunBufs][kHalves][kGroup][32];
@@ -395,103 +379,104 @@ rabin_scan_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict
     const uint32_t laneR = base | (lane * 4);
     const uint32_t laneW = laneR + 128;
     const bool a32 = (reinterpret_cast<uintptr_t>(bytes) & 31) == 0;
+    // The bytes at offA / offB for the two chains (zero past the batch end).
+    auto fetch = [&](uint32_t offA, uint32_t offB, bool okA, bool okB, uint32_t (&vA)[8],
+                     uint32_t (&vB)[8]) {
+        if (okA) load32_v8(bytes, offA, lim16, a32, vA);
+        if (okB) load32_v8(bytes, offB, lim16, a32, vB);
+    };
     int par = 0;
     for (uint32_t g = g0; g < n_groups; g += gstride, par ^= 1) {
-        uint32_t t[kChains], q[kChains];
+        const uint32_t tA = g * kGroup + hw, tB = tA + kGroupWarps;
+        const uint32_t qA = tA * kSelTile + lane * kLaneBytes;
+        const uint32_t qB = tB * kSelTile + lane * kLaneBytes;
+        uint32_t prevA[8], curA[8], prevB[8], curB[8];
 #pragma unroll
-        for (int c = 0; c < kChains; ++c) {
-            t[c] = g * kGroup + hw + c * kGroupWarps;
-            q[c] = t[c] * kSelTile + lane * kLaneBytes;
+        for (int i = 0; i < 8; ++i) prevA[i] = curA[i] = prevB[i] = curB[i] = 0;
+        // both tiles inside the batch and 32-byte aligned loads: no guards
+        const bool full = a32 && (tB + 1) * kSelTile <= nbytes;
+        fetch(qA - 32, qB - 32, qA >= 32 && qA < nbytes, qB >= 32 && qB < nbytes, prevA, prevB);
+        fetch(qA, qB, qA < nbytes, qB < nbytes, curA, curB);
+        uint32_t hA = 0, hB = 0, pbA = 0, pbB = 0;
+        {   // warm-up of both chains: the windows ending at q-1
+            const uint32_t zero[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+            uint32_t bA, bB;
+            roll32x2<kZeroValue>(hA, prevA, zero, bA, hB, prevB, zero, bB, laneR, laneW, mask,
+                                 value);
+            pbA = qA >= 32 ? bA : 0;
+            pbB = qB >= 32 ? bB : 0;
+            if (qA < 32) hA = 0;
+            if (qB < 32) hB = 0;
         }
-        uint32_t prev[kChains][8], cur[kChains][8];
-#pragma unroll
-        for (int c = 0; c < kChains; ++c)
-#pragma unroll
-            for (int i = 0; i < 8; ++i) prev[c][i] = cur[c][i] = 0;
-        // every tile inside the batch and 32-byte aligned loads: no guards
-        const bool full = a32 && (t[kChains - 1] + 1) * kSelTile <= nbytes;
-#pragma unroll
-        for (int c = 0; c < kChains; ++c) {
-            if (q[c] >= 32 && q[c] < nbytes) load32_v8(bytes, q[c] - 32, lim16, a32, prev[c]);
-            if (q[c] < nbytes) load32_v8(bytes, q[c], lim16, a32, cur[c]);
-        }
-        uint32_t h[kChains], pb[kChains];
-        {   // warm-up of the chains: the windows ending at q - 1
-            uint32_t zero[kChains][8], b0[kChains];
-#pragma unroll
-            for (int c = 0; c < kChains; ++c) {
-                h[c] = 0;
-#pragma unroll
-                for (int i = 0; i < 8; ++i) zero[c][i] = 0;
-            }
-            roll_step<kMul, 0, 8>(h, prev, zero, b0, laneR, laneW, mask, value, mul);
-#pragma unroll
-            for (int c = 0; c < kChains; ++c) {
-                pb[c] = q[c] >= 32 ? b0[c] : 0;
-                if (q[c] < 32) h[c] = 0;
-            }
-        }
-        // One 32-byte step of the chains, then the bits in e-space.  Once
-        // `old` has been rolled out, its registers receive the NEXT step's
-        // bytes, so `in` and `old` swap roles every step (the loop body holds
-        // two steps) and no extra registers are needed.
-        auto step = [&](int j, uint32_t (&in)[kChains][8], uint32_t (&old)[kChains][8]) {
-            uint32_t bits[kChains];
-            roll_step<kMul, 0, 4>(h, in, old, bits, laneR, laneW, mask, value, mul);
-            roll_step<kMul, 4, 8>(h, in, old, bits, laneR, laneW, mask, value, mul);
+        // One 32-byte step of both chains: roll `in` against `old`, then the
+        // bits in e-space.  Once `old` has been rolled out, its registers
+        // receive the NEXT step's bytes, so `in` and `old`
+        // swap roles every step (the loop body holds two steps) and no extra
+        // registers are needed.
+        auto step = [&](int j, uint32_t (&inA)[8], uint32_t (&oldA)[8], uint32_t (&inB)[8],
+                        uint32_t (&oldB)[8]) {
+            const uint32_t bA0 = qA + 32 * j, bB0 = qB + 32 * j;
+            uint32_t bitsA, bitsB;
+            roll32x2<kZeroValue, 0, 4>(hA, inA, oldA, bitsA, hB, inB, oldB, bitsB, laneR, laneW,
+                                       mask, value);
+            roll32x2<kZeroValue, 4, 8>(hA, inA, oldA, bitsA, hB, inB, oldB, bitsB, laneR, laneW,
+                                       mask, value);
             if (j < 7) {  // the next step's bytes into the registers `old` just freed
+                if (full) {
+                    ldg_v8(bytes + bA0 + 32, oldA);
+                    ldg_v8(bytes + bB0 + 32, oldB);
+                } else {
 #pragma unroll
-                for (int c = 0; c < kChains; ++c) {
-                    const uint32_t nq = q[c] + 32 * (j + 1);
-                    if (full) {
-                        ldg_v8(bytes + nq, old[c]);
-                    } else {
-#pragma unroll
-                        for (int i = 0; i < 8; ++i) old[c][i] = 0;
-                        if (nq < nbytes) load32_v8(bytes, nq, lim16, a32, old[c]);
-                    }
+                    for (int i = 0; i < 8; ++i) oldA[i] = oldB[i] = 0;
+                    fetch(bA0 + 32, bB0 + 32, bA0 + 32 < nbytes, bB0 + 32 < nbytes, oldA, oldB);
                 }
             }
-#pragma unroll
-            for (int c = 0; c < kChains; ++c) {
-                const uint32_t b0 = q[c] + 32 * j;
-                uint32_t ew = __funnelshift_l(pb[c], bits[c], 1);
-                if (!full) {  // the batch's ragged end
-                    if (b0 >= nbytes) ew = 0;
-                    else if (b0 + 32 > nbytes) ew &= (1u << (uint32_t)(nbytes - b0)) - 1u;
-                    if (b0 + 32 > nbytes)
-                        bits[c] &= b0 < nbytes ? (1u << (uint32_t)(nbytes - b0)) - 1u : 0u;
-                }
-                if (full || t[c] < n_tiles) bitmap[t[c] * kSelTileWords + lane * 8 + j] = ew;
-                pb[c] = bits[c];
+            uint32_t ewA = __funnelshift_l(pbA, bitsA, 1), ewB = __funnelshift_l(pbB, bitsB, 1);
+            if (!full) {  // the batch's ragged end
+                if (bA0 >= nbytes) ewA = 0;
+                else if (bA0 + 32 > nbytes) ewA &= (1u << (uint32_t)(nbytes - bA0)) - 1u;
+                if (bB0 >= nbytes) ewB = 0;
+                else if (bB0 + 32 > nbytes) ewB &= (1u << (uint32_t)(nbytes - bB0)) - 1u;
+                if (bA0 + 32 > nbytes)
+                    bitsA &= bA0 < nbytes ? (1u << (uint32_t)(nbytes - bA0)) - 1u : 0u;
+                if (bB0 + 32 > nbytes)
+                    bitsB &= bB0 < nbytes ? (1u << (uint32_t)(nbytes - bB0)) - 1u : 0u;
             }
+            sm.cand[lane * 8 + j] = ewA;
+            if (full || tA < n_tiles) bitmap[tA * kSelTileWords + lane * 8 + j] = ewA;
+            if (full || tB < n_tiles) bitmap[tB * kSelTileWords + lane * 8 + j] = ewB;
+            pbA = bitsA;
+            pbB = bitsB;
         };
 #pragma unroll 1
         for (int j = 0; j < 8; j += 2) {
-            step(j, cur, prev);      // prev now holds step j+1's bytes
-            step(j + 1, prev, cur);  // cur now holds step j+2's bytes
+            step(j, curA, prevA, curB, prevB);      // prev now holds step j+1's bytes
+            step(j + 1, prevA, curA, prevB, curB);  // cur now holds step j+2's bytes
+        }
+        // transfer functions of tile A (candidate words already in smem), then B
+        uint32_t fA = (uint32_t)lane << 27, fB = fA;
+        if (tA < n_tiles) {
+            const uint32_t n_ev = apply_items(sm, tA * kSelTile, nbytes, items, n_items, lane);
+            store_events(sm, n_ev, evbuf + (size_t)tA * kEvWords, lane);
+            uint32_t ex;
+            const uint32_t cnt = walk_any(sm, n_ev, lane, ex, nullptr, 0, 0, 0);
+            fA = (ex << 27) | cnt;
+            agg[32 * tA + lane] = fA;
         }
         __syncwarp();
-        // transfer functions of the warp's tiles (entry state = lane)
-#pragma unroll 1
-        for (int c = 0; c < kChains; ++c) {
-            const uint32_t tc = g * kGroup + hw + c * kGroupWarps;
-            uint32_t f = (uint32_t)lane << 27;
-            if (tc < n_tiles) {
+        if (tB < n_tiles) {
 #pragma unroll
-                for (int k = 0; k < 8; ++k)
-                    sm.cand[lane * 8 + k] = bitmap[tc * kSelTileWords + lane * 8 + k];
-                const uint32_t n_ev = apply_items(sm, (uint64_t)tc * kSelTile, nbytes, items,
-                                                  n_items, lane);
-                store_events(sm, n_ev, evbuf + (size_t)tc * kEvWords, lane);
-                uint32_t ex;
-                const uint32_t cnt = walk_any(sm, n_ev, lane, ex, nullptr, 0, 0, 0);
-                f = (ex << 27) | cnt;
-                agg[32 * tc + lane] = f;
-            }
-            fun[par][half][hw + c * kGroupWarps][lane] = f;
-            __syncwarp();
+            for (int k = 0; k < 8; ++k)
+                sm.cand[lane * 8 + k] = bitmap[tB * kSelTileWords + lane * 8 + k];
+            const uint32_t n_ev = apply_items(sm, tB * kSelTile, nbytes, items, n_items, lane);
+            store_events(sm, n_ev, evbuf + (size_t)tB * kEvWords, lane);
+            uint32_t ex;
+            const uint32_t cnt = walk_any(sm, n_ev, lane, ex, nullptr, 0, 0, 0);
+            fB = (ex << 27) | cnt;
+            agg[32 * tB + lane] = fB;
         }
+        fun[par][half][hw][lane] = fA;
+        fun[par][half][hw + kGroupWarps][lane] = fB;
         if (kHalves == 1) __syncthreads();
         else asm volatile("bar.sync %0, %1;" ::"r"(1 + half), "r"(kGroupWarps * 32) : "memory");
         if (hw == 0) {
@@ -723,7 +708,8 @@ void chunk_set_attrs() {
     const uint64_t bit = 1ull << (dev & 63);
     std::lock_guard<std::mutex> lock(mu);
     if (done_mask & bit) return;
-    for (const void* f : {(const void*)rabin_scan_kernel<true>, (const void*)rabin_scan_kernel<false>})
+    for (const void* f : {(const void*)rabin_scan_agg2_kernel<true>,
+                          (const void*)rabin_scan_agg2_kernel<false>})
         cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
     cudaFuncSetAttribute(select_emit_ev_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)sizeof(EmitEvSmem));
@@ -733,8 +719,9 @@ void chunk_set_attrs() {
 
 const char* chunk_unlaunchable() {
     chunk_set_attrs();
-    for (const void* f : {(const void*)rabin_scan_kernel<true>, (const void*)rabin_scan_kernel<false>})
-        if (!fits(f, kScanThreads, kScanSmem)) return "rabin_scan_kernel";
+    for (const void* f : {(const void*)rabin_scan_agg2_kernel<true>,
+                          (const void*)rabin_scan_agg2_kernel<false>})
+        if (!fits(f, kScanThreads, kScanSmem)) return "rabin_scan_agg2_kernel";
     if (!fits((const void*)select_scan_kernel, 1024, 0)) return "select_scan_kernel";
     if (!fits((const void*)select_emit_ev_kernel, kEmitEvWarps * 32, sizeof(EmitEvSmem)))
         return "select_emit_ev_kernel";
@@ -758,12 +745,8 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
     uint64_t gneed = (groups + kHalves - 1) / kHalves;
     gneed = (gneed + DEDUP_SCAN_GROUPS_PER_CTA - 1) / DEDUP_SCAN_GROUPS_PER_CTA;
     const unsigned grid = (unsigned)(gneed < (uint64_t)num_sms ? (gneed ? gneed : 1) : num_sms);
-    // (h & mask) == value for a low-bit mask and value 0 as an IMAD test
-    const bool low = value == 0 && (mask & (mask + 1u)) == 0;
-    const int kbits = __builtin_popcount(mask);  // low: mask = 2^kbits - 1
-    const uint32_t mul = kbits == 0 ? 0u : (kbits == 32 ? 1u : (1u << (32 - kbits)));
-    auto k = low ? rabin_scan_kernel<true> : rabin_scan_kernel<false>;
-    k<<<grid, kScanThreads, kScanSmem, s>>>(d, d_tab, mask, value, mul, bitmap, agg, gagg, evbuf);
+    auto k = value == 0 ? rabin_scan_agg2_kernel<true> : rabin_scan_agg2_kernel<false>;
+    k<<<grid, kScanThreads, kScanSmem, s>>>(d, d_tab, mask, value, bitmap, agg, gagg, evbuf);
     if (after_scan) cudaEventRecordWithFlags(after_scan, s, cudaEventRecordExternal);
     // NEXT-2 max_chunk: the state machine's cuts go to a scratch list first
     uint32_t* final_cut = cut_pos;
