@@ -20,6 +20,10 @@
 //   * unaligned chunk data is read with five 16-byte loads (the next block's
 //     window prefetched during the compression) and realigned with two
 //     select stages + one PRMT per word (PRMT also does the big-endian swap).
+//     Measured alternative (C3, 672 MiB): staging the window in shared memory
+//     with cp.async and reading it back with 17 LDS at the lane's offset saves
+//     the 34 selects (isolated 805 vs 750 GB/s) but its 40 KiB per CTA keeps
+//     SHA-1 CTAs off the SMs that hold a scan CTA: bench 744 vs 790 GB/s.
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -136,47 +140,6 @@ __device__ __forceinline__ void realign(const uint32_t raw[20], uint32_t o, uint
     const uint32_t sel = 0x0123u + (o & 3) * 0x1111u;
 #pragma unroll
     for (int j = 0; j < 16; ++j) M[j] = __byte_perm(v[j], v[j + 1], sel);
-}
-
-#ifndef DEDUP_SHA_SMEM
-#define DEDUP_SHA_SMEM 0
-#endif
-// Staging variant (DEDUP_SHA_SMEM): the next block's 80-byte window goes to a
-// per-lane shared-memory stage with cp.async (LDGSTS, no registers); the
-// message words are read back with 17 LDS at the lane's 4-byte offset, so the
-// two select stages of realign() disappear (34 ALU ops per block).  Stages
-// are stage-major ([stage][thread][80 B]: lane stride 20 words, 8 bank
-// groups).
-constexpr uint32_t kStageBytes = 80;
-__device__ __forceinline__ void cp16(uint32_t dst, const void* src, uint32_t n) {
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(n)
-                 : "memory");
-}
-template <bool kGuard>
-__device__ __forceinline__ void stage_block(uint32_t dst, const uint8_t* __restrict__ bytes,
-                                            uint64_t p, uint64_t lim16) {
-    const uint64_t base = p & ~uint64_t(15);
-#pragma unroll
-    for (int i = 0; i < 5; ++i) {
-        const uint64_t a = base + 16 * i;
-        const bool ok = !kGuard || a < lim16;
-        cp16(dst + 16 * i, bytes + (ok ? a : 0), ok ? 16u : 0u);
-    }
-    asm volatile("cp.async.commit_group;" ::: "memory");
-}
-__device__ __forceinline__ uint32_t lds32(uint32_t a) {
-    uint32_t v;
-    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
-    return v;
-}
-__device__ __forceinline__ void read_block(uint32_t stage, uint32_t o, uint32_t M[16]) {
-    const uint32_t a = stage + (o & ~3u);
-    uint32_t w[17];
-#pragma unroll
-    for (int j = 0; j < 17; ++j) w[j] = lds32(a + 4 * j);
-    const uint32_t sel = 0x0123u + (o & 3) * 0x1111u;
-#pragma unroll
-    for (int j = 0; j < 16; ++j) M[j] = __byte_perm(w[j], w[j + 1], sel);
 }
 
 // FIPS 180-4 5.1.1 padding of the block whose data starts r bytes before the
@@ -300,10 +263,6 @@ sha1_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ cut
     const uint32_t ntasks = (n + 31) >> 5;
     const uint32_t* __restrict__ order = ws + kOrderOff;
     const uint32_t lane = threadIdx.x & 31;
-#if DEDUP_SHA_SMEM
-    __shared__ __align__(16) uint8_t stages[2 * kShaThreads * kStageBytes];
-    const uint32_t smem_base = (uint32_t)__cvta_generic_to_shared(stages);
-#endif
     for (;;) {
         uint32_t task = 0;
         if (lane == 0) task = atomicAdd(&ws[2 * kBuckets], 1u);
@@ -323,40 +282,6 @@ sha1_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ cut
         const uint32_t nbulk = nb_min >= 3 ? nb_min - 2 : 0;
         const uint32_t o = s & 15;
         uint32_t H[5] = {0x67452301u, 0xEFCDAB89u, 0x98BADCFEu, 0x10325476u, 0xC3D2E1F0u};
-#if DEDUP_SHA_SMEM
-        uint64_t p = s;
-        uint32_t M[16];
-        const uint32_t st0 = smem_base + threadIdx.x * kStageBytes;
-        const uint32_t st1 = st0 + kShaThreads * kStageBytes;
-        if (nbulk > 0) stage_block<false>(st0, bytes, p, lim16);
-        else stage_block<true>(st0, bytes, p, lim16);
-        for (uint32_t i = 0; i < nbulk; ++i) {
-            const uint32_t cur = (i & 1) ? st1 : st0, nxt = (i & 1) ? st0 : st1;
-            p += 64;
-            // the next block's window while this one compresses
-            if (i + 1 < nbulk) stage_block<false>(nxt, bytes, p, lim16);
-            else stage_block<true>(nxt, bytes, p, lim16);
-            asm volatile("cp.async.wait_group 1;" ::: "memory");
-            read_block(cur, o, M);
-            sha1_compress(H, M, one);
-        }
-        for (uint32_t i = nbulk; i < nb_max; ++i) {
-            if (i < nb) {
-                const uint32_t cur = (i & 1) ? st1 : st0, nxt = (i & 1) ? st0 : st1;
-                p += 64;
-                if (i + 1 < nb) {
-                    stage_block<true>(nxt, bytes, p, lim16);
-                    asm volatile("cp.async.wait_group 1;" ::: "memory");
-                } else {
-                    asm volatile("cp.async.wait_group 0;" ::: "memory");
-                }
-                read_block(cur, o, M);
-                pad_block(M, (int32_t)L - (int32_t)(64 * i), i + 1 == nb, L);
-                sha1_compress(H, M, one);
-            }
-        }
-        asm volatile("cp.async.wait_group 0;" ::: "memory");
-#else
         uint32_t raw[20];
         uint64_t p = s;
         if (nbulk > 0) load_raw<false>(bytes, p, lim16, raw);
@@ -379,7 +304,6 @@ sha1_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ cut
                 sha1_compress(H, M, one);
             }
         }
-#endif
         if (act) {
             uint32_t* out = reinterpret_cast<uint32_t*>(digest + 20 * (uint64_t)k);
 #pragma unroll

@@ -23,10 +23,20 @@ def cuda():
     return torch.device("cuda:0")
 
 
-def make_ctx(**kw):
+# The engine tests run through dedup_init on every engine of include/dedup.h:
+# the single-GPU engine, and the multi-GPU engine (csrc/mg.cpp) with one rank
+# over NCCL and with 2 / 4 logical ranks on this GPU (copy transport).
+ENGINES = ["single", "nccl1", "copy2", "copy4"]
+
+
+def make_ctx(engine="single", **kw):
     from paper_conf_ipps_rockenbachsgmtd19_b200 import Dedup
     base = dict(batch_bytes=8 << 20, batch_items=1024, slots=3, table_capacity=1 << 18)
     base.update(kw)
+    if engine != "single":
+        G = {"nccl1": 1, "copy2": 2, "copy4": 4}[engine]
+        base.update(num_devices=G, device_ids=[0] * G, transport=1 if engine == "nccl1" else 2,
+                    slots=min(base["slots"], 4))
     return Dedup(0, **base)
 
 
@@ -173,12 +183,13 @@ def test_op_table_min_id_semantics(cuda):
 
 
 # -------------------------------------------------------- full pipeline ----
-def test_engine_c1_bit_exact_device(cuda):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_engine_c1_bit_exact_device(cuda, engine):
     data = synthgen.config_stream("C1")
     off = synthgen.split_items(data)
     want, counts = U.oracle_results(data, off)
     assert 0.3 < counts["dup_chunks"] / counts["chunks"] < 0.7
-    with make_ctx(batch_bytes=4 << 20) as d:
+    with make_ctx(engine, batch_bytes=4 << 20) as d:
         got = U.run_device(d, torch.from_numpy(data).to(cuda), off, 4 << 20)
         st = d.stats()
     U.assert_same(got, want)
@@ -186,11 +197,12 @@ def test_engine_c1_bit_exact_device(cuda):
     assert st["dup_bytes"] == counts["dup_bytes"] and st["bytes"] == counts["bytes"]
 
 
-def test_engine_c1_host_fed(cuda):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_engine_c1_host_fed(cuda, engine):
     data = synthgen.config_stream("C1")
     off = synthgen.split_items(data)
     want, _ = U.oracle_results(data, off)
-    with make_ctx(batch_bytes=3 << 20) as d:
+    with make_ctx(engine, batch_bytes=3 << 20) as d:
         items = U.items_of(data, off)
         got = []
         for k in range(0, len(items), 3):
@@ -208,31 +220,34 @@ def test_engine_c1_host_fed(cuda):
     U.assert_same(got2, want2)
 
 
+@pytest.mark.parametrize("engine", ENGINES)
 @pytest.mark.parametrize("batch_mb", [1, 2, 8])
-def test_batch_size_invariance(cuda, batch_mb):
+def test_batch_size_invariance(cuda, batch_mb, engine):
     data = U.stream(12 << 20, seed=21, dup_frac=0.5)
     off = synthgen.split_items(data)
     want, _ = U.oracle_results(data, off)
-    with make_ctx(batch_bytes=batch_mb << 20, slots=2) as d:
+    with make_ctx(engine, batch_bytes=batch_mb << 20, slots=2) as d:
         got = U.run_device(d, torch.from_numpy(data).to(cuda), off, batch_mb << 20)
     U.assert_same(got, want)
 
 
-def test_tiny_and_empty_items_pipeline(cuda):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_tiny_and_empty_items_pipeline(cuda, engine):
     rng = np.random.default_rng(4)
     lens = [0, 5, 0, 5, 31, 32, 33, 0, 64, 1000, 0, 5]
     base = rng.integers(0, 256, 2000, dtype=np.uint8)
     data = np.concatenate([base[:L] for L in lens]) if sum(lens) else np.zeros(0, np.uint8)
     off = np.concatenate([[0], np.cumsum(lens)]).astype(np.uint64)
     want, _ = U.oracle_results(data, off)
-    with make_ctx(batch_bytes=1 << 16, batch_items=4) as d:
+    with make_ctx(engine, batch_bytes=1 << 16, batch_items=4) as d:
         got = U.run_device(d, torch.from_numpy(np.concatenate([data, np.zeros(16, np.uint8)]))
                            .to(cuda), off, 1 << 16, 4)
     U.assert_same(got, want)
 
 
+@pytest.mark.parametrize("engine", ENGINES)
 @pytest.mark.parametrize("kind", ["all_zero", "hit", "no_hit", "all_dup"])
-def test_adversarial_streams(cuda, kind):
+def test_adversarial_streams(cuda, kind, engine):
     n = 4 << 20
     if kind == "all_zero":
         data = np.zeros(n, np.uint8)
@@ -244,7 +259,7 @@ def test_adversarial_streams(cuda, kind):
         data = synthgen.all_duplicate(n, 52)
     off = synthgen.split_items(data)
     want, _ = U.oracle_results(data, off)
-    with make_ctx(batch_bytes=2 << 20) as d:
+    with make_ctx(engine, batch_bytes=2 << 20) as d:
         got = U.run_device(d, torch.from_numpy(data).to(cuda), off, 2 << 20)
     U.assert_same(got, want)
     if kind in ("all_zero", "hit"):
@@ -253,7 +268,8 @@ def test_adversarial_streams(cuda, kind):
         assert all(g.n_chunks == 1 for g in got)
 
 
-def test_table_chain_orders_batches(cuda):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_table_chain_orders_batches(cuda, engine):
     """Batch 0 = one 1 MiB no-anchor item (a long sequential SHA-1 chain) +
     small item B; batch 1 = a copy of B, submitted right behind it.  Batch 1's
     lookup must wait for batch 0's inserts: B' is a duplicate of B."""
@@ -261,7 +277,7 @@ def test_table_chain_orders_batches(cuda):
     b = np.random.default_rng(8).integers(0, 256, 100, dtype=np.uint8)
     d0 = torch.from_numpy(np.concatenate([long_item, b, np.zeros(12, np.uint8)])).to(cuda)
     d1 = torch.from_numpy(np.concatenate([b, np.zeros(12, np.uint8)])).to(cuda)
-    with make_ctx(batch_bytes=2 << 20, slots=4) as d:
+    with make_ctx(engine, batch_bytes=2 << 20, slots=4) as d:
         for rep in range(4):
             s0 = d.submit_device(d0, np.array([0, 1 << 20, (1 << 20) + 100], np.uint64))
             d.submit_device(d1, np.array([0, 100], np.uint64))
@@ -272,10 +288,11 @@ def test_table_chain_orders_batches(cuda):
             d.end_stream()
 
 
-def test_end_stream_fresh_table(cuda):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_end_stream_fresh_table(cuda, engine):
     data = U.stream(6 << 20, seed=31, dup_frac=0.6)
     off = synthgen.split_items(data)
-    with make_ctx(batch_bytes=2 << 20) as d:
+    with make_ctx(engine, batch_bytes=2 << 20) as d:
         dev = torch.from_numpy(data).to(cuda)
         got1 = U.run_device(d, dev, off, 2 << 20)
         d.end_stream()
@@ -289,14 +306,15 @@ def test_end_stream_fresh_table(cuda):
         U.assert_same(g, want)
 
 
-def test_full_size_c2_bench_config(cuda):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_full_size_c2_bench_config(cuda, engine):
     """BASELINE configs[1] (184 MiB) in the launch configuration bench.py
     times: full bit-exact comparison with the oracle (~3 s of CPU)."""
     import bench
     data = synthgen.config_stream("C2")
     off = synthgen.split_items(data)
     want, counts = U.oracle_results(data, off)
-    with make_ctx(**bench.engine_kwargs(len(data))) as d:
+    with make_ctx(engine, **bench.engine_kwargs(len(data))) as d:
         got = U.run_device(d, torch.from_numpy(data).to(cuda), off, bench.BATCH_BYTES,
                            bench.BATCH_ITEMS)
     U.assert_same(got, want)

@@ -1,12 +1,15 @@
-# One GPU call: build, GPU tests (all or $TESTS), smoke, the bench in the
-# driver's configuration, a long step-only run (steady-state check).
+# One GPU call: build, all GPU tests, smoke, the bench in the driver's
+# configuration, a long step-only run (steady-state check), the reference
+# arm, the N>1 bench path at world 1, launch list + ncu captures.
 mkdir -p gpurun_out
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv > gpurun_out/gpu.txt 2>&1
 nproc > gpurun_out/host.txt; lscpu | grep "Model name" >> gpurun_out/host.txt
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
-timeout 1200 python -m pytest tests -m gpu -x -q ${TESTS:-} > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log
+timeout 1500 python -m pytest tests -m gpu -x -q ${TESTS:-} > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log
 timeout 120 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?" >> gpurun_out/smoke.log
 timeout 900 python bench.py --gpus 1 --steps 20 --warmup 5 > gpurun_out/bench.log 2>&1; echo "bench rc=$?" >> gpurun_out/bench.log
 timeout 300 python bench.py --steps 600 --warmup 5 --step-only > gpurun_out/bench_600.log 2>&1; echo "rc=$?" >> gpurun_out/bench_600.log
-timeout 300 python bench.py --steps 20 --warmup 5 --step-only > gpurun_out/bench_20.log 2>&1; echo "rc=$?" >> gpurun_out/bench_20.log
+timeout 300 python bench.py --impl reference --steps 20 --warmup 5 > gpurun_out/bench_ref.log 2>&1; echo "rc=$?" >> gpurun_out/bench_ref.log
+timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 1 --master-addr 127.0.0.1 --master-port 29533 bench.py --gpus 2 --steps 20 --warmup 5 --no-cpu-baseline > gpurun_out/dist_bench_w1.log 2>&1; echo "rc=$?" >> gpurun_out/dist_bench_w1.log
+${PROFILES:-true} && bash tools/gpu_profiles.sh
 echo done
