@@ -286,7 +286,8 @@ def batch_sweep(data, sizes=(1, 2, 4, 8, 16, 32, 64), target_bytes=2 << 30):
         with Dedup(0, batch_bytes=bb, batch_items=max(mb, 1) + 1, slots=SLOTS,
                    table_capacity=max(1 << 16, len(data) // 2048), host_fed=False) as d:
             prod = torch.cuda.current_stream().cuda_stream
-            passes = max(2, int(target_bytes // len(data)))
+            # enough batches that the SLOTS in flight reach steady state
+            passes = max(2, int(max(target_bytes, 4 * SLOTS * bb) // len(data)))
             ms, ds, _ = timed_passes(
                 d, lambda b: d.submit_device(subs[b][0], subs[b][1], prod), len(plan),
                 passes, 1)

@@ -590,6 +590,8 @@ dedup_status apply_resets(Engine* E, Rank& r, uint64_t w) {
 dedup_status rank_complete(Engine* E, Rank& r, uint64_t w) {
     Slot& sl = *r.slots[w % E->nslots];
     const uint32_t G = E->G;
+    if (sl.wave != w || r.done_wave != w || r.next_wave <= w)
+        return E->fail(DEDUP_ECUDA, "protocol: completion of a wave this rank did not submit");
     MCU(cudaSetDevice(r.dev));
     sl.timed = (w % E->time_every) == 0;
     if (E->copy) {
@@ -1154,6 +1156,9 @@ dedup_status drain(CtxEngine* e, uint32_t max_items, int32_t wait_ms, dedup_item
         if (!sl.parsed) {
             if (w >= e->complete_issued) {
                 if (!may_block) break;
+                // a wave completes only once every rank has its batch: pad
+                // the partly filled one first (its other ranks get empty batches)
+                if (w >= e->fill_wave && !e->close_partial()) break;
                 while (e->complete_issued <= w)
                     e->push_all({CtxEngine::Cmd::COMPLETE, e->complete_issued++});
             }
