@@ -100,7 +100,20 @@ typedef struct {
                                    devices), 2 in-process copy (peer loads over NVLink, or
                                    the loopback when device ids repeat) */
     const int32_t* device_ids;  /* [num_devices] CUDA ordinals, may repeat; NULL = 0..G-1 */
-    uint32_t reserved[2];
+    /* Carry-over mode (row NEXT-2; north_star: "the chunking is identical when
+     * the input is split at arbitrary batch cuts"): 1 = the bytes of a dedup
+     * stream form ONE chunking domain and every submitted item is a PIECE of
+     * it, cut anywhere (pieces of 0 bytes allowed); one piece per GPU batch.
+     * A piece's results are the chunks that END in it: chunk 0 may have begun
+     * in earlier pieces (dedup_item_result.carried = its bytes there), the
+     * chunk open at the piece end is reported by a later piece, and
+     * dedup_end_stream submits a closing item (0 bytes, seq = the next seq)
+     * that reports the stream's last chunk.  Ids are (piece seq << 32) |
+     * index: stream order.  Requires the single-GPU engine, min_chunk 32,
+     * max_chunk 0 and slots >= 2 (EUNSUPPORTED otherwise); at most slots - 1
+     * pieces are in flight. */
+    uint32_t carry_over;
+    uint32_t reserved[1];
 } dedup_config;
 
 /* Fills *cfg with the defaults above (struct_size set). */
@@ -153,14 +166,18 @@ dedup_status dedup_submit_device(dedup_ctx* c, const uint8_t* d_bytes, uint64_t 
 dedup_status dedup_join(dedup_ctx* c, void* stream);
 
 /* Marks the end of the current dedup stream: items submitted afterwards are
- * checked against a fresh (empty) digest table.  Sequence numbers continue. */
+ * checked against a fresh (empty) digest table.  Sequence numbers continue.
+ * Carry-over mode: first submits the stream's closing item (see carry_over;
+ * EAGAIN if no slot is free for it). */
 dedup_status dedup_end_stream(dedup_ctx* c);
 
 typedef struct {
     uint64_t seq;             /* sequence number (submission order) */
     uint64_t item_len;        /* bytes */
     uint32_t n_chunks;        /* 0 for an empty item */
-    uint32_t reserved;
+    uint32_t carried;         /* carry-over mode: bytes of chunk 0 that lie in earlier pieces
+                                 (chunk 0 then starts `carried` bytes before this item,
+                                 chunk_start[0] = 0; saturated at 2^32 - 1); else 0 */
     const uint32_t* chunk_start; /* [n_chunks] item-relative starts, [0] = 0, increasing (startPos) */
     const uint8_t* digest;    /* [n_chunks * 20] SHA-1, FIPS byte order */
     const uint8_t* is_dup;    /* [n_chunks] 1 iff an earlier chunk of the stream has the same digest */

@@ -79,14 +79,15 @@ class Config(ctypes.Structure):
         ("owner_rank", ctypes.c_uint32), ("num_owners", ctypes.c_uint32),
         ("host_fed", ctypes.c_uint32), ("sha_lane_bytes", ctypes.c_uint32),
         ("num_devices", ctypes.c_uint32), ("transport", ctypes.c_uint32),
-        ("device_ids", ctypes.POINTER(ctypes.c_int32)), ("reserved", ctypes.c_uint32 * 2),
+        ("device_ids", ctypes.POINTER(ctypes.c_int32)), ("carry_over", ctypes.c_uint32),
+        ("reserved", ctypes.c_uint32 * 1),
     ]
 
 
 class ItemResult(ctypes.Structure):
     _fields_ = [
         ("seq", ctypes.c_uint64), ("item_len", ctypes.c_uint64),
-        ("n_chunks", ctypes.c_uint32), ("reserved", ctypes.c_uint32),
+        ("n_chunks", ctypes.c_uint32), ("carried", ctypes.c_uint32),
         ("chunk_start", ctypes.POINTER(ctypes.c_uint32)),
         ("digest", ctypes.POINTER(ctypes.c_uint8)),
         ("is_dup", ctypes.POINTER(ctypes.c_uint8)),

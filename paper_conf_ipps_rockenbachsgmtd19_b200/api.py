@@ -26,6 +26,7 @@ class ItemResult:
     digest: np.ndarray       # u8 [n, 20]
     is_dup: np.ndarray       # u8 [n]
     first_id: np.ndarray     # u64 [n]
+    carried: int = 0         # carry-over mode: bytes of chunk 0 in earlier pieces
 
     @property
     def n_chunks(self) -> int:
@@ -55,14 +56,14 @@ def result_from_c(r: N.ItemResult, copy: bool = True) -> ItemResult:
     if n == 0:
         z = np.zeros(0, np.uint32)
         return ItemResult(int(r.seq), int(r.item_len), z, np.zeros((0, 20), np.uint8),
-                          np.zeros(0, np.uint8), np.zeros(0, np.uint64))
+                          np.zeros(0, np.uint8), np.zeros(0, np.uint64), int(r.carried))
     cs = np.ctypeslib.as_array(r.chunk_start, (n,))
     dg = np.ctypeslib.as_array(r.digest, (n * 20,)).reshape(n, 20)
     dup = np.ctypeslib.as_array(r.is_dup, (n,))
     fid = np.ctypeslib.as_array(r.first_id, (n,))
     if copy:
         cs, dg, dup, fid = cs.copy(), dg.copy(), dup.copy(), fid.copy()
-    return ItemResult(int(r.seq), int(r.item_len), cs, dg, dup, fid)
+    return ItemResult(int(r.seq), int(r.item_len), cs, dg, dup, fid, int(r.carried))
 
 
 def probe_int_rates(device: int = 0) -> dict:
@@ -82,7 +83,7 @@ class Dedup:
                  anchor_value: int = 0, min_chunk: int = 32, max_chunk: int = 0,
                  owner_rank: int = 0, num_owners: int = 1, max_drain: int = 65536,
                  sha_lane_bytes: int = 0, num_devices: int = 0, device_ids=None,
-                 transport: int = 0):
+                 transport: int = 0, carry_over: bool = False):
         """num_devices >= 2 (or transport != 0) selects the multi-GPU engine
         (include/dedup.h): G ranks on device_ids (default 0..G-1; ids may
         repeat: then the ranks share a GPU and exchange through the in-process
@@ -97,7 +98,8 @@ class Dedup:
                          anchor_mask=anchor_mask, anchor_value=anchor_value,
                          min_chunk=min_chunk, max_chunk=max_chunk, owner_rank=owner_rank,
                          num_owners=num_owners, sha_lane_bytes=sha_lane_bytes,
-                         num_devices=num_devices, transport=transport).items():
+                         num_devices=num_devices, transport=transport,
+                         carry_over=int(carry_over)).items():
             setattr(cfg, k, v)
         self._dev_ids = None
         if device_ids is not None:

@@ -57,6 +57,9 @@ struct Slot {
     cudaEvent_t ev_host = nullptr, ev_start = nullptr, ev_h2d = nullptr, ev_scan = nullptr,
                 ev_chunk = nullptr, ev_sha = nullptr, ev_table = nullptr, ev_done = nullptr;
     cudaEvent_t ev_prod = nullptr;  // producer-stream dependency (no timing)
+    // carry-over mode: this slot's batch done with its history / selection /
+    // continued chunk (the next slot's batch waits on them)
+    cudaEvent_t ev_hist = nullptr, ev_sel = nullptr, ev_carry = nullptr;
     cudaGraphExec_t graph = nullptr;
     BatchDesc* d_desc = nullptr;    // device descriptor (graph copies h_desc into it)
     BatchDesc* h_desc = nullptr;    // pinned staging
@@ -85,6 +88,7 @@ struct Slot {
     std::vector<uint64_t> item_len;
     std::vector<uint32_t> item_first, item_n;
     uint32_t next_item = 0;  // next item of this batch to hand out
+    uint32_t carried = 0;    // carry-over: bytes of chunk 0 in earlier pieces (saturated)
 };
 
 struct TableBuf {
@@ -107,6 +111,11 @@ struct dedup_ctx {
     TableBuf local;                   // local-combine table (dedup_op_local_combine)
     TableView* d_local_view = nullptr;
     bool stream_fresh = false;  // next batch starts a new dedup stream
+    // carry-over mode (row NEXT-2): one CarryState per slot (batch in slot i
+    // writes d_carry[i], reads d_carry[i - 1]); carry_started: the current
+    // dedup stream has bytes (its next piece continues it, end_stream closes it)
+    CarryState* d_carry = nullptr;
+    bool carry_started = false;
     uint64_t chunk_cap = 0;     // chunks per slot
     std::deque<int> inflight;   // slot indices in seq order
     std::vector<int> to_release;
@@ -218,12 +227,6 @@ bool usable(const dedup_ctx* c) { return c != nullptr && c->sticky == DEDUP_OK; 
         if ((c)->mg) return fail(c, DEDUP_EUNSUPPORTED, "dedup_op_* need a single-GPU ctx"); \
     } while (0)
 
-// Attribution builds (tools/attrib.sh) only: 1 = omit the SHA-1 kernels,
-// 2 = omit the table kernels, 4 = omit chunk selection.  Results are invalid;
-// the product build has 0.
-#ifndef DEDUP_ATTRIB_SKIP
-#define DEDUP_ATTRIB_SKIP 0
-#endif
 
 TableView table_view(const dedup_ctx* c) {
     const TableBuf& t = c->tables[c->cur_table];
@@ -236,8 +239,7 @@ void enqueue_chunk_sha(dedup_ctx* c, Workspace& w, cudaStream_t s, const BatchDe
                        uint8_t* digest, cudaEvent_t ev_scan, cudaEvent_t ev_chunk,
                        uint32_t* chunk_start, uint64_t* chunk_id, uint32_t* item_first,
                        uint32_t max_items) {
-    if (!(DEDUP_ATTRIB_SKIP & 4))
-        launch_chunk_select(d, c->d_tab, c->cfg.anchor_mask, c->cfg.anchor_value, w.bitmap,
+    launch_chunk_select(d, c->d_tab, c->cfg.anchor_mask, c->cfg.anchor_value, w.bitmap,
                             w.agg, w.gagg, w.gentry, w.evbuf,
                             (max_bytes + kSelTile - 1) / kSelTile, cut_pos, cap, n_chunks,
                             c->num_sms, s, ev_scan, c->cfg.max_chunk, w.mc_ws,
@@ -246,9 +248,33 @@ void enqueue_chunk_sha(dedup_ctx* c, Workspace& w, cudaStream_t s, const BatchDe
         launch_chunk_meta(d, cut_pos, n_chunks, cap, chunk_start, chunk_id, item_first,
                           max_items, c->num_sms, s);
     if (ev_chunk) cudaEventRecordWithFlags(ev_chunk, s, cudaEventRecordExternal);
-    if (digest && !(DEDUP_ATTRIB_SKIP & 1))
+    if (digest)
         launch_sha1(d, max_bytes, cut_pos, n_chunks, cap, w.sha_ws, digest, c->num_sms, s,
                     c->cfg.sha_lane_bytes);
+}
+
+// Carry-over mode (row NEXT-2, csrc/carry.cu): the piece's rows A2-A4, chained
+// to the previous slot's piece through its CarryState and three events.
+// d_small: [0] reported chunks, [4..8] table status, [9] cuts, [10..12] extra.
+void enqueue_carry_chunk_sha(dedup_ctx* c, Slot& sl, Slot& prev, cudaStream_t s, bool se) {
+    const uint64_t cap = c->chunk_cap;
+    uint32_t* n_cuts = sl.d_small + 9;
+    cudaStreamWaitEvent(s, prev.ev_hist, cudaEventWaitExternal);
+    launch_carry_hist(sl.d_desc, s);  // (the scan reads the previous piece's history)
+    cudaEventRecordWithFlags(sl.ev_hist, s, cudaEventRecordExternal);
+    launch_chunk_select(sl.d_desc, c->d_tab, c->cfg.anchor_mask, c->cfg.anchor_value,
+                        sl.ws.bitmap, sl.ws.agg, sl.ws.gagg, sl.ws.gentry, sl.ws.evbuf,
+                        (c->cfg.batch_bytes + kSelTile - 1) / kSelTile, sl.d_cut_pos, cap, n_cuts,
+                        c->num_sms, s, se ? sl.ev_scan : nullptr, 0, nullptr, 0, 32, prev.ev_sel);
+    launch_carry_meta(sl.d_desc, n_cuts, sl.d_cut_pos, cap, sl.d_small, sl.d_chunk_start,
+                      sl.d_chunk_id, sl.d_item_first, sl.d_small + 10, s);
+    cudaEventRecordWithFlags(sl.ev_sel, s, cudaEventRecordExternal);
+    if (se) cudaEventRecordWithFlags(sl.ev_chunk, s, cudaEventRecordExternal);
+    launch_sha1(sl.d_desc, c->cfg.batch_bytes, sl.d_cut_pos, n_cuts, cap, sl.ws.sha_ws,
+                sl.d_digest, c->num_sms, s, c->cfg.sha_lane_bytes);
+    cudaStreamWaitEvent(s, prev.ev_carry, cudaEventWaitExternal);
+    launch_carry_cont(sl.d_desc, n_cuts, sl.d_cut_pos, cap, sl.d_digest, s);
+    cudaEventRecordWithFlags(sl.ev_carry, s, cudaEventRecordExternal);
 }
 
 // Records the per-batch graph of slot i (capture of the slot's stream).
@@ -258,6 +284,7 @@ dedup_status build_graph(dedup_ctx* c, int i) {
     const uint64_t cap = c->chunk_cap;
     cudaStream_t s = sl.stream;
     const bool se = c->stage_events;  // per-stage timing events (DEDUP_STAGE_EVENTS=0: off)
+    const bool carry = c->cfg.carry_over != 0;
     CU(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
     if (se) cudaEventRecordWithFlags(sl.ev_start, s, cudaEventRecordExternal);
     cudaMemcpyAsync(sl.d_desc, sl.h_desc, sizeof(BatchDesc), cudaMemcpyHostToDevice, s);
@@ -265,26 +292,28 @@ dedup_status build_graph(dedup_ctx* c, int i) {
                     cudaMemcpyHostToDevice, s);
     cudaMemsetAsync(sl.d_small, 0, sizeof(uint32_t) * 16, s);  // counts + batch statistics
     if (se) cudaEventRecordWithFlags(sl.ev_h2d, s, cudaEventRecordExternal);
-    enqueue_chunk_sha(c, sl.ws, s, sl.d_desc, c->cfg.batch_bytes, sl.d_cut_pos, cap,
-                      sl.d_small, sl.d_digest, se ? sl.ev_scan : nullptr,
-                      se ? sl.ev_chunk : nullptr, sl.d_chunk_start, sl.d_chunk_id,
-                      sl.d_item_first, c->cfg.batch_items);
+    if (carry)
+        enqueue_carry_chunk_sha(c, sl, prev, s, se);
+    else
+        enqueue_chunk_sha(c, sl.ws, s, sl.d_desc, c->cfg.batch_bytes, sl.d_cut_pos, cap,
+                          sl.d_small, sl.d_digest, se ? sl.ev_scan : nullptr,
+                          se ? sl.ev_chunk : nullptr, sl.d_chunk_start, sl.d_chunk_id,
+                          sl.d_item_first, c->cfg.batch_items);
     if (se) cudaEventRecordWithFlags(sl.ev_sha, s, cudaEventRecordExternal);
     // table work waits for the previous batch's table work (global chain)
     cudaStreamWaitEvent(s, prev.ev_table, cudaEventWaitExternal);
     const TableView* tv = &sl.d_desc->table;
-    if (!(DEDUP_ATTRIB_SKIP & 2)) {
-        launch_table_prepare(sl.d_desc, c->tables[0].capacity, c->num_sms, s);
-        launch_table_insert(tv, sl.d_digest, sl.d_chunk_id, nullptr, sl.d_small, 0, cap,
-                            sl.ws.slot_idx, c->num_sms, s);
-    }
-    if (!(DEDUP_ATTRIB_SKIP & 2)) launch_table_lookup(tv, sl.d_chunk_id, nullptr, sl.d_small, 0, cap, sl.ws.slot_idx,
-                        sl.d_first_id, sl.d_is_dup, sl.d_small + 4, sl.d_cut_pos, sl.d_desc,
-                        c->num_sms, s);
+    launch_table_prepare(sl.d_desc, c->tables[0].capacity, c->num_sms, s);
+    launch_table_insert(tv, sl.d_digest, sl.d_chunk_id, nullptr, sl.d_small, 0, cap,
+                        sl.ws.slot_idx, c->num_sms, s);
+    // (carry-over: the batch statistics are computed on the host, parse_slot)
+    launch_table_lookup(tv, sl.d_chunk_id, nullptr, sl.d_small, 0, cap, sl.ws.slot_idx,
+                            sl.d_first_id, sl.d_is_dup, sl.d_small + 4,
+                            carry ? nullptr : sl.d_cut_pos, sl.d_desc, c->num_sms, s);
     cudaEventRecordWithFlags(sl.ev_table, s, cudaEventRecordExternal);
     launch_pack(sl.d_desc, sl.d_small, cap, c->cfg.batch_items, sl.d_chunk_start, sl.d_first_id,
                 sl.d_digest, sl.d_is_dup, sl.d_item_first, sl.d_small + 4, sl.hdev, c->num_sms,
-                s);
+                s, carry ? sl.d_small + 10 : nullptr);
     cudaEventRecordWithFlags(sl.ev_done, s, cudaEventRecordExternal);
     cudaGraph_t g = nullptr;
     cudaError_t e = cudaStreamEndCapture(s, &g);
@@ -317,6 +346,8 @@ dedup_status slot_alloc(dedup_ctx* c, Slot& sl) {
                            &sl.ev_sha, &sl.ev_table, &sl.ev_done})
         CU(cudaEventCreate(e));
     CU(cudaEventCreateWithFlags(&sl.ev_prod, cudaEventDisableTiming));
+    for (cudaEvent_t* e : {&sl.ev_hist, &sl.ev_sel, &sl.ev_carry})
+        CU(cudaEventCreateWithFlags(e, cudaEventDisableTiming));
     TRY(dalloc(c, &sl.d_desc, 1));
     TRY(halloc(c, &sl.h_desc, 1));
     std::memset(sl.h_desc, 0, sizeof(BatchDesc));
@@ -359,7 +390,7 @@ void slot_free(Slot& sl) {
     if (sl.stream) cudaStreamSynchronize(sl.stream);
     if (sl.graph) cudaGraphExecDestroy(sl.graph);
     for (cudaEvent_t e : {sl.ev_host, sl.ev_start, sl.ev_h2d, sl.ev_scan, sl.ev_chunk, sl.ev_sha,
-                          sl.ev_table, sl.ev_done, sl.ev_prod})
+                          sl.ev_table, sl.ev_done, sl.ev_prod, sl.ev_hist, sl.ev_sel, sl.ev_carry})
         if (e) cudaEventDestroy(e);
     cudaFree(sl.d_desc);
     if (sl.h_desc) cudaFreeHost(sl.h_desc);
@@ -380,10 +411,20 @@ void slot_free(Slot& sl) {
     sl = Slot{};
 }
 
+// Carry-over flags of the next piece (nbytes long); a non-empty piece starts
+// (or continues) the stream's chunking domain.
+uint32_t carry_flags(dedup_ctx* c, uint64_t nbytes) {
+    if (!c->cfg.carry_over) return 0;
+    const uint32_t f = kCarryMode | (c->carry_started ? kCarryCont : 0u);
+    if (nbytes > 0) c->carry_started = true;
+    return f;
+}
+
 // Prepare slot i's descriptor for a batch and launch its graph.
-dedup_status launch_batch(dedup_ctx* c, int i, const uint8_t* d_bytes) {
+dedup_status launch_batch(dedup_ctx* c, int i, const uint8_t* d_bytes, uint32_t carry = 0) {
     Slot& sl = c->slots[i];
     BatchDesc& d = *sl.h_desc;
+    d.carry = carry;
     d.bytes = d_bytes;
     d.nbytes = sl.nbytes;
     d.first_seq = sl.first_seq;
@@ -392,6 +433,12 @@ dedup_status launch_batch(dedup_ctx* c, int i, const uint8_t* d_bytes) {
     d.fresh = c->stream_fresh ? 1u : 0u;
     d.table = table_view(c);
     c->stream_fresh = false;
+    if (c->cfg.carry_over) {
+        const int np = (int)c->slots.size();
+        d.carry_in = c->d_carry + (i + np - 1) % np;
+        d.carry_out = c->d_carry + i;
+        // (carry flags: set by the submitting call)
+    }
     const auto t0 = std::chrono::steady_clock::now();
     CU(cudaGraphLaunch(sl.graph, sl.stream));
     c->st.ms_host_launch +=
@@ -417,6 +464,9 @@ dedup_status check_cfg(const dedup_config* g) {
         return DEDUP_EINVAL;
     if (g->table_capacity < 1 || g->table_capacity > (1ull << 31)) return DEDUP_EINVAL;
     if (g->num_devices > 64 || g->transport > 2) return DEDUP_EINVAL;
+    if (g->carry_over && (mg::wanted(g) || g->min_chunk != 32 || g->max_chunk != 0 ||
+                          g->slots < 2 || g->num_owners != 1))
+        return DEDUP_EUNSUPPORTED;  // carry-over: single-GPU engine, the 32-state selection
     if (mg::wanted(g) && (g->owner_rank != 0 || g->num_owners != 1)) return DEDUP_EINVAL;
     if (g->sha_lane_bytes != 0 && (g->sha_lane_bytes < 64 || g->sha_lane_bytes > (1u << 24)))
         return DEDUP_EINVAL;
@@ -448,8 +498,26 @@ dedup_status parse_slot(dedup_ctx* c, Slot& sl) {
         }
     }
     // batch statistics reduced on the device by the lookup kernel
-    const uint64_t dups = sl.hhost.header[3], dup_bytes = sl.hhost.header[4];
+    uint64_t dups = sl.hhost.header[3], dup_bytes = sl.hhost.header[4];
     c->st.sha1_blocks += sl.hhost.header[5];
+    sl.carried = 0;
+    if (c->cfg.carry_over) {
+        // one piece: chunk 0 may continue from earlier pieces (carried bytes);
+        // the last reported chunk ends at header[8] (the open chunk's start)
+        const HostResultLayout& h = sl.hhost;
+        const uint64_t carried = (uint64_t)h.header[6] | ((uint64_t)h.header[7] << 32);
+        sl.carried = carried > 0xFFFFFFFFull ? 0xFFFFFFFFu : (uint32_t)carried;
+        dups = dup_bytes = 0;
+        for (uint32_t r = 0; r < n; ++r) {
+            const uint64_t e = r + 1 < n ? h.chunk_start[r + 1] : h.header[8];
+            const uint64_t len = e - h.chunk_start[r] + (r == 0 ? carried : 0);
+            c->st.sha1_blocks += (len + 9 + 63) / 64;
+            if (h.is_dup[r]) {
+                ++dups;
+                dup_bytes += len;
+            }
+        }
+    }
     c->st.chunks += n;
     c->st.dup_chunks += dups;
     c->st.unique_chunks += n - dups;
@@ -579,6 +647,11 @@ dedup_status dedup_init(const dedup_config* cfg, dedup_ctx** out) {
             return bail(DEDUP_ECUDA);
     }
     if ((s = ws_alloc(c, c->op_ws, cfg->batch_bytes, c->chunk_cap)) != DEDUP_OK) return bail(s);
+    if (cfg->carry_over) {
+        if ((s = dalloc(c, &c->d_carry, cfg->slots)) != DEDUP_OK) return bail(s);
+        if (cudaMemset(c->d_carry, 0, sizeof(CarryState) * cfg->slots) != cudaSuccess)
+            return bail(DEDUP_ECUDA);
+    }
     if ((s = dalloc(c, &c->op_d_desc, kOpRing)) != DEDUP_OK) return bail(s);
     if ((s = halloc(c, &c->op_h_desc, kOpRing)) != DEDUP_OK) return bail(s);
     for (cudaEvent_t& e : c->op_ev)
@@ -626,6 +699,7 @@ void dedup_destroy(dedup_ctx* c) {
     cudaFree(c->local.status);
     cudaFree(c->d_local_view);
     cudaFree(c->d_tab);
+    cudaFree(c->d_carry);
     if (c->ev_ref) cudaEventDestroy(c->ev_ref);
     delete c;
 }
@@ -655,7 +729,9 @@ dedup_status dedup_submit_batch(dedup_ctx* c, uint32_t n_items, const uint8_t* c
         if (L > c->cfg.batch_bytes || L > 0xFFFFFFFFull)
             return fail(c, DEDUP_EINVAL, "item larger than batch_bytes");
         if (L > 0 && item_ptr[k] == nullptr) return fail(c, DEDUP_EINVAL, "null item pointer");
-        if (k > b0 && (bytes + L > c->cfg.batch_bytes || k - b0 >= c->cfg.batch_items)) {
+        // (carry-over: one piece per batch)
+        if (k > b0 && (bytes + L > c->cfg.batch_bytes || k - b0 >= c->cfg.batch_items ||
+                       c->cfg.carry_over)) {
             plan.emplace_back(b0, k);
             b0 = k;
             bytes = 0;
@@ -663,7 +739,10 @@ dedup_status dedup_submit_batch(dedup_ctx* c, uint32_t n_items, const uint8_t* c
         bytes += L;
     }
     if (n_items > b0) plan.emplace_back(b0, n_items);
-    for (size_t j = 0; j < plan.size(); ++j)  // round-robin slots must all be free
+    // round-robin slots must all be free (carry-over: and the slot after the
+    // last, whose batch reads the state the last one overwrites)
+    const size_t need = plan.size() + (c->cfg.carry_over && !plan.empty() ? 1 : 0);
+    for (size_t j = 0; j < need; ++j)
         if (j >= c->slots.size() || c->slots[(c->next_slot + j) % c->slots.size()].busy)
             return fail(c, DEDUP_EAGAIN, "no free batch slot");
     if (first_seq_out) *first_seq_out = c->next_seq;
@@ -691,7 +770,7 @@ dedup_status dedup_submit_batch(dedup_ctx* c, uint32_t n_items, const uint8_t* c
                 CU(cudaMemcpyAsync(sl.d_bytes + dst, p, len, cudaMemcpyHostToDevice, sl.stream));
             k = j;
         }
-        TRY(launch_batch(c, i, sl.d_bytes));
+        TRY(launch_batch(c, i, sl.d_bytes, carry_flags(c, sl.nbytes)));
         c->next_seq += sl.n_items;
     }
     return DEDUP_OK;
@@ -719,6 +798,11 @@ dedup_status dedup_submit_device(dedup_ctx* c, const uint8_t* d_bytes, uint64_t 
         if (item_off[k + 1] < item_off[k]) return fail(c, DEDUP_EINVAL, "item_off decreasing");
     const int i = (int)c->next_slot;
     if (c->slots[i].busy) return fail(c, DEDUP_EAGAIN, "no free batch slot");
+    if (c->cfg.carry_over) {
+        if (n_items != 1) return fail(c, DEDUP_EINVAL, "carry-over: one piece per batch");
+        if (c->slots[(i + 1) % c->slots.size()].busy)
+            return fail(c, DEDUP_EAGAIN, "no free batch slot");
+    }
     CU(cudaSetDevice(c->cfg.device));
     Slot& sl = c->slots[i];
     sl.host_fed = false;
@@ -731,7 +815,7 @@ dedup_status dedup_submit_device(dedup_ctx* c, const uint8_t* d_bytes, uint64_t 
     CU(cudaEventRecord(sl.ev_prod, static_cast<cudaStream_t>(producer)));
     CU(cudaStreamWaitEvent(sl.stream, sl.ev_prod, 0));
     if (first_seq_out) *first_seq_out = c->next_seq;
-    TRY(launch_batch(c, i, d_bytes));
+    TRY(launch_batch(c, i, d_bytes, carry_flags(c, nbytes)));
     c->next_seq += n_items;
     return DEDUP_OK;
 }
@@ -750,6 +834,25 @@ dedup_status dedup_end_stream(dedup_ctx* c) {
     if (c == nullptr) return DEDUP_EINVAL;
     if (c->mg) return mg::end_stream(c->mg);
     if (!usable(c)) return c->sticky;
+    if (c->cfg.carry_over && c->carry_started) {
+        // the closing batch: an empty piece that reports the stream's last
+        // (open) chunk, checked against the stream's table
+        const int i = (int)c->next_slot;
+        if (c->slots[i].busy || c->slots[(i + 1) % c->slots.size()].busy)
+            return fail(c, DEDUP_EAGAIN, "no free batch slot for the closing batch");
+        CU(cudaSetDevice(c->cfg.device));
+        Slot& sl = c->slots[i];
+        sl.host_fed = false;
+        sl.first_seq = c->next_seq;
+        sl.n_items = 1;
+        sl.nbytes = 0;
+        sl.item_len.assign(1, 0);
+        sl.h_item_off[0] = sl.h_item_off[1] = 0;
+        TRY(launch_batch(c, i, reinterpret_cast<const uint8_t*>(c->d_tab),
+                         kCarryMode | kCarryCont | kCarryClose));
+        c->next_seq += 1;
+        c->carry_started = false;
+    }
     c->cur_table ^= 1;
     c->stream_fresh = true;
     return DEDUP_OK;
@@ -793,7 +896,7 @@ dedup_status dedup_drain(dedup_ctx* c, uint32_t max_items, int32_t wait_ms,
             r.seq = sl.first_seq + k;
             r.item_len = sl.item_len[k];
             r.n_chunks = sl.item_n[k];
-            r.reserved = 0;
+            r.carried = sl.carried;
             if (r.n_chunks) {
                 const uint32_t f = sl.item_first[k];
                 r.chunk_start = sl.hhost.chunk_start + f;

@@ -22,6 +22,23 @@ struct TableView {
 
 // Per-batch parameters, read by the kernels from device memory so that the
 // launch sequence of a batch slot is a fixed CUDA graph.
+// Carry-over mode (row NEXT-2, dedup_config.carry_over): the state of the
+// chunker after a piece of the stream, passed to the next piece's batch.
+struct CarryState {
+    uint32_t H[5];        // SHA-1 state of the open chunk (after its full blocks)
+    uint32_t exit_state;  // positions still blocked at the piece end (0..32)
+    uint64_t open_len;    // bytes of the open chunk so far
+    uint32_t left_n;      // bytes of it not yet compressed (< 64), in left[]
+    uint32_t pad_;
+    uint8_t left[64];
+    uint8_t hist[32];     // the last 32 bytes of the stream so far
+};
+
+// BatchDesc.carry flags
+constexpr uint32_t kCarryMode = 1;   // the batch is one piece of a carry-over stream
+constexpr uint32_t kCarryCont = 2;   // ... continuing the previous piece (not the stream start)
+constexpr uint32_t kCarryClose = 4;  // ... the (empty) closing batch of the stream
+
 struct alignas(64) BatchDesc {
     const uint8_t* bytes;      // batch bytes (16-byte aligned)
     uint64_t nbytes;
@@ -30,6 +47,10 @@ struct alignas(64) BatchDesc {
     uint32_t n_items;
     uint32_t fresh;            // 1: clear the table before inserting
     TableView table;
+    uint32_t carry;            // kCarry* flags (0: the item model, reading O8)
+    uint32_t pad_c;
+    const CarryState* carry_in;  // the previous piece's state (kCarryCont)
+    CarryState* carry_out;       // this piece's state
 };
 
 // ---- product-side Rabin tables (independent of the oracle) ---------------
@@ -81,7 +102,7 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
                          uint32_t* cut_pos, uint64_t cap, uint32_t* n_chunks, int num_sms,
                          cudaStream_t s, cudaEvent_t after_scan, uint32_t max_chunk = 0,
                          uint32_t* mc_ws = nullptr, uint32_t max_items = 0,
-                         uint32_t min_chunk = 32);
+                         uint32_t min_chunk = 32, cudaEvent_t before_select = nullptr);
 // max_chunk workspace words: fsm count (1) + fsm cuts (cap) + item counts and
 // flags (2 x (max_items + 1)).
 inline uint64_t maxchunk_ws_words(uint64_t cap, uint64_t max_items) {
@@ -151,6 +172,16 @@ void launch_local_combine(TableView local, const uint8_t* digest, const uint32_t
                           uint64_t cap, uint32_t* slot_idx, uint32_t* rep, int num_sms,
                           cudaStream_t s, const TableView* d_local);
 
+// ---- carry-over mode (carry.cu, row NEXT-2) ---------------------------------
+void launch_carry_hist(const BatchDesc* d, cudaStream_t s);
+// m_out = reported chunks; extra[0..1] = bytes of chunk 0 in earlier pieces,
+// extra[2] = end of the last reported chunk (piece-relative)
+void launch_carry_meta(const BatchDesc* d, const uint32_t* n_cuts, const uint32_t* cut_pos,
+                       uint64_t cap, uint32_t* m_out, uint32_t* chunk_start, uint64_t* chunk_id,
+                       uint32_t* item_first, uint32_t* extra, cudaStream_t s);
+void launch_carry_cont(const BatchDesc* d, const uint32_t* n_cuts, const uint32_t* cut_pos,
+                       uint64_t cap, uint8_t* digest, cudaStream_t s);
+
 // ---- LZSS FindMatch (lzss.cu, row NEXT-1) ----------------------------------
 uint32_t findmatch_smem(uint32_t window, uint32_t max_coded);
 const char* findmatch_unlaunchable(uint32_t window, uint32_t max_coded);
@@ -174,10 +205,11 @@ struct HostResultLayout {
     uint8_t* is_dup;
     uint32_t* item_first_chunk;
 };
+// extra (optional, carry-over mode): 3 words copied to header[6..8]
 void launch_pack(const BatchDesc* d, const uint32_t* n_chunks, uint64_t cap, uint32_t max_items,
                  const uint32_t* chunk_start, const uint64_t* first_id, const uint8_t* digest,
                  const uint8_t* is_dup, const uint32_t* item_first_chunk,
                  const uint32_t* table_status, HostResultLayout h, int num_sms,
-                 cudaStream_t s);
+                 cudaStream_t s, const uint32_t* extra = nullptr);
 
 }  // namespace dd

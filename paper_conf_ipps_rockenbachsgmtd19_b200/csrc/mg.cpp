@@ -1193,7 +1193,7 @@ dedup_status drain(CtxEngine* e, uint32_t max_items, int32_t wait_ms, dedup_item
             o.seq = sl.first_seq + k;
             o.item_len = sl.item_len[k];
             o.n_chunks = sl.item_n[k];
-            o.reserved = 0;
+            o.carried = 0;
             if (o.n_chunks) {
                 const uint32_t f = sl.item_first_v[k];
                 o.chunk_start = sl.hhost.chunk_start + f;

@@ -236,10 +236,13 @@ __device__ __forceinline__ uint32_t first_item(uint64_t T0, const uint64_t* item
 // Lane's 8 e-space candidate words (already in sm.cand) get the item rules:
 // no candidate at e in [q, q+32) (the window would leave the item), a forced
 // cut at q for every non-empty item; then the summaries and the event list.
-// Returns the number of events (kInf: use the bitmap walker).
+// Returns the number of events (kInf: use the bitmap walker).  first_rule:
+// the first item whose start gets the rules (1 for a carry-over piece that
+// continues the stream: its start is not a cut and its windows reach back
+// into the previous piece).
 __device__ __forceinline__ uint32_t apply_items(SelWarpSmem& sm, uint64_t T0, uint64_t nbytes,
                                                 const uint64_t* item_off, uint32_t n_items,
-                                                int lane) {
+                                                int lane, uint32_t first_rule = 0) {
     uint32_t cw[8], fw[8];
 #pragma unroll
     for (int j = 0; j < 8; ++j) {
@@ -247,7 +250,7 @@ __device__ __forceinline__ uint32_t apply_items(SelWarpSmem& sm, uint64_t T0, ui
         fw[j] = 0;
     }
     const uint64_t E0 = T0 + (uint64_t)lane * kLaneBytes;  // this lane's e-range
-    const uint32_t lo = first_item(T0, item_off, n_items, lane);
+    const uint32_t lo = max(first_item(T0, item_off, n_items, lane), first_rule);
     if (E0 < nbytes && n_items > 0) {
         for (uint32_t it = lo; it < n_items; ++it) {
             const uint64_t q = item_off[it];
@@ -368,6 +371,7 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
     if (threadIdx.x < 512) src[threadIdx.x] = gtab[threadIdx.x];
     const uint64_t* items = cache_items(icache, desc);
     const uint32_t n_items = desc->n_items;
+    const bool cont = (desc->carry & kCarryCont) != 0;
     __syncthreads();
     {
         uint32_t* t32 = reinterpret_cast<uint32_t*>(smem + pad);
@@ -397,15 +401,22 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
         const bool full = a32 && (tB + 1) * kSelTile <= nbytes;
         fetch(qA - 32, qB - 32, qA >= 32 && qA < nbytes, qB >= 32 && qB < nbytes, prevA, prevB);
         fetch(qA, qB, qA < nbytes, qB < nbytes, curA, curB);
+        // carry-over continuation: the stream's 32 bytes before this piece
+        const bool contA = cont && qA == 0;
+        if (contA) {
+            const uint32_t* hw32 = reinterpret_cast<const uint32_t*>(desc->carry_in->hist);
+#pragma unroll
+            for (int i = 0; i < 8; ++i) prevA[i] = hw32[i];
+        }
         uint32_t hA = 0, hB = 0, pbA = 0, pbB = 0;
         {   // warm-up of both chains: the windows ending at q-1
             const uint32_t zero[8] = {0, 0, 0, 0, 0, 0, 0, 0};
             uint32_t bA, bB;
             roll32x2<kZeroValue>(hA, prevA, zero, bA, hB, prevB, zero, bB, laneR, laneW, mask,
                                  value);
-            pbA = qA >= 32 ? bA : 0;
+            pbA = (qA >= 32 || contA) ? bA : 0;
             pbB = qB >= 32 ? bB : 0;
-            if (qA < 32) hA = 0;
+            if (qA < 32 && !contA) hA = 0;
             if (qB < 32) hB = 0;
         }
         // One 32-byte step of both chains: roll `in` against `old`, then the
@@ -456,7 +467,8 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
         // transfer functions of tile A (candidate words already in smem), then B
         uint32_t fA = (uint32_t)lane << 27, fB = fA;
         if (tA < n_tiles) {
-            const uint32_t n_ev = apply_items(sm, tA * kSelTile, nbytes, items, n_items, lane);
+            const uint32_t n_ev =
+                apply_items(sm, tA * kSelTile, nbytes, items, n_items, lane, cont ? 1u : 0u);
             store_events(sm, n_ev, evbuf + (size_t)tA * kEvWords, lane);
             uint32_t ex;
             const uint32_t cnt = walk_any(sm, n_ev, lane, ex, nullptr, 0, 0, 0);
@@ -468,7 +480,8 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
 #pragma unroll
             for (int k = 0; k < 8; ++k)
                 sm.cand[lane * 8 + k] = bitmap[tB * kSelTileWords + lane * 8 + k];
-            const uint32_t n_ev = apply_items(sm, tB * kSelTile, nbytes, items, n_items, lane);
+            const uint32_t n_ev =
+                apply_items(sm, tB * kSelTile, nbytes, items, n_items, lane, cont ? 1u : 0u);
             store_events(sm, n_ev, evbuf + (size_t)tB * kEvWords, lane);
             uint32_t ex;
             const uint32_t cnt = walk_any(sm, n_ev, lane, ex, nullptr, 0, 0, 0);
@@ -523,7 +536,9 @@ select_scan_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restric
     fc[w][lane] = Gc;
     __syncthreads();
     if (threadIdx.x == 0) {
-        uint32_t s = 0, c = 0;  // the batch starts with a forced cut: entry state 0
+        // the batch starts with a forced cut (entry state 0), or continues a
+        // carry-over stream from the previous piece's exit state
+        uint32_t s = (desc->carry & kCarryCont) ? desc->carry_in->exit_state : 0u, c = 0;
         for (int r = 0; r < 32; ++r) {
             es[r] = s;
             ec[r] = c;
@@ -640,7 +655,8 @@ select_emit_ev_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __rest
             for (int k = 0; k < 8; ++k)
                 w.cand[lane * 8 + k] = bitmap[(size_t)td * kSelTileWords + lane * 8 + k];
             const uint32_t n_ev = apply_items(w, (uint64_t)td * kSelTile, nbytes, items,
-                                              n_items, lane);
+                                              n_items, lane,
+                                              (desc->carry & kCarryCont) ? 1u : 0u);
             const uint32_t st = sm.te_state[wid][j];
             if (lane == (int)st) {
                 uint32_t ex;
@@ -734,7 +750,8 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
                          uint32_t* gentry, uint32_t* evbuf, uint64_t max_tiles,
                          uint32_t* cut_pos, uint64_t cap, uint32_t* n_chunks, int num_sms,
                          cudaStream_t s, cudaEvent_t after_scan, uint32_t max_chunk,
-                         uint32_t* mc_ws, uint32_t max_items, uint32_t min_chunk) {
+                         uint32_t* mc_ws, uint32_t max_items, uint32_t min_chunk,
+                         cudaEvent_t before_select) {
     chunk_set_attrs();
     const uint64_t groups = select_groups(max_tiles);
     // A persistent scan CTA takes several groups: fewer, longer-lived CTAs
@@ -756,6 +773,8 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
         n_chunks = mc_ws;
         cut_pos = mc_ws + 1;
     }
+    // carry-over: the entry state is the previous piece's exit state
+    if (before_select) cudaStreamWaitEvent(s, before_select, cudaEventWaitExternal);
     select_scan_kernel<<<1, 1024, 0, s>>>(d, gagg, gentry, n_chunks);
     uint64_t blocks = (groups + kEmitEvWarps - 1) / kEmitEvWarps;
     if (blocks > (uint64_t)num_sms * 4) blocks = (uint64_t)num_sms * 4;

@@ -175,6 +175,16 @@ __device__ __forceinline__ void chunk_bounds(const uint32_t* __restrict__ cut_po
     L = (uint32_t)(e - s);
 }
 
+// Carry-over mode (row NEXT-2): the last chunk of a piece (from its last cut
+// to the piece end) is OPEN -- it continues into the next piece, so only its
+// full 64-byte blocks are compressed here and its state goes to carry_out.
+__device__ __forceinline__ bool last_is_open(const BatchDesc* desc) {
+    return (desc->carry & kCarryMode) && !(desc->carry & kCarryClose);
+}
+__device__ __forceinline__ uint32_t task_blocks(uint64_t L, bool open) {
+    return open ? (uint32_t)(L >> 6) : sha_blocks(L);
+}
+
 // ---- counting sort of the chunks by compressions, longest first ----------
 __global__ void sha_hist_kernel(const BatchDesc* __restrict__ desc,
                                 const uint32_t* __restrict__ cut_pos,
@@ -182,10 +192,11 @@ __global__ void sha_hist_kernel(const BatchDesc* __restrict__ desc,
                                 uint32_t* __restrict__ ws) {
     const uint32_t n = (uint32_t)min((uint64_t)*n_chunks_p, cap);
     const uint64_t nbytes = desc->nbytes;
+    const bool open_last = last_is_open(desc);
     for (uint32_t k = blockIdx.x * blockDim.x + threadIdx.x; k < n; k += gridDim.x * blockDim.x) {
         uint32_t s, L;
         chunk_bounds(cut_pos, k, n, nbytes, s, L);
-        const uint32_t b = bucket_of(sha_blocks(L));
+        const uint32_t b = bucket_of(task_blocks(L, open_last && k + 1 == n));
         const uint32_t peers = __match_any_sync(__activemask(), b);
         if ((threadIdx.x & 31) == (uint32_t)(__ffs(peers) - 1)) atomicAdd(&ws[b], __popc(peers));
     }
@@ -237,10 +248,11 @@ __global__ void sha_scatter_kernel(const BatchDesc* __restrict__ desc,
     const uint32_t n = (uint32_t)min((uint64_t)*n_chunks_p, cap);
     const uint64_t nbytes = desc->nbytes;
     uint32_t* order = ws + kOrderOff;
+    const bool open_last = last_is_open(desc);
     for (uint32_t k = blockIdx.x * blockDim.x + threadIdx.x; k < n; k += gridDim.x * blockDim.x) {
         uint32_t s, L;
         chunk_bounds(cut_pos, k, n, nbytes, s, L);
-        const uint32_t b = bucket_of(sha_blocks(L));
+        const uint32_t b = bucket_of(task_blocks(L, open_last && k + 1 == n));
         const uint32_t peers = __match_any_sync(__activemask(), b);
         const uint32_t lane = threadIdx.x & 31;
         const int leader = __ffs(peers) - 1;
@@ -263,6 +275,10 @@ sha1_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ cut
     const uint32_t ntasks = (n + 31) >> 5;
     const uint32_t* __restrict__ order = ws + kOrderOff;
     const uint32_t lane = threadIdx.x & 31;
+    const bool open_last = last_is_open(desc);
+    // carry-over continuation: reported chunk 0 is the one continued from the
+    // previous piece (hashed by carry_cont_kernel); the cut list's chunks follow
+    const uint32_t shift = (desc->carry & kCarryCont) ? 1u : 0u;
     for (;;) {
         uint32_t task = 0;
         if (lane == 0) task = atomicAdd(&ws[2 * kBuckets], 1u);
@@ -271,10 +287,12 @@ sha1_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ cut
         const uint32_t idx = 32 * task + lane;
         const bool act = idx < n;
         uint32_t k = 0, s = 0, L = 0, nb = 0;
+        bool open = false;
         if (act) {
             k = order[idx];
             chunk_bounds(cut_pos, k, n, nbytes, s, L);
-            nb = sha_blocks(L);
+            open = open_last && k + 1 == n;
+            nb = task_blocks(L, open);
         }
         const uint32_t nb_max = __reduce_max_sync(kFull, nb);
         const uint32_t nb_min = __reduce_min_sync(kFull, act ? nb : kFull);
@@ -300,14 +318,22 @@ sha1_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ cut
                 realign(raw, o, M);
                 p += 64;
                 if (i + 1 < nb) load_raw<true>(bytes, p, lim16, raw);
-                pad_block(M, (int32_t)L - (int32_t)(64 * i), i + 1 == nb, L);
+                pad_block(M, (int32_t)L - (int32_t)(64 * i), i + 1 == nb && !open, L);
                 sha1_compress(H, M, one);
             }
         }
-        if (act) {
-            uint32_t* out = reinterpret_cast<uint32_t*>(digest + 20 * (uint64_t)k);
+        if (act && !open) {
+            uint32_t* out = reinterpret_cast<uint32_t*>(digest + 20 * (uint64_t)(k + shift));
 #pragma unroll
             for (int i = 0; i < 5; ++i) out[i] = __byte_perm(H[i], 0, 0x0123);
+        } else if (act) {  // the open chunk's state for the next piece
+            CarryState* co = desc->carry_out;
+#pragma unroll
+            for (int i = 0; i < 5; ++i) co->H[i] = H[i];
+            co->open_len = L;
+            const uint32_t done = 64 * nb;
+            co->left_n = L - done;
+            for (uint32_t j = done; j < L; ++j) co->left[j - done] = bytes[s + j];
         }
     }
 }

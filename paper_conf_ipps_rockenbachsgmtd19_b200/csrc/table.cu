@@ -316,7 +316,8 @@ __global__ void pack_kernel(const BatchDesc* __restrict__ desc,
                             const uint64_t* __restrict__ first_id,
                             const uint8_t* __restrict__ digest, const uint8_t* __restrict__ is_dup,
                             const uint32_t* __restrict__ item_first_chunk,
-                            const uint32_t* __restrict__ table_status, HostResultLayout h) {
+                            const uint32_t* __restrict__ table_status, HostResultLayout h,
+                            const uint32_t* __restrict__ extra) {
     const uint64_t n = min((uint64_t)*n_chunks_p, cap);
     const uint32_t n_items = desc->n_items;
     const uint64_t tid = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
@@ -328,6 +329,7 @@ __global__ void pack_kernel(const BatchDesc* __restrict__ desc,
         h.header[3] = table_status[2];  // duplicate chunks
         h.header[4] = table_status[3];  // duplicate bytes
         h.header[5] = table_status[4];  // SHA-1 blocks
+        for (int i = 0; i < 3; ++i) h.header[6 + i] = extra != nullptr ? extra[i] : 0u;
     }
     for (uint64_t r = tid; r < n; r += stride) {
         h.chunk_start[r] = chunk_start[r];
@@ -430,10 +432,10 @@ void launch_pack(const BatchDesc* d, const uint32_t* n_chunks, uint64_t cap, uin
                  const uint32_t* chunk_start, const uint64_t* first_id, const uint8_t* digest,
                  const uint8_t* is_dup, const uint32_t* item_first_chunk,
                  const uint32_t* table_status, HostResultLayout h, int num_sms,
-                 cudaStream_t s) {
+                 cudaStream_t s, const uint32_t* extra) {
     pack_kernel<<<grid_for(cap / 4 + max_items + 1, 256, 64, 1), 256, 0, s>>>(
         d, n_chunks, cap, chunk_start, first_id, digest, is_dup, item_first_chunk, table_status,
-        h);
+        h, extra);
 }
 
 }  // namespace dd
