@@ -154,8 +154,16 @@ def submit_pass(d, submit, n_batches, new_stream=True):
     slot ring is relieved by a non-blocking drain (results of the batches
     handed out by the previous drain are released), blocking only if nothing
     has completed."""
-    if new_stream:
-        d.end_stream()
+    if new_stream:  # (carry-over mode: may need a slot for the closing item)
+        while True:
+            try:
+                d.end_stream()
+                break
+            except Exception as e:
+                if "EAGAIN" not in str(e):
+                    raise
+                if d.drain_raw(wait_ms=0) == 0:
+                    d.drain_raw(wait_ms=-1)
     for b in range(n_batches):
         while True:
             try:
@@ -236,6 +244,32 @@ def stream_throughput(name, data, steps=3, warmup=1, distinct=None):
             "chunks_per_pass": ds["chunks"] // steps,
             "dup_ratio": ds["dup_chunks"] / max(ds["chunks"], 1),
             "bytes_per_pass": ds["bytes"] // steps, "passes": steps}
+
+
+def carry_throughput(data, piece=61 * MiB + 48, steps=4, warmup=1):
+    """Row NEXT-2, carry-over mode: the stream as ONE chunking domain cut into
+    pieces of `piece` bytes (not item- or chunk-aligned), device-resident,
+    one piece per batch, each pass a new dedup stream closed by end_stream."""
+    import torch
+
+    from paper_conf_ipps_rockenbachsgmtd19_b200 import Dedup
+    dd = torch.from_numpy(data).cuda()
+    bounds = [(a, min(a + piece, len(data))) for a in range(0, len(data), piece)]
+    subs = [(dd[a:b], np.array([0, b - a], np.uint64)) for a, b in bounds]
+    with Dedup(0, batch_bytes=piece, batch_items=1, slots=SLOTS, carry_over=True,
+               table_capacity=max(1 << 16, len(data) // 2048), host_fed=False) as d:
+        prod = torch.cuda.current_stream().cuda_stream
+
+        def submit(b):
+            d.submit_device(subs[b][0], subs[b][1], prod)
+
+        ms, ds, _ = timed_passes(d, submit, len(subs), steps, warmup)
+    del dd, subs
+    torch.cuda.empty_cache()
+    return {"gbs": ds["bytes"] / (ms * 1e-3) / 1e9, "chunks_per_s": ds["chunks"] / (ms * 1e-3),
+            "chunks_per_pass": ds["chunks"] // steps, "piece_bytes": piece, "passes": steps,
+            "workload": "C3 as one chunking domain (carry-over mode, row NEXT-2), cut into "
+                        f"{len(bounds)} pieces of {piece} B, one piece per batch"}
 
 
 def config_lines(steps):
@@ -695,6 +729,10 @@ def main():
     # ---- the other BASELINE.json configs ----
     cfgs = config_lines(args.steps)
     cfgs["C2_batch_sweep_gbs"] = batch_sweep(synthgen.config_stream("C2"))
+    try:
+        cfgs["C3_carry_over"] = carry_throughput(data)
+    except Exception as e:  # report, keep the bench line
+        cfgs["C3_carry_over"] = {"error": str(e)[:200]}
 
     # ---- end-to-end through the host-fed C ABI ----
     e2e_steps = args.e2e_steps or args.steps

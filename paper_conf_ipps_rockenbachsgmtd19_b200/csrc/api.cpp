@@ -273,7 +273,7 @@ void enqueue_carry_chunk_sha(dedup_ctx* c, Slot& sl, Slot& prev, cudaStream_t s,
     launch_sha1(sl.d_desc, c->cfg.batch_bytes, sl.d_cut_pos, n_cuts, cap, sl.ws.sha_ws,
                 sl.d_digest, c->num_sms, s, c->cfg.sha_lane_bytes);
     cudaStreamWaitEvent(s, prev.ev_carry, cudaEventWaitExternal);
-    launch_carry_cont(sl.d_desc, n_cuts, sl.d_cut_pos, cap, sl.d_digest, s);
+    launch_carry_cont(sl.d_desc, n_cuts, sl.d_cut_pos, cap, sl.d_digest, sl.d_small + 10, s);
     cudaEventRecordWithFlags(sl.ev_carry, s, cudaEventRecordExternal);
 }
 

@@ -129,9 +129,8 @@ __global__ void carry_meta_kernel(const BatchDesc* __restrict__ desc,
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         *m_out = m;
         item_first[0] = m ? 0u : 0xFFFFFFFFu;
-        const uint64_t carried = has_cont ? desc->carry_in->open_len : 0;
-        extra[0] = (uint32_t)carried;
-        extra[1] = (uint32_t)(carried >> 32);
+        // (extra[0..1], the carried bytes, come from carry_cont_kernel: the
+        // previous piece's open length is final only after its SHA-1)
         extra[2] = n > 0 ? cut_pos[n - 1] : 0u;
         uint32_t ex = 0;  // positions still blocked after the piece
         if (n > 0) {
@@ -145,14 +144,40 @@ __global__ void carry_meta_kernel(const BatchDesc* __restrict__ desc,
     }
 }
 
+// 16 big-endian message words at byte offset p of a 16-byte aligned buffer
+// readable to its length rounded up to 16: five 16-byte loads, two word-select
+// stages and a PRMT per word (as sha1_kernel).
+__device__ __forceinline__ void load_block(const uint8_t* __restrict__ bytes, uint64_t p,
+                                           uint32_t W[16]) {
+    const uint64_t base = p & ~uint64_t(15);
+    uint32_t v[20];
+#pragma unroll
+    for (int i = 0; i < 5; ++i) {
+        uint4 x = make_uint4(0, 0, 0, 0);
+        if (i < 4 || (p & 15)) x = __ldg(reinterpret_cast<const uint4*>(bytes + base + 16 * i));
+        v[4 * i] = x.x;
+        v[4 * i + 1] = x.y;
+        v[4 * i + 2] = x.z;
+        v[4 * i + 3] = x.w;
+    }
+    const uint32_t o = (uint32_t)(p & 15), wsh = o >> 2;
+#pragma unroll
+    for (int i = 0; i < 18; ++i) v[i] = (wsh & 2) ? v[i + 2] : v[i];
+#pragma unroll
+    for (int i = 0; i < 17; ++i) v[i] = (wsh & 1) ? v[i + 1] : v[i];
+    const uint32_t sel = 0x0123u + (o & 3) * 0x1111u;
+#pragma unroll
+    for (int j = 0; j < 16; ++j) W[j] = __byte_perm(v[j], v[j + 1], sel);
+}
+
 // The continued chunk: the previous piece's open state + this piece's bytes
 // up to its first cut (the whole piece if it has none).  Finished (digest =
-// reported chunk 0) if the piece has a cut or closes the stream; else the
-// open state moves on to carry_out.
+// reported chunk 0, carried bytes to extra[0..1]) if the piece has a cut or
+// closes the stream; else the open state moves on to carry_out.
 __global__ void carry_cont_kernel(const BatchDesc* __restrict__ desc,
                                   const uint32_t* __restrict__ n_cuts_p,
                                   const uint32_t* __restrict__ cut_pos, uint64_t cap,
-                                  uint8_t* __restrict__ digest) {
+                                  uint8_t* __restrict__ digest, uint32_t* __restrict__ extra) {
     if (threadIdx.x != 0) return;
     const uint32_t fl = desc->carry;
     if (!(fl & kCarryCont)) return;
@@ -162,20 +187,33 @@ __global__ void carry_cont_kernel(const BatchDesc* __restrict__ desc,
     const bool finish = n > 0 || (fl & kCarryClose);
     const uint8_t* __restrict__ bytes = desc->bytes;
     const uint64_t plen = n > 0 ? (uint64_t)cut_pos[0] : desc->nbytes;
+    const uint64_t open_len = in.open_len;
     uint32_t H[5];
 #pragma unroll
     for (int i = 0; i < 5; ++i) H[i] = in.H[i];
     uint8_t buf[64];
     uint32_t bn = in.left_n;
     for (uint32_t i = 0; i < bn; ++i) buf[i] = in.left[i];
-    for (uint64_t i = 0; i < plen; ++i) {
-        buf[bn++] = bytes[i];
+    uint64_t pos = 0;
+    if (bn > 0) {  // complete the buffered block first
+        const uint64_t take = min((uint64_t)(64 - bn), plen);
+        for (uint64_t i = 0; i < take; ++i) buf[bn + i] = bytes[i];
+        bn += (uint32_t)take;
+        pos = take;
         if (bn == 64) {
             compress_bytes(H, buf);
             bn = 0;
         }
     }
-    const uint64_t total = in.open_len + plen;
+    if (bn == 0) {
+        for (; pos + 64 <= plen; pos += 64) {  // full blocks straight from the piece
+            uint32_t W[16];
+            load_block(bytes, pos, W);
+            compress(H, W);
+        }
+        for (; pos < plen; ++pos) buf[bn++] = bytes[pos];
+    }
+    const uint64_t total = open_len + plen;
     if (finish) {  // FIPS 180-4 5.1.1 padding with the chunk's total length
         buf[bn++] = 0x80;
         if (bn > 56) {
@@ -193,6 +231,8 @@ __global__ void carry_cont_kernel(const BatchDesc* __restrict__ desc,
             digest[4 * i + 2] = (uint8_t)(H[i] >> 8);
             digest[4 * i + 3] = (uint8_t)H[i];
         }
+        extra[0] = (uint32_t)open_len;  // bytes of chunk 0 in earlier pieces
+        extra[1] = (uint32_t)(open_len >> 32);
     } else {
 #pragma unroll
         for (int i = 0; i < 5; ++i) out.H[i] = H[i];
@@ -216,8 +256,8 @@ void launch_carry_meta(const BatchDesc* d, const uint32_t* n_cuts, const uint32_
 }
 
 void launch_carry_cont(const BatchDesc* d, const uint32_t* n_cuts, const uint32_t* cut_pos,
-                       uint64_t cap, uint8_t* digest, cudaStream_t s) {
-    carry_cont_kernel<<<1, 32, 0, s>>>(d, n_cuts, cut_pos, cap, digest);
+                       uint64_t cap, uint8_t* digest, uint32_t* extra, cudaStream_t s) {
+    carry_cont_kernel<<<1, 32, 0, s>>>(d, n_cuts, cut_pos, cap, digest, extra);
 }
 
 }  // namespace dd

@@ -180,7 +180,7 @@ void launch_carry_meta(const BatchDesc* d, const uint32_t* n_cuts, const uint32_
                        uint64_t cap, uint32_t* m_out, uint32_t* chunk_start, uint64_t* chunk_id,
                        uint32_t* item_first, uint32_t* extra, cudaStream_t s);
 void launch_carry_cont(const BatchDesc* d, const uint32_t* n_cuts, const uint32_t* cut_pos,
-                       uint64_t cap, uint8_t* digest, cudaStream_t s);
+                       uint64_t cap, uint8_t* digest, uint32_t* extra, cudaStream_t s);
 
 // ---- LZSS FindMatch (lzss.cu, row NEXT-1) ----------------------------------
 uint32_t findmatch_smem(uint32_t window, uint32_t max_coded);
