@@ -34,6 +34,9 @@ namespace dd {
 namespace {
 
 constexpr int kShaThreads = 256;
+#ifndef DEDUP_SHA_FMASEL
+#define DEDUP_SHA_FMASEL 0
+#endif
 #ifndef DEDUP_SHA_MINB
 #define DEDUP_SHA_MINB 4
 #endif
@@ -125,6 +128,15 @@ __device__ __forceinline__ void load_raw(const uint8_t* __restrict__ bytes, uint
     }
 }
 
+// a + (b - a) * m for m in {0, 1}, as two IMADs (inline PTX: ptxas would turn
+// the arithmetic back into a SEL on the ALU pipe)
+__device__ __forceinline__ uint32_t fma_select(uint32_t a, uint32_t b, uint32_t m) {
+    uint32_t d, r;
+    asm("mad.lo.u32 %0, %1, 0xFFFFFFFF, %2;" : "=r"(d) : "r"(a), "r"(b));
+    asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(r) : "r"(d), "r"(m), "r"(a));
+    return r;
+}
+
 // Realign the raw window to byte offset o = p & 15 and byte-swap to 16
 // big-endian message words: two select stages for the word offset, one PRMT
 // per word for the byte offset + endianness.
@@ -133,10 +145,20 @@ __device__ __forceinline__ void realign(const uint32_t raw[20], uint32_t o, uint
 #pragma unroll
     for (int i = 0; i < 20; ++i) v[i] = raw[i];
     const uint32_t wsh = o >> 2;
+#if DEDUP_SHA_FMASEL
+    // word-select stages on the FMA pipe: v = v + (v' - v) * bit (IMAD x 2),
+    // the ALU pipe being the kernel's binding pipe
+    const uint32_t m2 = (wsh >> 1) & 1, m1 = wsh & 1;
+#pragma unroll
+    for (int i = 0; i < 18; ++i) v[i] = fma_select(v[i], v[i + 2], m2);
+#pragma unroll
+    for (int i = 0; i < 17; ++i) v[i] = fma_select(v[i], v[i + 1], m1);
+#else
 #pragma unroll
     for (int i = 0; i < 18; ++i) v[i] = (wsh & 2) ? v[i + 2] : v[i];
 #pragma unroll
     for (int i = 0; i < 17; ++i) v[i] = (wsh & 1) ? v[i + 1] : v[i];
+#endif
     const uint32_t sel = 0x0123u + (o & 3) * 0x1111u;
 #pragma unroll
     for (int j = 0; j < 16; ++j) M[j] = __byte_perm(v[j], v[j + 1], sel);
