@@ -119,7 +119,11 @@ typedef struct {
 /* Fills *cfg with the defaults above (struct_size set). */
 void dedup_config_default(dedup_config* cfg);
 
-/* Creates a ctx on cfg->device: copies the config, builds the Rabin tables,
+/* Creates a ctx (the GPU side of the paper's Dedup pipeline, stages 1-3 of
+ * P:211-215 plus the reorder of P:217) on cfg->device -- or, with
+ * num_devices >= 2, on G GPUs (memory spaces assigned to GPUs
+ * round-robin; one host thread per device): copies the config,
+ * builds the Rabin tables,
  * allocates `slots` batch slots (device + pinned host result buffers) and two
  * digest tables of >= 2 * table_capacity slots (power of two).
  * Errors: EINVAL (bad config), EUNSUPPORTED (window other than 32, or
@@ -136,15 +140,21 @@ const char* dedup_last_error(const dedup_ctx* c);
 /* 1. Streaming API                                                         */
 /* ------------------------------------------------------------------------ */
 
-/* Submits n_items host items (item k = item_len[k] bytes at item_ptr[k]).
- * Items receive consecutive sequence numbers *first_seq_out + k.  Items are
+/* Submits n_items host items (item k = item_len[k] bytes at item_ptr[k]): the
+ * paper's stream of fixed-size batches read by the first pipeline stage
+ * ("read the input file and generate batches of 1MB"), each item a
+ * chunking domain (reading O8).  Items receive consecutive sequence numbers
+ * *first_seq_out + k (the order P:217's reorder stage restores).  Items are
  * packed in order into GPU batches of <= batch_bytes / batch_items; every
- * batch needs a free slot, otherwise nothing is submitted and DEDUP_EAGAIN is
- * returned.  An item longer than batch_bytes or 2^32-1 is EINVAL.
- * Ownership: item buffers are BORROWED until the item is returned by
- * dedup_drain (copies are asynchronous).  Buffers from dedup_host_alloc (or
- * otherwise pinned) are DMA'd directly; other memory goes through the CUDA
- * driver's staging copy (slower).  Requires cfg.host_fed = 1. */
+ * batch needs a free slot ("memory space"), otherwise nothing is
+ * submitted and DEDUP_EAGAIN is returned.  An item longer than batch_bytes or
+ * 2^32-1 is EINVAL.
+ * Ownership: buffers from dedup_host_alloc (or otherwise page-locked) are
+ * DMA'd directly and BORROWED until the item is returned by dedup_drain;
+ * other (pageable) memory is first copied by the calling thread into the
+ * slot's internal page-locked bounce buffer (allocated on first use, one
+ * batch_bytes buffer per slot), so it may be reused as soon as the call
+ * returns.  Requires cfg.host_fed = 1. */
 dedup_status dedup_submit_batch(dedup_ctx* c, uint32_t n_items, const uint8_t* const* item_ptr,
                                 const uint64_t* item_len, uint64_t* first_seq_out);
 
@@ -223,7 +233,10 @@ typedef struct {
     uint32_t num_devices, reserved_;
 } dedup_stats_t;
 
-/* Counters over all drained batches of the ctx (all streams). */
+/* Counters over all drained batches of the ctx (all streams): items, bytes,
+ * chunks and duplicates (the paper's stage-3 outcome; duplicate ratio
+ * by chunk count and by bytes, reading O15), per-stage CUDA-event times and,
+ * for the multi-GPU engine, the bytes of the digest exchange. */
 dedup_status dedup_stats(const dedup_ctx* c, dedup_stats_t* out);
 
 /* Pinned, portable host memory usable as zero-copy DMA source for

@@ -64,6 +64,7 @@ struct Slot {
     BatchDesc* d_desc = nullptr;    // device descriptor (graph copies h_desc into it)
     BatchDesc* h_desc = nullptr;    // pinned staging
     uint8_t* d_bytes = nullptr;     // host-fed input copy
+    uint8_t* h_bounce = nullptr;    // page-locked bounce buffer for pageable items (lazy)
     uint64_t* d_item_off = nullptr;
     uint64_t* h_item_off = nullptr;  // pinned staging of item offsets
     Workspace ws;
@@ -407,6 +408,7 @@ void slot_free(Slot& sl) {
     cudaFree(sl.d_digest);
     cudaFree(sl.d_is_dup);
     if (sl.h_res) cudaFreeHost(sl.h_res);
+    if (sl.h_bounce) cudaFreeHost(sl.h_bounce);
     if (sl.stream) cudaStreamDestroy(sl.stream);
     sl = Slot{};
 }
@@ -766,8 +768,19 @@ dedup_status dedup_submit_batch(dedup_ctx* c, uint32_t n_items, const uint8_t* c
             uint64_t len = sl.item_len[k];
             uint32_t j = k + 1;
             while (j < sl.n_items && item_ptr[r.first + j] == p + len) len += sl.item_len[j++];
-            if (len)
+            if (len) {
+                cudaPointerAttributes pa{};
+                const bool locked = cudaPointerGetAttributes(&pa, p) == cudaSuccess &&
+                                    pa.type == cudaMemoryTypeHost;
+                cudaGetLastError();
+                if (!locked) {  // pageable: through the slot's page-locked bounce buffer
+                    if (sl.h_bounce == nullptr)
+                        TRY(halloc(c, &sl.h_bounce, c->cfg.batch_bytes));
+                    std::memcpy(sl.h_bounce + dst, p, len);
+                    p = sl.h_bounce + dst;
+                }
                 CU(cudaMemcpyAsync(sl.d_bytes + dst, p, len, cudaMemcpyHostToDevice, sl.stream));
+            }
             k = j;
         }
         TRY(launch_batch(c, i, sl.d_bytes, carry_flags(c, sl.nbytes)));
