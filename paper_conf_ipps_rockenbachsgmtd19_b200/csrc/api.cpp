@@ -545,15 +545,17 @@ dedup_status parse_slot(dedup_ctx* c, Slot& sl) {
         c->st.timed_sha1_blocks += sl.hhost.header[5];
     }
     if (c->trace && c->stage_events) {  // DEDUP_TRACE=1: per-batch event timeline (ms)
-        float t[7] = {0, 0, 0, 0, 0, 0, 0};
-        const cudaEvent_t ev[7] = {sl.ev_start, sl.ev_h2d, sl.ev_scan, sl.ev_chunk,
-                                   sl.ev_sha, sl.ev_table, sl.ev_done};
-        for (int k = 0; k < 7; ++k) cudaEventElapsedTime(&t[k], c->ev_ref, ev[k]);
+        // host: the items' H2D starts at `host` (host-fed batches; else = start)
+        float t[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+        const cudaEvent_t ev[8] = {sl.host_fed ? sl.ev_host : sl.ev_start, sl.ev_start,
+                                   sl.ev_h2d, sl.ev_scan, sl.ev_chunk, sl.ev_sha, sl.ev_table,
+                                   sl.ev_done};
+        for (int k = 0; k < 8; ++k) cudaEventElapsedTime(&t[k], c->ev_ref, ev[k]);
         std::fprintf(stderr,
-                     "trace seq=%llu bytes=%llu start=%.3f h2d=%.3f scan=%.3f chunk=%.3f "
-                     "sha=%.3f table=%.3f done=%.3f\n",
+                     "trace seq=%llu bytes=%llu host=%.3f start=%.3f h2d=%.3f scan=%.3f "
+                     "chunk=%.3f sha=%.3f table=%.3f done=%.3f\n",
                      (unsigned long long)sl.first_seq, (unsigned long long)sl.nbytes, t[0], t[1],
-                     t[2], t[3], t[4], t[5], t[6]);
+                     t[2], t[3], t[4], t[5], t[6], t[7]);
     }
     cudaGetLastError();  // clear a possible error from a timing query
     sl.parsed = true;
