@@ -1,11 +1,13 @@
 """bench.py --gpus N (N > 1) under torchrun: one process per GPU, NCCL.
 
-Strong scaling on the headline workload (BASELINE.json configs[2]: the
+Weak scaling on the headline workload (BASELINE.json configs[2]: the
 672 MiB native-sized stream C3 "at 1/2/4/8 GPUs with all-to-all digest
-routing"): a step is one pass over the whole C3 stream as a new dedup
+routing"): a pass is one pass over the whole C3 stream as a new dedup
 stream, its items cut into a multiple of N GPU batches (<= 64 MiB, whole
 items, balanced) that go to the ranks round-robin -- wave v of a pass holds
-batches vN .. vN + N - 1, one per rank.  Every rank runs the C++ wave
+batches vN .. vN + N - 1, one per rank; a step is N passes, so every GPU
+processes one stream's worth (672 MiB) per step at any N, as the single-GPU
+step does.  Every rank runs the C++ wave
 pipeline of the multi-GPU engine (csrc/mg.cpp through dedup_dist_*,
 dist.NativeWavePipeline): local rows of up to DEPTH waves in flight, digests
 routed to their owner rank over NCCL (rows A5-A8).  Consecutive passes run
@@ -116,6 +118,10 @@ def main(args, data, off, B):
                 counted["bytes"] += int(nbytes)
                 counted["chunks"] += int(nchunks)
 
+    def run_step(st, timed, submit_one):  # N passes: one stream's worth per GPU
+        for p in range(st * world, (st + 1) * world):
+            run_pass(p, timed, submit_one)
+
     def run_pass(p, timed, submit_one):
         take(pipe.end_stream(collect=False, drain=False), timed)   # new dedup stream
         for _, k, j, seq in rank_schedule(plan, world, rank, p, n_items):
@@ -125,8 +131,8 @@ def main(args, data, off, B):
         return pipe.submit([(views[(k, j)], off[k:j + 1] - off[k], seq)], collect=False)
 
     def timed_run(submit_one, steps):
-        for p in range(args.warmup):
-            run_pass(p, False, submit_one)
+        for st in range(args.warmup):
+            run_step(st, False, submit_one)
         take(pipe.flush(collect=False), False)
         torch.cuda.synchronize()
         dist.barrier()
@@ -134,8 +140,8 @@ def main(args, data, off, B):
         l0 = pipe.kernel_launches()
         start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         start.record()
-        for p in range(args.warmup, args.warmup + steps):
-            run_pass(p, True, submit_one)
+        for st in range(args.warmup, args.warmup + steps):
+            run_step(st, True, submit_one)
         take(pipe.flush(collect=False), True)
         pipe.join()
         end.record()
@@ -176,12 +182,14 @@ def main(args, data, off, B):
         line = {
             "metric": B.METRIC, "value": value, "unit": "GB/s",
             "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": t / args.steps, "higher_is_better": True, "scaling": "strong",
+            "ms_per_step": t / args.steps, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "u32", "data": "synthetic",
             "chunks_per_s": tot_chunks / (t / 1e3),
-            "config": {"workload": B.WORKLOAD_DESC + f"; the pass split into {len(plan)} "
-                                                     f"batches, {len(plan) // world} waves of "
-                                                     f"one batch per GPU",
+            "config": {"workload": B.WORKLOAD_DESC + f"; at N GPUs a step is N such passes "
+                                                     f"(each a new dedup stream), a pass split "
+                                                     f"into {len(plan)} batches, "
+                                                     f"{len(plan) // world} waves of one batch "
+                                                     "per GPU",
                        "batch_bytes": wave_bytes, "waves_in_flight": DEPTH,
                        "parallelism": f"{world} GPUs (one process each), digest-prefix table "
                                       "sharding, NCCL grouped send/recv (C++ engine)",
