@@ -484,6 +484,9 @@ dedup_status dedup_dist_last_counts(const dedup_dist* d, uint32_t* n_items, uint
 
 /* Kernels this rank's pipeline has launched so far. */
 uint64_t dedup_dist_kernel_launches(const dedup_dist* d);
+/* Bytes this rank has sent to OTHER ranks so far (32-byte records of row A6
+ * and 8-byte replies of row A8, counted at completion). */
+uint64_t dedup_dist_a2a_bytes(const dedup_dist* d);
 
 /* Number of kernels this ctx has launched so far (all layers). */
 uint64_t dedup_kernel_launches(const dedup_ctx* c);

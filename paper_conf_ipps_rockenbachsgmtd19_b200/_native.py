@@ -39,7 +39,7 @@ EXPORTS = [
     "dedup_archive_decode",
     "dedup_nccl_unique_id", "dedup_dist_create", "dedup_dist_destroy", "dedup_dist_last_error",
     "dedup_dist_submit", "dedup_dist_flush", "dedup_dist_join", "dedup_dist_end_stream",
-    "dedup_dist_result", "dedup_dist_kernel_launches",
+    "dedup_dist_result", "dedup_dist_kernel_launches", "dedup_dist_a2a_bytes",
     "dedup_dist_last_counts", "dedup_probe_int_rates",
 ]
 # every symbol declared in include/mandel.h (row NEXT-4)
@@ -175,6 +175,7 @@ def lib():
         "dedup_dist_flush": (st, [vp, P(u32)]),
         "dedup_dist_join": (st, [vp, vp]),
         "dedup_dist_kernel_launches": (u64, [vp]),
+        "dedup_dist_a2a_bytes": (u64, [vp]),
         "dedup_dist_end_stream": (st, [vp]),
         "dedup_dist_result": (st, [vp, P(WaveResult)]),
         "dedup_dist_last_counts": (st, [vp, P(u32), P(u32), P(u64)]),

@@ -190,6 +190,7 @@ struct Engine {
     std::string err = "no error";
     std::atomic<int> sticky{0};
     std::atomic<uint64_t> launches{0};
+    std::atomic<uint64_t> a2a_sent{0};  // NCCL: record + reply bytes sent to other ranks
     uint32_t graph_kernels = 0;
     double timeout_s = 600.0;
 
@@ -627,6 +628,12 @@ dedup_status rank_complete(Engine* E, Rank& r, uint64_t w) {
             ro[p + 1] = ro[p] + rcnt[p];
         }
         if (ro[G] > E->cap * G) return E->fail(DEDUP_ECUDA, "received records exceed capacity");
+        uint64_t sent = 0;
+        for (uint32_t p = 0; p < G; ++p)
+            if (p != r.me)
+                sent += (uint64_t)(soff[p + 1] - soff[p]) * sizeof(dedup_record) +
+                        rcnt[p] * sizeof(uint64_t);
+        E->a2a_sent += sent;
         MTRY(apply_resets(E, r, w));
         MCU(cudaStreamWaitEvent(r.os, sl.e_cnt, 0));
         if (sl.timed) MCU(cudaEventRecord(sl.e_a0, r.os));
@@ -1380,6 +1387,8 @@ dedup_status dedup_dist_join(dedup_dist* d, void* stream) {
 uint64_t dedup_dist_kernel_launches(const dedup_dist* d) {
     return d ? d->E.launches.load() : 0;
 }
+
+uint64_t dedup_dist_a2a_bytes(const dedup_dist* d) { return d ? d->E.a2a_sent.load() : 0; }
 
 dedup_status dedup_dist_end_stream(dedup_dist* d) {
     if (d == nullptr) return DEDUP_EINVAL;

@@ -159,6 +159,10 @@ class NativeWavePipeline:
     def kernel_launches(self) -> int:
         return int(self.N.lib().dedup_dist_kernel_launches(self._d))
 
+    def a2a_bytes(self) -> int:
+        """Record + reply bytes this rank sent to other ranks so far."""
+        return int(self.N.lib().dedup_dist_a2a_bytes(self._d))
+
     def close(self):
         if self._d:
             self.N.lib().dedup_dist_destroy(self._d)

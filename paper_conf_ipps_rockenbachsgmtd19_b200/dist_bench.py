@@ -137,7 +137,7 @@ def main(args, data, off, B):
         torch.cuda.synchronize()
         dist.barrier()
         counted["bytes"] = counted["chunks"] = 0
-        l0 = pipe.kernel_launches()
+        l0, a0 = pipe.kernel_launches(), pipe.a2a_bytes()
         start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         start.record()
         for st in range(args.warmup, args.warmup + steps):
@@ -148,15 +148,15 @@ def main(args, data, off, B):
         torch.cuda.synchronize()
         dist.barrier()
         return reduce_timed(start.elapsed_time(end),
-                            [counted["bytes"], counted["chunks"], pipe.kernel_launches() - l0],
-                            dev)
+                            [counted["bytes"], counted["chunks"], pipe.kernel_launches() - l0,
+                             pipe.a2a_bytes() - a0], dev)
 
     # untimed priming pass: every slot's graph and the NCCL channels set up
     run_pass(0, False, sub_device)
     take(pipe.flush(collect=False), False)
     clk = B.ClockSampler(local)
     with clk:
-        t, (tot_bytes, tot_chunks, launches) = timed_run(sub_device, args.steps)
+        t, (tot_bytes, tot_chunks, launches, a2a) = timed_run(sub_device, args.steps)
     # ---- e2e: the same passes with every batch copied H2D from pinned host
     # memory on the producer stream inside the timed region ----
     mine = [(k, j) for v, k, j, _ in rank_schedule(plan, world, rank, 0, n_items)]
@@ -174,7 +174,7 @@ def main(args, data, off, B):
         return pipe.submit([(buf[:n], off[k:j + 1] - off[k], seq)], collect=False)
 
     e2e_steps = max(3, min(args.steps, 10))
-    te, (e_bytes, e_chunks, _) = timed_run(sub_host, e2e_steps)
+    te, (e_bytes, e_chunks, _, _) = timed_run(sub_host, e2e_steps)
     pipe.close()
     line = None
     if rank == 0:
@@ -195,6 +195,12 @@ def main(args, data, off, B):
                                       "sharding, NCCL grouped send/recv (C++ engine)",
                        "l2": "inputs larger than L2 (672 MiB stream)"},
             "clocks": clk.summary(), "gpu_launches": int(launches),
+            # rows A6 + A8 over NVLink: bytes that left each GPU per second,
+            # against NVLink5's 900 GB/s per direction per GPU (nominal)
+            "a2a": {"bytes_per_step": a2a / args.steps,
+                    "gbs_per_gpu": a2a / world / (t / 1e3) / 1e9,
+                    "nvlink_frac": a2a / world / (t / 1e3) / 1e9 / 900.0,
+                    "peak_source": "nominal NVLink5 900 GB/s per direction per GPU"},
             "e2e": {"value": e_bytes / (te / 1e3) / 1e9, "unit": "GB/s",
                     "h2d_bytes_per_step": e_bytes / e2e_steps,
                     "d2h_bytes_per_step": 33 * e_chunks / e2e_steps, "steps": e2e_steps,
