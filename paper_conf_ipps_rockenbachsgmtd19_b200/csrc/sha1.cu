@@ -35,7 +35,10 @@ namespace {
 
 constexpr int kShaThreads = 256;
 #ifndef DEDUP_SHA_FMASEL
-#define DEDUP_SHA_FMASEL 0
+#define DEDUP_SHA_FMASEL 1
+#endif
+#ifndef DEDUP_SHA_FMAROT
+#define DEDUP_SHA_FMAROT 0  // A/B: bit 0 rotl30, bit 1 the schedule's rotl1 on the FMA pipe
 #endif
 #ifndef DEDUP_SHA_MINB
 #define DEDUP_SHA_MINB 4
@@ -59,6 +62,15 @@ __device__ __forceinline__ uint32_t bucket_of(uint32_t nb) {
 
 __device__ __forceinline__ uint32_t rotl(uint32_t x, int s) { return __funnelshift_l(x, x, s); }
 
+// rotl(x, s) = x * 2^s + hi(x * 2^s) on the FMA pipe (IMAD.HI is half rate);
+// m = 2^s at run time so that ptxas keeps the IMADs
+__device__ __forceinline__ uint32_t rotl_fma(uint32_t x, uint32_t m) {
+    uint32_t h, r;
+    asm("mad.hi.u32 %0, %1, %2, 0;" : "=r"(h) : "r"(x), "r"(m));
+    asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(r) : "r"(x), "r"(m), "r"(h));
+    return r;
+}
+
 // `one` is a runtime 1 (kernel argument): w * one + ... compiles to an IMAD
 // on the FMA pipe, which balances the ALU pipe (LOP3 f, LEA.HI rotl5 + add,
 // SHF rotl30, the schedule's LOP3/SHF) against the FMA pipe (the other adds;
@@ -71,7 +83,8 @@ __device__ __forceinline__ void sha1_compress(uint32_t H[5], uint32_t W[16], uin
         if (t < 16) {
             w = W[t];
         } else {
-            w = rotl(W[(t - 3) & 15] ^ W[(t - 8) & 15] ^ W[(t - 14) & 15] ^ W[t & 15], 1);
+            const uint32_t xw = W[(t - 3) & 15] ^ W[(t - 8) & 15] ^ W[(t - 14) & 15] ^ W[t & 15];
+            w = (DEDUP_SHA_FMAROT & 2) ? rotl_fma(xw, one << 1) : rotl(xw, 1);
             W[t & 15] = w;
         }
         uint32_t f, K;
@@ -96,7 +109,7 @@ __device__ __forceinline__ void sha1_compress(uint32_t H[5], uint32_t W[16], uin
         const uint32_t T = rotl(a, 5) + x;
         e = d;
         d = c;
-        c = rotl(b, 30);
+        c = (DEDUP_SHA_FMAROT & 1) ? rotl_fma(b, one << 30) : rotl(b, 30);
         b = a;
         a = T;
     }
