@@ -104,6 +104,7 @@ struct Slot {
     BatchDesc *d_desc = nullptr, *h_desc = nullptr;
     uint64_t *d_item_off = nullptr, *h_item_off = nullptr;
     uint8_t* d_in = nullptr;  // host-fed input
+    uint8_t* h_bounce = nullptr;  // page-locked bounce buffer for pageable items (lazy)
     // chunking / SHA-1 workspace (as the single-GPU engine's)
     uint32_t *bitmap = nullptr, *agg = nullptr, *gagg = nullptr, *gentry = nullptr,
              *evbuf = nullptr, *counters = nullptr, *slot_idx = nullptr, *sha_ws = nullptr,
@@ -268,7 +269,7 @@ void slot_free(Slot& sl) {
                     (void*)sl.p_rec_off})
         if (p) cudaFree(p);
     for (void* p : {(void*)sl.h_desc, (void*)sl.h_item_off, (void*)sl.h_cnt, (void*)sl.h_self,
-                    (void*)sl.h_res})
+                    (void*)sl.h_res, (void*)sl.h_bounce})
         if (p) cudaFreeHost(p);
     if (sl.s) cudaStreamDestroy(sl.s);
 }
@@ -1078,6 +1079,24 @@ dedup_status submit_host(CtxEngine* e, uint32_t n_items, const uint8_t* const* i
             const uint64_t dst = off[k];
             uint32_t j = k + 1;
             while (j < n && item_ptr[pr.first + j] == p + len) len += item_len[pr.first + j++];
+            if (len) {
+                cudaPointerAttributes pa{};
+                const bool locked = cudaPointerGetAttributes(&pa, p) == cudaSuccess &&
+                                    pa.type == cudaMemoryTypeHost;
+                cudaGetLastError();
+                if (!locked) {  // pageable: into the slot's page-locked bounce buffer now
+                    if (sl.h_bounce == nullptr) {
+                        cudaSetDevice(E.ranks[r]->dev);
+                        if (cudaHostAlloc(reinterpret_cast<void**>(&sl.h_bounce), E.batch_bytes,
+                                          cudaHostAllocPortable) != cudaSuccess) {
+                            sl.h_bounce = nullptr;
+                            return E.fail(DEDUP_ENOMEM, "bounce buffer allocation failed");
+                        }
+                    }
+                    std::memcpy(sl.h_bounce + dst, p, len);
+                    p = sl.h_bounce + dst;
+                }
+            }
             sl.h2d.push_back({p, dst, len});
             k = j;
         }

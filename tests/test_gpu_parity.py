@@ -320,16 +320,17 @@ def test_full_size_c2_bench_config(cuda, engine):
     U.assert_same(got, want)
 
 
-def test_pageable_items_bounce_copied(cuda):
-    """Single-GPU engine: pageable host items go through the slot's page-locked
-    bounce buffer, so the caller may overwrite them as soon as submit returns
-    (include/dedup.h dedup_submit_batch)."""
+@pytest.mark.parametrize("engine", ENGINES)
+def test_pageable_items_bounce_copied(cuda, engine):
+    """Pageable host items go through the slot's page-locked bounce buffer, so
+    the caller may overwrite them as soon as submit returns (include/dedup.h
+    dedup_submit_batch), on every engine."""
     data = U.stream(6 << 20, seed=91, dup_frac=0.5)
     off = synthgen.split_items(data)
     want, _ = U.oracle_results(data, off)
     scratch = data.copy()
     got = []
-    with make_ctx(batch_bytes=2 << 20, slots=2) as d:
+    with make_ctx(engine, batch_bytes=2 << 20, slots=2) as d:
         for k in range(0, len(off) - 1, 2):
             j = min(k + 2, len(off) - 1)
             items = [scratch[int(off[i]):int(off[i + 1])] for i in range(k, j)]
