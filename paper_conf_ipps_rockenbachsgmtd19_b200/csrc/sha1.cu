@@ -37,9 +37,6 @@ constexpr int kShaThreads = 256;
 #ifndef DEDUP_SHA_FMASEL
 #define DEDUP_SHA_FMASEL 1
 #endif
-#ifndef DEDUP_SHA_FMAROT
-#define DEDUP_SHA_FMAROT 0  // A/B: bit 0 rotl30, bit 1 the schedule's rotl1 on the FMA pipe
-#endif
 #ifndef DEDUP_SHA_MINB
 #define DEDUP_SHA_MINB 4
 #endif
@@ -62,19 +59,14 @@ __device__ __forceinline__ uint32_t bucket_of(uint32_t nb) {
 
 __device__ __forceinline__ uint32_t rotl(uint32_t x, int s) { return __funnelshift_l(x, x, s); }
 
-// rotl(x, s) = x * 2^s + hi(x * 2^s) on the FMA pipe (IMAD.HI is half rate);
-// m = 2^s at run time so that ptxas keeps the IMADs
-__device__ __forceinline__ uint32_t rotl_fma(uint32_t x, uint32_t m) {
-    uint32_t h, r;
-    asm("mad.hi.u32 %0, %1, %2, 0;" : "=r"(h) : "r"(x), "r"(m));
-    asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(r) : "r"(x), "r"(m), "r"(h));
-    return r;
-}
-
 // `one` is a runtime 1 (kernel argument): w * one + ... compiles to an IMAD
 // on the FMA pipe, which balances the ALU pipe (LOP3 f, LEA.HI rotl5 + add,
 // SHF rotl30, the schedule's LOP3/SHF) against the FMA pipe (the other adds;
 // measured on B200: LOP3/SHF/LEA.HI/IMAD 16 lanes/clk/SMSP each, IMAD.HI 8).
+// Measured alternative (C3 bench, 300 steps): the rotates as IMAD.HI +
+// IMAD on the FMA pipe (x * 2^s + hi(x * 2^s)) -- rotl30: 773 GB/s, the
+// schedule's rotl1: 781, SHF (kept): 805; IMAD.HI's half rate costs more
+// than the ALU slot it frees.
 __device__ __forceinline__ void sha1_compress(uint32_t H[5], uint32_t W[16], uint32_t one) {
     uint32_t a = H[0], b = H[1], c = H[2], d = H[3], e = H[4];
 #pragma unroll
@@ -84,7 +76,7 @@ __device__ __forceinline__ void sha1_compress(uint32_t H[5], uint32_t W[16], uin
             w = W[t];
         } else {
             const uint32_t xw = W[(t - 3) & 15] ^ W[(t - 8) & 15] ^ W[(t - 14) & 15] ^ W[t & 15];
-            w = (DEDUP_SHA_FMAROT & 2) ? rotl_fma(xw, one << 1) : rotl(xw, 1);
+            w = rotl(xw, 1);
             W[t & 15] = w;
         }
         uint32_t f, K;
@@ -109,7 +101,7 @@ __device__ __forceinline__ void sha1_compress(uint32_t H[5], uint32_t W[16], uin
         const uint32_t T = rotl(a, 5) + x;
         e = d;
         d = c;
-        c = (DEDUP_SHA_FMAROT & 1) ? rotl_fma(b, one << 30) : rotl(b, 30);
+        c = rotl(b, 30);
         b = a;
         a = T;
     }
