@@ -47,7 +47,16 @@ namespace {
 // SM.  Measured (round 2, C3, 672 MiB chunk stage): 4 chains per lane (8
 // warps per group, two groups per CTA) 1220 GB/s at 128 registers and 1171
 // at 96; the anchor test as IMAD + predicated add (FMA pipe) 1341; this
-// kernel 1480 -- neither kept.
+// kernel 1480 -- neither kept.  Measured and not kept (round 2, C3 bench at
+// 300 steps, interleaved reps; this kernel 806-818 GB/s, chunk stage
+// 1486-1504): a 32-warp CTA, two groups (chunk stage 1077, bench 565); the
+// next step's bytes as two 16-byte loads issued half a step earlier (each
+// lane-strided 16-byte load fetches its whole sector: 1179, bench 698); L2 or
+// L1 prefetch of the next step's sector (1339, bench 757); L2 prefetch of the
+// next group's first bytes (1468, bench 801); the next group's warm-up bytes
+// loaded into registers before this group's tail (1479, bench 806); the
+// warm-up without the (zero) W lookups (1472, bench 810); the candidate bit
+// insert as a predicated IMAD on the FMA pipe (1461, bench 797).
 #ifndef DEDUP_SCAN_GROUPS_PER_CTA
 #define DEDUP_SCAN_GROUPS_PER_CTA 4  // select groups per scan CTA (launch_chunk_select)
 #endif
