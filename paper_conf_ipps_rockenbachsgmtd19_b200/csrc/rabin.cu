@@ -57,9 +57,7 @@ namespace {
 // loaded into registers before this group's tail (1479, bench 806); the
 // warm-up without the (zero) W lookups (1472, bench 810); the candidate bit
 // insert as a predicated IMAD on the FMA pipe (1461, bench 797).
-#ifndef DEDUP_SCAN_GROUPS_PER_CTA
-#define DEDUP_SCAN_GROUPS_PER_CTA 4  // select groups per scan CTA (launch_chunk_select)
-#endif
+constexpr int kScanGroupsPerCta = 4;  // select groups per scan CTA (launch_chunk_select)
 constexpr int kScanWarps = 16;
 constexpr int kScanThreads = kScanWarps * 32;
 constexpr int kGroupWarps = 16;                    // warps per select group
@@ -769,7 +767,7 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
     // Measured (bench, C2, 64 MiB batches = 256 groups, SHA lane 32 KiB,
     // 40 slots): 1 group per CTA 632, 2 640, 4 709-716, 8 702, 16 700 GB/s.
     uint64_t gneed = (groups + kHalves - 1) / kHalves;
-    gneed = (gneed + DEDUP_SCAN_GROUPS_PER_CTA - 1) / DEDUP_SCAN_GROUPS_PER_CTA;
+    gneed = (gneed + kScanGroupsPerCta - 1) / kScanGroupsPerCta;
     const unsigned grid = (unsigned)(gneed < (uint64_t)num_sms ? (gneed ? gneed : 1) : num_sms);
     auto k = value == 0 ? rabin_scan_agg2_kernel<true> : rabin_scan_agg2_kernel<false>;
     k<<<grid, kScanThreads, kScanSmem, s>>>(d, d_tab, mask, value, bitmap, agg, gagg, evbuf);

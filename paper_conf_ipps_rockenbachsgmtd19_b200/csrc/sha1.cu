@@ -34,13 +34,7 @@ namespace dd {
 namespace {
 
 constexpr int kShaThreads = 256;
-#ifndef DEDUP_SHA_FMASEL
-#define DEDUP_SHA_FMASEL 1
-#endif
-#ifndef DEDUP_SHA_MINB
-#define DEDUP_SHA_MINB 4
-#endif
-constexpr int kShaMinBlocks = DEDUP_SHA_MINB;
+constexpr int kShaMinBlocks = 4;  // CTAs per SM (launch bounds: <= 64 registers)
 constexpr uint32_t kFull = 0xFFFFFFFFu;
 
 // Sort keys: the number of compressions nb of a chunk; nb < kExact gets its
@@ -150,7 +144,6 @@ __device__ __forceinline__ void realign(const uint32_t raw[20], uint32_t o, uint
 #pragma unroll
     for (int i = 0; i < 20; ++i) v[i] = raw[i];
     const uint32_t wsh = o >> 2;
-#if DEDUP_SHA_FMASEL
     // word-select stages on the FMA pipe: v = v + (v' - v) * bit (IMAD x 2),
     // the ALU pipe being the kernel's binding pipe
     const uint32_t m2 = (wsh >> 1) & 1, m1 = wsh & 1;
@@ -158,12 +151,6 @@ __device__ __forceinline__ void realign(const uint32_t raw[20], uint32_t o, uint
     for (int i = 0; i < 18; ++i) v[i] = fma_select(v[i], v[i + 2], m2);
 #pragma unroll
     for (int i = 0; i < 17; ++i) v[i] = fma_select(v[i], v[i + 1], m1);
-#else
-#pragma unroll
-    for (int i = 0; i < 18; ++i) v[i] = (wsh & 2) ? v[i + 2] : v[i];
-#pragma unroll
-    for (int i = 0; i < 17; ++i) v[i] = (wsh & 1) ? v[i + 1] : v[i];
-#endif
     const uint32_t sel = 0x0123u + (o & 3) * 0x1111u;
 #pragma unroll
     for (int j = 0; j < 16; ++j) M[j] = __byte_perm(v[j], v[j + 1], sel);
