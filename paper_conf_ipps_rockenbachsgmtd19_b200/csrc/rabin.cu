@@ -56,7 +56,13 @@ namespace {
 // next group's first bytes (1468, bench 801); the next group's warm-up bytes
 // loaded into registers before this group's tail (1479, bench 806); the
 // warm-up without the (zero) W lookups (1472, bench 810); the candidate bit
-// insert as a predicated IMAD on the FMA pipe (1461, bench 797).
+// insert as a predicated IMAD on the FMA pipe (1461, bench 797); two
+// positions per dependent step (h2 = (h << 16 | a << 8 | b) ^ RA[h3] ^ R[h2]
+// ^ W8[oa] ^ W[ob] with RA = x t^40, W8 = o t^264 in a second 64 KiB table
+// pair, h1 computed off the chain for its test: half the chain latency per
+// byte, 3 LDS and 12.3 instructions per byte instead of 2 and 10.6; bit-exact,
+// 1279, bench 731) -- so the kernel is bound by issue / pipe throughput
+// rather than by the rolling chain's latency.
 constexpr int kScanGroupsPerCta = 4;  // select groups per scan CTA (launch_chunk_select)
 constexpr int kScanWarps = 16;
 constexpr int kScanThreads = kScanWarps * 32;
