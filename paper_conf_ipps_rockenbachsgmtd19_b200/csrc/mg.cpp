@@ -99,6 +99,7 @@ struct Barrier {
 struct Slot {
     cudaStream_t s = nullptr;
     cudaEvent_t e_local = nullptr, e_cnt = nullptr, e_done = nullptr, e_prod = nullptr;
+    cudaEvent_t e_rep = nullptr;  // NCCL: this wave's replies are in (owner stream)
     cudaEvent_t e_a0 = nullptr, e_a1 = nullptr;  // exchange + owner phase (timed)
     cudaGraphExec_t graph = nullptr;
     BatchDesc *d_desc = nullptr, *h_desc = nullptr;
@@ -194,6 +195,12 @@ struct Engine {
     std::atomic<uint64_t> a2a_sent{0};  // NCCL: record + reply bytes sent to other ranks
     uint32_t graph_kernels = 0;
     double timeout_s = 600.0;
+    // DEDUP_MG_PROFILE=1: host seconds per section of the NCCL wave path,
+    // printed to stderr when the engine is destroyed (kProf* below)
+    bool profile = false;
+    bool nccl_self = false;  // DEDUP_MG_NCCL_SELF: the own share through NCCL too
+    double prof[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    uint64_t prof_n[8] = {0, 0, 0, 0, 0, 0, 0, 0};
 
     dedup_status fail(dedup_status st, const std::string& m) {
         {
@@ -217,6 +224,22 @@ struct Engine {
         return err;
     }
     ~Engine();
+};
+
+enum { kProfLocal, kProfCounts, kProfWaitCnt, kProfRecords, kProfOwner, kProfReplies,
+       kProfFinish, kProfSubmit };
+struct ProfScope {  // accumulates the scope's host time into E->prof[i]
+    Engine* E;
+    int i;
+    Clock::time_point t0;
+    ProfScope(Engine* e, int k) : E(e), i(k) {
+        if (E->profile) t0 = Clock::now();
+    }
+    ~ProfScope() {
+        if (!E->profile) return;
+        E->prof[i] += std::chrono::duration<double>(Clock::now() - t0).count();
+        E->prof_n[i] += 1;
+    }
 };
 
 #define MCU(x)                                                                        \
@@ -255,7 +278,7 @@ dedup_status hmalloc(Engine* E, T** p, uint64_t n, unsigned flags = cudaHostAllo
 void slot_free(Slot& sl) {
     if (sl.s) cudaStreamSynchronize(sl.s);
     if (sl.graph) cudaGraphExecDestroy(sl.graph);
-    for (cudaEvent_t e : {sl.e_local, sl.e_cnt, sl.e_done, sl.e_prod, sl.e_a0, sl.e_a1,
+    for (cudaEvent_t e : {sl.e_local, sl.e_cnt, sl.e_done, sl.e_prod, sl.e_rep, sl.e_a0, sl.e_a1,
                           sl.e_prod_foreign})
         if (e) cudaEventDestroy(e);
     for (void* p : {(void*)sl.d_desc, (void*)sl.d_item_off, (void*)sl.d_in, (void*)sl.bitmap,
@@ -292,7 +315,21 @@ void rank_free(Rank& r) {
     if (r.cs) cudaStreamDestroy(r.cs);
 }
 
+void prof_dump(Engine* E) {  // DEDUP_MG_PROFILE: print and reset
+    if (!E->profile || E->prof_n[kProfSubmit] + E->prof_n[kProfLocal] == 0) return;
+    static const char* names[8] = {"local rows", "counts exchange", "wait counts", "records",
+                                   "owner", "replies", "finish", "submit call"};
+    for (int i = 0; i < 8; ++i) {
+        if (E->prof_n[i])
+            std::fprintf(stderr, "mg profile: %-16s %8llu calls %8.1f us/call\n", names[i],
+                         (unsigned long long)E->prof_n[i], 1e6 * E->prof[i] / E->prof_n[i]);
+        E->prof[i] = 0;
+        E->prof_n[i] = 0;
+    }
+}
+
 Engine::~Engine() {
+    prof_dump(this);
     for (auto& r : ranks) rank_free(*r);
 }
 
@@ -349,7 +386,7 @@ dedup_status slot_alloc(Engine* E, Rank& r, Slot& sl) {
     const uint64_t cap = E->cap, bb = E->batch_bytes;
     const uint32_t G = E->G, bi = E->batch_items;
     MCU(cudaStreamCreateWithFlags(&sl.s, cudaStreamNonBlocking));
-    for (cudaEvent_t* e : {&sl.e_local, &sl.e_cnt, &sl.e_done, &sl.e_prod})
+    for (cudaEvent_t* e : {&sl.e_local, &sl.e_cnt, &sl.e_done, &sl.e_prod, &sl.e_rep})
         MCU(cudaEventCreateWithFlags(e, cudaEventDisableTiming));
     MCU(cudaEventCreate(&sl.e_a0));
     MCU(cudaEventCreate(&sl.e_a1));
@@ -438,8 +475,13 @@ dedup_status rank_alloc(Engine* E, Rank& r, uint64_t shard_capacity) {
     rabin_tables(E->cfg.poly, tab);
     MTRY(dmalloc(E, &r.d_rtab, 512));
     MCU(cudaMemcpy(r.d_rtab, tab, sizeof(tab), cudaMemcpyHostToDevice));
-    MCU(cudaStreamCreateWithFlags(&r.os, cudaStreamNonBlocking));
-    MCU(cudaStreamCreateWithFlags(&r.cs, cudaStreamNonBlocking));
+    // the owner stream is serial across waves (exchange + table work), the
+    // counts gate the host: both at the highest priority, so that their small
+    // kernels take SMs ahead of the next waves' scan / SHA-1 CTAs
+    int prio_lo = 0, prio_hi = 0;
+    MCU(cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi));
+    MCU(cudaStreamCreateWithPriority(&r.os, cudaStreamNonBlocking, prio_hi));
+    MCU(cudaStreamCreateWithPriority(&r.cs, cudaStreamNonBlocking, prio_hi));
     MCU(cudaEventCreateWithFlags(&r.e_rdy, cudaEventDisableTiming));
     MCU(cudaEventCreateWithFlags(&r.e_fin, cudaEventDisableTiming));
     r.tab_cap = next_pow2(2 * shard_capacity);
@@ -535,17 +577,30 @@ dedup_status rank_submit(Engine* E, Rank& r, uint64_t w) {
             sl.e_prod_foreign = nullptr;
         }
     }
-    MCU(cudaGraphLaunch(sl.graph, sl.s));
+    {
+        ProfScope ps(E, kProfLocal);
+        MCU(cudaGraphLaunch(sl.graph, sl.s));
+    }
     E->launches += E->graph_kernels;
     if (!E->copy) {
+        ProfScope ps(E, kProfCounts);
         // counts of this wave to every peer right behind its local rows (ccomm, cs)
         MCU(cudaStreamWaitEvent(r.cs, sl.e_local, 0));
-        MNC(ncclGroupStart());
-        for (uint32_t p = 0; p < G; ++p) {
-            MNC(ncclSend(sl.send_off + p, 2, ncclUint32, (int)p, r.ccomm, r.cs));
-            MNC(ncclRecv(sl.cnt_recv + 2 * p, 2, ncclUint32, (int)p, r.ccomm, r.cs));
+        // (the rank's own share is a device copy: no NCCL kernel for it,
+        // unless DEDUP_MG_NCCL_SELF -- the tests' way to drive the NCCL calls
+        // at world size 1)
+        if (!E->nccl_self)
+            MCU(cudaMemcpyAsync(sl.cnt_recv + 2 * r.me, sl.send_off + r.me,
+                                2 * sizeof(uint32_t), cudaMemcpyDeviceToDevice, r.cs));
+        if (G > 1 || E->nccl_self) {
+            MNC(ncclGroupStart());
+            for (uint32_t p = 0; p < G; ++p) {
+                if (p == r.me && !E->nccl_self) continue;
+                MNC(ncclSend(sl.send_off + p, 2, ncclUint32, (int)p, r.ccomm, r.cs));
+                MNC(ncclRecv(sl.cnt_recv + 2 * p, 2, ncclUint32, (int)p, r.ccomm, r.cs));
+            }
+            MNC(ncclGroupEnd());
         }
-        MNC(ncclGroupEnd());
         MCU(cudaMemcpyAsync(sl.h_cnt, sl.cnt_recv, sizeof(uint32_t) * 2 * G,
                             cudaMemcpyDeviceToHost, r.cs));
         MCU(cudaEventRecord(sl.e_cnt, r.cs));
@@ -564,16 +619,28 @@ dedup_status owner_work(Engine* E, Rank& r, const uint32_t* d_n, uint64_t n_host
     return DEDUP_OK;
 }
 
-dedup_status finish(Engine* E, Rank& r, Slot& sl) {
-    // this shard's overflow flag and used slots -> small[4..5]; a reply of ~0
-    // (any owner overflowed) also sets small[4] (scatter)
+// Rows A8 (scatter of the replies) and A9 (pack to pinned host memory) of a
+// wave.  The shard's overflow flag and used slots are copied on the owner
+// stream (before a later wave's reset can clear them) -> small[4..5]; a
+// reply of ~0 (any owner overflowed) also sets small[4] (scatter).  With
+// on_slot the scatter and pack run on the slot's stream behind the wave's
+// replies, so the owner stream -- serial across waves -- carries only the
+// exchange and the table work.
+dedup_status finish(Engine* E, Rank& r, Slot& sl, bool on_slot = false) {
     MCU(cudaMemcpyAsync(sl.small + 4, r.tab_status, 2 * sizeof(uint32_t),
                         cudaMemcpyDeviceToDevice, r.os));
+    cudaStream_t st = r.os;
+    if (on_slot) {
+        if (sl.timed) MCU(cudaEventRecord(sl.e_a1, r.os));
+        MCU(cudaEventRecord(sl.e_rep, r.os));
+        MCU(cudaStreamWaitEvent(sl.s, sl.e_rep, 0));
+        st = sl.s;
+    }
     launch_scatter(sl.reply_back, sl.send_pos, sl.rep, sl.chunk_id, sl.small, E->cap,
-                   sl.first_id, sl.is_dup, r.num_sms, r.os, sl.small + 4);
-    if (sl.timed) MCU(cudaEventRecord(sl.e_a1, r.os));
+                   sl.first_id, sl.is_dup, r.num_sms, st, sl.small + 4);
+    if (sl.timed && !on_slot) MCU(cudaEventRecord(sl.e_a1, r.os));
     launch_pack(sl.d_desc, sl.small, E->cap, E->batch_items, sl.chunk_start, sl.first_id,
-                sl.digest, sl.is_dup, sl.item_first, sl.small + 4, sl.hdev, r.num_sms, r.os);
+                sl.digest, sl.is_dup, sl.item_first, sl.small + 4, sl.hdev, r.num_sms, st);
     E->launches += 2;
     MCU(cudaGetLastError());
     return DEDUP_OK;
@@ -621,7 +688,10 @@ dedup_status rank_complete(Engine* E, Rank& r, uint64_t w) {
         if (!E->bar.wait(E->abort)) return (dedup_status)E->sticky.load();  // all pulled
         for (auto& q : E->ranks) MCU(cudaStreamWaitEvent(r.os, q->e_fin, 0));
     } else {
-        MTRY(wait_event(E, r, sl.e_cnt));  // sizes of the payload (host)
+        {
+            ProfScope ps(E, kProfWaitCnt);
+            MTRY(wait_event(E, r, sl.e_cnt));  // sizes of the payload (host)
+        }
         const uint32_t* soff = sl.h_self;
         std::vector<uint64_t> rcnt(G), ro(G + 1, 0);
         for (uint32_t p = 0; p < G; ++p) {
@@ -638,26 +708,54 @@ dedup_status rank_complete(Engine* E, Rank& r, uint64_t w) {
         MTRY(apply_resets(E, r, w));
         MCU(cudaStreamWaitEvent(r.os, sl.e_cnt, 0));
         if (sl.timed) MCU(cudaEventRecord(sl.e_a0, r.os));
-        MNC(ncclGroupStart());  // row A6
-        for (uint32_t p = 0; p < G; ++p) {
-            const uint64_t ns = soff[p + 1] - soff[p], nr = rcnt[p];
-            if (ns) MNC(ncclSend(sl.send + soff[p], ns * sizeof(dedup_record), ncclUint8, (int)p,
-                                 r.comm, r.os));
-            if (nr) MNC(ncclRecv(r.recv + ro[p], nr * sizeof(dedup_record), ncclUint8, (int)p,
-                                 r.comm, r.os));
+        {
+            ProfScope ps(E, kProfRecords);
+            const uint64_t nself = soff[r.me + 1] - soff[r.me];  // == rcnt[me]
+            if (nself && !E->nccl_self)  // own records: a device copy
+                MCU(cudaMemcpyAsync(r.recv + ro[r.me], sl.send + soff[r.me],
+                                    nself * sizeof(dedup_record), cudaMemcpyDeviceToDevice, r.os));
+            if (G > 1 || E->nccl_self) {
+                MNC(ncclGroupStart());  // row A6
+                for (uint32_t p = 0; p < G; ++p) {
+                    const uint64_t ns = soff[p + 1] - soff[p], nr = rcnt[p];
+                    if (p == r.me && !E->nccl_self) continue;
+                    if (ns) MNC(ncclSend(sl.send + soff[p], ns * sizeof(dedup_record), ncclUint8,
+                                         (int)p, r.comm, r.os));
+                    if (nr) MNC(ncclRecv(r.recv + ro[p], nr * sizeof(dedup_record), ncclUint8,
+                                         (int)p, r.comm, r.os));
+                }
+                MNC(ncclGroupEnd());
+            }
         }
-        MNC(ncclGroupEnd());
-        if (ro[G]) MTRY(owner_work(E, r, nullptr, ro[G], ro[G]));  // row A7
-        MNC(ncclGroupStart());  // row A8
-        for (uint32_t p = 0; p < G; ++p) {
-            const uint64_t ns = soff[p + 1] - soff[p], nr = rcnt[p];
-            if (nr) MNC(ncclSend(r.reply + ro[p], nr, ncclUint64, (int)p, r.comm, r.os));
-            if (ns) MNC(ncclRecv(sl.reply_back + soff[p], ns, ncclUint64, (int)p, r.comm, r.os));
+        {
+            ProfScope ps(E, kProfOwner);
+            if (ro[G]) MTRY(owner_work(E, r, nullptr, ro[G], ro[G]));  // row A7
         }
-        MNC(ncclGroupEnd());
-        MTRY(finish(E, r, sl));
+        {
+            ProfScope ps(E, kProfReplies);
+            const uint64_t nself = soff[r.me + 1] - soff[r.me];
+            if (nself && !E->nccl_self)  // replies to the own records: a device copy
+                MCU(cudaMemcpyAsync(sl.reply_back + soff[r.me], r.reply + ro[r.me],
+                                    nself * sizeof(uint64_t), cudaMemcpyDeviceToDevice, r.os));
+            if (G > 1 || E->nccl_self) {
+                MNC(ncclGroupStart());  // row A8
+                for (uint32_t p = 0; p < G; ++p) {
+                    const uint64_t ns = soff[p + 1] - soff[p], nr = rcnt[p];
+                    if (p == r.me && !E->nccl_self) continue;
+                    if (nr) MNC(ncclSend(r.reply + ro[p], nr, ncclUint64, (int)p, r.comm, r.os));
+                    if (ns)
+                        MNC(ncclRecv(sl.reply_back + soff[p], ns, ncclUint64, (int)p, r.comm,
+                                     r.os));
+                }
+                MNC(ncclGroupEnd());
+            }
+        }
+        {
+            ProfScope ps(E, kProfFinish);
+            MTRY(finish(E, r, sl, true));
+        }
     }
-    MCU(cudaEventRecord(sl.e_done, r.os));
+    MCU(cudaEventRecord(sl.e_done, E->copy ? r.os : sl.s));
     sl.done_wave.store(w, std::memory_order_release);
     ++r.done_wave;
     return DEDUP_OK;
@@ -796,6 +894,8 @@ dedup_status engine_init(Engine* E, const dedup_config* cfg, uint32_t G, uint32_
     if (const char* v = std::getenv("DEDUP_TIME_EVERY"))
         E->time_every = std::atoi(v) > 0 ? (uint32_t)std::atoi(v) : 1u;
     if (const char* v = std::getenv("DEDUP_MG_TIMEOUT_S")) E->timeout_s = std::atof(v);
+    E->profile = std::getenv("DEDUP_MG_PROFILE") != nullptr;
+    E->nccl_self = std::getenv("DEDUP_MG_NCCL_SELF") != nullptr;
     return DEDUP_OK;
 }
 
@@ -1347,6 +1447,7 @@ dedup_status dedup_dist_submit(dedup_dist* d, const uint8_t* d_bytes, uint64_t n
     *completed = 0;
     Engine* E = &d->E;
     if (E->sticky.load()) return E->sticky.load();
+    ProfScope ps(E, kProfSubmit);
     // argument checks before anything is enqueued (every rank then issues
     // the same NCCL sequence or none)
     if (n_items > E->batch_items || nbytes > E->batch_bytes ||
@@ -1381,7 +1482,10 @@ dedup_status dedup_dist_flush(dedup_dist* d, uint32_t* completed) {
     Engine* E = &d->E;
     if (E->sticky.load()) return E->sticky.load();
     Rank& rk = *E->ranks[0];
-    if (rk.done_wave == rk.next_wave) return DEDUP_OK;
+    if (rk.done_wave == rk.next_wave) {
+        prof_dump(E);  // drained: one profile per drained run
+        return DEDUP_OK;
+    }
     MTRY(rank_complete(E, rk, rk.done_wave));
     d->last_done = (int)((rk.done_wave - 1) % E->nslots);
     Slot& ds = *rk.slots[d->last_done];

@@ -1,6 +1,6 @@
 """GPU tests of the routing ops (row A5: owner split by digest prefix, local
 combine) and of the one-process-per-GPU front end of the multi-GPU engine
-(dedup_dist_*, NCCL at world size 1).  The engine at G > 1 is tested in
+(dedup_dist_*, world size 1: own share by device copy or NCCL).  G > 1 is tested in
 tests/test_gpu_mg.py (G logical ranks on one GPU, the copy transport)."""
 import numpy as np
 import pytest
@@ -70,15 +70,28 @@ def test_local_combine_representatives():
             assert ovf == 0
 
 
+@pytest.fixture(params=["self_copy", "nccl_self"])
+def self_path(request, monkeypatch):
+    """The rank's own share of the exchange: a device copy (the product
+    path), or through NCCL send/recv to itself (DEDUP_MG_NCCL_SELF), which
+    is how the NCCL calls of the exchange run at world size 1."""
+    if request.param == "nccl_self":
+        monkeypatch.setenv("DEDUP_MG_NCCL_SELF", "1")
+    else:
+        monkeypatch.delenv("DEDUP_MG_NCCL_SELF", raising=False)
+    return request.param
+
+
 @pytest.mark.parametrize("drain", [True, False])
 @pytest.mark.parametrize("depth", [1, 3])
-def test_native_wave_pipeline_world1(depth, drain):
+def test_native_wave_pipeline_world1(depth, drain, self_path):
     """The one-process-per-GPU front end of the multi-GPU engine (csrc/mg.cpp,
-    dedup_dist_*) through NCCL with one rank: the exchange sends every record
-    to itself.  Three dedup streams: the first half of the batches, the second
-    half, then the first half again from the same device buffers; bit-exact vs
-    the oracle each time.  drain=False: end_stream with waves in flight (the
-    table reset deferred to the next stream's first wave)."""
+    dedup_dist_*) with one rank: the exchange sends every record to itself
+    (a device copy, or NCCL send/recv to itself).  Three dedup streams: the
+    first half of the batches, the second half, then the first half again
+    from the same device buffers; bit-exact vs the oracle each time.
+    drain=False: end_stream with waves in flight (the table reset deferred to
+    the next stream's first wave)."""
     assert torch.cuda.is_available()
     from paper_conf_ipps_rockenbachsgmtd19_b200 import dist as D
     data = U.stream(10 * MiB, seed=71 + depth, dup_frac=0.6)
@@ -127,7 +140,7 @@ def test_native_wave_pipeline_world1(depth, drain):
 
 
 @pytest.mark.parametrize("depth", [2, 4])
-def test_native_wave_pipeline_deferred_resets(depth):
+def test_native_wave_pipeline_deferred_resets(depth, self_path):
     """end_stream twice in a row with waves in flight (an empty dedup stream
     between two), then a stream that repeats the first one's data: every
     deferred reset lands before the right wave, so the repeat is all-new

@@ -141,10 +141,17 @@ def test_mg_all_duplicate_sends_one_record_per_digest():
     assert st["a2a_bytes"] > 0
 
 
-def test_mg_nccl_world1_matches_oracle():
+@pytest.mark.parametrize("nccl_self", [False, True])
+def test_mg_nccl_world1_matches_oracle(nccl_self, monkeypatch):
     """transport = NCCL with one rank (ncclCommInitAll on device 0): the NCCL
-    code path of the engine (counts on their own communicator, grouped
-    send/recv of records and replies) end to end."""
+    code path of the engine end to end.  The rank's own share of the
+    exchange is a device copy; with DEDUP_MG_NCCL_SELF it goes through NCCL
+    send/recv to itself (counts on their own communicator, grouped send/recv
+    of records and replies)."""
+    if nccl_self:
+        monkeypatch.setenv("DEDUP_MG_NCCL_SELF", "1")
+    else:
+        monkeypatch.delenv("DEDUP_MG_NCCL_SELF", raising=False)
     data, off = ragged_stream(6 * MiB, seed=303)
     dev = torch.from_numpy(data).cuda()
     n = len(off) - 1
