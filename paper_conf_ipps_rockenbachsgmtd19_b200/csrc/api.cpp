@@ -191,7 +191,8 @@ dedup_status halloc(dedup_ctx* c, T** p, uint64_t count, unsigned flags = cudaHo
 
 dedup_status ws_alloc(dedup_ctx* c, Workspace& w, uint64_t batch_bytes, uint64_t cap) {
     w.max_tiles = (batch_bytes + kSelTile - 1) / kSelTile + 1;
-    TRY(dalloc(c, &w.bitmap, batch_bytes / 32 + 2));
+    // whole tiles: the scan writes every word of the last (partial) tile
+    TRY(dalloc(c, &w.bitmap, w.max_tiles * kSelTileWords + 2));
     TRY(dalloc(c, &w.agg, w.max_tiles * 32));
     TRY(dalloc(c, &w.gagg, (select_groups(w.max_tiles) + 1) * 32));
     TRY(dalloc(c, &w.gentry, (select_groups(w.max_tiles) + 1) * 2));

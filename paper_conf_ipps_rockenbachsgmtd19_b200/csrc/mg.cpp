@@ -398,7 +398,7 @@ dedup_status slot_alloc(Engine* E, Rank& r, Slot& sl) {
     std::memset(sl.h_item_off, 0, sizeof(uint64_t) * (bi + 1));
     if (E->host_fed) MTRY(dmalloc(E, &sl.d_in, bb + 256));
     sl.max_tiles = (bb + kSelTile - 1) / kSelTile + 1;
-    MTRY(dmalloc(E, &sl.bitmap, bb / 32 + 2));
+    MTRY(dmalloc(E, &sl.bitmap, sl.max_tiles * kSelTileWords + 2));  // whole tiles
     MTRY(dmalloc(E, &sl.agg, sl.max_tiles * 32));
     MTRY(dmalloc(E, &sl.gagg, (select_groups(sl.max_tiles) + 1) * 32));
     MTRY(dmalloc(E, &sl.gentry, (select_groups(sl.max_tiles) + 1) * 2));

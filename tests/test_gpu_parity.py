@@ -232,6 +232,22 @@ def test_batch_size_invariance(cuda, batch_mb, engine):
 
 
 @pytest.mark.parametrize("engine", ENGINES)
+def test_full_batches_not_a_tile_multiple(cuda, engine):
+    """Batches of exactly batch_bytes where batch_bytes is not a multiple of
+    the scan's 8 KiB selection tile: the last, partial tile of every batch is
+    written whole into the candidate bitmap (sized in whole tiles), and the
+    results stay bit-exact (run under compute-sanitizer memcheck by
+    tools/gpu_sanitize.sh)."""
+    bb = 1_000_003
+    data = U.stream(4 * bb, seed=33, dup_frac=0.5)
+    off = np.array([0, bb, 2 * bb, 2 * bb + 5, 3 * bb, 4 * bb], np.uint64)
+    want, _ = U.oracle_results(data, off)
+    with make_ctx(engine, batch_bytes=bb, batch_items=4, slots=2) as d:
+        got = U.run_device(d, torch.from_numpy(data).to(cuda), off, bb, 4)
+    U.assert_same(got, want)
+
+
+@pytest.mark.parametrize("engine", ENGINES)
 def test_tiny_and_empty_items_pipeline(cuda, engine):
     rng = np.random.default_rng(4)
     lens = [0, 5, 0, 5, 31, 32, 33, 0, 64, 1000, 0, 5]
