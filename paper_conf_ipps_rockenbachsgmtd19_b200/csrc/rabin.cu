@@ -62,7 +62,9 @@ namespace {
 // pair, h1 computed off the chain for its test: half the chain latency per
 // byte, 3 LDS and 12.3 instructions per byte instead of 2 and 10.6; bit-exact,
 // 1279, bench 731) -- so the kernel is bound by issue / pipe throughput
-// rather than by the rolling chain's latency.
+// rather than by the rolling chain's latency; 16 KiB selection tiles (512
+// bytes per lane: half the warm-up and per-tile tail per byte; bit-exact)
+// 1415 vs 1480 chunk stage, bench equal (814 vs 816).
 constexpr int kScanGroupsPerCta = 4;  // select groups per scan CTA (launch_chunk_select)
 constexpr int kScanWarps = 16;
 constexpr int kScanThreads = kScanWarps * 32;
