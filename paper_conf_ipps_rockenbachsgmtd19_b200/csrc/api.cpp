@@ -326,26 +326,10 @@ dedup_status build_graph(dedup_ctx* c, int i) {
     std::vector<cudaGraphNode_t> nodes(n_nodes);
     cudaGraphGetNodes(g, nodes.data(), &n_nodes);
     uint32_t kern = 0;
-    // the table chain is serial across batches: its kernels take SMs ahead of
-    // the other in-flight batches' scan / SHA-1 CTAs (DEDUP_TABLE_PRIO=0: off)
-    int prio_lo = 0, prio_hi = 0;
-    cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
-    const char* tp = std::getenv("DEDUP_TABLE_PRIO");
-    const bool table_prio = tp == nullptr || std::atoi(tp) != 0;
     for (auto& nd : nodes) {
         cudaGraphNodeType ty;
         cudaGraphNodeGetType(nd, &ty);
-        if (ty != cudaGraphNodeTypeKernel) continue;
-        ++kern;
-        cudaKernelNodeParams kp{};
-        if (table_prio && cudaGraphKernelNodeGetParams(nd, &kp) == cudaSuccess &&
-            is_table_chain_kernel(kp.func)) {
-            cudaKernelNodeAttrValue v{};
-            v.priority = prio_hi;
-            if (cudaGraphKernelNodeSetAttribute(nd, cudaKernelNodeAttributePriority, &v) !=
-                cudaSuccess)
-                return fail(c, DEDUP_ECUDA, "graph: kernel node priority");
-        }
+        kern += ty == cudaGraphNodeTypeKernel ? 1 : 0;
     }
     c->graph_kernels = kern;
     e = cudaGraphInstantiate(&sl.graph, g, 0);

@@ -136,9 +136,6 @@ void launch_sha1(const BatchDesc* d, uint64_t max_bytes, const uint32_t* cut_pos
 // id) arrays or as packed 32-byte records (rec != nullptr).
 // The table is read from *tv (device memory) at run time.
 void launch_table_prepare(const BatchDesc* d, uint64_t max_slots, int num_sms, cudaStream_t s);
-// True for the kernels of the per-batch table chain (prepare, insert, lookup):
-// their graph nodes run at the highest priority (api.cpp build_graph).
-bool is_table_chain_kernel(const void* fn);
 void launch_table_insert(const TableView* tv, const uint8_t* digest, const uint64_t* id,
                          const void* rec, const uint32_t* d_n, uint64_t n_host, uint64_t cap,
                          uint32_t* slot_idx, int num_sms, cudaStream_t s);

@@ -438,9 +438,4 @@ void launch_pack(const BatchDesc* d, const uint32_t* n_chunks, uint64_t cap, uin
         h, extra);
 }
 
-bool is_table_chain_kernel(const void* fn) {
-    return fn == (const void*)table_prepare_kernel || fn == (const void*)table_insert_kernel ||
-           fn == (const void*)table_lookup_kernel;
-}
-
 }  // namespace dd
