@@ -104,9 +104,10 @@ constexpr int kScanSmem = kAuxInPad ? 65536 + kTabBytes : 2 * 65536 - kStaticMin
 // Group buffers in the scan (double buffering across the group barrier).
 constexpr int kFunBufs = 2;
 
+template <uint32_t kOff = 0>
 __device__ __forceinline__ uint32_t lds(uint32_t addr) {
     uint32_t v;
-    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(addr));
+    asm volatile("ld.shared.u32 %0, [%1+%2];" : "=r"(v) : "r"(addr), "n"(kOff));
     return v;
 }
 
@@ -322,7 +323,7 @@ __device__ __forceinline__ uint32_t walk_any(const SelWarpSmem& sm, uint32_t n_e
 // Two independent rolling chains per lane (ILP 2): the LDS -> LOP3 -> PRMT
 // dependency of one chain overlaps with the other's.
 // Words [W0, W1) of the 32-byte step; bits accumulate into bitsA / bitsB.
-template <bool kZeroValue, int W0 = 0, int W1 = 8>
+template <bool kZeroValue, int W0 = 0, int W1 = 8, uint32_t kOff = 0>
 __device__ __forceinline__ void roll32x2(uint32_t& hA, const uint32_t curA[8],
                                          const uint32_t oldA[8], uint32_t& bitsA, uint32_t& hB,
                                          const uint32_t curB[8], const uint32_t oldB[8],
@@ -339,8 +340,8 @@ __device__ __forceinline__ void roll32x2(uint32_t& hA, const uint32_t curA[8],
             const uint32_t aWB = __byte_perm(oldB[w], laneW, 0x7604 | (k << 4));
             const uint32_t hsA = __byte_perm(curA[w], hA, 0x6540 | k);
             const uint32_t hsB = __byte_perm(curB[w], hB, 0x6540 | k);
-            hA = hsA ^ lds(aRA) ^ lds(aWA);
-            hB = hsB ^ lds(aRB) ^ lds(aWB);
+            hA = hsA ^ lds<kOff>(aRA) ^ lds<kOff>(aWA);
+            hB = hsB ^ lds<kOff>(aRB) ^ lds<kOff>(aWB);
             const uint32_t tA = kZeroValue ? (hA & mask) : ((hA & mask) ^ value);
             const uint32_t tB = kZeroValue ? (hB & mask) : ((hB & mask) ^ value);
             asm("{\n\t.reg .pred p;\n\tsetp.eq.u32 p, %1, 0;\n\t@p or.b32 %0, %0, %2;\n\t}"
@@ -474,7 +475,11 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
             pbA = bitsA;
             pbB = bitsB;
         };
+#ifdef DEDUP_SCAN_U8
+#pragma unroll
+#else
 #pragma unroll 1
+#endif
         for (int j = 0; j < 8; j += 2) {
             step(j, curA, prevA, curB, prevB);      // prev now holds step j+1's bytes
             step(j + 1, prevA, curA, prevB, curB);  // cur now holds step j+2's bytes
@@ -519,6 +524,199 @@ rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __res
             }
             gagg[32 * g + lane] = (Gs << 27) | Gc;
         }
+    }
+}
+
+// ---- decoupled scan: roll kernel (candidate bitmap) + per-tile selection ----
+//
+// rabin_roll_kernel: a warp task is 64 KiB of the batch (two chains of 32
+// lanes x kRollLane bytes: chain B follows chain A); every lane rolls its
+// kRollLane bytes after a 32-byte warm-up and stores one e-space candidate
+// word per 32-byte step.  No item knowledge, no selection, no barrier: the
+// hot loop is the whole kernel.  The 64 KiB table is the only shared memory
+// (the kernel has no static shared memory, so the dynamic window starts on a
+// 64 KiB boundary and the PRMT address trick needs no pad): two CTAs per SM.
+constexpr uint32_t kRollLane = 1024;             // bytes per lane per chain
+constexpr uint32_t kRollChain = 32 * kRollLane;  // 32 KiB
+constexpr uint32_t kRollTask = 2 * kRollChain;   // 64 KiB per warp task
+constexpr int kRollWarps = 16;
+constexpr int kRollThreads = kRollWarps * 32;
+constexpr int kRollSteps = kRollLane / 32;
+constexpr int kRollTasksPerCta = 16;  // one task per warp: a CTA covers 1 MiB
+constexpr uint32_t kRollWin = 1024;   // shared-window offset of the dynamic smem (1 KiB reserved)
+static_assert(kSelTile % kRollLane == 0, "a lane's range lies inside one tile");
+
+template <bool kZeroValue>
+__global__ void __launch_bounds__(kRollThreads, 2)  // <= 64 registers
+rabin_roll_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ gtab,
+                  uint32_t mask, uint32_t value, uint32_t* __restrict__ bitmap) {
+    extern __shared__ __align__(16) uint8_t smem[];
+    // layout assumption: no static shared memory, so the table (the dynamic
+    // window) starts at kRollWin; the LDS immediate adds it to the PRMT-built
+    // offset x * 256 + lane * 4 (+ 128 for W)
+    if ((uint32_t)__cvta_generic_to_shared(smem) != kRollWin) __trap();
+    {
+        uint32_t* t32 = reinterpret_cast<uint32_t*>(smem);
+        for (int idx = threadIdx.x; idx < kTabBytes / 4; idx += blockDim.x)
+            t32[idx] = __ldg(gtab + ((idx >> 5) & 1) * 256 + (idx >> 6));
+    }
+    __syncthreads();
+    const uint8_t* __restrict__ bytes = desc->bytes;
+    const uint32_t nbytes = (uint32_t)desc->nbytes;  // <= 2^30 (check_cfg)
+    if (nbytes == 0) return;
+    const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t cover = ((nbytes + kSelTile - 1) / kSelTile) * kSelTile;  // bitmap e-range
+    const uint32_t n_tasks = (cover + kRollTask - 1) / kRollTask;
+    const uint32_t lim16 = (nbytes + 15) & ~15u;
+    const bool cont = (desc->carry & kCarryCont) != 0;
+    const uint32_t laneR = lane * 4;
+    const uint32_t laneW = laneR + 128;
+    const bool a32 = (reinterpret_cast<uintptr_t>(bytes) & 31) == 0;
+    auto fetch = [&](uint32_t offA, uint32_t offB, bool okA, bool okB, uint32_t (&vA)[8],
+                     uint32_t (&vB)[8]) {
+        if (okA) load32_v8(bytes, offA, lim16, a32, vA);
+        if (okB) load32_v8(bytes, offB, lim16, a32, vB);
+    };
+    for (uint32_t task = blockIdx.x * kRollWarps + wid; task < n_tasks;
+         task += gridDim.x * kRollWarps) {
+        const uint32_t qA = task * kRollTask + lane * kRollLane;
+        const uint32_t qB = qA + kRollChain;
+        const bool actA = qA < cover, actB = qB < cover;
+        uint32_t prevA[8], curA[8], prevB[8], curB[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) prevA[i] = curA[i] = prevB[i] = curB[i] = 0;
+        // the whole task inside the batch and 32-byte aligned loads: no guards
+        const bool full = a32 && (task + 1) * kRollTask <= nbytes;
+        fetch(qA - 32, qB - 32, qA >= 32 && qA < nbytes, qB < nbytes, prevA, prevB);
+        fetch(qA, qB, qA < nbytes, qB < nbytes, curA, curB);
+        const bool contA = cont && qA == 0;  // carry-over: the stream's 32 bytes before
+        if (contA) {
+            const uint32_t* hw32 = reinterpret_cast<const uint32_t*>(desc->carry_in->hist);
+#pragma unroll
+            for (int i = 0; i < 8; ++i) prevA[i] = hw32[i];
+        }
+        uint32_t hA = 0, hB = 0, pbA = 0, pbB = 0;
+        {   // warm-up of both chains: the windows ending at q-1
+            const uint32_t zero[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+            uint32_t bA, bB;
+            roll32x2<kZeroValue, 0, 8, kRollWin>(hA, prevA, zero, bA, hB, prevB, zero, bB, laneR,
+                                                 laneW, mask, value);
+            pbA = (qA >= 32 || contA) ? bA : 0;
+            pbB = bB;  // qB >= 32 always
+            if (qA < 32 && !contA) hA = 0;
+        }
+        // one 32-byte step of both chains (`in` and `old` swap roles every
+        // step, as in the fused scan)
+        auto step = [&](int j, uint32_t (&inA)[8], uint32_t (&oldA)[8], uint32_t (&inB)[8],
+                        uint32_t (&oldB)[8]) {
+            const uint32_t bA0 = qA + 32 * j, bB0 = qB + 32 * j;
+            uint32_t bitsA, bitsB;
+            roll32x2<kZeroValue, 0, 4, kRollWin>(hA, inA, oldA, bitsA, hB, inB, oldB, bitsB, laneR,
+                                                 laneW, mask, value);
+            roll32x2<kZeroValue, 4, 8, kRollWin>(hA, inA, oldA, bitsA, hB, inB, oldB, bitsB, laneR,
+                                                 laneW, mask, value);
+            if (j < kRollSteps - 1) {  // the next step's bytes into the freed `old`
+                if (full) {
+                    ldg_v8(bytes + bA0 + 32, oldA);
+                    ldg_v8(bytes + bB0 + 32, oldB);
+                } else {
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) oldA[i] = oldB[i] = 0;
+                    fetch(bA0 + 32, bB0 + 32, bA0 + 32 < nbytes, bB0 + 32 < nbytes, oldA, oldB);
+                }
+            }
+            uint32_t ewA = __funnelshift_l(pbA, bitsA, 1), ewB = __funnelshift_l(pbB, bitsB, 1);
+            if (!full) {  // the batch's ragged end
+                if (bA0 >= nbytes) ewA = 0;
+                else if (bA0 + 32 > nbytes) ewA &= (1u << (nbytes - bA0)) - 1u;
+                if (bB0 >= nbytes) ewB = 0;
+                else if (bB0 + 32 > nbytes) ewB &= (1u << (nbytes - bB0)) - 1u;
+                if (bA0 + 32 > nbytes) bitsA &= bA0 < nbytes ? (1u << (nbytes - bA0)) - 1u : 0u;
+                if (bB0 + 32 > nbytes) bitsB &= bB0 < nbytes ? (1u << (nbytes - bB0)) - 1u : 0u;
+            }
+            if (full || actA) bitmap[(bA0 >> 5)] = ewA;
+            if (full || actB) bitmap[(bB0 >> 5)] = ewB;
+            pbA = bitsA;
+            pbB = bitsB;
+        };
+#pragma unroll 1
+        for (int j = 0; j < kRollSteps; j += 2) {
+            step(j, curA, prevA, curB, prevB);
+            step(j + 1, prevA, curA, prevB, curB);
+        }
+    }
+}
+
+// Per-tile selection from the candidate bitmap (the fused scan's epilogue):
+// a warp takes a group of 32 tiles; per tile it applies the item rules,
+// stores the tile's event list for the emit kernel and the tile's transfer
+// function, then composes the group's function.  The next tile's candidate
+// words are loaded while the current one is processed.
+constexpr int kSelWarps = 4;
+struct SelCtaSmem {
+    SelWarpSmem w[kSelWarps];
+    uint32_t fun[kSelWarps][kGroup][33];
+};
+
+__global__ void __launch_bounds__(kSelWarps * 32)
+select_tiles_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ bitmap,
+                    uint32_t* __restrict__ agg, uint32_t* __restrict__ gagg,
+                    uint32_t* __restrict__ evbuf) {
+    extern __shared__ __align__(16) uint8_t smraw[];
+    SelCtaSmem& cs = *reinterpret_cast<SelCtaSmem*>(smraw);
+    const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    SelWarpSmem& sm = cs.w[wid];
+    const uint64_t nbytes = desc->nbytes;
+    const uint32_t n_tiles = (uint32_t)((nbytes + kSelTile - 1) / kSelTile);
+    const uint32_t n_groups = (n_tiles + kGroup - 1) / kGroup;
+    const uint64_t* items = desc->item_off;
+    const uint32_t n_items = desc->n_items;
+    const uint32_t first_rule = (desc->carry & kCarryCont) ? 1u : 0u;
+    for (uint32_t g = blockIdx.x * kSelWarps + wid; g < n_groups; g += gridDim.x * kSelWarps) {
+        const uint32_t t0 = g * kGroup;
+        uint4 na = make_uint4(0, 0, 0, 0), nb = na;
+        if (t0 < n_tiles) {
+            const uint4* src = reinterpret_cast<const uint4*>(bitmap + (size_t)t0 * kSelTileWords);
+            na = src[2 * lane];
+            nb = src[2 * lane + 1];
+        }
+        for (int j = 0; j < kGroup; ++j) {
+            const uint32_t t = t0 + j;
+            uint32_t f = (uint32_t)lane << 27;
+            if (t < n_tiles) {
+                uint4* dst = reinterpret_cast<uint4*>(sm.cand);
+                dst[2 * lane] = na;
+                dst[2 * lane + 1] = nb;
+                if (t + 1 < n_tiles && j + 1 < kGroup) {  // prefetch the next tile's words
+                    const uint4* src =
+                        reinterpret_cast<const uint4*>(bitmap + (size_t)(t + 1) * kSelTileWords);
+                    na = src[2 * lane];
+                    nb = src[2 * lane + 1];
+                }
+                __syncwarp();
+                const uint32_t n_ev = apply_items(sm, (uint64_t)t * kSelTile, nbytes, items,
+                                                  n_items, lane, first_rule);
+                store_events(sm, n_ev, evbuf + (size_t)t * kEvWords, lane);
+                uint32_t ex;
+                const uint32_t cnt = walk_any(sm, n_ev, lane, ex, nullptr, 0, 0, 0);
+                f = (ex << 27) | cnt;
+                agg[32 * t + lane] = f;
+                __syncwarp();
+            }
+            cs.fun[wid][j][lane] = f;
+        }
+        __syncwarp();
+        uint32_t Gs = lane, Gc = 0;
+#pragma unroll 8
+        for (int j = 0; j < kGroup; ++j) {
+            const uint32_t a = cs.fun[wid][j][lane];
+            const uint32_t ns = __shfl_sync(kFull, a >> 27, Gs);
+            const uint32_t nc = Gc + __shfl_sync(kFull, a & kM27, Gs);
+            Gs = ns;
+            Gc = nc;
+        }
+        gagg[32 * g + lane] = (Gs << 27) | Gc;
+        __syncwarp();
     }
 }
 
@@ -744,6 +942,10 @@ void chunk_set_attrs() {
         cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
     cudaFuncSetAttribute(select_emit_ev_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)sizeof(EmitEvSmem));
+    for (const void* f : {(const void*)rabin_roll_kernel<true>, (const void*)rabin_roll_kernel<false>})
+        cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kTabBytes);
+    cudaFuncSetAttribute(select_tiles_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)sizeof(SelCtaSmem));
     done_mask |= bit;
 }
 }  // namespace
@@ -753,6 +955,10 @@ const char* chunk_unlaunchable() {
     for (const void* f : {(const void*)rabin_scan_agg2_kernel<true>,
                           (const void*)rabin_scan_agg2_kernel<false>})
         if (!fits(f, kScanThreads, kScanSmem)) return "rabin_scan_agg2_kernel";
+    for (const void* f : {(const void*)rabin_roll_kernel<true>, (const void*)rabin_roll_kernel<false>})
+        if (!fits(f, kRollThreads, kTabBytes)) return "rabin_roll_kernel";
+    if (!fits((const void*)select_tiles_kernel, kSelWarps * 32, sizeof(SelCtaSmem)))
+        return "select_tiles_kernel";
     if (!fits((const void*)select_scan_kernel, 1024, 0)) return "select_scan_kernel";
     if (!fits((const void*)select_emit_ev_kernel, kEmitEvWarps * 32, sizeof(EmitEvSmem)))
         return "select_emit_ev_kernel";
@@ -774,11 +980,27 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
     // share the SMs better with the other in-flight batches' SHA-1 CTAs.
     // Measured (bench, C2, 64 MiB batches = 256 groups, SHA lane 32 KiB,
     // 40 slots): 1 group per CTA 632, 2 640, 4 709-716, 8 702, 16 700 GB/s.
+#ifdef DEDUP_SCAN_FUSED
     uint64_t gneed = (groups + kHalves - 1) / kHalves;
     gneed = (gneed + kScanGroupsPerCta - 1) / kScanGroupsPerCta;
     const unsigned grid = (unsigned)(gneed < (uint64_t)num_sms ? (gneed ? gneed : 1) : num_sms);
     auto k = value == 0 ? rabin_scan_agg2_kernel<true> : rabin_scan_agg2_kernel<false>;
     k<<<grid, kScanThreads, kScanSmem, s>>>(d, d_tab, mask, value, bitmap, agg, gagg, evbuf);
+#else
+    {
+        const uint64_t tasks = (max_tiles * kSelTile + kRollTask - 1) / kRollTask;
+        uint64_t grid = (tasks + kRollTasksPerCta - 1) / kRollTasksPerCta;
+        if (grid > (uint64_t)num_sms * 2) grid = (uint64_t)num_sms * 2;
+        if (grid < 1) grid = 1;
+        auto k = value == 0 ? rabin_roll_kernel<true> : rabin_roll_kernel<false>;
+        k<<<(unsigned)grid, kRollThreads, kTabBytes, s>>>(d, d_tab, mask, value, bitmap);
+        uint64_t sb = (groups + kSelWarps - 1) / kSelWarps;
+        if (sb > (uint64_t)num_sms * 8) sb = (uint64_t)num_sms * 8;
+        if (sb < 1) sb = 1;
+        select_tiles_kernel<<<(unsigned)sb, kSelWarps * 32, sizeof(SelCtaSmem), s>>>(
+            d, bitmap, agg, gagg, evbuf);
+    }
+#endif
     if (after_scan) cudaEventRecordWithFlags(after_scan, s, cudaEventRecordExternal);
     // NEXT-2 max_chunk: the state machine's cuts go to a scratch list first
     uint32_t* final_cut = cut_pos;

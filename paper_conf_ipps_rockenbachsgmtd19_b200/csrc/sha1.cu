@@ -319,6 +319,9 @@ sha1_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ cut
         if (nbulk > 0) load_raw<false>(bytes, p, lim16, raw);
         else load_raw<true>(bytes, p, lim16, raw);
         uint32_t M[16];
+#ifdef DEDUP_SHA_U2
+#pragma unroll 2
+#endif
         for (uint32_t i = 0; i < nbulk; ++i) {
             realign(raw, o, M);
             p += 64;

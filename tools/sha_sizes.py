@@ -17,7 +17,9 @@ reps = int(os.environ.get("REPS", "5"))
 nb = mb * MiB
 data = synthgen.make_stream(nb, seed=3, dup_frac=0.5)
 dev = torch.from_numpy(data).cuda()
-d = Dedup(0, batch_bytes=nb, batch_items=mb + 1, slots=1, table_capacity=1 << 16, host_fed=False)
+lane = int(os.environ.get("LANE", "0"))  # SHA-1 bytes per lane (grid size); 0 = default
+d = Dedup(0, batch_bytes=nb, batch_items=mb + 1, slots=1, table_capacity=1 << 16, host_fed=False,
+          sha_lane_bytes=lane)
 cap = nb // 32 + mb + 2
 for case in cases:
     cut = torch.zeros(cap, dtype=torch.int32, device="cuda")
@@ -51,5 +53,5 @@ for case in cases:
     k = int(n.item())
     cp = cut[:k].cpu().numpy().astype(np.int64)
     lens = np.diff(np.append(cp, nb))
-    print(f"{case}: {mb} MiB, {k} chunks (max {lens.max()} B): sha1 {ms * 1e3:.1f} us -> "
+    print(f"{case} lane={lane}: {mb} MiB, {k} chunks (max {lens.max()} B): sha1 {ms * 1e3:.1f} us -> "
           f"{nb / ms / 1e6:.1f} GB/s", flush=True)
