@@ -3,29 +3,36 @@
 // fragmentation of fixed batches, "saved all the indexes where the algorithm
 // would fragment the data"), P:199 / Fig. 2 (startPos).
 //
-// The paper ran this on the CPU; here it is three sm_100a kernels:
+// The paper ran this on the CPU; here it is four sm_100a kernels:
 //
-//  rabin_scan_agg2_kernel  persistent, one CTA of 16 warps per SM.  A CTA
-//      takes groups of 32 tiles of 8 KiB; warp w rolls tiles w and w + 16 of
-//      the group together (two independent chains per lane, ILP 2); each lane
-//      rolls the 32-byte window hash over its 256 bytes (after a 32-byte
-//      warm-up) with the post-shift recurrence
+//  rabin_roll_kernel      persistent, two CTAs of 16 warps per SM.  A warp
+//      task is 64 lanes-worth of contiguous ranges (two independent chains
+//      per lane, ILP 2); each lane rolls the 32-byte window hash over its
+//      range (after a 32-byte warm-up) with the post-shift recurrence
 //          h' = ((h << 8) | in) ^ R[h >> 24] ^ W256[out]
-//      and records one candidate bit per byte.  R and W256 are replicated per
-//      lane in shared memory ([x][lane] layout: bank = lane, conflict-free);
-//      the table sits on a 64 KiB boundary of the shared window so that one
-//      PRMT builds the whole LDS address.  Greedy cut selection is then a
-//      32-state machine (with min chunk = window = 32 the only state crossing
-//      a position is "positions still blocked", 0..31): the warp simulates all
-//      32 entry states over its tile (lane s = state s) and stores the tile's
-//      transfer function and its sorted event list (candidates + forced
-//      cuts); the CTA composes each group's 32 functions (warp shuffles).
+//      and stores one candidate bit per byte (e-space bitmap words).  R and
+//      W256 are replicated per lane in shared memory ([x][lane] layout: bank
+//      = lane, conflict-free); one PRMT builds the LDS offset, the LDS
+//      immediate adds the table base.
+//  select_tiles_kernel    greedy cut selection is a 32-state machine (with
+//      min chunk = window = 32 the only state crossing a position is
+//      "positions still blocked", 0..31): per 8 KiB tile a warp applies the
+//      item rules, simulates all 32 entry states (lane s = state s) and
+//      stores the tile's transfer function and sorted event list (candidates
+//      + forced cuts); it composes each group of 32 tiles (warp shuffles).
 //  select_scan_kernel     one CTA composes the group functions in order (a
 //      prefix over an associative operator) -> entry state and cut offset of
 //      every group, and the batch's chunk count.
 //  select_emit_ev_kernel  one warp per group derives its tiles' entry states;
 //      lane j walks tile j's stored event list from its real entry state,
 //      writing the cut positions (the paper's startPos).
+// Measured (round 2, C3 bench at 300 steps): the roll and the selection were
+// one kernel (selection as the scan CTA's per-group epilogue, 128 KiB of
+// shared memory per CTA with the table on a 64 KiB boundary) -- 813 GB/s;
+// split, the roll kernel is the hot loop alone -- 872 GB/s.  Measured and not
+// kept: L1 / L2 prefetch of the step after next (838 / 841), the two chains
+// rolled one after the other so that each chain's load flies during the
+// other's half step (854).
 // Item starts are forced cuts and reset the state; a candidate is valid only
 // if its 32-byte window lies inside one item.
 #include <cuda_runtime.h>
@@ -39,45 +46,12 @@ namespace dd {
 
 namespace {
 
-// Scan CTA: 16 warps (64 registers each).  A select group is 32 tiles rolled
-// by 16 warps (2 tiles per warp, ILP 2).  Measured (round 1): a 32-warp CTA
-// running two groups at once scans faster alone (736 MiB chunk stage 1647 vs
-// 1527 GB/s) but takes a whole SM, and the pipelined bench is faster with 16
-// warps (590 vs 576 GB/s): other batches' SHA-1 / table / emit CTAs share the
-// SM.  Measured (round 2, C3, 672 MiB chunk stage): 4 chains per lane (8
-// warps per group, two groups per CTA) 1220 GB/s at 128 registers and 1171
-// at 96; the anchor test as IMAD + predicated add (FMA pipe) 1341; this
-// kernel 1480 -- neither kept.  Measured and not kept (round 2, C3 bench at
-// 300 steps, interleaved reps; this kernel 806-818 GB/s, chunk stage
-// 1486-1504): a 32-warp CTA, two groups (chunk stage 1077, bench 565); the
-// next step's bytes as two 16-byte loads issued half a step earlier (each
-// lane-strided 16-byte load fetches its whole sector: 1179, bench 698); L2 or
-// L1 prefetch of the next step's sector (1339, bench 757); L2 prefetch of the
-// next group's first bytes (1468, bench 801); the next group's warm-up bytes
-// loaded into registers before this group's tail (1479, bench 806); the
-// warm-up without the (zero) W lookups (1472, bench 810); the candidate bit
-// insert as a predicated IMAD on the FMA pipe (1461, bench 797); two
-// positions per dependent step (h2 = (h << 16 | a << 8 | b) ^ RA[h3] ^ R[h2]
-// ^ W8[oa] ^ W[ob] with RA = x t^40, W8 = o t^264 in a second 64 KiB table
-// pair, h1 computed off the chain for its test: half the chain latency per
-// byte, 3 LDS and 12.3 instructions per byte instead of 2 and 10.6; bit-exact,
-// 1279, bench 731) -- so the kernel is bound by issue / pipe throughput
-// rather than by the rolling chain's latency; 16 KiB selection tiles (512
-// bytes per lane: half the warm-up and per-tile tail per byte; bit-exact)
-// 1415 vs 1480 chunk stage, bench equal (814 vs 816).
-constexpr int kScanGroupsPerCta = 4;  // select groups per scan CTA (launch_chunk_select)
-constexpr int kScanWarps = 16;
-constexpr int kScanThreads = kScanWarps * 32;
-constexpr int kGroupWarps = 16;                    // warps per select group
-constexpr int kHalves = kScanWarps / kGroupWarps;  // groups in flight per CTA
-static_assert(kHalves == 1, "one group per scan CTA");
 constexpr int kTabBytes = 256 * 256;  // [x][R|W][lane] u32 = 64 KiB
-constexpr uint32_t kLaneBytes = kSelTile / 32;  // 256 bytes per lane per tile
+constexpr uint32_t kLaneBytes = kSelTile / 32;  // 256 bytes of a tile per lane (selection)
 constexpr uint32_t kFull = 0xFFFFFFFFu;
 constexpr uint32_t kInf = 0xFFFFFFFFu;
 constexpr uint32_t kM27 = (1u << 27) - 1;
-constexpr int kGroup = kGroupWarps * 2;  // tiles per select group (2 per warp)
-constexpr int kItemCache = 1024;  // item offsets cached in shared memory
+constexpr int kGroup = 32;  // tiles per select group
 
 constexpr uint32_t kListCap = 128;  // events per tile kept as a sorted list
 
@@ -88,21 +62,6 @@ struct SelWarpSmem {
     uint32_t fsum[8];
     uint32_t list[kListCap];
 };
-
-// scan: [pad to a 64 KiB shared-window boundary][table][aux?]; the per-warp
-// walk buffers and the item cache (aux) live in the pad when it is large
-// enough (16-warp CTA: the CTA then needs only 128 KiB of dynamic shared
-// memory and other batches' kernels can share the SM), else after the table
-// (32-warp CTA).  The pad is 64 KiB minus the static smem, so the request
-// assumes at least kStaticMin bytes of static smem; the kernel traps if the
-// runtime layout disagrees.
-constexpr int kScanAux = kScanWarps * (int)sizeof(SelWarpSmem) + kItemCache * 8;
-constexpr int kStaticMin = kHalves == 1 ? 8192 : 16384;
-constexpr bool kAuxInPad = kScanAux <= 65536 - 1024 - 10752;
-constexpr int kScanSmem = kAuxInPad ? 65536 + kTabBytes : 2 * 65536 - kStaticMin + kScanAux;
-
-// Group buffers in the scan (double buffering across the group barrier).
-constexpr int kFunBufs = 2;
 
 template <uint32_t kOff = 0>
 __device__ __forceinline__ uint32_t lds(uint32_t addr) {
@@ -175,14 +134,6 @@ __device__ __forceinline__ uint32_t walk_tile(const SelWarpSmem& sm, uint32_t s,
     }
     exit_state = E > kSelTile ? E - kSelTile : 0;
     return cnt;
-}
-
-// Item offsets: cached in shared memory when they fit.
-__device__ __forceinline__ const uint64_t* cache_items(uint64_t* cache, const BatchDesc* desc) {
-    const uint32_t n = desc->n_items + 1;
-    if (n > kItemCache) return desc->item_off;
-    for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) cache[i] = desc->item_off[i];
-    return cache;
 }
 
 // Events of a tile as a sorted compact list (bit 31 = forced cut), when there
@@ -354,202 +305,25 @@ __device__ __forceinline__ void roll32x2(uint32_t& hA, const uint32_t curA[8],
     }
 }
 
-// ILP-2 scan: a CTA of kScanWarps warps takes groups of 2 x kScanWarps tiles;
-// warp w rolls tiles w and w + kScanWarps of the group together.
-template <bool kZeroValue>
-__global__ void __launch_bounds__(kScanThreads, 1024 / kScanThreads)  // <= 64 registers
-rabin_scan_agg2_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ gtab,
-                       uint32_t mask, uint32_t value, uint32_t* __restrict__ bitmap,
-                       uint32_t* __restrict__ agg, uint32_t* __restrict__ gagg,
-                       uint32_t* __restrict__ evbuf) {
-    extern __shared__ __align__(16) uint8_t smem[];
-    __shared__ uint32_t src[512];
-    __shared__ uint32_t fun[kFunBufs][kHalves][kGroup][32];
-    const uint8_t* __restrict__ bytes = desc->bytes;
-    const uint32_t nbytes = (uint32_t)desc->nbytes;  // <= 2^30 (check_cfg)
-    const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int half = wid / kGroupWarps, hw = wid % kGroupWarps;  // group slot, warp in group
-    const uint32_t win = (uint32_t)__cvta_generic_to_shared(smem);
-    const uint32_t pad = (0x10000u - (win & 0xFFFFu)) & 0xFFFFu;
-    const uint32_t base = win + pad;
-    // layout assumptions (see kScanSmem)
-    if (kAuxInPad ? pad < (uint32_t)kScanAux
-                  : base + kTabBytes + kScanAux > win + (uint32_t)kScanSmem)
-        __trap();
-    SelWarpSmem* wsm = reinterpret_cast<SelWarpSmem*>(kAuxInPad ? smem : smem + pad + kTabBytes);
-    uint64_t* icache = reinterpret_cast<uint64_t*>(wsm + kScanWarps);
-    SelWarpSmem& sm = wsm[wid];
-    const uint32_t n_tiles = (nbytes + kSelTile - 1) / kSelTile;
-    const uint32_t n_groups = (n_tiles + kGroup - 1) / kGroup;
-    const uint32_t lim16 = (nbytes + 15) & ~15u;
-    // CTA b, half h takes groups b * kHalves + h + k * gridDim.x * kHalves
-    const uint32_t g0 = blockIdx.x * kHalves + half, gstride = gridDim.x * kHalves;
-    if (threadIdx.x < 512) src[threadIdx.x] = gtab[threadIdx.x];
-    const uint64_t* items = cache_items(icache, desc);
-    const uint32_t n_items = desc->n_items;
-    const bool cont = (desc->carry & kCarryCont) != 0;
-    __syncthreads();
-    {
-        uint32_t* t32 = reinterpret_cast<uint32_t*>(smem + pad);
-        for (int idx = threadIdx.x; idx < kTabBytes / 4; idx += blockDim.x)
-            t32[idx] = src[((idx >> 5) & 1) * 256 + (idx >> 6)];
-    }
-    __syncthreads();
-    if (nbytes == 0) return;
-    const uint32_t laneR = base | (lane * 4);
-    const uint32_t laneW = laneR + 128;
-    const bool a32 = (reinterpret_cast<uintptr_t>(bytes) & 31) == 0;
-    // The bytes at offA / offB for the two chains (zero past the batch end).
-    auto fetch = [&](uint32_t offA, uint32_t offB, bool okA, bool okB, uint32_t (&vA)[8],
-                     uint32_t (&vB)[8]) {
-        if (okA) load32_v8(bytes, offA, lim16, a32, vA);
-        if (okB) load32_v8(bytes, offB, lim16, a32, vB);
-    };
-    int par = 0;
-    for (uint32_t g = g0; g < n_groups; g += gstride, par ^= 1) {
-        const uint32_t tA = g * kGroup + hw, tB = tA + kGroupWarps;
-        const uint32_t qA = tA * kSelTile + lane * kLaneBytes;
-        const uint32_t qB = tB * kSelTile + lane * kLaneBytes;
-        uint32_t prevA[8], curA[8], prevB[8], curB[8];
-#pragma unroll
-        for (int i = 0; i < 8; ++i) prevA[i] = curA[i] = prevB[i] = curB[i] = 0;
-        // both tiles inside the batch and 32-byte aligned loads: no guards
-        const bool full = a32 && (tB + 1) * kSelTile <= nbytes;
-        fetch(qA - 32, qB - 32, qA >= 32 && qA < nbytes, qB >= 32 && qB < nbytes, prevA, prevB);
-        fetch(qA, qB, qA < nbytes, qB < nbytes, curA, curB);
-        // carry-over continuation: the stream's 32 bytes before this piece
-        const bool contA = cont && qA == 0;
-        if (contA) {
-            const uint32_t* hw32 = reinterpret_cast<const uint32_t*>(desc->carry_in->hist);
-#pragma unroll
-            for (int i = 0; i < 8; ++i) prevA[i] = hw32[i];
-        }
-        uint32_t hA = 0, hB = 0, pbA = 0, pbB = 0;
-        {   // warm-up of both chains: the windows ending at q-1
-            const uint32_t zero[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-            uint32_t bA, bB;
-            roll32x2<kZeroValue>(hA, prevA, zero, bA, hB, prevB, zero, bB, laneR, laneW, mask,
-                                 value);
-            pbA = (qA >= 32 || contA) ? bA : 0;
-            pbB = qB >= 32 ? bB : 0;
-            if (qA < 32 && !contA) hA = 0;
-            if (qB < 32) hB = 0;
-        }
-        // One 32-byte step of both chains: roll `in` against `old`, then the
-        // bits in e-space.  Once `old` has been rolled out, its registers
-        // receive the NEXT step's bytes, so `in` and `old`
-        // swap roles every step (the loop body holds two steps) and no extra
-        // registers are needed.
-        auto step = [&](int j, uint32_t (&inA)[8], uint32_t (&oldA)[8], uint32_t (&inB)[8],
-                        uint32_t (&oldB)[8]) {
-            const uint32_t bA0 = qA + 32 * j, bB0 = qB + 32 * j;
-            uint32_t bitsA, bitsB;
-            roll32x2<kZeroValue, 0, 4>(hA, inA, oldA, bitsA, hB, inB, oldB, bitsB, laneR, laneW,
-                                       mask, value);
-            roll32x2<kZeroValue, 4, 8>(hA, inA, oldA, bitsA, hB, inB, oldB, bitsB, laneR, laneW,
-                                       mask, value);
-            if (j < 7) {  // the next step's bytes into the registers `old` just freed
-                if (full) {
-                    ldg_v8(bytes + bA0 + 32, oldA);
-                    ldg_v8(bytes + bB0 + 32, oldB);
-                } else {
-#pragma unroll
-                    for (int i = 0; i < 8; ++i) oldA[i] = oldB[i] = 0;
-                    fetch(bA0 + 32, bB0 + 32, bA0 + 32 < nbytes, bB0 + 32 < nbytes, oldA, oldB);
-                }
-            }
-            uint32_t ewA = __funnelshift_l(pbA, bitsA, 1), ewB = __funnelshift_l(pbB, bitsB, 1);
-            if (!full) {  // the batch's ragged end
-                if (bA0 >= nbytes) ewA = 0;
-                else if (bA0 + 32 > nbytes) ewA &= (1u << (uint32_t)(nbytes - bA0)) - 1u;
-                if (bB0 >= nbytes) ewB = 0;
-                else if (bB0 + 32 > nbytes) ewB &= (1u << (uint32_t)(nbytes - bB0)) - 1u;
-                if (bA0 + 32 > nbytes)
-                    bitsA &= bA0 < nbytes ? (1u << (uint32_t)(nbytes - bA0)) - 1u : 0u;
-                if (bB0 + 32 > nbytes)
-                    bitsB &= bB0 < nbytes ? (1u << (uint32_t)(nbytes - bB0)) - 1u : 0u;
-            }
-            sm.cand[lane * 8 + j] = ewA;
-            if (full || tA < n_tiles) bitmap[tA * kSelTileWords + lane * 8 + j] = ewA;
-            if (full || tB < n_tiles) bitmap[tB * kSelTileWords + lane * 8 + j] = ewB;
-            pbA = bitsA;
-            pbB = bitsB;
-        };
-#ifdef DEDUP_SCAN_U8
-#pragma unroll
-#else
-#pragma unroll 1
-#endif
-        for (int j = 0; j < 8; j += 2) {
-            step(j, curA, prevA, curB, prevB);      // prev now holds step j+1's bytes
-            step(j + 1, prevA, curA, prevB, curB);  // cur now holds step j+2's bytes
-        }
-        // transfer functions of tile A (candidate words already in smem), then B
-        uint32_t fA = (uint32_t)lane << 27, fB = fA;
-        if (tA < n_tiles) {
-            const uint32_t n_ev =
-                apply_items(sm, tA * kSelTile, nbytes, items, n_items, lane, cont ? 1u : 0u);
-            store_events(sm, n_ev, evbuf + (size_t)tA * kEvWords, lane);
-            uint32_t ex;
-            const uint32_t cnt = walk_any(sm, n_ev, lane, ex, nullptr, 0, 0, 0);
-            fA = (ex << 27) | cnt;
-            agg[32 * tA + lane] = fA;
-        }
-        __syncwarp();
-        if (tB < n_tiles) {
-#pragma unroll
-            for (int k = 0; k < 8; ++k)
-                sm.cand[lane * 8 + k] = bitmap[tB * kSelTileWords + lane * 8 + k];
-            const uint32_t n_ev =
-                apply_items(sm, tB * kSelTile, nbytes, items, n_items, lane, cont ? 1u : 0u);
-            store_events(sm, n_ev, evbuf + (size_t)tB * kEvWords, lane);
-            uint32_t ex;
-            const uint32_t cnt = walk_any(sm, n_ev, lane, ex, nullptr, 0, 0, 0);
-            fB = (ex << 27) | cnt;
-            agg[32 * tB + lane] = fB;
-        }
-        fun[par][half][hw][lane] = fA;
-        fun[par][half][hw + kGroupWarps][lane] = fB;
-        if (kHalves == 1) __syncthreads();
-        else asm volatile("bar.sync %0, %1;" ::"r"(1 + half), "r"(kGroupWarps * 32) : "memory");
-        if (hw == 0) {
-            uint32_t Gs = lane, Gc = 0;
-#pragma unroll
-            for (int j = 0; j < kGroup; ++j) {
-                const uint32_t a = fun[par][half][j][lane];
-                const uint32_t ns = __shfl_sync(kFull, a >> 27, Gs);
-                const uint32_t nc = Gc + __shfl_sync(kFull, a & kM27, Gs);
-                Gs = ns;
-                Gc = nc;
-            }
-            gagg[32 * g + lane] = (Gs << 27) | Gc;
-        }
-    }
-}
-
 // ---- decoupled scan: roll kernel (candidate bitmap) + per-tile selection ----
 //
-// rabin_roll_kernel: a warp task is 64 KiB of the batch (two chains of 32
-// lanes x kRollLane bytes: chain B follows chain A); every lane rolls its
-// kRollLane bytes after a 32-byte warm-up and stores one e-space candidate
-// word per 32-byte step.  No item knowledge, no selection, no barrier: the
-// hot loop is the whole kernel.  The 64 KiB table is the only shared memory
-// (the kernel has no static shared memory, so the dynamic window starts on a
-// 64 KiB boundary and the PRMT address trick needs no pad): two CTAs per SM.
-constexpr uint32_t kRollLane = 1024;             // bytes per lane per chain
-constexpr uint32_t kRollChain = 32 * kRollLane;  // 32 KiB
-constexpr uint32_t kRollTask = 2 * kRollChain;   // 64 KiB per warp task
+// rabin_roll_kernel: a warp task is 64 x lane_bytes of the batch (two chains
+// of 32 lanes x lane_bytes: chain B follows chain A); every lane rolls its
+// lane_bytes after a 32-byte warm-up and stores one e-space candidate word
+// per 32-byte step.  lane_bytes (a power of two, 256 .. kSelTile) is chosen
+// per launch (launch_chunk_select).  No item knowledge, no selection, no
+// barrier: the hot loop is the whole kernel.  The 64 KiB table is the only
+// shared memory (no static shared memory: the dynamic window starts right
+// after the 1 KiB the driver reserves), so two CTAs fit per SM.
 constexpr int kRollWarps = 16;
 constexpr int kRollThreads = kRollWarps * 32;
-constexpr int kRollSteps = kRollLane / 32;
-constexpr int kRollTasksPerCta = 16;  // one task per warp: a CTA covers 1 MiB
-constexpr uint32_t kRollWin = 1024;   // shared-window offset of the dynamic smem (1 KiB reserved)
-static_assert(kSelTile % kRollLane == 0, "a lane's range lies inside one tile");
+constexpr uint32_t kRollWin = 1024;  // shared-window offset of the dynamic smem (1 KiB reserved)
 
 template <bool kZeroValue>
 __global__ void __launch_bounds__(kRollThreads, 2)  // <= 64 registers
 rabin_roll_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ gtab,
-                  uint32_t mask, uint32_t value, uint32_t* __restrict__ bitmap) {
+                  uint32_t mask, uint32_t value, uint32_t* __restrict__ bitmap,
+                  uint32_t lane_bytes) {
     extern __shared__ __align__(16) uint8_t smem[];
     // layout assumption: no static shared memory, so the table (the dynamic
     // window) starts at kRollWin; the LDS immediate adds it to the PRMT-built
@@ -566,7 +340,9 @@ rabin_roll_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict
     if (nbytes == 0) return;
     const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t cover = ((nbytes + kSelTile - 1) / kSelTile) * kSelTile;  // bitmap e-range
-    const uint32_t n_tasks = (cover + kRollTask - 1) / kRollTask;
+    const uint32_t chain_bytes = 32 * lane_bytes, task_bytes = 2 * chain_bytes;
+    const int steps = (int)(lane_bytes >> 5);
+    const uint32_t n_tasks = (cover + task_bytes - 1) / task_bytes;
     const uint32_t lim16 = (nbytes + 15) & ~15u;
     const bool cont = (desc->carry & kCarryCont) != 0;
     const uint32_t laneR = lane * 4;
@@ -579,14 +355,14 @@ rabin_roll_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict
     };
     for (uint32_t task = blockIdx.x * kRollWarps + wid; task < n_tasks;
          task += gridDim.x * kRollWarps) {
-        const uint32_t qA = task * kRollTask + lane * kRollLane;
-        const uint32_t qB = qA + kRollChain;
+        const uint32_t qA = task * task_bytes + lane * lane_bytes;
+        const uint32_t qB = qA + chain_bytes;
         const bool actA = qA < cover, actB = qB < cover;
         uint32_t prevA[8], curA[8], prevB[8], curB[8];
 #pragma unroll
         for (int i = 0; i < 8; ++i) prevA[i] = curA[i] = prevB[i] = curB[i] = 0;
         // the whole task inside the batch and 32-byte aligned loads: no guards
-        const bool full = a32 && (task + 1) * kRollTask <= nbytes;
+        const bool full = a32 && (task + 1) * task_bytes <= nbytes;
         fetch(qA - 32, qB - 32, qA >= 32 && qA < nbytes, qB < nbytes, prevA, prevB);
         fetch(qA, qB, qA < nbytes, qB < nbytes, curA, curB);
         const bool contA = cont && qA == 0;  // carry-over: the stream's 32 bytes before
@@ -615,7 +391,7 @@ rabin_roll_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict
                                                  laneW, mask, value);
             roll32x2<kZeroValue, 4, 8, kRollWin>(hA, inA, oldA, bitsA, hB, inB, oldB, bitsB, laneR,
                                                  laneW, mask, value);
-            if (j < kRollSteps - 1) {  // the next step's bytes into the freed `old`
+            if (j < steps - 1) {  // the next step's bytes into the freed `old`
                 if (full) {
                     ldg_v8(bytes + bA0 + 32, oldA);
                     ldg_v8(bytes + bB0 + 32, oldB);
@@ -640,7 +416,7 @@ rabin_roll_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict
             pbB = bitsB;
         };
 #pragma unroll 1
-        for (int j = 0; j < kRollSteps; j += 2) {
+        for (int j = 0; j < steps; j += 2) {
             step(j, curA, prevA, curB, prevB);
             step(j + 1, prevA, curA, prevB, curB);
         }
@@ -937,9 +713,6 @@ void chunk_set_attrs() {
     const uint64_t bit = 1ull << (dev & 63);
     std::lock_guard<std::mutex> lock(mu);
     if (done_mask & bit) return;
-    for (const void* f : {(const void*)rabin_scan_agg2_kernel<true>,
-                          (const void*)rabin_scan_agg2_kernel<false>})
-        cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, kScanSmem);
     cudaFuncSetAttribute(select_emit_ev_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)sizeof(EmitEvSmem));
     for (const void* f : {(const void*)rabin_roll_kernel<true>, (const void*)rabin_roll_kernel<false>})
@@ -952,9 +725,6 @@ void chunk_set_attrs() {
 
 const char* chunk_unlaunchable() {
     chunk_set_attrs();
-    for (const void* f : {(const void*)rabin_scan_agg2_kernel<true>,
-                          (const void*)rabin_scan_agg2_kernel<false>})
-        if (!fits(f, kScanThreads, kScanSmem)) return "rabin_scan_agg2_kernel";
     for (const void* f : {(const void*)rabin_roll_kernel<true>, (const void*)rabin_roll_kernel<false>})
         if (!fits(f, kRollThreads, kTabBytes)) return "rabin_roll_kernel";
     if (!fits((const void*)select_tiles_kernel, kSelWarps * 32, sizeof(SelCtaSmem)))
@@ -975,32 +745,28 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
                          cudaEvent_t before_select) {
     chunk_set_attrs();
     const uint64_t groups = select_groups(max_tiles);
-    // A persistent scan CTA takes several groups: fewer, longer-lived CTAs
-    // per batch (a CTA holds 128 KiB of shared memory and 32K registers)
-    // share the SMs better with the other in-flight batches' SHA-1 CTAs.
-    // Measured (bench, C2, 64 MiB batches = 256 groups, SHA lane 32 KiB,
-    // 40 slots): 1 group per CTA 632, 2 640, 4 709-716, 8 702, 16 700 GB/s.
-#ifdef DEDUP_SCAN_FUSED
-    uint64_t gneed = (groups + kHalves - 1) / kHalves;
-    gneed = (gneed + kScanGroupsPerCta - 1) / kScanGroupsPerCta;
-    const unsigned grid = (unsigned)(gneed < (uint64_t)num_sms ? (gneed ? gneed : 1) : num_sms);
-    auto k = value == 0 ? rabin_scan_agg2_kernel<true> : rabin_scan_agg2_kernel<false>;
-    k<<<grid, kScanThreads, kScanSmem, s>>>(d, d_tab, mask, value, bitmap, agg, gagg, evbuf);
-#else
     {
-        const uint64_t tasks = (max_tiles * kSelTile + kRollTask - 1) / kRollTask;
-        uint64_t grid = (tasks + kRollTasksPerCta - 1) / kRollTasksPerCta;
-        if (grid > (uint64_t)num_sms * 2) grid = (uint64_t)num_sms * 2;
+        // 2 KiB per lane when one task per warp covers the batch on <= 2 CTAs
+        // per SM (the pipeline's 64 MiB batches: 32 CTAs, 1.5 % warm-up);
+        // bigger launches take 512 B lanes, several tasks per warp, for balance.
+        // Measured (C3, 300-step bench / isolated chunk stage over 672 MiB):
+        // 512 B 837 / 1562, 1 KiB 867 / 1468, 2 KiB 876 / 1305 GB/s.
+        const uint64_t span = max_tiles * kSelTile, cap = (uint64_t)num_sms * 2;
+        uint32_t lane_bytes = 2048;
+        if ((span + 64 * 2048 - 1) / (64 * 2048) > cap * kRollWarps) lane_bytes = 512;
+        const uint64_t tasks = (span + 64 * lane_bytes - 1) / (64 * lane_bytes);
+        uint64_t grid = (tasks + kRollWarps - 1) / kRollWarps;
+        if (grid > cap) grid = cap;
         if (grid < 1) grid = 1;
         auto k = value == 0 ? rabin_roll_kernel<true> : rabin_roll_kernel<false>;
-        k<<<(unsigned)grid, kRollThreads, kTabBytes, s>>>(d, d_tab, mask, value, bitmap);
+        k<<<(unsigned)grid, kRollThreads, kTabBytes, s>>>(d, d_tab, mask, value, bitmap,
+                                                          lane_bytes);
         uint64_t sb = (groups + kSelWarps - 1) / kSelWarps;
         if (sb > (uint64_t)num_sms * 8) sb = (uint64_t)num_sms * 8;
         if (sb < 1) sb = 1;
         select_tiles_kernel<<<(unsigned)sb, kSelWarps * 32, sizeof(SelCtaSmem), s>>>(
             d, bitmap, agg, gagg, evbuf);
     }
-#endif
     if (after_scan) cudaEventRecordWithFlags(after_scan, s, cudaEventRecordExternal);
     // NEXT-2 max_chunk: the state machine's cuts go to a scratch list first
     uint32_t* final_cut = cut_pos;

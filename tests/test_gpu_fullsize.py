@@ -87,3 +87,28 @@ def test_fullsize_all_zero():
         assert (g.digest == d0).all(), k
         assert (g.first_id == 0).all(), k
         assert g.is_dup.sum() == len(starts) - (k == 0), k
+
+
+def test_fullsize_op_chunk_one_launch():
+    """The whole 672 MiB C3 stream chunked by ONE op_chunk launch: the roll
+    kernel's many-tasks-per-warp configuration (512-byte lanes; the engine's
+    64 MiB batches use 2 KiB lanes), every cut position against the oracle."""
+    from paper_conf_ipps_rockenbachsgmtd19_b200 import Dedup
+    data = synthgen.config_stream("C3")
+    off = synthgen.split_items(data)
+    nbytes, n_items = len(data), len(off) - 1
+    with Dedup(0, batch_bytes=nbytes, batch_items=n_items + 1, slots=1, table_capacity=1 << 12,
+               host_fed=False) as d:
+        dev = torch.from_numpy(data).cuda()
+        offt = torch.from_numpy(off.astype(np.int64)).cuda()
+        cap = nbytes // 32 + n_items + 2
+        cut = torch.zeros(cap, dtype=torch.int32, device="cuda")
+        n = torch.zeros(1, dtype=torch.int32, device="cuda")
+        d.op_chunk(dev, nbytes, offt, n_items, cut, cap, n)
+        torch.cuda.synchronize()
+        got = cut[:int(n.item())].cpu().numpy().astype(np.int64)
+    s = oracle.Stream()
+    want = s.items_parallel(0, data, off)
+    s.close()
+    exp = np.concatenate([int(off[k]) + want.item(k)[0].astype(np.int64) for k in range(n_items)])
+    assert np.array_equal(got, exp)

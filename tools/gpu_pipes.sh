@@ -7,6 +7,6 @@ M=sm__inst_executed_pipe_alu.sum,sm__inst_executed_pipe_fma.sum,sm__inst_execute
 timeout 300 ncu --metrics $M --csv /tmp/mbp > gpurun_out/pipes_ncu.csv 2>&1
 for L in 32768 8192 4096; do MB=672 CASES=real REPS=3 LANE=$L timeout 300 python tools/sha_sizes.py >> gpurun_out/sha_lane.txt 2>&1; done
 MB=672 CASES=real REPS=1 LANE=4096 timeout 300 ncu --metrics $M --csv -k regex:sha1_kernel -s 1 -c 1 python tools/sha_sizes.py > gpurun_out/sha_ncu.csv 2>&1
-NBATCH=2 timeout 300 ncu --metrics $M --csv -k regex:"rabin_scan_agg2|sha1_kernel" -s 2 -c 2 python tools/one_batch.py > gpurun_out/batch_ncu.csv 2>&1
+NBATCH=2 timeout 300 ncu --metrics $M --csv -k regex:"rabin_roll|sha1_kernel" -s 2 -c 2 python tools/one_batch.py > gpurun_out/batch_ncu.csv 2>&1
 timeout 600 python bench.py --steps 20 --warmup 5 > gpurun_out/bench20.json 2> gpurun_out/bench20.err
 echo done
