@@ -209,7 +209,8 @@ __device__ __forceinline__ uint32_t first_item(uint64_t T0, const uint64_t* item
 // into the previous piece).
 __device__ __forceinline__ uint32_t apply_items(SelWarpSmem& sm, uint64_t T0, uint64_t nbytes,
                                                 const uint64_t* item_off, uint32_t n_items,
-                                                int lane, uint32_t first_rule = 0) {
+                                                int lane, uint32_t first_rule = 0,
+                                                uint32_t first = kInf) {
     uint32_t cw[8], fw[8];
 #pragma unroll
     for (int j = 0; j < 8; ++j) {
@@ -217,7 +218,8 @@ __device__ __forceinline__ uint32_t apply_items(SelWarpSmem& sm, uint64_t T0, ui
         fw[j] = 0;
     }
     const uint64_t E0 = T0 + (uint64_t)lane * kLaneBytes;  // this lane's e-range
-    const uint32_t lo = max(first_item(T0, item_off, n_items, lane), first_rule);
+    if (first == kInf) first = first_item(T0, item_off, n_items, lane);
+    const uint32_t lo = max(first, first_rule);
     if (E0 < nbytes && n_items > 0) {
         for (uint32_t it = lo; it < n_items; ++it) {
             const uint64_t q = item_off[it];
@@ -423,15 +425,17 @@ rabin_roll_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict
     }
 }
 
-// Per-tile selection from the candidate bitmap (the fused scan's epilogue):
-// a warp takes a group of 32 tiles; per tile it applies the item rules,
-// stores the tile's event list for the emit kernel and the tile's transfer
-// function, then composes the group's function.  The next tile's candidate
-// words are loaded while the current one is processed.
-constexpr int kSelWarps = 4;
+// Per-tile selection from the candidate bitmap: a CTA of kSelWarps warps
+// takes a group of 32 tiles, warp w its tiles w, w + kSelWarps, ...; per tile
+// a warp applies the item rules, stores the tile's event list for the emit
+// kernel and the tile's transfer function; warp 0 then composes the group's
+// function.  A warp's tiles increase, so its first-item index advances
+// incrementally (one binary search per warp and group); the next tile's
+// candidate words are loaded while the current one is processed.
+constexpr int kSelWarps = 8;
 struct SelCtaSmem {
     SelWarpSmem w[kSelWarps];
-    uint32_t fun[kSelWarps][kGroup][33];
+    uint32_t fun[kGroup][33];
 };
 
 __global__ void __launch_bounds__(kSelWarps * 32)
@@ -448,30 +452,39 @@ select_tiles_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restri
     const uint64_t* items = desc->item_off;
     const uint32_t n_items = desc->n_items;
     const uint32_t first_rule = (desc->carry & kCarryCont) ? 1u : 0u;
-    for (uint32_t g = blockIdx.x * kSelWarps + wid; g < n_groups; g += gridDim.x * kSelWarps) {
-        const uint32_t t0 = g * kGroup;
+    for (uint32_t g = blockIdx.x; g < n_groups; g += gridDim.x) {
+        const uint32_t t0 = g * kGroup + wid;
         uint4 na = make_uint4(0, 0, 0, 0), nb = na;
         if (t0 < n_tiles) {
             const uint4* src = reinterpret_cast<const uint4*>(bitmap + (size_t)t0 * kSelTileWords);
             na = src[2 * lane];
             nb = src[2 * lane + 1];
         }
-        for (int j = 0; j < kGroup; ++j) {
-            const uint32_t t = t0 + j;
+        uint32_t first = first_item((uint64_t)t0 * kSelTile, items, n_items, lane);
+        for (int j = wid; j < kGroup; j += kSelWarps) {
+            const uint32_t t = g * kGroup + j;
             uint32_t f = (uint32_t)lane << 27;
             if (t < n_tiles) {
                 uint4* dst = reinterpret_cast<uint4*>(sm.cand);
                 dst[2 * lane] = na;
                 dst[2 * lane + 1] = nb;
-                if (t + 1 < n_tiles && j + 1 < kGroup) {  // prefetch the next tile's words
+                const uint32_t tn = t + kSelWarps;
+                if (tn < n_tiles && j + kSelWarps < kGroup) {  // the next tile's words
                     const uint4* src =
-                        reinterpret_cast<const uint4*>(bitmap + (size_t)(t + 1) * kSelTileWords);
+                        reinterpret_cast<const uint4*>(bitmap + (size_t)tn * kSelTileWords);
                     na = src[2 * lane];
                     nb = src[2 * lane + 1];
                 }
+                // first item whose start is > T0 - 32 (first_item), advanced from
+                // the previous tile of this warp
+                const uint64_t T0 = (uint64_t)t * kSelTile;
+                const uint64_t key = T0 >= 31 ? T0 - 31 : 0;
+                if (lane == 0)
+                    while (first < n_items && items[first] < key) ++first;
+                first = __shfl_sync(kFull, first, 0);
                 __syncwarp();
-                const uint32_t n_ev = apply_items(sm, (uint64_t)t * kSelTile, nbytes, items,
-                                                  n_items, lane, first_rule);
+                const uint32_t n_ev =
+                    apply_items(sm, T0, nbytes, items, n_items, lane, first_rule, first);
                 store_events(sm, n_ev, evbuf + (size_t)t * kEvWords, lane);
                 uint32_t ex;
                 const uint32_t cnt = walk_any(sm, n_ev, lane, ex, nullptr, 0, 0, 0);
@@ -479,20 +492,22 @@ select_tiles_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restri
                 agg[32 * t + lane] = f;
                 __syncwarp();
             }
-            cs.fun[wid][j][lane] = f;
+            cs.fun[j][lane] = f;
         }
-        __syncwarp();
-        uint32_t Gs = lane, Gc = 0;
+        __syncthreads();
+        if (wid == 0) {
+            uint32_t Gs = lane, Gc = 0;
 #pragma unroll 8
-        for (int j = 0; j < kGroup; ++j) {
-            const uint32_t a = cs.fun[wid][j][lane];
-            const uint32_t ns = __shfl_sync(kFull, a >> 27, Gs);
-            const uint32_t nc = Gc + __shfl_sync(kFull, a & kM27, Gs);
-            Gs = ns;
-            Gc = nc;
+            for (int j = 0; j < kGroup; ++j) {
+                const uint32_t a = cs.fun[j][lane];
+                const uint32_t ns = __shfl_sync(kFull, a >> 27, Gs);
+                const uint32_t nc = Gc + __shfl_sync(kFull, a & kM27, Gs);
+                Gs = ns;
+                Gc = nc;
+            }
+            gagg[32 * g + lane] = (Gs << 27) | Gc;
         }
-        gagg[32 * g + lane] = (Gs << 27) | Gc;
-        __syncwarp();
+        __syncthreads();
     }
 }
 
@@ -761,7 +776,7 @@ void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mas
         auto k = value == 0 ? rabin_roll_kernel<true> : rabin_roll_kernel<false>;
         k<<<(unsigned)grid, kRollThreads, kTabBytes, s>>>(d, d_tab, mask, value, bitmap,
                                                           lane_bytes);
-        uint64_t sb = (groups + kSelWarps - 1) / kSelWarps;
+        uint64_t sb = groups;  // one CTA per group of 32 tiles
         if (sb > (uint64_t)num_sms * 8) sb = (uint64_t)num_sms * 8;
         if (sb < 1) sb = 1;
         select_tiles_kernel<<<(unsigned)sb, kSelWarps * 32, sizeof(SelCtaSmem), s>>>(

@@ -42,7 +42,8 @@ M = ['gpu__time_duration.sum', 'smsp__inst_executed.sum', 'sm__inst_executed.avg
      'sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active',
      'sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active',
      'smsp__thread_inst_executed_per_inst_executed.ratio', 'dram__bytes_read.sum', 'dram__bytes_write.sum',
-     'launch__registers_per_thread', 'launch__grid_size', 'launch__block_size', 'sm__cycles_active.avg']
+     'launch__registers_per_thread', 'launch__grid_size', 'launch__block_size', 'sm__cycles_active.avg',
+     'sm__inst_executed_pipe_alu.sum', 'sm__inst_executed_pipe_fmaheavy.sum']
 
 
 def full_table(rep):
@@ -80,6 +81,11 @@ if os.path.exists('gpurun_out/prof_sha.ncu-rep'):
     md += ['', '## ncu --set full, the SHA-1 kernel alone on all 672 MiB of C3 chunks '
                '(tools/sha_sizes.py, one launch)', '']
     md += sh
+if os.path.exists('gpurun_out/prof_roll.ncu-rep'):
+    rl, _ = full_table('gpurun_out/prof_roll.ncu-rep')
+    md += ['', '## ncu --set full, the roll and tile-selection kernels over all 672 MiB of C3 '
+               '(tools/scan_sizes.py, one op_chunk launch: 512-byte lanes)', '']
+    md += rl
 if os.path.exists('gpurun_out/prof_fm.ncu-rep'):
     fm, fm_traffic = full_table('gpurun_out/prof_fm.ncu-rep')
     md += ['', '## ncu --set full, row NEXT-1 FindMatch, one 64 MiB batch of C2 (tools/fm_sizes.py)', '']
@@ -88,7 +94,7 @@ if os.path.exists('gpurun_out/prof_fm.ncu-rep'):
 open(f'profiles/{tag}_ncu_summary.md', 'w').write('\n'.join(md) + '\n')
 tj = {"_source": "ncu --set full, tools/one_batch.py (64 MiB batches of C3); DRAM read+write bytes per "
                  "launch; bench scales per input byte", "capture_batch_bytes": BATCH}
-name_map = {'sha1_kernel': 'sha1', 'rabin_scan_kernel': 'rabin_scan', 'select_emit_ev_kernel': 'select_emit',
+name_map = {'sha1_kernel': 'sha1', 'rabin_roll_kernel': 'rabin_roll', 'select_emit_ev_kernel': 'select_emit',
             'table_insert_kernel': 'table_insert'}
 for k, v in traffic.items():
     tj[name_map.get(k, k)] = v
