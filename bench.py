@@ -346,14 +346,16 @@ def sha1_peak(r):
     return SHA1_OPS_PER_BLOCK / t
 
 
-def isolated_kernels(dd, off, int_peak, alu_peak, reps=3, streams=4):
+def isolated_kernels(dd, off, int_peak, alu_peak, reps=3, streams=12):
     """Live per-kernel throughput with the GPU filled by one kernel type, on
     the C3 stream.  chunk stage: one op_chunk call (scan + cut selection)
     over the whole stream.  SHA-1: one launch's duration is floored by its
     longest chunk's serial chain of 64-byte compressions (latency, not
     throughput), so `streams` contexts launch the same SHA-1 work
     concurrently on their own streams and the throughput is all their blocks
-    over the joint elapsed time.  CUDA events on torch's stream bracket both."""
+    over the joint elapsed time.  12 launches of 84 CTAs keep every SM's 4
+    SHA-1 CTA slots busy through each launch's tail (measured: 4 / 8 / 12
+    concurrent launches 1.64-1.67 / 1.72-1.74 / 1.82-1.85 TB/s).  CUDA events on torch's stream bracket both."""
     import torch
 
     from paper_conf_ipps_rockenbachsgmtd19_b200 import Dedup
@@ -724,7 +726,7 @@ def main():
                                f"{rates['mix_lop3_imad']:.1f} T ops/s",
                 "launch": f"{kd['launch_bytes'] / MiB:.0f} MiB of C3 chunks per launch, "
                           f"{kd['launch_us']:.0f} us per launch (CUDA events, "
-                          "4 concurrent streams)"}
+                          "12 concurrent launches on their own streams)"}
 
     # ---- the other BASELINE.json configs ----
     cfgs = config_lines(args.steps)
