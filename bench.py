@@ -140,7 +140,7 @@ def plan_batches(off, batch_bytes=None, batch_items=None):
     return out
 
 
-SHA_LANE = 0                     # batch bytes per SHA-1 lane (0: the engine's 32 KiB)
+SHA_LANE = 0                     # batch bytes per SHA-1 lane (0: the engine's 16 KiB)
 
 
 def engine_kwargs(stream_bytes: int) -> dict:
@@ -353,9 +353,10 @@ def isolated_kernels(dd, off, int_peak, alu_peak, reps=3, streams=12):
     longest chunk's serial chain of 64-byte compressions (latency, not
     throughput), so `streams` contexts launch the same SHA-1 work
     concurrently on their own streams and the throughput is all their blocks
-    over the joint elapsed time.  12 launches of 84 CTAs keep every SM's 4
-    SHA-1 CTA slots busy through each launch's tail (measured: 4 / 8 / 12
-    concurrent launches 1.64-1.67 / 1.72-1.74 / 1.82-1.85 TB/s).  CUDA events on torch's stream bracket both."""
+    over the joint elapsed time.  12 concurrent launches keep every SM's 4
+    SHA-1 CTA slots busy through each launch's tail (measured with 32 KiB
+    lanes, 84 CTAs per launch: 4 / 8 / 12 launches 1.64-1.67 / 1.72-1.74 /
+    1.82-1.85 TB/s; 8 launches of 16 KiB lanes 1.83-1.86).  CUDA events on torch's stream bracket both."""
     import torch
 
     from paper_conf_ipps_rockenbachsgmtd19_b200 import Dedup

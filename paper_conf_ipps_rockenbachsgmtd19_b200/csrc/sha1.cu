@@ -381,7 +381,7 @@ void launch_sha1(const BatchDesc* d, uint64_t max_bytes, const uint32_t* cut_pos
     // lanes to finish the batch's bulk within its longest chunk's latency:
     // one lane per lane_bytes of input keeps the per-batch footprint small
     // and leaves the SMs to the other in-flight batches.
-    const uint64_t per_lane = lane_bytes ? lane_bytes : 32768;
+    const uint64_t per_lane = lane_bytes ? lane_bytes : 16384;
     uint64_t lanes = max_bytes / per_lane;
     if (lanes < 2048) lanes = 2048;
     uint64_t blocks = (lanes + kShaThreads - 1) / kShaThreads;
