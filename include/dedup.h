@@ -98,7 +98,10 @@ typedef struct {
     uint32_t transport;         /* exchange of rows A6/A8: 0 auto (NCCL if the devices are
                                    distinct, else copy), 1 NCCL (ncclCommInitAll; distinct
                                    devices), 2 in-process copy (peer loads over NVLink, or
-                                   the loopback when device ids repeat) */
+                                   the loopback when device ids repeat), 3 in-process p2p
+                                   (the exchange fused into the table kernels: records
+                                   inserted into and first ids read from the owners' shards
+                                   with system-scope atomics / loads on peer memory) */
     const int32_t* device_ids;  /* [num_devices] CUDA ordinals, may repeat; NULL = 0..G-1 */
     /* Carry-over mode (row NEXT-2; north_star: "the chunking is identical when
      * the input is split at arbitrary batch cuts"): 1 = the bytes of a dedup

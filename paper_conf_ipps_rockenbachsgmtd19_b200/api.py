@@ -87,7 +87,7 @@ class Dedup:
         """num_devices >= 2 (or transport != 0) selects the multi-GPU engine
         (include/dedup.h): G ranks on device_ids (default 0..G-1; ids may
         repeat: then the ranks share a GPU and exchange through the in-process
-        copy transport), transport 0 auto / 1 NCCL / 2 copy; `slots` is then
+        copy transport), transport 0 auto / 1 NCCL / 2 copy / 3 p2p; `slots` is then
         the waves in flight per rank."""
         L = N.lib()
         cfg = N.Config()

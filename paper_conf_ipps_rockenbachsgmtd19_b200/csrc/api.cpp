@@ -466,7 +466,7 @@ dedup_status check_cfg(const dedup_config* g) {
     if (g->num_owners < 1 || g->num_owners > 64 || g->owner_rank >= g->num_owners)
         return DEDUP_EINVAL;
     if (g->table_capacity < 1 || g->table_capacity > (1ull << 31)) return DEDUP_EINVAL;
-    if (g->num_devices > 64 || g->transport > 2) return DEDUP_EINVAL;
+    if (g->num_devices > 64 || g->transport > 3) return DEDUP_EINVAL;
     if (g->carry_over && (mg::wanted(g) || g->min_chunk != 32 || g->max_chunk != 0 ||
                           g->slots < 2 || g->num_owners != 1))
         return DEDUP_EUNSUPPORTED;  // carry-over: single-GPU engine, the 32-state selection

@@ -139,6 +139,18 @@ void launch_table_prepare(const BatchDesc* d, uint64_t max_slots, int num_sms, c
 void launch_table_insert(const TableView* tv, const uint8_t* digest, const uint64_t* id,
                          const void* rec, const uint32_t* d_n, uint64_t n_host, uint64_t cap,
                          uint32_t* slot_idx, int num_sms, cudaStream_t s);
+// Transport 3 (p2p, one process): the routed records of a rank (send,
+// grouped by owner, send_off[G] of them, <= cap) inserted directly into the
+// owners' shards (views: device array of the G owners' TableViews, peer
+// memory), and after every rank's inserts their first ids read back into
+// reply_back (send order).  slot_idx: cap words of scratch kept between the
+// two calls.
+void launch_p2p_insert(const TableView* views, uint32_t G, const void* send,
+                       const uint32_t* send_off, uint64_t cap, uint32_t* slot_idx, int num_sms,
+                       cudaStream_t s);
+void launch_p2p_lookup(const TableView* views, uint32_t G, const void* send,
+                       const uint32_t* send_off, uint64_t cap, const uint32_t* slot_idx,
+                       uint64_t* reply_back, int num_sms, cudaStream_t s);
 void launch_table_lookup(const TableView* tv, const uint64_t* id, const void* rec,
                          const uint32_t* d_n, uint64_t n_host, uint64_t cap,
                          const uint32_t* slot_idx, uint64_t* first_id, uint8_t* is_dup,

@@ -34,6 +34,13 @@
 //     needs no host synchronisation.  Host barriers of the rank threads order
 //     the events: all ranks submitted the wave; all owners looked up; all
 //     pulls done (before any buffer of the wave is reused).
+//   * p2p (in-process, transport 3): the exchange fused into the table
+//     kernels -- a rank inserts its routed records straight into the owners'
+//     shards (system-scope atomics on peer memory over NVLink, or the
+//     loopback) and, once every rank's inserts of the wave are done, reads
+//     its first ids back from them: no record or reply copies, 2 kernels per
+//     wave instead of 4.  Barriers as for copy (all submitted + resets
+//     issued; all inserted; all looked up).
 // Uses: dedup_init with num_devices >= 2 (one process, one worker thread per
 // rank, results merged in seq order by dedup_drain) and dedup_dist_* (one
 // process per GPU, NCCL, driven by the caller's thread).
@@ -166,6 +173,8 @@ struct Rank {
     TableSlot* tab = nullptr;
     uint32_t* tab_status = nullptr;
     TableView* d_tabv = nullptr;
+    TableView* d_views = nullptr;  // p2p: the G owners' shards (peer memory)
+    cudaEvent_t e_rst = nullptr;   // p2p: this wave's table resets issued
     uint64_t tab_cap = 0;
     dedup_record* recv = nullptr;
     uint64_t* reply = nullptr;
@@ -183,6 +192,7 @@ struct Engine {
     uint32_t nslots = 1;        // slots per rank (dist: depth + 1, so a completed wave's
                                 // results stay readable while the next one is submitted)
     bool copy = false, host_fed = false;
+    bool p2p = false;  // transport 3: remote insert / lookup on the owners' shards
     uint64_t batch_bytes = 0, cap = 0;
     uint32_t batch_items = 0, lane_bytes = 16384, time_every = 1;
     std::vector<std::unique_ptr<Rank>> ranks;  // local ranks
@@ -305,9 +315,10 @@ void rank_free(Rank& r) {
     r.slots.clear();
     if (r.ccomm) ncclCommDestroy(r.ccomm);
     if (r.comm) ncclCommDestroy(r.comm);
-    for (cudaEvent_t e : {r.e_rdy, r.e_fin})
+    for (cudaEvent_t e : {r.e_rdy, r.e_fin, r.e_rst})
         if (e) cudaEventDestroy(e);
     for (void* p : {(void*)r.d_rtab, (void*)r.tab, (void*)r.tab_status, (void*)r.d_tabv,
+                    (void*)r.d_views,
                     (void*)r.recv, (void*)r.reply, (void*)r.roff, (void*)r.o_slot_idx,
                     (void*)r.p_rep_src, (void*)r.p_rep_off})
         if (p) cudaFree(p);
@@ -484,6 +495,7 @@ dedup_status rank_alloc(Engine* E, Rank& r, uint64_t shard_capacity) {
     MCU(cudaStreamCreateWithPriority(&r.cs, cudaStreamNonBlocking, prio_hi));
     MCU(cudaEventCreateWithFlags(&r.e_rdy, cudaEventDisableTiming));
     MCU(cudaEventCreateWithFlags(&r.e_fin, cudaEventDisableTiming));
+    MCU(cudaEventCreateWithFlags(&r.e_rst, cudaEventDisableTiming));
     r.tab_cap = next_pow2(2 * shard_capacity);
     MTRY(dmalloc(E, &r.tab, r.tab_cap));
     MTRY(dmalloc(E, &r.tab_status, 4));
@@ -493,16 +505,21 @@ dedup_status rank_alloc(Engine* E, Rank& r, uint64_t shard_capacity) {
     const TableView tv{r.tab, r.tab_cap - 1, r.tab_status};
     MCU(cudaMemcpy(r.d_tabv, &tv, sizeof(tv), cudaMemcpyHostToDevice));
     // an owner receives at most every rank's whole batch (distinct digests)
+    // (p2p: no records or replies are copied; o_slot_idx holds the rank's
+    // own records' slots between its insert and lookup)
     const uint64_t rcap = E->cap * E->G;
-    MTRY(dmalloc(E, &r.recv, rcap));
-    MTRY(dmalloc(E, &r.reply, rcap));
-    MTRY(dmalloc(E, &r.o_slot_idx, rcap));
+    if (!E->p2p) {
+        MTRY(dmalloc(E, &r.recv, rcap));
+        MTRY(dmalloc(E, &r.reply, rcap));
+    }
+    MTRY(dmalloc(E, &r.o_slot_idx, E->p2p ? E->cap : rcap));
     MTRY(dmalloc(E, &r.roff, E->G + 1));
     MCU(cudaMemset(r.roff, 0, sizeof(uint32_t) * (E->G + 1)));
     if (E->copy) {
         MTRY(dmalloc(E, &r.p_rep_src, E->G));
         MTRY(dmalloc(E, &r.p_rep_off, E->G));
     }
+    if (E->p2p) MTRY(dmalloc(E, &r.d_views, E->G));
     r.slots.resize(E->nslots);
     for (auto& sl : r.slots) {
         sl.reset(new Slot());
@@ -525,6 +542,13 @@ dedup_status wire_copy(Engine* E) {
         }
         MCU(cudaMemcpy(r.p_rep_src, a.data(), sizeof(void*) * G, cudaMemcpyHostToDevice));
         MCU(cudaMemcpy(r.p_rep_off, b.data(), sizeof(void*) * G, cudaMemcpyHostToDevice));
+        if (E->p2p) {  // every owner's shard, as this rank's kernels address it
+            std::vector<TableView> v(G);
+            for (uint32_t s = 0; s < G; ++s)
+                v[s] = TableView{E->ranks[s]->tab, E->ranks[s]->tab_cap - 1,
+                                 E->ranks[s]->tab_status};
+            MCU(cudaMemcpy(r.d_views, v.data(), sizeof(TableView) * G, cudaMemcpyHostToDevice));
+        }
         for (uint32_t i = 0; i < E->nslots; ++i) {
             for (uint32_t s = 0; s < G; ++s) {
                 a[s] = E->ranks[s]->slots[i]->send;
@@ -663,7 +687,30 @@ dedup_status rank_complete(Engine* E, Rank& r, uint64_t w) {
         return E->fail(DEDUP_ECUDA, "protocol: completion of a wave this rank did not submit");
     MCU(cudaSetDevice(r.dev));
     sl.timed = (w % E->time_every) == 0;
-    if (E->copy) {
+    if (E->p2p) {
+        // own shard's resets for this wave first (others insert into it next)
+        MTRY(apply_resets(E, r, w));
+        MCU(cudaEventRecord(r.e_rst, r.os));
+        if (!E->bar.wait(E->abort)) return (dedup_status)E->sticky.load();  // submitted, reset
+        MCU(cudaStreamWaitEvent(r.os, sl.e_local, 0));
+        for (auto& q : E->ranks) MCU(cudaStreamWaitEvent(r.os, q->e_rst, 0));
+        if (sl.timed) MCU(cudaEventRecord(sl.e_a0, r.os));
+        launch_p2p_insert(r.d_views, G, sl.send, sl.send_off, E->cap, r.o_slot_idx, r.num_sms,
+                          r.os);  // rows A6 + A7 (insert) over peer memory
+        E->launches += 1;
+        MCU(cudaGetLastError());
+        MCU(cudaEventRecord(r.e_rdy, r.os));
+        if (!E->bar.wait(E->abort)) return (dedup_status)E->sticky.load();  // all inserted
+        for (auto& q : E->ranks) MCU(cudaStreamWaitEvent(r.os, q->e_rdy, 0));
+        launch_p2p_lookup(r.d_views, G, sl.send, sl.send_off, E->cap, r.o_slot_idx,
+                          sl.reply_back, r.num_sms, r.os);  // rows A7 (lookup) + A8
+        E->launches += 1;
+        MCU(cudaGetLastError());
+        MTRY(finish(E, r, sl));
+        MCU(cudaEventRecord(r.e_fin, r.os));
+        if (!E->bar.wait(E->abort)) return (dedup_status)E->sticky.load();  // all looked up
+        for (auto& q : E->ranks) MCU(cudaStreamWaitEvent(r.os, q->e_fin, 0));
+    } else if (E->copy) {
         if (!E->bar.wait(E->abort)) return (dedup_status)E->sticky.load();  // all submitted w
         MTRY(apply_resets(E, r, w));
         for (auto& q : E->ranks)
@@ -1039,7 +1086,8 @@ dedup_status create(const dedup_config* cfg, CtxEngine** out, const char** why) 
         }
         for (uint32_t q = 0; q < r; ++q) distinct = distinct && devs[q] != devs[r];
     }
-    bool copy = cfg->transport == 2 || (cfg->transport == 0 && !distinct);
+    const bool p2p = cfg->transport == 3;
+    bool copy = cfg->transport == 2 || p2p || (cfg->transport == 0 && !distinct);
     if (!copy && !distinct) {
         *why = "NCCL needs distinct devices (one rank per GPU)";
         return DEDUP_EUNSUPPORTED;
@@ -1047,6 +1095,7 @@ dedup_status create(const dedup_config* cfg, CtxEngine** out, const char** why) 
     auto* e = new CtxEngine();
     Engine& E = e->E;
     E.copy = copy;
+    E.p2p = p2p;
     engine_init(&E, cfg, G, cfg->slots, cfg->batch_bytes, cfg->batch_items);
     E.bar.n = G;
     e->lag = E.depth > 1 ? E.depth - 1 : 1;

@@ -165,6 +165,90 @@ __device__ __forceinline__ uint32_t owner_of(const uint8_t* digest, uint64_t r, 
     return (uint32_t)(((uint64_t)be * G) >> 32);
 }
 
+// ---- transport 3 (p2p): the exchange fused into the table kernels ----
+// One process, G ranks with peer access (NVLink) or sharing a GPU: a rank
+// inserts its routed records directly into the owner ranks' shards and later
+// reads the first ids back from them (remote atomics / loads on peer memory),
+// instead of copying records to the owners and replies back.  System-scope
+// atomics and fences: the shards are touched by the SMs of several GPUs.
+__device__ __forceinline__ uint32_t ld_acquire_sys(const uint32_t* p) {
+    uint32_t v;
+    asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ uint32_t owner_of_key(uint32_t k0, uint32_t G) {
+    const uint32_t be = __byte_perm(k0, 0, 0x0123);  // BE32(digest[0..3])
+    return (uint32_t)(((uint64_t)be * G) >> 32);
+}
+
+__global__ void p2p_insert_kernel(const TableView* __restrict__ views, uint32_t G,
+                                  const uint8_t* __restrict__ send,
+                                  const uint32_t* __restrict__ send_off, uint64_t cap,
+                                  uint32_t* __restrict__ slot_idx) {
+    const uint64_t n = min((uint64_t)send_off[G], cap);
+    for (uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; r < n;
+         r += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t* rec = reinterpret_cast<const uint32_t*>(send + 32 * r);  // dedup_record
+        uint32_t key[5];
+#pragma unroll
+        for (int i = 0; i < 5; ++i) key[i] = rec[i];
+        const uint64_t myid = *reinterpret_cast<const uint64_t*>(rec + 6);
+        const TableView t = views[owner_of_key(key[0], G)];
+        uint64_t idx = (((uint64_t)key[2] << 32) | key[1]) & t.mask;
+        uint32_t found = 0xFFFFFFFFu;
+        for (uint64_t probe = 0; probe <= t.mask; ++probe) {
+            TableSlot* sl = t.slots + idx;
+            uint32_t st = ld_acquire_sys(&sl->state);
+            if (st == 0) {
+                const uint32_t old = atomicCAS_system(&sl->state, 0u, 1u);
+                if (old == 0) {
+#pragma unroll
+                    for (int i = 0; i < 5; ++i) sl->key[i] = key[i];
+                    __threadfence_system();
+                    atomicExch_system(&sl->state, 2u);
+                    atomicAdd_system(&t.status[1], 1u);
+                    atomicMax_system(reinterpret_cast<unsigned long long*>(&sl->inv_min),
+                                     (unsigned long long)~myid);
+                    found = (uint32_t)idx;
+                    break;
+                }
+                st = old;
+            }
+            while (st == 1) st = ld_acquire_sys(&sl->state);
+            bool eq = true;
+#pragma unroll
+            for (int i = 0; i < 5; ++i) eq = eq && (ld_acquire_sys(&sl->key[i]) == key[i]);
+            if (eq) {
+                atomicMax_system(reinterpret_cast<unsigned long long*>(&sl->inv_min),
+                                 (unsigned long long)~myid);
+                found = (uint32_t)idx;
+                break;
+            }
+            idx = (idx + 1) & t.mask;
+        }
+        if (found == 0xFFFFFFFFu) atomicExch_system(&t.status[0], 1u);
+        slot_idx[r] = found;
+    }
+}
+
+// After every rank's inserts of the wave: the first id of each routed record
+// read from its owner's shard (~0 if the shard overflowed).
+__global__ void p2p_lookup_kernel(const TableView* __restrict__ views, uint32_t G,
+                                  const uint8_t* __restrict__ send,
+                                  const uint32_t* __restrict__ send_off, uint64_t cap,
+                                  const uint32_t* __restrict__ slot_idx,
+                                  uint64_t* __restrict__ reply_back) {
+    const uint64_t n = min((uint64_t)send_off[G], cap);
+    for (uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; r < n;
+         r += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t si = slot_idx[r];
+        const TableView t =
+            views[owner_of_key(*reinterpret_cast<const uint32_t*>(send + 32 * r), G)];
+        reply_back[r] = si == 0xFFFFFFFFu ? ~0ull : ~t.slots[si].inv_min;
+    }
+}
+
 // rep (optional, local combine): only records with rep[r] == r are routed.
 __device__ __forceinline__ bool routed(const uint32_t* rep, uint64_t r) {
     return rep == nullptr || rep[r] == (uint32_t)r;
@@ -375,6 +459,22 @@ void launch_table_lookup(const TableView* t, const uint64_t* id, const void* rec
     const uint64_t n = d_n != nullptr ? cap : n_host;
     table_lookup_kernel<<<grid_for(n, 256, num_sms, 1), 256, 0, s>>>(
         t, id, rec, d_n, n_host, cap, slot_idx, first_id, is_dup, status_out, cut_pos, desc);
+}
+
+void launch_p2p_insert(const TableView* views, uint32_t G, const void* send,
+                       const uint32_t* send_off, uint64_t cap, uint32_t* slot_idx, int num_sms,
+                       cudaStream_t s) {
+    if (cap == 0) return;
+    p2p_insert_kernel<<<grid_for(cap, 256, num_sms, 1), 256, 0, s>>>(
+        views, G, static_cast<const uint8_t*>(send), send_off, cap, slot_idx);
+}
+
+void launch_p2p_lookup(const TableView* views, uint32_t G, const void* send,
+                       const uint32_t* send_off, uint64_t cap, const uint32_t* slot_idx,
+                       uint64_t* reply_back, int num_sms, cudaStream_t s) {
+    if (cap == 0) return;
+    p2p_lookup_kernel<<<grid_for(cap, 256, num_sms, 1), 256, 0, s>>>(
+        views, G, static_cast<const uint8_t*>(send), send_off, cap, slot_idx, reply_back);
 }
 
 void launch_route(const uint8_t* digest, const uint64_t* id, const uint32_t* d_n, uint64_t cap,

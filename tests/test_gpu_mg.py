@@ -59,8 +59,9 @@ def submit_device_batches(d, dev, off, k0, k1, batch_bytes, batch_items, got):
                 got.extend(d.drain(wait_ms=-1))
 
 
+@pytest.mark.parametrize("transport", [2, 3])
 @pytest.mark.parametrize("G,depth", [(2, 1), (2, 3), (4, 2), (8, 3), (3, 4)])
-def test_mg_loopback_device_matches_oracle(G, depth):
+def test_mg_loopback_device_matches_oracle(G, depth, transport):
     """Device-resident batches through G ranks: two dedup streams (an
     end_stream between them with waves in flight) then the first stream's
     bytes again (all new again after the reset); every output bit-exact."""
@@ -69,7 +70,7 @@ def test_mg_loopback_device_matches_oracle(G, depth):
     n = len(off) - 1
     h = n // 2
     got = []
-    with mg(G, depth) as d:
+    with mg(G, depth, transport=transport) as d:
         submit_device_batches(d, dev, off, 0, h, MiB, 8, got)
         d.end_stream()
         submit_device_batches(d, dev, off, h, n, MiB, 8, got)
@@ -119,7 +120,8 @@ def test_mg_loopback_host_fed_matches_oracle(G):
     U.assert_same(got, oracle_stream(data, off))
 
 
-def test_mg_all_duplicate_sends_one_record_per_digest():
+@pytest.mark.parametrize("transport", [0, 3])
+def test_mg_all_duplicate_sends_one_record_per_digest(transport):
     """C5b-like: every item equal.  The local combine sends one record per
     distinct digest per batch; a2a bytes count what left each rank."""
     item = U.stream(MiB // 2, seed=77, dup_frac=0.0)
@@ -128,7 +130,7 @@ def test_mg_all_duplicate_sends_one_record_per_digest():
     dev = torch.from_numpy(data).cuda()
     G = 4
     got = []
-    with mg(G, 2, batch_bytes=MiB, batch_items=2) as d:
+    with mg(G, 2, batch_bytes=MiB, batch_items=2, transport=transport) as d:
         submit_device_batches(d, dev, off, 0, len(off) - 1, MiB, 2, got)
         got.extend(d.drain_all())
         st = d.stats()
@@ -180,13 +182,14 @@ def test_mg_join_brackets_all_work():
     U.assert_same(got, oracle_stream(data, off))
 
 
-def test_mg_table_overflow_is_sticky():
+@pytest.mark.parametrize("transport", [2, 3])
+def test_mg_table_overflow_is_sticky(transport):
     """A full shard is DEDUP_ETABLEFULL (sticky), never wrong dup flags."""
     from paper_conf_ipps_rockenbachsgmtd19_b200._native import DedupError
     data = U.stream(48 * MiB, seed=505, dup_frac=0.0)      # ~12 k distinct chunks
     off = synthgen.split_items(data, MiB // 2)
     dev = torch.from_numpy(data).cuda()
-    with mg(2, 2, table_capacity=16) as d:                  # 2 shards of 4096 slots
+    with mg(2, 2, table_capacity=16, transport=transport) as d:  # 2 shards of 4096 slots
         with pytest.raises(DedupError, match="ETABLEFULL"):
             got = []
             submit_device_batches(d, dev, off, 0, len(off) - 1, MiB, 8, got)
@@ -201,6 +204,8 @@ def test_mg_rejects_op_layer_and_bad_config():
         mg(2, 2, owner_rank=1, num_owners=2)
     with pytest.raises(DedupError):
         mg(2, 2, transport=1)           # NCCL needs distinct devices
+    with pytest.raises(DedupError):
+        mg(2, 2, transport=4)           # no such transport
     with mg(2, 1) as d:
         cut = torch.zeros(16, dtype=torch.int32, device="cuda")
         with pytest.raises(DedupError, match="EUNSUPPORTED"):

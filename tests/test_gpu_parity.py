@@ -25,8 +25,10 @@ def cuda():
 
 # The engine tests run through dedup_init on every engine of include/dedup.h:
 # the single-GPU engine, and the multi-GPU engine (csrc/mg.cpp) with one rank
-# over NCCL and with 2 / 4 logical ranks on this GPU (copy transport).
-ENGINES = ["single", "nccl1", "copy2", "copy4"]
+# over NCCL, with 2 / 4 logical ranks on this GPU (copy transport) and with 2 /
+# 8 logical ranks exchanging through the owners' shards (p2p transport: remote
+# insert / lookup kernels; on one GPU the peer pointers are local).
+ENGINES = ["single", "nccl1", "copy2", "copy4", "p2p2", "p2p8"]
 
 
 def make_ctx(engine="single", **kw):
@@ -34,8 +36,9 @@ def make_ctx(engine="single", **kw):
     base = dict(batch_bytes=8 << 20, batch_items=1024, slots=3, table_capacity=1 << 18)
     base.update(kw)
     if engine != "single":
-        G = {"nccl1": 1, "copy2": 2, "copy4": 4}[engine]
-        base.update(num_devices=G, device_ids=[0] * G, transport=1 if engine == "nccl1" else 2,
+        G = {"nccl1": 1, "copy2": 2, "copy4": 4, "p2p2": 2, "p2p8": 8}[engine]
+        transport = 1 if engine == "nccl1" else (3 if engine.startswith("p2p") else 2)
+        base.update(num_devices=G, device_ids=[0] * G, transport=transport,
                     slots=min(base["slots"], 4))
     return Dedup(0, **base)
 
