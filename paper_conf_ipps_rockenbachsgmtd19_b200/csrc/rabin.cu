@@ -742,6 +742,14 @@ const char* chunk_unlaunchable() {
     chunk_set_attrs();
     for (const void* f : {(const void*)rabin_roll_kernel<true>, (const void*)rabin_roll_kernel<false>})
         if (!fits(f, kRollThreads, kTabBytes)) return "rabin_roll_kernel";
+    // the roll kernel addresses its table at window offset kRollWin (the shared
+    // memory the driver reserves per block; the kernel traps if it differs)
+    int dev = 0, reserved = -1;
+    cudaGetDevice(&dev);
+    if (cudaDeviceGetAttribute(&reserved, cudaDevAttrReservedSharedMemoryPerBlock, dev) !=
+            cudaSuccess ||
+        reserved != (int)kRollWin)
+        return "rabin_roll_kernel (reserved shared memory per block != 1 KiB)";
     if (!fits((const void*)select_tiles_kernel, kSelWarps * 32, sizeof(SelCtaSmem)))
         return "select_tiles_kernel";
     if (!fits((const void*)select_scan_kernel, 1024, 0)) return "select_scan_kernel";
