@@ -17,9 +17,12 @@
 //     lanes already done) take the guarded path;
 //   * the 16-word message schedule lives in registers (fully unrolled
 //     rounds, circular W[16]) and rotates are funnel shifts (SHF);
-//   * unaligned chunk data is read with five 16-byte loads (the next block's
-//     window prefetched during the compression) and realigned with two
-//     select stages + one PRMT per word (PRMT also does the big-endian swap).
+//   * unaligned chunk data is read as an 80-byte window of five 16-byte
+//     vectors (the next block's window prefetched during the compression;
+//     its first vector is this window's last, kept in registers, so a block
+//     costs four loads: isolated SHA-1 1.82 -> 1.89 TB/s) and realigned with
+//     two select stages + one PRMT per word (PRMT also does the big-endian
+//     swap).
 //     Measured alternative (C3, 672 MiB): staging the window in shared memory
 //     with cp.async and reading it back with 17 LDS at the lane's offset saves
 //     the 34 selects (isolated 805 vs 750 GB/s) but its 40 KiB per CTA keeps
@@ -115,6 +118,36 @@ __device__ __forceinline__ void load_raw(const uint8_t* __restrict__ bytes, uint
     const bool need5 = (p & 15) != 0;
 #pragma unroll
     for (int i = 0; i < 5; ++i) {
+        uint4 x = make_uint4(0, 0, 0, 0);
+        const uint64_t a = base + 16 * i;
+        bool ok = (i < 4) || need5;
+        if (kGuard) ok = ok && (a < lim16);
+        if (ok) x = __ldg(reinterpret_cast<const uint4*>(bytes + a));
+        v[4 * i] = x.x;
+        v[4 * i + 1] = x.y;
+        v[4 * i + 2] = x.z;
+        v[4 * i + 3] = x.w;
+    }
+}
+
+// The next block's window, base + 64: its vector 0 is this window's vector 4
+// when that one was loaded (p & 15 != 0, the same for every block of a chunk),
+// so only 4 vectors are loaded per block either way.
+template <bool kGuard>
+__device__ __forceinline__ void load_next(const uint8_t* __restrict__ bytes, uint64_t p,
+                                          uint64_t lim16, uint32_t v[20], bool need5) {
+    const uint64_t base = p & ~uint64_t(15);
+    uint4 x0 = make_uint4(v[16], v[17], v[18], v[19]);
+    if (!need5) {
+        x0 = make_uint4(0, 0, 0, 0);
+        if (!kGuard || base < lim16) x0 = __ldg(reinterpret_cast<const uint4*>(bytes + base));
+    }
+    v[0] = x0.x;
+    v[1] = x0.y;
+    v[2] = x0.z;
+    v[3] = x0.w;
+#pragma unroll
+    for (int i = 1; i < 5; ++i) {
         uint4 x = make_uint4(0, 0, 0, 0);
         const uint64_t a = base + 16 * i;
         bool ok = (i < 4) || need5;
@@ -326,15 +359,15 @@ sha1_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ cut
             realign(raw, o, M);
             p += 64;
             // prefetch the next block's window while this one compresses
-            if (i + 1 < nbulk) load_raw<false>(bytes, p, lim16, raw);
-            else load_raw<true>(bytes, p, lim16, raw);
+            if (i + 1 < nbulk) load_next<false>(bytes, p, lim16, raw, o != 0);
+            else load_next<true>(bytes, p, lim16, raw, o != 0);
             sha1_compress(H, M, one);
         }
         for (uint32_t i = nbulk; i < nb_max; ++i) {
             if (i < nb) {
                 realign(raw, o, M);
                 p += 64;
-                if (i + 1 < nb) load_raw<true>(bytes, p, lim16, raw);
+                if (i + 1 < nb) load_next<true>(bytes, p, lim16, raw, o != 0);
                 pad_block(M, (int32_t)L - (int32_t)(64 * i), i + 1 == nb && !open, L);
                 sha1_compress(H, M, one);
             }
