@@ -630,6 +630,7 @@ dedup_status dedup_init(const dedup_config* cfg, dedup_ctx** out) {
     if (cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, cfg->device) !=
         cudaSuccess)
         return bail(DEDUP_ECUDA);
+    set_pipeline_carveout();
     for (const char* bad : {chunk_unlaunchable(), sha1_unlaunchable()}) {
         if (bad) {
             std::fprintf(stderr, "dedup_init: %s cannot launch on device %d\n", bad,

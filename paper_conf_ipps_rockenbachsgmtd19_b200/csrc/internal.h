@@ -96,6 +96,13 @@ inline bool fits(const void* fn, int threads, size_t dyn_smem) {
 // configuration, or nullptr.
 const char* chunk_unlaunchable();
 const char* sha1_unlaunchable();
+// Preferred shared-memory carveout (percent) of the pipeline's kernels;
+// set_pipeline_carveout applies the engine's setting (table.cu) to all of
+// them on the current device.
+void set_pipeline_carveout();
+void sha1_set_carveout(int pct);
+void chunk_set_carveout(int pct);
+void table_set_carveout(int pct);
 void launch_chunk_select(const BatchDesc* d, const uint32_t* d_tab, uint32_t mask,
                          uint32_t value, uint32_t* bitmap, uint32_t* agg, uint32_t* gagg,
                          uint32_t* gentry, uint32_t* evbuf, uint64_t max_tiles,

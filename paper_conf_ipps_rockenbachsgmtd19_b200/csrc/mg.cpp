@@ -478,6 +478,7 @@ dedup_status slot_alloc(Engine* E, Rank& r, Slot& sl) {
 dedup_status rank_alloc(Engine* E, Rank& r, uint64_t shard_capacity) {
     MCU(cudaSetDevice(r.dev));
     MCU(cudaDeviceGetAttribute(&r.num_sms, cudaDevAttrMultiProcessorCount, r.dev));
+    set_pipeline_carveout();
     if (const char* bad = chunk_unlaunchable())
         return E->fail(DEDUP_ECUDA, std::string(bad) + " cannot launch");
     if (const char* bad = sha1_unlaunchable())

@@ -738,6 +738,13 @@ void chunk_set_attrs() {
 }
 }  // namespace
 
+void chunk_set_carveout(int pct) {
+    for (const void* f : {(const void*)rabin_roll_kernel<true>, (const void*)rabin_roll_kernel<false>,
+                          (const void*)select_tiles_kernel, (const void*)select_scan_kernel,
+                          (const void*)select_emit_ev_kernel, (const void*)chunk_meta_kernel})
+        cudaFuncSetAttribute(f, cudaFuncAttributePreferredSharedMemoryCarveout, pct);
+}
+
 const char* chunk_unlaunchable() {
     chunk_set_attrs();
     for (const void* f : {(const void*)rabin_roll_kernel<true>, (const void*)rabin_roll_kernel<false>})

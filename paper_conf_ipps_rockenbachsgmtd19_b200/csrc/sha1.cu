@@ -390,6 +390,12 @@ sha1_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ cut
 
 }  // namespace
 
+void sha1_set_carveout(int pct) {
+    for (const void* f : {(const void*)sha_hist_kernel, (const void*)sha_scan_kernel,
+                          (const void*)sha_scatter_kernel, (const void*)sha1_kernel})
+        cudaFuncSetAttribute(f, cudaFuncAttributePreferredSharedMemoryCarveout, pct);
+}
+
 const char* sha1_unlaunchable() {
     if (!fits((const void*)sha_hist_kernel, 256, 0)) return "sha_hist_kernel";
     if (!fits((const void*)sha_scan_kernel, 1024, 0)) return "sha_scan_kernel";

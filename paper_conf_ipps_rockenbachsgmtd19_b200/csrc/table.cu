@@ -13,6 +13,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <cstdlib>
+
 #include "internal.h"
 
 namespace dd {
@@ -459,6 +461,35 @@ void launch_table_lookup(const TableView* t, const uint64_t* id, const void* rec
     const uint64_t n = d_n != nullptr ? cap : n_host;
     table_lookup_kernel<<<grid_for(n, 256, num_sms, 1), 256, 0, s>>>(
         t, id, rec, d_n, n_host, cap, slot_idx, first_id, is_dup, status_out, cut_pos, desc);
+}
+
+// One shared-memory / L1 split for every kernel of the batch pipeline, so
+// that co-resident CTAs of different kernels never force an SM to
+// reconfigure (the driver's per-kernel default picks max L1 for the kernels
+// without shared memory and a large carve-out for the roll kernel).
+// Measured (C3 bench, 300 / 20 steps, interleaved reps): no preference
+// 899-903 / 840-860 GB/s; 44-52 % 923-925 / 865-884; 58 % 913-916 / 861-876;
+// 72 % 907; 86-100 % 688-693 (too little L1 for SHA-1's 16-byte loads);
+// 36-40 % 890-901; 0 % (max L1) 768-773 at 20 steps.  DEDUP_CARVEOUT=<pct>
+// overrides (A/B runs); -1 keeps the driver's choice.
+void set_pipeline_carveout() {
+    int pct = 48;
+    if (const char* cv = std::getenv("DEDUP_CARVEOUT")) pct = std::atoi(cv);
+    if (pct < 0) return;
+    sha1_set_carveout(pct);
+    chunk_set_carveout(pct);
+    table_set_carveout(pct);
+}
+
+void table_set_carveout(int pct) {
+    for (const void* f :
+         {(const void*)table_prepare_kernel, (const void*)table_insert_kernel,
+          (const void*)table_lookup_kernel, (const void*)pack_kernel, (const void*)scatter_kernel,
+          (const void*)route_count_kernel, (const void*)route_scan_kernel,
+          (const void*)route_scatter_kernel, (const void*)combine_rep_kernel,
+          (const void*)gather_rows_kernel, (const void*)gather_counts_kernel,
+          (const void*)p2p_insert_kernel, (const void*)p2p_lookup_kernel})
+        cudaFuncSetAttribute(f, cudaFuncAttributePreferredSharedMemoryCarveout, pct);
 }
 
 void launch_p2p_insert(const TableView* views, uint32_t G, const void* send,
