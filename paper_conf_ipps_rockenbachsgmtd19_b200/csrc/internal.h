@@ -4,6 +4,23 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+// DEDUP_CHECK builds (tools/gpu_checked.sh): device-side bounds checks in
+// the kernels, a trap with the failed condition printed; nothing otherwise.
+#ifdef DEDUP_CHECK
+#include <cstdio>
+#define DD_CHECK(cond)                                                                \
+    do {                                                                              \
+        if (!(cond)) {                                                                \
+            printf("DD_CHECK failed: %s (%s:%d)\n", #cond, __FILE__, __LINE__);       \
+            __trap();                                                                 \
+        }                                                                             \
+    } while (0)
+#else
+#define DD_CHECK(cond) \
+    do {               \
+    } while (0)
+#endif
+
 namespace dd {
 
 // ---- digest table --------------------------------------------------------

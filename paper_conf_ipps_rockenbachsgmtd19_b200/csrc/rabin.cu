@@ -395,6 +395,7 @@ rabin_roll_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict
                                                  laneW, mask, value);
             if (j < steps - 1) {  // the next step's bytes into the freed `old`
                 if (full) {
+                    DD_CHECK(bB0 + 64 <= nbytes && bA0 + 64 <= nbytes);
                     ldg_v8(bytes + bA0 + 32, oldA);
                     ldg_v8(bytes + bB0 + 32, oldB);
                 } else {
@@ -412,6 +413,8 @@ rabin_roll_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict
                 if (bA0 + 32 > nbytes) bitsA &= bA0 < nbytes ? (1u << (nbytes - bA0)) - 1u : 0u;
                 if (bB0 + 32 > nbytes) bitsB &= bB0 < nbytes ? (1u << (nbytes - bB0)) - 1u : 0u;
             }
+            DD_CHECK(!(full || actA) || bA0 < cover);
+            DD_CHECK(!(full || actB) || bB0 < cover);
             if (full || actA) bitmap[(bA0 >> 5)] = ewA;
             if (full || actB) bitmap[(bB0 >> 5)] = ewB;
             pbA = bitsA;
@@ -483,6 +486,8 @@ select_tiles_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restri
                     while (first < n_items && items[first] < key) ++first;
                 first = __shfl_sync(kFull, first, 0);
                 __syncwarp();
+                DD_CHECK(first <= n_items && (first == n_items || items[first] >= key) &&
+                         (first == 0 || items[first - 1] < key));
                 const uint32_t n_ev =
                     apply_items(sm, T0, nbytes, items, n_items, lane, first_rule, first);
                 store_events(sm, n_ev, evbuf + (size_t)t * kEvWords, lane);

@@ -116,6 +116,7 @@ __device__ __forceinline__ void load_raw(const uint8_t* __restrict__ bytes, uint
                                          uint64_t lim16, uint32_t v[20]) {
     const uint64_t base = p & ~uint64_t(15);
     const bool need5 = (p & 15) != 0;
+    DD_CHECK(kGuard || base + (need5 ? 80 : 64) <= lim16);
 #pragma unroll
     for (int i = 0; i < 5; ++i) {
         uint4 x = make_uint4(0, 0, 0, 0);
@@ -137,6 +138,7 @@ template <bool kGuard>
 __device__ __forceinline__ void load_next(const uint8_t* __restrict__ bytes, uint64_t p,
                                           uint64_t lim16, uint32_t v[20], bool need5) {
     const uint64_t base = p & ~uint64_t(15);
+    DD_CHECK(kGuard || base + (need5 ? 80 : 64) <= lim16);
     uint4 x0 = make_uint4(v[16], v[17], v[18], v[19]);
     if (!need5) {
         x0 = make_uint4(0, 0, 0, 0);
@@ -343,8 +345,13 @@ sha1_kernel(const BatchDesc* __restrict__ desc, const uint32_t* __restrict__ cut
         }
         const uint32_t nb_max = __reduce_max_sync(kFull, nb);
         const uint32_t nb_min = __reduce_min_sync(kFull, act ? nb : kFull);
-        // blocks [0, nbulk) hold 64 data bytes on every active lane
-        const uint32_t nbulk = nb_min >= 3 ? nb_min - 2 : 0;
+        // blocks [0, nbulk) hold 64 data bytes on every active lane.  Idle
+        // lanes (the last task, past the last chunk) run them from byte 0 of
+        // the batch: one bulk block less then keeps their unguarded window
+        // loads below 64 nb_min - 112 <= the shortest active chunk, so inside
+        // the batch (the guarded tail path takes that block)
+        uint32_t nbulk = nb_min >= 3 ? nb_min - 2 : 0;
+        if (32 * task + 31 >= n && nbulk > 0) --nbulk;
         const uint32_t o = s & 15;
         uint32_t H[5] = {0x67452301u, 0xEFCDAB89u, 0x98BADCFEu, 0x10325476u, 0xC3D2E1F0u};
         uint32_t raw[20];

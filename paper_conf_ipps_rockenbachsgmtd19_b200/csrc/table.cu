@@ -196,6 +196,7 @@ __global__ void p2p_insert_kernel(const TableView* __restrict__ views, uint32_t 
 #pragma unroll
         for (int i = 0; i < 5; ++i) key[i] = rec[i];
         const uint64_t myid = *reinterpret_cast<const uint64_t*>(rec + 6);
+        DD_CHECK(owner_of_key(key[0], G) < G);
         const TableView t = views[owner_of_key(key[0], G)];
         uint64_t idx = (((uint64_t)key[2] << 32) | key[1]) & t.mask;
         uint32_t found = 0xFFFFFFFFu;
@@ -247,6 +248,7 @@ __global__ void p2p_lookup_kernel(const TableView* __restrict__ views, uint32_t 
         const uint32_t si = slot_idx[r];
         const TableView t =
             views[owner_of_key(*reinterpret_cast<const uint32_t*>(send + 32 * r), G)];
+        DD_CHECK(si == 0xFFFFFFFFu || si <= t.mask);
         reply_back[r] = si == 0xFFFFFFFFu ? ~0ull : ~t.slots[si].inv_min;
     }
 }

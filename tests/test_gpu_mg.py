@@ -86,8 +86,8 @@ def test_mg_loopback_device_matches_oracle(G, depth, transport):
     assert st["dup_chunks"] == sum(int(w.is_dup.sum()) for w in want)
 
 
-@pytest.mark.parametrize("G", [2, 5])
-def test_mg_loopback_host_fed_matches_oracle(G):
+@pytest.mark.parametrize("G,transport", [(2, 2), (5, 2), (3, 3)])
+def test_mg_loopback_host_fed_matches_oracle(G, transport):
     """Host items (dedup_submit_batch, pinned and pageable buffers) through G
     ranks, submissions of several batches per call and drains in between
     (partial waves padded with empty batches)."""
@@ -95,7 +95,7 @@ def test_mg_loopback_host_fed_matches_oracle(G):
     data, off = ragged_stream(6 * MiB, seed=200 + G)
     items = U.items_of(data, off)
     got = []
-    with mg(G, 3, host_fed=True) as d:
+    with mg(G, 3, host_fed=True, transport=transport) as d:
         pin = d.host_empty(len(data))
         pin[:] = data
         k = 0
